@@ -1,0 +1,125 @@
+/*
+ * include/ipt.h -- C ABI of the B200 (sm_100a) decomposed in-place transpose.
+ *
+ * Method: Catanzaro, Keller, Garland, "A Decomposition for In-place Matrix
+ * Transposition", PPoPP'14.  Citations are PAPER.md lines + equation/section.
+ *
+ * Every entry point is asynchronous on `stream` (a cudaStream_t of the current device,
+ * passed as void* so that this header needs no CUDA include; NULL = legacy default
+ * stream).  Arguments are validated synchronously before anything is enqueued; an
+ * argument error leaves the buffer untouched.  No entry point allocates device memory
+ * that outlives the call, throws, or synchronises the stream.  All entry points are
+ * thread-safe and reentrant.
+ *
+ * Memory: `ptr` is caller-owned device memory on the current device, aligned to
+ * elem_bytes (16-byte alignment is NOT required).  The caller must not read or write it
+ * until the stream reaches the end of the call.  The operation is not atomic: if a
+ * launch fails mid-sequence (IPT_ERR_CUDA) the buffer content is unspecified.
+ *
+ * Element size: elem_bytes in {4, 8, 16}.  Elements are opaque words (bit-exact moves,
+ * no floating-point semantics; NaN payloads, -0.0 and subnormals are preserved).
+ */
+#ifndef IPT_H_
+#define IPT_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    IPT_ROW_MAJOR = 0, /* element (i, j) of the m x n matrix at offset i*n + j (Eq. 1, :85)  */
+    IPT_COL_MAJOR = 1  /* element (i, j) of the m x n matrix at offset i + j*m (Eq. 4, :99)  */
+} ipt_layout_t;
+
+typedef enum {
+    IPT_OK = 0,
+    IPT_ERR_INVALID_ARGUMENT = 1, /* negative dims, bad elem_bytes/layout, NULL or misaligned
+                                     ptr, stride < m*n, size overflow; buffer untouched      */
+    IPT_ERR_UNSUPPORTED = 2,      /* shape beyond the implemented on-chip staging limits, or
+                                     the device is not sm_100; buffer untouched              */
+    IPT_ERR_OUT_OF_MEMORY = 3,    /* scratch allocation failed; buffer untouched            */
+    IPT_ERR_CUDA = 4              /* a launch failed; buffer contents unspecified            */
+} ipt_status_t;
+
+/*
+ * ipt_c2r -- in-place transpose.
+ *   In:  an m x n matrix stored in `layout` at ptr.
+ *   Out: its n x m transpose, stored in the same layout, in the same memory.
+ * Row-major input is the paper's C2R (Theorem 1: "The C2R transpose
+ * implements transposition for row-major arrays"); column-major input swaps m and n
+ * (Theorem 2, :227-255).  Internally the library runs the decomposed algorithm
+ * (Algorithm 1, :569-599; gather forms §4.2-4.3, :669-743) on whichever engine the
+ * heuristic of :959 selects (C2R if the array has more rows than columns, else R2C; both
+ * induce the same permutation, Theorem 2/7).  Passes: [column rotation if gcd > 1]
+ * (Eq. 23), row shuffle (Eq. 31 / 24), column shuffle (Eq. 26 = p_j o q, Eqs. 32-33).
+ * Auxiliary space: O(max(m, n)) elements per worker (Theorem 6, :605), on chip; see
+ * ipt_scratch_bytes.  m or n in {0, 1} is the identity: IPT_OK, nothing enqueued.
+ */
+ipt_status_t ipt_c2r(void *ptr, int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
+                     void *stream);
+
+/*
+ * ipt_r2c -- the exact inverse of ipt_c2r with the same arguments ("The R2C
+ * and C2R transposes are inverses of each other"; :603).  In: the n x m matrix produced
+ * by ipt_c2r(ptr, m, n, elem_bytes, layout); out: the original m x n matrix.
+ */
+ipt_status_t ipt_r2c(void *ptr, int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
+                     void *stream);
+
+/*
+ * Batched variants: `batch` independent matrices, matrix k at
+ * (char*)base + k * stride_elems * elem_bytes, stride_elems >= m*n.  One plan, one launch
+ * per pass for the whole batch (the paper's rows and columns are independent units,
+ * Theorem 4, :479; batches add a third independent axis).  Matrices must not overlap.
+ */
+ipt_status_t ipt_c2r_batched(void *base, int64_t batch, int64_t stride_elems, int64_t m,
+                             int64_t n, int elem_bytes, ipt_layout_t layout, void *stream);
+ipt_status_t ipt_r2c_batched(void *base, int64_t batch, int64_t stride_elems, int64_t m,
+                             int64_t n, int elem_bytes, ipt_layout_t layout, void *stream);
+
+/*
+ * Skinny AoS <-> SoA conversion (§6.1).  An Array of Structures of
+ * `count` structs, each of `fields` fields of field_bytes bytes, is a row-major
+ * count x fields array; ipt_aos_to_soa transposes it in place into `fields` arrays of
+ * `count` (the Structure of Arrays).  ipt_soa_to_aos is the exact inverse.  Equivalent to
+ * ipt_c2r / ipt_r2c(ptr, count, fields, field_bytes, IPT_ROW_MAJOR, stream), routed to the
+ * specialised skinny engine when fields <= 32.
+ */
+ipt_status_t ipt_aos_to_soa(void *ptr, int64_t count, int64_t fields, int field_bytes,
+                            void *stream);
+ipt_status_t ipt_soa_to_aos(void *ptr, int64_t count, int64_t fields, int field_bytes,
+                            void *stream);
+
+/*
+ * Auxiliary-space statement for ipt_c2r(m, n, elem_bytes, ...) (Theorem 6, PAPER.md:605:
+ * O(max(m, n)) auxiliary space).  *global_bytes: device scratch the call allocates
+ * (stream-ordered, freed before the call's work completes); *onchip_per_cta: the largest
+ * shared-memory staging buffer of any launched CTA.  Either pointer may be NULL.
+ */
+ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *global_bytes,
+                               size_t *onchip_per_cta);
+
+/* Static description of a status code. */
+const char *ipt_status_string(ipt_status_t s);
+
+/*
+ * Introspection for tests and benchmarks (no side effects).  Fills `out` with the plan
+ * the library would run for ipt_c2r(m, n, elem_bytes, layout): out[0] engine (0 none,
+ * 1 C2R, 2 R2C, 3 skinny), out[1] M (engine rows), out[2] N (engine columns), out[3] c =
+ * gcd(M, N), out[4] number of kernel launches, out[5] column-tile cluster size, out[6]
+ * column-tile width in elements.  Returns IPT_ERR_UNSUPPORTED for shapes beyond limits.
+ */
+ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
+                           int64_t out[8]);
+
+/* Number of kernel launches this library has enqueued since load (all threads). */
+uint64_t ipt_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* IPT_H_ */

@@ -1,0 +1,153 @@
+"""B200-native decomposed in-place transpose (Catanzaro, Keller, Garland, PPoPP'14).
+
+Thin Python binding of the C ABI in include/ipt.h: argument marshalling only.  Every
+step of the transpose runs in the CUDA kernels of libipt.so (built in-tree for sm_100a
+by __graft_entry__.build()).  There is no CPU fallback: importing this package without
+the built library raises.
+
+Buffers are torch CUDA tensors (any dtype; elem_bytes defaults to the element size, so
+complex128 carries 16-byte elements) or raw device pointers (int).  Calls are
+asynchronous on the given stream (default: torch's current stream of the tensor's
+device).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libipt.so")
+
+ROW_MAJOR = 0
+COL_MAJOR = 1
+_LAYOUTS = {"row": ROW_MAJOR, "col": COL_MAJOR, ROW_MAJOR: ROW_MAJOR, COL_MAJOR: COL_MAJOR}
+
+STATUS = {0: "IPT_OK", 1: "IPT_ERR_INVALID_ARGUMENT", 2: "IPT_ERR_UNSUPPORTED",
+          3: "IPT_ERR_OUT_OF_MEMORY", 4: "IPT_ERR_CUDA"}
+
+# Every symbol declared in include/ipt.h.
+EXPORTS = ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
+           "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_status_string", "ipt_plan_info",
+           "ipt_launch_count")
+
+
+class IptError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        super().__init__(f"{where}: {STATUS.get(status, status)}")
+        self.status = status
+
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() (nvcc, sm_100a). "
+                      "There is no CPU fallback.")
+
+_lib = ctypes.CDLL(LIB_PATH)
+_i64, _int, _vp = ctypes.c_int64, ctypes.c_int, ctypes.c_void_p
+_lib.ipt_c2r.argtypes = [_vp, _i64, _i64, _int, _int, _vp]
+_lib.ipt_r2c.argtypes = [_vp, _i64, _i64, _int, _int, _vp]
+_lib.ipt_c2r_batched.argtypes = [_vp, _i64, _i64, _i64, _i64, _int, _int, _vp]
+_lib.ipt_r2c_batched.argtypes = [_vp, _i64, _i64, _i64, _i64, _int, _int, _vp]
+_lib.ipt_aos_to_soa.argtypes = [_vp, _i64, _i64, _int, _vp]
+_lib.ipt_soa_to_aos.argtypes = [_vp, _i64, _i64, _int, _vp]
+_lib.ipt_scratch_bytes.argtypes = [_i64, _i64, _int, ctypes.POINTER(ctypes.c_size_t), ctypes.POINTER(ctypes.c_size_t)]
+_lib.ipt_status_string.argtypes = [_int]
+_lib.ipt_status_string.restype = ctypes.c_char_p
+_lib.ipt_plan_info.argtypes = [_i64, _i64, _int, _int, ctypes.POINTER(_i64)]
+_lib.ipt_launch_count.argtypes = []
+_lib.ipt_launch_count.restype = ctypes.c_uint64
+for _f in ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
+           "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_plan_info"):
+    getattr(_lib, _f).restype = _int
+
+
+def library() -> ctypes.CDLL:
+    return _lib
+
+
+def _ptr_eb_stream(buf, elem_bytes, stream):
+    """(device pointer, element bytes, stream handle) of a tensor or raw pointer."""
+    if isinstance(buf, int):
+        if elem_bytes is None:
+            raise ValueError("elem_bytes is required with a raw pointer")
+        ptr, eb, dev = buf, elem_bytes, None
+    else:
+        if not buf.is_cuda:
+            raise ValueError("buffer must be a CUDA tensor (no CPU fallback)")
+        if not buf.is_contiguous():
+            raise ValueError("buffer must be contiguous")
+        ptr, dev = buf.data_ptr(), buf.device
+        eb = elem_bytes if elem_bytes is not None else buf.element_size()
+    if stream is None:
+        import torch
+        stream = torch.cuda.current_stream(dev).cuda_stream
+    elif not isinstance(stream, int):
+        stream = stream.cuda_stream
+    return ptr, eb, stream
+
+
+def _check(status: int, where: str):
+    if status != 0:
+        raise IptError(status, where)
+
+
+def c2r(buf, m: int, n: int, elem_bytes: int | None = None, layout="row", stream=None):
+    """In place: the m x n matrix in `layout` becomes its n x m transpose (same layout)."""
+    p, eb, st = _ptr_eb_stream(buf, elem_bytes, stream)
+    _check(_lib.ipt_c2r(p, m, n, eb, _LAYOUTS[layout], st), "ipt_c2r")
+    return buf
+
+
+def r2c(buf, m: int, n: int, elem_bytes: int | None = None, layout="row", stream=None):
+    """Exact inverse of c2r with the same arguments."""
+    p, eb, st = _ptr_eb_stream(buf, elem_bytes, stream)
+    _check(_lib.ipt_r2c(p, m, n, eb, _LAYOUTS[layout], st), "ipt_r2c")
+    return buf
+
+
+def c2r_batched(buf, batch: int, stride_elems: int, m: int, n: int, elem_bytes: int | None = None,
+                layout="row", stream=None):
+    p, eb, st = _ptr_eb_stream(buf, elem_bytes, stream)
+    _check(_lib.ipt_c2r_batched(p, batch, stride_elems, m, n, eb, _LAYOUTS[layout], st), "ipt_c2r_batched")
+    return buf
+
+
+def r2c_batched(buf, batch: int, stride_elems: int, m: int, n: int, elem_bytes: int | None = None,
+                layout="row", stream=None):
+    p, eb, st = _ptr_eb_stream(buf, elem_bytes, stream)
+    _check(_lib.ipt_r2c_batched(p, batch, stride_elems, m, n, eb, _LAYOUTS[layout], st), "ipt_r2c_batched")
+    return buf
+
+
+def aos_to_soa(buf, count: int, fields: int, field_bytes: int | None = None, stream=None):
+    p, eb, st = _ptr_eb_stream(buf, field_bytes, stream)
+    _check(_lib.ipt_aos_to_soa(p, count, fields, eb, st), "ipt_aos_to_soa")
+    return buf
+
+
+def soa_to_aos(buf, count: int, fields: int, field_bytes: int | None = None, stream=None):
+    p, eb, st = _ptr_eb_stream(buf, field_bytes, stream)
+    _check(_lib.ipt_soa_to_aos(p, count, fields, eb, st), "ipt_soa_to_aos")
+    return buf
+
+
+def scratch_bytes(m: int, n: int, elem_bytes: int):
+    g, o = ctypes.c_size_t(), ctypes.c_size_t()
+    _check(_lib.ipt_scratch_bytes(m, n, elem_bytes, ctypes.byref(g), ctypes.byref(o)), "ipt_scratch_bytes")
+    return int(g.value), int(o.value)
+
+
+def plan_info(m: int, n: int, elem_bytes: int, layout="row"):
+    out = (_i64 * 8)()
+    _check(_lib.ipt_plan_info(m, n, elem_bytes, _LAYOUTS[layout], out), "ipt_plan_info")
+    keys = ("engine", "M", "N", "c", "launches", "cluster", "tile_w", "onchip_bytes")
+    d = dict(zip(keys, (int(v) for v in out)))
+    d["engine"] = {0: "none", 1: "c2r", 2: "r2c", 3: "skinny"}[d["engine"]]
+    return d
+
+
+def launch_count() -> int:
+    return int(_lib.ipt_launch_count())
+
+
+def status_string(s: int) -> str:
+    return _lib.ipt_status_string(s).decode()

@@ -1,0 +1,350 @@
+// C ABI (include/ipt.h): argument validation, the host planner and pass dispatch.
+//
+// Planner:
+//  * export + layout -> buffer permutation P_{x,y} ("transpose the row-major x-by-y
+//    buffer"), Theorems 1-2, reading C18;
+//  * engine: C2R(M=x, N=y) if x > y, else R2C(M=y, N=x) -- the paper's heuristic "if
+//    m > n, use the C2R algorithm, otherwise use the R2C algorithm" (:959, reading C11):
+//    the row length N = min(x, y) is the dimension staged on chip;
+//  * constants c = gcd, a, b (:275-277), a^{-1} = mmi(a, b), b^{-1} = mmi(b, a)
+//    (:673-685, :719), strength-reduced divisors (§4.4, :745-749);
+//  * pass list and launch geometry (row kernel, column-tile cluster size K and width W).
+#include <atomic>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+
+#include "ipt.h"
+#include "plan.h"
+
+namespace ipt {
+namespace {
+
+std::atomic<uint64_t> g_launches{0};
+
+struct DevInfo {
+    int ok = 0;
+    int sms = 0, smem_optin = 0, major = 0, minor = 0;
+};
+
+DevInfo device_info() {
+    static std::mutex mu;
+    static DevInfo cache[64];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) {
+        cudaGetLastError();
+        return DevInfo{};
+    }
+    std::lock_guard<std::mutex> lk(mu);
+    DevInfo &d = cache[dev];
+    if (!d.ok) {
+        cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaDeviceGetAttribute(&d.smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        cudaDeviceGetAttribute(&d.major, cudaDevAttrComputeCapabilityMajor, dev);
+        cudaDeviceGetAttribute(&d.minor, cudaDevAttrComputeCapabilityMinor, dev);
+        d.ok = cudaGetLastError() == cudaSuccess ? 1 : 0;
+    }
+    return d;
+}
+
+int64_t gcd64(int64_t x, int64_t y) {
+    while (y) {
+        int64_t t = x % y;
+        x = y;
+        y = t;
+    }
+    return x;
+}
+
+// Modular multiplicative inverse; mmi(x, 1) = 0.
+int64_t mmi64(int64_t x, int64_t y) {
+    if (y == 1) return 0;
+    int64_t r0 = y, r1 = x % y, t0 = 0, t1 = 1;
+    while (r1) {
+        int64_t q = r0 / r1, t;
+        t = r0 - q * r1; r0 = r1; r1 = t;
+        t = t0 - q * t1; t0 = t1; t1 = t;
+    }
+    t0 %= y;
+    return t0 < 0 ? t0 + y : t0;
+}
+
+int env_int(const char *name, int dflt) {
+    const char *v = std::getenv(name);
+    return v && *v ? std::atoi(v) : dflt;
+}
+
+struct ColPlan {
+    ColParams p;
+    size_t smem = 0;
+    int mode = 0;
+};
+
+struct Plan {
+    int engine = ENG_NONE;
+    int64_t M = 0, N = 0, c = 1, a = 1, b = 1;
+    int eb = 4;
+    RowParams row{};
+    int row_dir = 0;
+    ColPlan shuf, rot;
+    bool has_rot = false;
+    int nlaunch = 0;
+    size_t onchip = 0;
+};
+
+int ilog2(int v) {
+    int l = 0;
+    while ((1 << l) < v) ++l;
+    return l;
+}
+
+// Column-tile geometry: the smallest cluster (K <= 16) whose CTAs can each stage their
+// band of the M x W tile; the width starts at IPT_TILE_BYTES (default 32 B = one sector)
+// and halves if no cluster fits.
+ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp) {
+    int tile_bytes = env_int("IPT_TILE_BYTES", 32);
+    if (tile_bytes < pl.eb) tile_bytes = pl.eb;
+    for (int W = tile_bytes / pl.eb; W >= 1; W /= 2) {
+        if (W & (W - 1)) continue;
+        for (int K = 1; K <= 16; ++K) {
+            const int64_t B = (pl.M + K - 1) / K;
+            const size_t smem = col_smem_bytes(B, W, pl.eb);
+            if (smem > static_cast<size_t>(dev.smem_optin)) continue;
+            if (K > 1 && col_max_active_clusters(mode, pl.eb, K, smem) < 1) continue;
+            ColParams &p = cp.p;
+            std::memset(&p, 0, sizeof(p));
+            p.M = static_cast<int32_t>(pl.M);
+            p.N = static_cast<int32_t>(pl.N);
+            p.c = static_cast<int32_t>(pl.c);
+            p.a = static_cast<int32_t>(pl.a);
+            p.b = static_cast<int32_t>(pl.b);
+            p.binv = static_cast<int32_t>(mmi64(pl.b, pl.a));
+            p.fd_c = make_fastdiv(static_cast<uint32_t>(pl.c));
+            p.fd_a = make_fastdiv(static_cast<uint32_t>(pl.a));
+            p.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
+            p.fd_M = make_fastdiv(static_cast<uint32_t>(pl.M));
+            p.W = W;
+            p.log2W = ilog2(W);
+            p.ntiles = static_cast<int32_t>((pl.N + W - 1) / W);
+            p.K = K;
+            p.B = static_cast<int32_t>(B);
+            p.rot_sign = 1;
+            p.wide_a = pl.a >= 65536 ? 1 : 0;
+            cp.smem = smem;
+            cp.mode = mode;
+            return IPT_OK;
+        }
+    }
+    return IPT_ERR_UNSUPPORTED;
+}
+
+// P_{x,y} on `batch` matrices.
+ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
+    pl = Plan{};
+    pl.eb = eb;
+    if (x <= 1 || y <= 1) return IPT_OK;  // P_{1,y} and P_{x,1} are the identity
+    const DevInfo dev = device_info();
+    if (!dev.ok) return IPT_ERR_CUDA;
+    if (dev.major != 10 || dev.minor != 0) return IPT_ERR_UNSUPPORTED;  // sm_100 only
+
+    int engine = x > y ? ENG_C2R : ENG_R2C;
+    const char *force = std::getenv("IPT_FORCE_ENGINE");
+    if (force && !std::strcmp(force, "c2r")) engine = ENG_C2R;
+    if (force && !std::strcmp(force, "r2c")) engine = ENG_R2C;
+    pl.engine = engine;
+    pl.M = engine == ENG_C2R ? x : y;  // C2R(x, y) = P_{x,y} = R2C(y, x)
+    pl.N = engine == ENG_C2R ? y : x;
+    if (pl.M >= (int64_t(1) << 31) || pl.N >= (int64_t(1) << 31)) return IPT_ERR_UNSUPPORTED;
+    pl.c = gcd64(pl.M, pl.N);
+    pl.a = pl.M / pl.c;
+    pl.b = pl.N / pl.c;
+
+    // Row pass: the whole row must fit one CTA's shared memory.
+    const size_t rsm = row_smem_bytes(pl.N, eb);
+    if (rsm > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
+    RowParams &rp = pl.row;
+    std::memset(&rp, 0, sizeof(rp));
+    rp.M = static_cast<int32_t>(pl.M);
+    rp.N = static_cast<int32_t>(pl.N);
+    rp.c = static_cast<int32_t>(pl.c);
+    rp.a = static_cast<int32_t>(pl.a);
+    rp.b = static_cast<int32_t>(pl.b);
+    rp.ainv = static_cast<int32_t>(mmi64(pl.a, pl.b));
+    rp.amodb = static_cast<int32_t>(pl.a % pl.b);
+    rp.fd_c = make_fastdiv(static_cast<uint32_t>(pl.c));
+    rp.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
+    rp.wide = pl.b >= 65536 ? 1 : 0;
+    pl.row_dir = engine == ENG_C2R ? ROW_C2R : ROW_R2C;
+
+    ipt_status_t s = plan_col(dev, pl, engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.shuf);
+    if (s != IPT_OK) return s;
+    pl.onchip = rsm > pl.shuf.smem ? rsm : pl.shuf.smem;
+    pl.nlaunch = 2;
+    if (pl.c > 1) {
+        s = plan_col(dev, pl, COL_ROT, pl.rot);
+        if (s != IPT_OK) return s;
+        pl.rot.p.rot_sign = engine == ENG_C2R ? 1 : -1;
+        pl.has_rot = true;
+        pl.nlaunch = 3;
+        if (pl.rot.smem > pl.onchip) pl.onchip = pl.rot.smem;
+    }
+    return IPT_OK;
+}
+
+ipt_status_t check(cudaError_t e) {
+    if (e == cudaSuccess) return IPT_OK;
+    cudaGetLastError();
+    return IPT_ERR_CUDA;
+}
+
+ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_bytes, cudaStream_t st) {
+    if (pl0.engine == ENG_NONE || batch == 0) return IPT_OK;
+    Plan pl = pl0;
+    pl.row.base = base;
+    pl.row.batch = batch;
+    pl.row.mat_stride_bytes = stride_bytes;
+    for (ColPlan *cp : {&pl.shuf, &pl.rot}) {
+        cp->p.base = base;
+        cp->p.batch = batch;
+        cp->p.mat_stride_bytes = stride_bytes;
+    }
+    // IPT_DEBUG_PASSES=k (tests only): stop after the first k passes, so that each pass
+    // can be compared with the oracle's snapshot of the same step.
+    int budget = env_int("IPT_DEBUG_PASSES", 1 << 30);
+    auto run = [&](auto &&launch) -> ipt_status_t {
+        if (budget-- <= 0) return IPT_OK;
+        ipt_status_t s = check(launch());
+        if (s == IPT_OK) g_launches++;
+        return s;
+    };
+    auto rot = [&] { return launch_col(pl.rot.p, COL_ROT, pl.eb, st, pl.rot.smem); };
+    auto row = [&] { return launch_row(pl.row, pl.row_dir, pl.eb, st); };
+    ipt_status_t s;
+    if (pl.engine == ENG_C2R) {
+        auto shuf = [&] { return launch_col(pl.shuf.p, COL_C2R_SHUF, pl.eb, st, pl.shuf.smem); };
+        if (pl.has_rot && (s = run(rot)) != IPT_OK) return s;  // Eq. 23 pre-rotation
+        if ((s = run(row)) != IPT_OK) return s;                  // Eq. 31 row gather
+        if ((s = run(shuf)) != IPT_OK) return s;                 // Eq. 26 = p_j o q
+    } else {
+        auto shuf = [&] { return launch_col(pl.shuf.p, COL_R2C_SHUF, pl.eb, st, pl.shuf.smem); };
+        if ((s = run(shuf)) != IPT_OK) return s;                 // Eqs. 34-35
+        if ((s = run(row)) != IPT_OK) return s;                  // Eq. 24 row gather
+        if (pl.has_rot && (s = run(rot)) != IPT_OK) return s;  // Eq. 36 post-rotation
+    }
+    return IPT_OK;
+}
+
+bool valid_eb(int eb) { return eb == 4 || eb == 8 || eb == 16; }
+
+// Validate and run P_{x,y} on `batch` matrices of x*y elements, `stride` elements apart.
+// stride < 0 means "packed" (stride = x*y), used by the single-matrix entry points.
+ipt_status_t run_perm(void *ptr, int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, void *stream) {
+    if (!valid_eb(eb) || x < 0 || y < 0 || batch < 0) return IPT_ERR_INVALID_ARGUMENT;
+    if (x != 0 && y > INT64_MAX / x) return IPT_ERR_INVALID_ARGUMENT;
+    const int64_t elems = x * y;
+    if (stride < 0) stride = elems;
+    if (stride < elems) return IPT_ERR_INVALID_ARGUMENT;
+    if (stride != 0 && batch > INT64_MAX / stride) return IPT_ERR_INVALID_ARGUMENT;
+    if (elems != 0 && batch * stride > INT64_MAX / eb) return IPT_ERR_INVALID_ARGUMENT;
+    if (elems == 0 || batch == 0) return IPT_OK;
+    if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % static_cast<uintptr_t>(eb) != 0)
+        return IPT_ERR_INVALID_ARGUMENT;
+    Plan pl;
+    ipt_status_t s = make_plan(x, y, eb, pl);
+    if (s != IPT_OK) return s;
+    return execute(pl, static_cast<char *>(ptr), batch, stride * eb, static_cast<cudaStream_t>(stream));
+}
+
+// Export -> P_{x,y} (reading C18): c2r(m,n,ROW) = P_{m,n}, c2r(m,n,COL) = P_{n,m};
+// r2c is the inverse: r2c(m,n,ROW) = P_{n,m}, r2c(m,n,COL) = P_{m,n}.
+bool perm_of(bool c2r, int64_t m, int64_t n, int layout, int64_t &x, int64_t &y) {
+    if (layout != IPT_ROW_MAJOR && layout != IPT_COL_MAJOR) return false;
+    const bool mn = (c2r == (layout == IPT_ROW_MAJOR));
+    x = mn ? m : n;
+    y = mn ? n : m;
+    return true;
+}
+
+}  // namespace
+}  // namespace ipt
+
+using namespace ipt;
+
+extern "C" {
+
+ipt_status_t ipt_c2r(void *ptr, int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout, void *stream) {
+    int64_t x, y;
+    if (!perm_of(true, m, n, layout, x, y)) return IPT_ERR_INVALID_ARGUMENT;
+    return run_perm(ptr, 1, -1, x, y, elem_bytes, stream);
+}
+
+ipt_status_t ipt_r2c(void *ptr, int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout, void *stream) {
+    int64_t x, y;
+    if (!perm_of(false, m, n, layout, x, y)) return IPT_ERR_INVALID_ARGUMENT;
+    return run_perm(ptr, 1, -1, x, y, elem_bytes, stream);
+}
+
+ipt_status_t ipt_c2r_batched(void *base, int64_t batch, int64_t stride_elems, int64_t m, int64_t n, int elem_bytes,
+                             ipt_layout_t layout, void *stream) {
+    int64_t x, y;
+    if (stride_elems < 0 || !perm_of(true, m, n, layout, x, y)) return IPT_ERR_INVALID_ARGUMENT;
+    return run_perm(base, batch, stride_elems, x, y, elem_bytes, stream);
+}
+
+ipt_status_t ipt_r2c_batched(void *base, int64_t batch, int64_t stride_elems, int64_t m, int64_t n, int elem_bytes,
+                             ipt_layout_t layout, void *stream) {
+    int64_t x, y;
+    if (stride_elems < 0 || !perm_of(false, m, n, layout, x, y)) return IPT_ERR_INVALID_ARGUMENT;
+    return run_perm(base, batch, stride_elems, x, y, elem_bytes, stream);
+}
+
+ipt_status_t ipt_aos_to_soa(void *ptr, int64_t count, int64_t fields, int field_bytes, void *stream) {
+    return run_perm(ptr, 1, -1, count, fields, field_bytes, stream);  // P_{count,fields}
+}
+
+ipt_status_t ipt_soa_to_aos(void *ptr, int64_t count, int64_t fields, int field_bytes, void *stream) {
+    return run_perm(ptr, 1, -1, fields, count, field_bytes, stream);  // P_{fields,count}
+}
+
+ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *global_bytes, size_t *onchip_per_cta) {
+    if (!valid_eb(elem_bytes) || m < 0 || n < 0) return IPT_ERR_INVALID_ARGUMENT;
+    Plan pl;
+    ipt_status_t s = make_plan(m, n, elem_bytes, pl);
+    if (s != IPT_OK) return s;
+    if (global_bytes) *global_bytes = 0;
+    if (onchip_per_cta) *onchip_per_cta = pl.onchip;
+    return IPT_OK;
+}
+
+ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout, int64_t out[8]) {
+    int64_t x, y;
+    if (!out || !valid_eb(elem_bytes) || m < 0 || n < 0 || !perm_of(true, m, n, layout, x, y))
+        return IPT_ERR_INVALID_ARGUMENT;
+    Plan pl;
+    ipt_status_t s = make_plan(x, y, elem_bytes, pl);
+    if (s != IPT_OK) return s;
+    out[0] = pl.engine;
+    out[1] = pl.M;
+    out[2] = pl.N;
+    out[3] = pl.c;
+    out[4] = pl.nlaunch;
+    out[5] = pl.engine ? pl.shuf.p.K : 0;
+    out[6] = pl.engine ? pl.shuf.p.W : 0;
+    out[7] = static_cast<int64_t>(pl.onchip);
+    return IPT_OK;
+}
+
+uint64_t ipt_launch_count(void) { return g_launches.load(); }
+
+const char *ipt_status_string(ipt_status_t s) {
+    switch (s) {
+        case IPT_OK: return "IPT_OK";
+        case IPT_ERR_INVALID_ARGUMENT: return "IPT_ERR_INVALID_ARGUMENT";
+        case IPT_ERR_UNSUPPORTED: return "IPT_ERR_UNSUPPORTED";
+        case IPT_ERR_OUT_OF_MEMORY: return "IPT_ERR_OUT_OF_MEMORY";
+        case IPT_ERR_CUDA: return "IPT_ERR_CUDA";
+        default: return "IPT_UNKNOWN_STATUS";
+    }
+}
+
+}  // extern "C"

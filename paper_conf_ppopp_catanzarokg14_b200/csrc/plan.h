@@ -1,0 +1,72 @@
+// Host planner and kernel parameter blocks of the CUDA path.
+//
+// An engine works on the buffer viewed as an M x N row-major array (rows of N contiguous
+// elements).  c = gcd(M, N), a = M / c, b = N / c.
+//   C2R(M, N) realises P_{M,N} ("transpose the row-major M x N buffer", Theorem 1):
+//       [column rotation r_j, Eq. 23, if c > 1] -> row gather d'^{-1}_i (Eq. 31)
+//       -> column gather s'_j = p_j o q (Eqs. 26, 32, 33)
+//   R2C(M, N) realises P_{N,M} = P_{M,N}^{-1} (§4.3):
+//       column gather q^{-1}((i - j) mod M) (Eqs. 34, 35) -> row gather d'_i (Eq. 24)
+//       -> [column rotation r^{-1}_j, Eq. 36, if c > 1]
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+
+namespace ipt {
+
+enum Engine : int { ENG_NONE = 0, ENG_C2R = 1, ENG_R2C = 2, ENG_SKINNY = 3 };
+
+// Column-tile kernel modes.
+enum ColMode : int {
+    COL_ROT = 0,       // out[i][j] = in[(i + sign*floor(j/b)) mod M][j]   (Eq. 23 / Eq. 36)
+    COL_C2R_SHUF = 1,  // out[i][j] = in[(j + q(i)) mod M][j]              (Eq. 26 = p_j o q)
+    COL_R2C_SHUF = 2,  // out[i][j] = in[q^{-1}((i - j) mod M)][j]         (Eqs. 34, 35)
+};
+
+// Row-shuffle directions.
+enum RowDir : int {
+    ROW_C2R = 0,  // out[i][j] = in[i][d'^{-1}_i(j)]  (Eq. 31)
+    ROW_R2C = 1,  // out[i][j] = in[i][d'_i(j)]       (Eq. 24 as a gather, §4.3 :717)
+};
+
+struct RowParams {
+    char *base;
+    int64_t mat_stride_bytes;  // distance between matrices of a batch
+    int64_t batch;
+    int32_t M, N, c, a, b;
+    int32_t ainv;   // mmi(a, b)
+    int32_t amodb;  // a mod b
+    FastDiv fd_c, fd_b;
+    int32_t wide;   // b >= 2^16: products need 64 bits
+};
+
+struct ColParams {
+    char *base;
+    int64_t mat_stride_bytes;
+    int64_t batch;
+    int32_t M, N, c, a, b;
+    int32_t binv;   // mmi(b, a)
+    FastDiv fd_c, fd_a, fd_b, fd_M;
+    int32_t W, log2W;   // tile width in elements (power of two)
+    int32_t ntiles;     // ceil(N / W)
+    int32_t K;          // cluster size (CTAs per tile)
+    int32_t B;          // rows per CTA band: ceil(M / K)
+    int32_t rot_sign;   // COL_ROT: +1 (C2R pre-rotation) or -1 (R2C post-rotation)
+    int32_t wide_a;     // a >= 2^16
+};
+
+// Launchers (col_tile.cu / row_shuffle.cu).  They return the CUDA error of the launch.
+size_t row_smem_bytes(int64_t N, int eb);
+int row_block_threads();
+cudaError_t launch_row(const RowParams &p, int dir, int eb, cudaStream_t st);
+
+size_t col_smem_bytes(int64_t B, int64_t W, int eb);
+int col_block_threads();
+cudaError_t launch_col(const ColParams &p, int mode, int eb, cudaStream_t st, size_t smem);
+int col_max_active_clusters(int mode, int eb, int K, size_t smem);
+
+}  // namespace ipt

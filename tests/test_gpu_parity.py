@@ -1,0 +1,213 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, bit-exact.
+
+Tolerance is zero: the transpose moves opaque words (north_star: "bit-exact against the
+oracle for every element type, including floats").  Inputs are random bit patterns from
+workloads.py (NaN payloads, -0.0 and subnormals included when viewed as floats).
+"""
+import os
+import random
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+import paper_conf_ppopp_catanzarokg14_b200 as ipt  # noqa: E402
+
+DEV = torch.device("cuda:0")
+
+
+def vwords(host, eb):
+    """numpy view of host words as opaque eb-byte elements."""
+    return np.ascontiguousarray(host).view(np.dtype((np.void, eb))).reshape(-1)
+
+
+def to_dev(host):
+    return torch.from_numpy(np.ascontiguousarray(host).view(np.uint8).reshape(-1).copy()).to(DEV)
+
+
+def dev_bytes(t):
+    return t.cpu().numpy().tobytes()
+
+
+class forced_engine:
+    def __init__(self, eng):
+        self.eng = eng
+
+    def __enter__(self):
+        self.old = os.environ.get("IPT_FORCE_ENGINE")
+        if self.eng:
+            os.environ["IPT_FORCE_ENGINE"] = self.eng
+        else:
+            os.environ.pop("IPT_FORCE_ENGINE", None)
+
+    def __exit__(self, *a):
+        if self.old is None:
+            os.environ.pop("IPT_FORCE_ENGINE", None)
+        else:
+            os.environ["IPT_FORCE_ENGINE"] = self.old
+
+
+class debug_passes:
+    def __init__(self, k):
+        self.k = k
+
+    def __enter__(self):
+        os.environ["IPT_DEBUG_PASSES"] = str(self.k)
+
+    def __exit__(self, *a):
+        os.environ.pop("IPT_DEBUG_PASSES", None)
+
+
+def run_packed(shapes, eb, op, layout, engine, seed):
+    """Pack every shape into one device buffer, run `op` on each slice, compare each slice
+    with the oracle, then run the inverse and compare with the input."""
+    offs, tot = [], 0
+    for m, n in shapes:
+        offs.append(tot)
+        tot += m * n + 3  # gaps between matrices must stay untouched
+    host = workloads.random_words(tot, eb, seed)
+    hv = vwords(host, eb)
+    buf = to_dev(host)
+    base = buf.data_ptr()
+    inv = ipt.r2c if op is ipt.c2r else ipt.c2r
+    with forced_engine(engine):
+        for (m, n), o in zip(shapes, offs):
+            op(base + o * eb, m, n, elem_bytes=eb, layout=layout)
+        got = vwords(buf.cpu().numpy(), eb)
+        oc = oracle.ipt_c2r if op is ipt.c2r else oracle.ipt_r2c
+        for (m, n), o in zip(shapes, offs):
+            want = oc(hv[o:o + m * n], m, n, {"row": oracle.ROW_MAJOR, "col": oracle.COL_MAJOR}[layout])
+            assert got[o:o + m * n].tobytes() == want.tobytes(), (m, n, eb, layout, engine)
+            assert got[o + m * n:o + m * n + 3].tobytes() == hv[o + m * n:o + m * n + 3].tobytes()
+        for (m, n), o in zip(shapes, offs):
+            inv(base + o * eb, m, n, elem_bytes=eb, layout=layout)
+    torch.cuda.synchronize()
+    assert dev_bytes(buf) == np.ascontiguousarray(host).tobytes()
+
+
+@pytest.mark.parametrize("engine", [None, "c2r", "r2c"])
+def test_bruteforce_all_shapes_to_64_fp32(engine):
+    shapes = workloads.small_shapes(64)
+    run_packed(shapes, 4, ipt.c2r, "row", engine, seed=11)
+
+
+@pytest.mark.parametrize("eb", [8, 16])
+@pytest.mark.parametrize("engine", ["c2r", "r2c"])
+def test_bruteforce_shapes_to_40_wide_elements(eb, engine):
+    run_packed(workloads.small_shapes(40), eb, ipt.c2r, "row", engine, seed=eb)
+
+
+@pytest.mark.parametrize("layout", ["row", "col"])
+@pytest.mark.parametrize("op", ["c2r", "r2c"])
+def test_layouts_and_directions(layout, op):
+    shapes = [(m, n) for m in (1, 2, 3, 7, 16, 33, 64, 100) for n in (1, 2, 5, 8, 31, 64, 97)]
+    run_packed(shapes, 4, getattr(ipt, op), layout, None, seed=3)
+    run_packed(shapes, 8, getattr(ipt, op), layout, None, seed=4)
+
+
+@pytest.mark.parametrize("engine", ["c2r", "r2c"])
+def test_config1_matches_algorithm1_and_each_pass(engine):
+    """BASELINE config 1: m=1200, n=1800, 4-byte elements, gcd 600 (pre-rotation)."""
+    m, n, eb = 1200, 1800, 4
+    host = workloads.random_words(m * n, eb, seed=1)
+    want = oracle.c2r_alg1(host, m, n)                       # Algorithm 1
+    assert want.tobytes() == oracle.transpose(host, m, n).tobytes()
+    with forced_engine(engine):
+        x = to_dev(host)
+        ipt.c2r(x, m, n, elem_bytes=eb)
+        assert dev_bytes(x) == want.tobytes()
+        ipt.r2c(x, m, n, elem_bytes=eb)
+        assert dev_bytes(x) == host.tobytes()
+        # per-pass parity against the oracle's §4.2 / §4.3 gather-form snapshots
+        if engine == "c2r":       # C2R(M=1200, N=1800): [r_j], d'^{-1}, p_j o q
+            _, snaps = oracle.c2r_gather_forms(host, m, n, snapshots=True)
+            expect = [snaps[0], snaps[1], snaps[3]]
+        else:                     # R2C(M=1800, N=1200): q^{-1} o p^{-1}, d', [r^{-1}]
+            _, snaps = oracle.r2c_gather_forms(host, n, m, snapshots=True)
+            expect = [snaps[1], snaps[2], snaps[3]]
+        for k, e in enumerate(expect, start=1):
+            x = to_dev(host)
+            with debug_passes(k):
+                ipt.c2r(x, m, n, elem_bytes=eb)
+            assert dev_bytes(x) == e.tobytes(), f"pass {k}"
+
+
+def test_misaligned_base_and_batched_with_gaps():
+    m, n = 37, 91
+    for eb in (4, 8):
+        for shift in (1, 2, 3):  # base not 16-byte aligned
+            batch, stride = 5, m * n + 7
+            tot = shift + batch * stride
+            host = workloads.random_words(tot, eb, seed=shift)
+            hv = vwords(host, eb)
+            x = to_dev(host)
+            ipt.c2r_batched(x.data_ptr() + shift * eb, batch, stride, m, n, elem_bytes=eb)
+            got = vwords(x.cpu().numpy(), eb)
+            want = hv.copy()
+            for k in range(batch):
+                o = shift + k * stride
+                want[o:o + m * n] = oracle.ipt_c2r(hv[o:o + m * n], m, n)
+            assert got.tobytes() == want.tobytes()
+            ipt.r2c_batched(x.data_ptr() + shift * eb, batch, stride, m, n, elem_bytes=eb)
+            assert dev_bytes(x) == np.ascontiguousarray(host).tobytes()
+
+
+def test_two_streams_disjoint_buffers():
+    shapes = [(300, 451), (512, 384)]
+    hosts = [workloads.random_words(m * n, 4, seed=i) for i, (m, n) in enumerate(shapes)]
+    xs = [to_dev(h) for h in hosts]
+    ss = [torch.cuda.Stream(), torch.cuda.Stream()]
+    for _ in range(3):
+        for (m, n), x, s in zip(shapes, xs, ss):
+            with torch.cuda.stream(s):
+                ipt.c2r(x, m, n, elem_bytes=4, stream=s)
+                ipt.r2c(x, m, n, elem_bytes=4, stream=s)
+                ipt.c2r(x, m, n, elem_bytes=4, stream=s)
+    torch.cuda.synchronize()
+    for (m, n), x, h in zip(shapes, xs, hosts):
+        assert dev_bytes(x) == oracle.transpose(h, m, n).tobytes()
+
+
+def test_degenerate_shapes():
+    """m or n = 1: identity; m = n: textbook swap; n | m (b = 1) and m | n (a = 1)."""
+    shapes = [(1, 1), (1, 500), (500, 1), (2, 2), (97, 97), (256, 256), (1000, 10), (10, 1000),
+              (4096, 64), (64, 4096), (2, 3000), (3000, 2), (6, 4), (4, 6), (1024, 1023), (1023, 1024)]
+    for eb in (4, 8, 16):
+        run_packed(shapes, eb, ipt.c2r, "row", None, seed=eb + 100)
+
+
+def _sampled_check(got_words, host_words, m, n, samples, rng):
+    """Check sampled outputs one by one with the oracle's Eqs. 7-8 source function:
+    ipt_c2r(m, n, ROW) is the C2R of the m x n buffer (Theorem 1), so output element
+    l = i*n + j (Eq. 1) holds input element s(i,j)*n + c(i,j) (Eq. 11)."""
+    for _ in range(samples):
+        l = rng.randrange(m * n)
+        i, j = divmod(l, n)                 # C2R output position on the m x n view
+        si, sj = oracle.c2r_source(m, n, i, j)
+        assert got_words[l] == host_words[si * n + sj], (m, n, l)
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_sweep_shapes_full_size(eb):
+    """Config-2 shapes at full size (the bench workload): full comparison with the oracle's
+    plain transpose for the first shapes, sampled one-by-one checks for the rest."""
+    rng = random.Random(eb)
+    for k, (m, n) in enumerate(workloads.sweep_shapes(6)):
+        host = workloads.random_words(m * n, eb, seed=k)
+        x = to_dev(host)
+        ipt.c2r(x, m, n, elem_bytes=eb)
+        got = x.cpu().numpy().view(host.dtype)
+        if k < 2:
+            assert got.tobytes() == oracle.transpose(host, m, n).tobytes(), (m, n)
+        else:
+            _sampled_check(got, host, m, n, 20000, rng)
+        ipt.r2c(x, m, n, elem_bytes=eb)
+        assert torch.equal(x, to_dev(host)), (m, n)
