@@ -1,0 +1,387 @@
+#!/usr/bin/env python3
+"""Benchmark of the B200 decomposed in-place transpose (driver contract).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+Workload (BASELINE.json configs[1], the metric's configuration): the paper's GPU sweep
+(Table 2) -- random m, n uniform in [1000, 20000] (workloads.sweep_shapes,
+seed 20140215), 4-byte (float32) and 8-byte (float64) elements, row-major.  One STEP is
+one in-place transpose of every one of the S shapes in both element sizes through the C
+ABI (ipt_c2r on even steps, ipt_r2c on odd steps, so both directions are timed and the
+data stay meaningful).  Every call is timed alone with CUDA events on the launching
+stream; L2 is flushed (a 256 MiB write, > the 126 MB L2) before every timed call, outside
+the events.  Throughput per call follows Eq. 37: 2 m n s / t, GB = 1e9 B.
+
+value   = median over all timed calls of the per-call GB/s (the paper's statistic);
+          with N ranks each rank transposes its own S independent shapes (weak scaling,
+          no collective on the data path) and value = the sum of the rank medians.
+e2e     = the same median, each call timed from a pinned-host H2D copy through ipt_c2r
+          to the D2H copy of the result (public API, host buffers).
+roofline= the dominant kernel's algorithmic bytes / its event-timed device time against
+          the measured HBM copy bandwidth (MEASURED_PEAKS.json).
+cpu_baseline = the C oracle's Algorithm 1 (oracle/, single thread) on a bounded sample.
+
+--impl reference: the reference arm of this tier is the oracle itself (the paper ships no
+code): rank 0 times oracle Algorithm 1 on host cores, one sweep shape per step.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads  # noqa: E402
+
+METRIC = "median in-place transpose GB/s over random m×n; fraction of B200 HBM peak"
+UNIT = "GB/s"
+FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
+FLUSH_BYTES = 256 << 20
+REF_MAX_ELEMS = 40_000_000  # reference-arm sample: sweep shapes with m*n <= this
+
+
+def parse_args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=6)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", choices=("ours", "reference"), default="ours")
+    p.add_argument("--shapes", type=int, default=48, help="sweep shapes per rank per step")
+    p.add_argument("--e2e-shapes", type=int, default=8)
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--profile-only", action="store_true", help="one short untimed pass (for ncu)")
+    return p.parse_args()
+
+
+def hbm_peak():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic():
+    """Per-launch DRAM bytes of the captured kernels (profiles/ncu_summary.json), if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(path) as f:
+            return json.load(f)
+    except Exception:
+        return {}
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_id: str):
+        self.gpu_id = gpu_id
+        self.proc = None
+        self.tmp = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "100", "-i", self.gpu_id], stdout=self.tmp,
+                                         stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        self.proc.wait()
+        self.tmp.flush()
+        rows = []
+        with open(self.tmp.name) as f:
+            for line in f:
+                v = [x.strip() for x in line.split(",")]
+                if len(v) >= 9 and v[1].isdigit():
+                    rows.append(v)
+        os.unlink(self.tmp.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm = [int(r[1]) for r in rows]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in rows for k in range(4) if r[5 + k].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": int(rows[0][2]), "reasons": reasons,
+                "samples": len(rows), "power_w_max": max(float(r[3]) for r in rows if r[3].replace(".", "").isdigit())
+                if any(r[3].replace(".", "").isdigit() for r in rows) else None}
+
+
+def cpu_info():
+    try:
+        cores = len(os.sched_getaffinity(0))
+    except Exception:
+        cores = os.cpu_count()
+    model = ""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except Exception:
+        pass
+    return cores, model
+
+
+def oracle_step(shape, eb, seed):
+    """One oracle Algorithm 1 C2R on host; returns (seconds, bytes)."""
+    import oracle
+    m, n = shape
+    host = workloads.random_words(m * n, eb, seed)
+    t0 = time.perf_counter()
+    oracle.c2r_alg1(host, m, n)
+    dt = time.perf_counter() - t0
+    return dt, 2.0 * m * n * eb
+
+
+def reference_sample_shapes(k):
+    out = []
+    for s in workloads.sweep_shapes(4096):
+        if s[0] * s[1] <= REF_MAX_ELEMS:
+            out.append(s)
+        if len(out) >= k:
+            break
+    return out
+
+
+def cpu_baseline(budget_s=20.0):
+    """The oracle as it stands (single-threaded C, Algorithm 1), fp32, on sweep shapes until
+    ~budget_s of CPU work."""
+    cores, model = cpu_info()
+    shapes, t_tot, rates = [], 0.0, []
+    for k, s in enumerate(workloads.sweep_shapes(64)):
+        dt, by = oracle_step(s, 4, seed=k)
+        shapes.append(s)
+        rates.append(by / dt / 1e9)
+        t_tot += dt
+        if t_tot >= budget_s:
+            break
+    return {"value": round(statistics.median(rates), 4), "unit": UNIT, "cores": 1, "kind": "oracle",
+            "host_cores_available": cores, "cpu_model": model,
+            "sample": f"oracle Algorithm 1 C2R, float32, first {len(shapes)} cfg2 sweep shapes {shapes}, "
+                      f"{t_tot:.1f} s CPU; median of per-shape Eq. 37 GB/s"}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    shapes = reference_sample_shapes(max(1, args.steps + args.warmup))
+    for k in range(args.warmup):
+        oracle_step(shapes[k % len(shapes)], 4, seed=k)
+    rates, secs = [], []
+    for k in range(args.steps):
+        s = shapes[(args.warmup + k) % len(shapes)]
+        dt, by = oracle_step(s, 4, seed=100 + k)
+        rates.append(by / dt / 1e9)
+        secs.append(dt)
+    cores, model = cpu_info()
+    value = statistics.median(rates)
+    sample = (f"oracle Algorithm 1 C2R (single thread), float32, one cfg2 sweep shape per step "
+              f"(shapes with m*n <= {REF_MAX_ELEMS}), {sum(secs):.1f} s CPU")
+    out = {"metric": METRIC, "value": round(value, 4), "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": round(1e3 * statistics.mean(secs), 3), "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+           "config": {"workload": "cfg2 paper sweep m,n~U[1000,20000] (reference arm: CPU oracle sample)",
+                      "seed": workloads.SWEEP_SEED},
+           "impl": "reference",
+           "cpu_baseline": {"value": round(value, 4), "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                            "host_cores_available": cores, "cpu_model": model},
+           "e2e": {"value": round(value, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def run_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ppopp_catanzarokg14_b200 as ipt
+
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    S = args.shapes
+    shapes = workloads.sweep_shapes(S * (rank + 1))[S * rank:]
+    ebs = (4, 8)
+    maxel = max(m * n for m, n in shapes)
+    bufs = {eb: torch.randint(0, 255, (maxel * eb,), dtype=torch.uint8, device=dev) for eb in ebs}
+    flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    def one_step(step, record):
+        op = ipt.c2r if step % 2 == 0 else ipt.r2c
+        for (m, n) in shapes:
+            for eb in ebs:
+                flush.zero_()
+                if record is not None:
+                    e0 = torch.cuda.Event(enable_timing=True)
+                    e1 = torch.cuda.Event(enable_timing=True)
+                    e0.record(stream)
+                op(bufs[eb], m, n, elem_bytes=eb, stream=stream.cuda_stream)
+                if record is not None:
+                    e1.record(stream)
+                    record.append((m, n, eb, e0, e1))
+
+    if args.profile_only:
+        one_step(0, None)
+        torch.cuda.synchronize()
+        return
+
+    for w in range(args.warmup):
+        one_step(w, None)
+    torch.cuda.synchronize()
+
+    gpu_id = "GPU-" + str(torch.cuda.get_device_properties(dev).uuid) if hasattr(
+        torch.cuda.get_device_properties(dev), "uuid") else str(local_rank)
+    clocks = Clocks(gpu_id)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    time.sleep(0.3)
+    launches0 = ipt.launch_count()
+    ipt.profile_enable(True)
+    ipt.profile_read()
+    rec = []
+    t_wall = time.perf_counter()
+    for k in range(args.steps):
+        one_step(args.warmup + k, rec)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    t_wall = time.perf_counter() - t_wall
+    ipt.profile_enable(False)
+    kern = ipt.profile_read()
+    launches = ipt.launch_count() - launches0
+    clk = clocks.stop()
+
+    per_call = []
+    by_eb = {eb: [] for eb in ebs}
+    dev_ms = 0.0
+    for (m, n, eb, e0, e1) in rec:
+        ms = e0.elapsed_time(e1)
+        dev_ms += ms
+        g = 2.0 * m * n * eb / (ms * 1e-3) / 1e9
+        per_call.append(g)
+        by_eb[eb].append(g)
+    median = statistics.median(per_call)
+    ms_step = dev_ms / args.steps
+
+    # ---- e2e through the public API with host buffers --------------------------------
+    e2e_shapes = shapes[:args.e2e_shapes]
+    e2e_rates, h2d = [], 0
+    for eb in ebs:
+        big = max(m * n for m, n in e2e_shapes) * eb
+        host = torch.empty(big, dtype=torch.uint8, pin_memory=True)
+        host.random_(0, 255)
+        for (m, n) in e2e_shapes:
+            nb = m * n * eb
+            d = bufs[eb][:nb]
+            h = host[:nb]
+            for rep in range(2):
+                flush.zero_()
+                e0 = torch.cuda.Event(enable_timing=True)
+                e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                d.copy_(h, non_blocking=True)
+                ipt.c2r(d, m, n, elem_bytes=eb, stream=stream.cuda_stream)
+                h.copy_(d, non_blocking=True)
+                e1.record(stream)
+                e1.synchronize()
+                if rep == 1:
+                    e2e_rates.append(2.0 * nb / (e0.elapsed_time(e1) * 1e-3) / 1e9)
+            h2d += nb
+    e2e = {"value": round(statistics.median(e2e_rates), 2), "unit": UNIT,
+           "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": h2d,
+           "note": f"median over {len(e2e_rates)} calls: pinned host -> H2D -> ipt_c2r -> D2H, first "
+                   f"{len(e2e_shapes)} sweep shapes x fp32/fp64"}
+
+    # ---- aggregate over ranks (max time, summed medians) ------------------------------
+    if world > 1:
+        t = torch.tensor([median, ms_step, e2e["value"]], dtype=torch.float64, device=dev)
+        tmax = t.clone()
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        value, ms_step, e2e_value = float(t[0]), float(tmax[1]), float(t[2])
+        e2e["value"] = round(e2e_value, 2)
+    else:
+        value = median
+    if rank != 0:
+        return
+
+    peak, peak_src = hbm_peak()
+    dom = max(kern.items(), key=lambda kv: kv[1][1]) if kern else None
+    roof = None
+    if dom:
+        name, (nl, ms, by) = dom
+        achieved = by / (ms * 1e-3) / 1e9
+        tr = ncu_traffic().get(name)
+        roof = {"bound": "hbm", "kernel": name, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "peak_source": peak_src,
+                "traffic": tr.get("dram_bytes_per_launch") if tr else None,
+                "traffic_algorithmic": tr.get("algorithmic_bytes_per_launch") if tr else None,
+                "traffic_source": tr.get("source") if tr else None,
+                "launches": nl, "share_of_device_time": round(ms / sum(v[1] for v in kern.values()), 3)}
+    kernels = {k: {"launches": v[0], "ms": round(v[1], 3), "GBps": round(v[2] / (v[1] * 1e-3) / 1e9, 1)}
+               for k, v in kern.items()}
+    out = {"metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": round(ms_step, 3), "higher_is_better": True, "scaling": "weak",
+           "vs_baseline": None, "dtype": "f32+f64", "data": "synthetic",
+           "config": {"workload": "cfg2 paper sweep: m,n ~ U[1000,20000] (seed 20140215), row-major, "
+                                  "float32+float64, ipt_c2r/ipt_r2c alternating steps",
+                      "shapes_per_rank": S, "elem_bytes": list(ebs), "calls_per_step": S * len(ebs),
+                      "l2": "flushed before every timed call (256 MiB write > 126 MB L2)",
+                      "parallelism": f"replicas x{world} (independent matrices per rank, no data-path collective)",
+                      "engine": "paper heuristic PAPER.md:959 (C2R if m > n else R2C)"},
+           "impl": "ours",
+           "median_GBps_fp32": round(statistics.median(by_eb[4]), 2),
+           "median_GBps_fp64": round(statistics.median(by_eb[8]), 2),
+           "p10_GBps": round(sorted(per_call)[len(per_call) // 10], 2),
+           "p90_GBps": round(sorted(per_call)[(9 * len(per_call)) // 10], 2),
+           "frac_of_hbm_peak": round(value / world / peak, 4),
+           "paper_context": {"K20c_median_GBps_fp64": 19.53, "K20c_median_GBps_fp32": 14.23,
+                             "source": "PAPER.md:1027-1033 Table 2 (other hardware; context only)"},
+           "roofline": roof, "kernels": kernels, "gpu_launches": launches, "e2e": e2e, "clocks": clk,
+           "wall_s_timed_region": round(t_wall, 3)}
+    if world == 1 and not args.no_cpu_baseline:
+        out["cpu_baseline"] = cpu_baseline()
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    args = parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -110,13 +110,28 @@ const char *ipt_status_string(ipt_status_t s);
  * the library would run for ipt_c2r(m, n, elem_bytes, layout): out[0] engine (0 none,
  * 1 C2R, 2 R2C, 3 skinny), out[1] M (engine rows), out[2] N (engine columns), out[3] c =
  * gcd(M, N), out[4] number of kernel launches, out[5] column-tile cluster size, out[6]
- * column-tile width in elements.  Returns IPT_ERR_UNSUPPORTED for shapes beyond limits.
+ * column-tile width in elements, out[7] largest on-chip staging bytes per CTA.  Returns
+ * IPT_ERR_UNSUPPORTED for shapes beyond limits.
  */
 ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
                            int64_t out[8]);
 
 /* Number of kernel launches this library has enqueued since load (all threads). */
 uint64_t ipt_launch_count(void);
+
+/*
+ * Per-kernel timing for benchmarks.  While enabled (process-wide), every launch is
+ * bracketed by two CUDA events recorded on the launch's own stream.  ipt_profile_read
+ * waits for those events and returns, per kernel kind k (0 row shuffle, 1 column
+ * shuffle, 2 column rotation, 3 skinny pass), launches[k], the summed device time ms[k]
+ * and the summed ALGORITHMIC bytes bytes[k] (what the pass must move: one read and one
+ * write of every element it permutes, Eq. 37's 2mns per full pass);
+ * then clears the record.  Arrays have IPT_PROFILE_KINDS entries.  Returns the number of
+ * launches read, or -1 on a CUDA error.
+ */
+#define IPT_PROFILE_KINDS 8
+void ipt_profile_enable(int on);
+int64_t ipt_profile_read(int64_t *launches, double *ms, double *bytes);
 
 #ifdef __cplusplus
 }

@@ -28,7 +28,9 @@ STATUS = {0: "IPT_OK", 1: "IPT_ERR_INVALID_ARGUMENT", 2: "IPT_ERR_UNSUPPORTED",
 # Every symbol declared in include/ipt.h.
 EXPORTS = ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_status_string", "ipt_plan_info",
-           "ipt_launch_count")
+           "ipt_launch_count", "ipt_profile_enable", "ipt_profile_read")
+PROFILE_KINDS = 8
+KERNEL_KINDS = ("row_shuffle", "col_shuffle", "col_rotate", "skinny")
 
 
 class IptError(RuntimeError):
@@ -55,6 +57,11 @@ _lib.ipt_status_string.restype = ctypes.c_char_p
 _lib.ipt_plan_info.argtypes = [_i64, _i64, _int, _int, ctypes.POINTER(_i64)]
 _lib.ipt_launch_count.argtypes = []
 _lib.ipt_launch_count.restype = ctypes.c_uint64
+_lib.ipt_profile_enable.argtypes = [_int]
+_lib.ipt_profile_enable.restype = None
+_lib.ipt_profile_read.argtypes = [ctypes.POINTER(_i64), ctypes.POINTER(ctypes.c_double),
+                                  ctypes.POINTER(ctypes.c_double)]
+_lib.ipt_profile_read.restype = _i64
 for _f in ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_plan_info"):
     getattr(_lib, _f).restype = _int
@@ -147,6 +154,22 @@ def plan_info(m: int, n: int, elem_bytes: int, layout="row"):
 
 def launch_count() -> int:
     return int(_lib.ipt_launch_count())
+
+
+def profile_enable(on: bool = True) -> None:
+    """Bracket every launch with CUDA events on its stream (see ipt_profile_read)."""
+    _lib.ipt_profile_enable(1 if on else 0)
+
+
+def profile_read():
+    """{kind: (launches, device ms, algorithmic bytes)} since the last read."""
+    n = (_i64 * PROFILE_KINDS)()
+    ms = (ctypes.c_double * PROFILE_KINDS)()
+    by = (ctypes.c_double * PROFILE_KINDS)()
+    if _lib.ipt_profile_read(n, ms, by) < 0:
+        raise IptError(4, "ipt_profile_read")
+    return {KERNEL_KINDS[k]: (int(n[k]), float(ms[k]), float(by[k]))
+            for k in range(len(KERNEL_KINDS)) if n[k]}
 
 
 def status_string(s: int) -> str:

@@ -13,6 +13,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
+#include <vector>
 
 #include "ipt.h"
 #include "plan.h"
@@ -197,6 +198,35 @@ ipt_status_t check(cudaError_t e) {
     return IPT_ERR_CUDA;
 }
 
+// ---- per-kernel event profiling (ipt_profile_enable / ipt_profile_read) ---------------
+enum ProfKind : int { PK_ROW = 0, PK_COL = 1, PK_ROT = 2, PK_SKINNY = 3 };
+struct ProfRec {
+    int kind = 0;
+    double bytes = 0;
+    cudaEvent_t start = nullptr, stop = nullptr;
+};
+std::atomic<int> g_prof_on{0};
+std::mutex g_prof_mu;
+std::vector<ProfRec> g_prof;
+
+bool profile_begin(ProfRec &r, int kind, double bytes, cudaStream_t st) {
+    if (!g_prof_on.load()) return false;
+    r.kind = kind;
+    r.bytes = bytes;
+    if (cudaEventCreate(&r.start) != cudaSuccess || cudaEventCreate(&r.stop) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    cudaEventRecord(r.start, st);
+    return true;
+}
+
+void profile_end(ProfRec &r, cudaStream_t st) {
+    cudaEventRecord(r.stop, st);
+    std::lock_guard<std::mutex> lk(g_prof_mu);
+    g_prof.push_back(r);
+}
+
 ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_bytes, cudaStream_t st) {
     if (pl0.engine == ENG_NONE || batch == 0) return IPT_OK;
     Plan pl = pl0;
@@ -211,25 +241,31 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
     // IPT_DEBUG_PASSES=k (tests only): stop after the first k passes, so that each pass
     // can be compared with the oracle's snapshot of the same step.
     int budget = env_int("IPT_DEBUG_PASSES", 1 << 30);
-    auto run = [&](auto &&launch) -> ipt_status_t {
+    const double full = 2.0 * static_cast<double>(pl.M) * static_cast<double>(pl.N) * pl.eb * static_cast<double>(batch);
+    auto run = [&](int kind, double bytes, auto &&launch) -> ipt_status_t {
         if (budget-- <= 0) return IPT_OK;
+        ProfRec rec;
+        const bool prof = profile_begin(rec, kind, bytes, st);
         ipt_status_t s = check(launch());
+        if (prof) profile_end(rec, st);
         if (s == IPT_OK) g_launches++;
         return s;
     };
+    // The rotation moves only the columns with a non-zero amount: (c - 1) / c of them.
+    const double rot_bytes = full * static_cast<double>(pl.c - 1) / static_cast<double>(pl.c);
     auto rot = [&] { return launch_col(pl.rot.p, COL_ROT, pl.eb, st, pl.rot.smem); };
     auto row = [&] { return launch_row(pl.row, pl.row_dir, pl.eb, st); };
     ipt_status_t s;
     if (pl.engine == ENG_C2R) {
         auto shuf = [&] { return launch_col(pl.shuf.p, COL_C2R_SHUF, pl.eb, st, pl.shuf.smem); };
-        if (pl.has_rot && (s = run(rot)) != IPT_OK) return s;  // Eq. 23 pre-rotation
-        if ((s = run(row)) != IPT_OK) return s;                  // Eq. 31 row gather
-        if ((s = run(shuf)) != IPT_OK) return s;                 // Eq. 26 = p_j o q
+        if (pl.has_rot && (s = run(PK_ROT, rot_bytes, rot)) != IPT_OK) return s;  // Eq. 23
+        if ((s = run(PK_ROW, full, row)) != IPT_OK) return s;                     // Eq. 31
+        if ((s = run(PK_COL, full, shuf)) != IPT_OK) return s;                    // Eq. 26
     } else {
         auto shuf = [&] { return launch_col(pl.shuf.p, COL_R2C_SHUF, pl.eb, st, pl.shuf.smem); };
-        if ((s = run(shuf)) != IPT_OK) return s;                 // Eqs. 34-35
-        if ((s = run(row)) != IPT_OK) return s;                  // Eq. 24 row gather
-        if (pl.has_rot && (s = run(rot)) != IPT_OK) return s;  // Eq. 36 post-rotation
+        if ((s = run(PK_COL, full, shuf)) != IPT_OK) return s;                    // Eqs. 34-35
+        if ((s = run(PK_ROW, full, row)) != IPT_OK) return s;                     // Eq. 24
+        if (pl.has_rot && (s = run(PK_ROT, rot_bytes, rot)) != IPT_OK) return s;  // Eq. 36
     }
     return IPT_OK;
 }
@@ -335,6 +371,39 @@ ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t la
 }
 
 uint64_t ipt_launch_count(void) { return g_launches.load(); }
+
+void ipt_profile_enable(int on) { g_prof_on.store(on ? 1 : 0); }
+
+int64_t ipt_profile_read(int64_t *launches, double *ms, double *bytes) {
+    std::vector<ProfRec> recs;
+    {
+        std::lock_guard<std::mutex> lk(g_prof_mu);
+        recs.swap(g_prof);
+    }
+    for (int k = 0; k < IPT_PROFILE_KINDS; ++k) {
+        if (launches) launches[k] = 0;
+        if (ms) ms[k] = 0;
+        if (bytes) bytes[k] = 0;
+    }
+    bool ok = true;
+    for (ProfRec &r : recs) {
+        float t = 0;
+        if (cudaEventSynchronize(r.stop) != cudaSuccess || cudaEventElapsedTime(&t, r.start, r.stop) != cudaSuccess)
+            ok = false;
+        if (r.kind >= 0 && r.kind < IPT_PROFILE_KINDS) {
+            if (launches) launches[r.kind] += 1;
+            if (ms) ms[r.kind] += t;
+            if (bytes) bytes[r.kind] += r.bytes;
+        }
+        cudaEventDestroy(r.start);
+        cudaEventDestroy(r.stop);
+    }
+    if (!ok) {
+        cudaGetLastError();
+        return -1;
+    }
+    return static_cast<int64_t>(recs.size());
+}
 
 const char *ipt_status_string(ipt_status_t s) {
     switch (s) {

@@ -72,6 +72,9 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     if (MODE == COL_ROT) {
         lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
         hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + Wt - 1), P.fd_b));
+        // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.  The
+        // whole cluster shares the tile, so the early exit is cluster-uniform.
+        if (hi_q == 0) return;
         ext = hi_q - lo_q;
         base_off = P.rot_sign > 0 ? lo_q : -hi_q;  // smallest rotation amount in the tile
     } else {
