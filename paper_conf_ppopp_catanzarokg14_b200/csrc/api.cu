@@ -14,6 +14,9 @@
 #include <cstring>
 #include <mutex>
 #include <vector>
+#include <algorithm>
+#include <string>
+#include <unordered_map>
 
 #include "ipt.h"
 #include "plan.h"
@@ -99,19 +102,24 @@ int ilog2(int v) {
     return l;
 }
 
-// Column-tile geometry: the smallest cluster (K <= 16) whose CTAs can each stage their
-// band of the M x W tile; the width starts at IPT_TILE_BYTES (default 32 B = one sector)
-// and halves if no cluster fits.
+// Column-tile geometry.  Tile width TWB = IPT_TILE_BYTES (32, 64 or 128; default 64 B =
+// two L2 sectors, the best of the three in the round-1 width study, profiles/).  Cluster size: the smallest K <= 16 whose per-CTA band fits the per-CTA
+// shared-memory target IPT_COL_SMEM (default 100 KiB, so that two CTAs -- one loading,
+// one storing -- share an SM), else the smallest K whose band fits the opt-in maximum.
 ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp) {
-    int tile_bytes = env_int("IPT_TILE_BYTES", 32);
-    if (tile_bytes < pl.eb) tile_bytes = pl.eb;
-    for (int W = tile_bytes / pl.eb; W >= 1; W /= 2) {
-        if (W & (W - 1)) continue;
+    int twb = env_int("IPT_TILE_BYTES", 64);
+    if (twb != 32 && twb != 64 && twb != 128) twb = 64;
+    if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
+    const size_t target = static_cast<size_t>(env_int("IPT_COL_SMEM", 100 * 1024));
+    const int W = twb / pl.eb;
+    for (int pass = 0; pass < 2; ++pass) {
+        const size_t limit = pass == 0 ? (target < static_cast<size_t>(dev.smem_optin) ? target : dev.smem_optin)
+                                       : static_cast<size_t>(dev.smem_optin);
         for (int K = 1; K <= 16; ++K) {
             const int64_t B = (pl.M + K - 1) / K;
             const size_t smem = col_smem_bytes(B, W, pl.eb);
-            if (smem > static_cast<size_t>(dev.smem_optin)) continue;
-            if (K > 1 && col_max_active_clusters(mode, pl.eb, K, smem) < 1) continue;
+            if (smem > limit) continue;
+            if (K > 1 && col_max_active_clusters(mode, pl.eb, twb, K, smem) < 1) continue;
             ColParams &p = cp.p;
             std::memset(&p, 0, sizeof(p));
             p.M = static_cast<int32_t>(pl.M);
@@ -190,6 +198,59 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         if (pl.rot.smem > pl.onchip) pl.onchip = pl.rot.smem;
     }
     return IPT_OK;
+}
+
+// Plan cache: planning queries the device (cluster occupancy) and must not sit between
+// the launches of a call.  Keyed by everything make_plan reads.
+struct PlanKey {
+    int64_t x, y;
+    int eb, dev;
+    std::string env;
+    bool operator==(const PlanKey &o) const {
+        return x == o.x && y == o.y && eb == o.eb && dev == o.dev && env == o.env;
+    }
+};
+struct PlanKeyHash {
+    size_t operator()(const PlanKey &k) const {
+        return std::hash<int64_t>()(k.x * 1000003 + k.y) ^ (std::hash<std::string>()(k.env) << 1) ^
+               static_cast<size_t>(k.eb * 131 + k.dev);
+    }
+};
+
+std::string tunables_key() {
+    std::string s;
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_FUSE_ROT"}) {
+        const char *v = std::getenv(n);
+        s += v ? v : "-";
+        s += '|';
+    }
+    return s;
+}
+
+ipt_status_t cached_plan(int64_t x, int64_t y, int eb, Plan &pl) {
+    static std::mutex mu;
+    static std::unordered_map<PlanKey, Plan, PlanKeyHash> cache;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) {
+        cudaGetLastError();
+        return IPT_ERR_CUDA;
+    }
+    PlanKey key{x, y, eb, dev, tunables_key()};
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) {
+            pl = it->second;
+            return IPT_OK;
+        }
+    }
+    ipt_status_t s = make_plan(x, y, eb, pl);
+    if (s == IPT_OK) {
+        std::lock_guard<std::mutex> lk(mu);
+        if (cache.size() >= 4096) cache.clear();
+        cache.emplace(std::move(key), pl);
+    }
+    return s;
 }
 
 ipt_status_t check(cudaError_t e) {
@@ -286,7 +347,7 @@ ipt_status_t run_perm(void *ptr, int64_t batch, int64_t stride, int64_t x, int64
     if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % static_cast<uintptr_t>(eb) != 0)
         return IPT_ERR_INVALID_ARGUMENT;
     Plan pl;
-    ipt_status_t s = make_plan(x, y, eb, pl);
+    ipt_status_t s = cached_plan(x, y, eb, pl);
     if (s != IPT_OK) return s;
     return execute(pl, static_cast<char *>(ptr), batch, stride * eb, static_cast<cudaStream_t>(stream));
 }
@@ -302,6 +363,53 @@ bool perm_of(bool c2r, int64_t m, int64_t n, int layout, int64_t &x, int64_t &y)
 }
 
 }  // namespace
+
+cudaError_t ensure_kernel_attrs(const void *kern, size_t smem, bool nonportable_cluster) {
+    static std::mutex mu;
+    static std::unordered_map<std::string, size_t> smem_set;  // "kern@dev" -> limit set
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const std::string key = std::to_string(reinterpret_cast<uintptr_t>(kern)) + "@" + std::to_string(dev);
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = smem_set.find(key);
+    const size_t want = smem | (nonportable_cluster ? (size_t(1) << 62) : 0);
+    if (it != smem_set.end() && (it->second & ~(size_t(1) << 62)) >= smem &&
+        (!nonportable_cluster || (it->second >> 62))) return cudaSuccess;
+    size_t have = it == smem_set.end() ? 0 : it->second;
+    const size_t lim = std::max(smem, have & ~(size_t(1) << 62));
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(lim));
+    if (e != cudaSuccess) return e;
+    if (nonportable_cluster) {
+        e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        if (e != cudaSuccess) return e;
+    }
+    smem_set[key] = lim | ((have | want) & (size_t(1) << 62));
+    return cudaSuccess;
+}
+
+int cached_resident_blocks(const void *kern, int threads, size_t smem) {
+    static std::mutex mu;
+    static std::unordered_map<std::string, int> cache;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const std::string key = std::to_string(reinterpret_cast<uintptr_t>(kern)) + "@" + std::to_string(dev) + "/" +
+                            std::to_string(threads) + "/" + std::to_string(smem);
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) return it->second;
+    }
+    int per_sm = 0, sms = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, smem) != cudaSuccess ||
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    std::lock_guard<std::mutex> lk(mu);
+    cache[key] = per_sm * sms;
+    return per_sm * sms;
+}
+
 }  // namespace ipt
 
 using namespace ipt;

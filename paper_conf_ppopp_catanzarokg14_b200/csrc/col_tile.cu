@@ -2,14 +2,14 @@
 // §4.6-4.7).
 //
 // A column operation permutes every column independently.  The B200 realisation stages a
-// whole column tile -- all M rows x W adjacent columns (W * eb bytes wide) -- on chip,
-// spread over the shared memory of a thread-block cluster of K CTAs (each CTA holds a
-// band of B = ceil(M/K) rows plus a halo), and makes the operation a single read + write
-// pass.  In-place safety: every CTA finishes reading its part of the tile before ANY CTA
-// of the cluster writes (cluster barrier with release/acquire); tiles are disjoint byte
-// ranges owned by exactly one cluster.  This replaces the paper's multi-pass
-// cache-aware rotate (coarse cycle following + fine on-chip rotation, §4.6) and cycle-
-// following row permute (§4.7) -- prior art for a K20c without clusters.
+// whole column tile -- all M rows x W adjacent columns (TWB = W * eb bytes wide) -- on
+// chip, spread over the shared memory of a thread-block cluster of K CTAs (each CTA holds
+// a band of B = ceil(M/K) rows plus a halo), and makes the operation a single read +
+// write pass.  In-place safety: every CTA finishes reading its part of the tile before
+// ANY CTA of the cluster writes (cluster barrier with release/acquire); tiles are
+// disjoint byte ranges owned by exactly one cluster.  This replaces the paper's
+// multi-pass cache-aware rotate (coarse cycle following + fine on-chip rotation, §4.6)
+// and cycle-following row permute (§4.7) -- prior art for a K20c without clusters.
 //
 // Tile-local forms (w = j - j0 is the column inside the tile [j0, j0 + W)):
 //  * COL_ROT, gather rotation rho_j = sign * floor(j/b) (Eq. 23 for sign = +1 as the C2R
@@ -26,6 +26,14 @@
 //        out[i][w] = in[q^{-1}((i - w - j0) mod M)][w].
 //    The CTA writing band [r0, r1) reads the rows q^{-1}((u - j0) mod M) for
 //    u in [r0 - W + 1, r1) (scattered whole sub-rows) and writes its band contiguously.
+//
+// Memory access: each staged row is fetched as its 16-byte-aligned hull (TWB/16 + 1
+// chunks) with cp.async (LDGSTS, global -> shared without a register round trip), so a
+// CTA has its whole band in flight at once; rows are 16-byte aligned only when
+// N*eb % 16 == 0, and the hull's extra bytes (neighbouring tiles of the same row) are
+// never used.  Chunks that would leave the matrix (row 0 head, row M-1 tail) are fetched
+// element by element.  Stores are element-wise (eb bytes per thread, a warp covers
+// 32*eb/TWB whole tile rows).
 #include "plan.h"
 
 namespace ipt {
@@ -33,6 +41,24 @@ namespace ipt {
 namespace {
 
 constexpr int kColThreads = 512;
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void *src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(src) : "memory");
+}
+template <int B>
+__device__ __forceinline__ void cp_async_small(uint32_t dst, const void *src) {
+    if constexpr (B == 16) {
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(src) : "memory");
+    } else {
+        asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" :: "r"(dst), "l"(src), "n"(B) : "memory");
+    }
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+}
 
 // q^{-1}(i) = (floor((c-1+i)/c) b^{-1}) mod a + (((c-1) i) mod c) a  (Eq. 34).
 __device__ __forceinline__ int32_t qinv_of(const ColParams &P, int32_t i) {
@@ -44,17 +70,26 @@ __device__ __forceinline__ int32_t qinv_of(const ColParams &P, int32_t i) {
     return static_cast<int32_t>(u + cm * static_cast<uint32_t>(P.a));
 }
 
-__device__ __forceinline__ int32_t mod_M(int64_t v, int32_t M) {
-    v %= M;
-    return static_cast<int32_t>(v < 0 ? v + M : v);
+// v mod M for v >= -kshift*M (kshift = 2 + W/M covers every caller; M < 2^30).
+__device__ __forceinline__ int32_t mod_M(int32_t v, uint32_t kshiftM, const FastDiv &fdM) {
+    return static_cast<int32_t>(fmod_(static_cast<uint32_t>(v) + kshiftM, fdM));
 }
 
-template <int EB, int MODE>
+template <int TWB>
+struct TileGeom {
+    static constexpr int SLOT = TWB + 16;  // hull bytes per staged row
+    static constexpr int CH = TWB / 16 + 1;  // hull chunks per staged row
+};
+
+template <int EB, int MODE, int TWB>
 __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     using T = typename Word<EB>::T;
+    constexpr int W = TWB / EB;
+    constexpr int LW = W == 1 ? 0 : W == 2 ? 1 : W == 4 ? 2 : W == 8 ? 3 : W == 16 ? 4 : 5;
+    constexpr int SLOT = TileGeom<TWB>::SLOT;
+    constexpr int CH = TileGeom<TWB>::CH;
     extern __shared__ __align__(16) unsigned char smem[];
 
-    const int32_t W = P.W, lw = P.log2W;
     const int64_t cid = blockIdx.x / P.K;  // cluster id
     const int32_t r = blockIdx.x - static_cast<int32_t>(cid * P.K);
     const int32_t tile = static_cast<int32_t>(cid % P.ntiles);
@@ -65,10 +100,11 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     const int32_t r0 = r * P.B;
     const int32_t r1 = min(P.M, r0 + P.B);
     const int32_t nrows = max(0, r1 - r0);
+    const char *Aend = A + static_cast<int64_t>(P.M) * P.N * EB;
+    const uint32_t kshM = static_cast<uint32_t>(2 + W / P.M) * static_cast<uint32_t>(P.M);
+    const int32_t j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j0), P.fd_M));
 
-    // Band geometry per mode.
-    int32_t ext, base_off = 0;
-    int32_t lo_q = 0, hi_q = 0;
+    int32_t ext, base_off = 0, lo_q = 0, hi_q = 0;
     if (MODE == COL_ROT) {
         lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
         hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + Wt - 1), P.fd_b));
@@ -82,110 +118,126 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     }
     const int32_t nslots = nrows > 0 ? nrows + ext : 0;
 
-    T *slot = reinterpret_cast<T *>(smem);                                       // [nslots][W]
-    int32_t *ridx = reinterpret_cast<int32_t *>(smem + static_cast<size_t>(nslots) * W * EB);  // [nslots]
+    unsigned char *stage = smem;                                  // [nslots][SLOT]
+    uint8_t *dlt = smem + static_cast<size_t>(nslots) * SLOT;    // [nslots] hull offsets
+    int32_t *ridx = reinterpret_cast<int32_t *>(smem + ((static_cast<size_t>(nslots) * (SLOT + 1) + 3) & ~size_t(3)));
 
-    // ---- phase 1: which global row feeds each slot (C2R: also the destination rows) --
-    for (int32_t t = threadIdx.x; t < nslots; t += blockDim.x) {
+    // ---- R2C: the scattered source rows of every slot ---------------------------------
+    if (MODE == COL_R2C_SHUF) {
+        for (int32_t t = threadIdx.x; t < nslots; t += blockDim.x) {
+            ridx[t] = qinv_of(P, mod_M(r0 - (W - 1) + t - j0m, kshM, P.fd_M));
+        }
+        __syncthreads();
+    }
+
+    // ---- load: cp.async of every staged row's 16-byte hull ------------------------------
+    const int32_t nch = nslots * CH;
+    for (int32_t e = threadIdx.x; e < nch; e += blockDim.x) {
+        const int32_t t = e / CH, k = e - t * CH;
         int32_t row;
-        if (MODE == COL_ROT) {
-            row = mod_M(static_cast<int64_t>(r0) + base_off + t, P.M);
-        } else if (MODE == COL_C2R_SHUF) {
-            row = mod_M(static_cast<int64_t>(r0) + t, P.M);
+        if (MODE == COL_ROT) row = mod_M(r0 + base_off + t, kshM, P.fd_M);
+        else if (MODE == COL_C2R_SHUF) row = mod_M(r0 + t, kshM, P.fd_M);
+        else row = ridx[t];
+        const char *ra = A + (static_cast<int64_t>(row) * P.N + j0) * EB;
+        const int d = static_cast<int>(reinterpret_cast<uintptr_t>(ra) & 15);
+        if (k == 0) dlt[t] = static_cast<uint8_t>(d);
+        const char *lo = ra - d + 16 * k;
+        const char *vend = ra + Wt * EB;
+        if (lo >= vend) continue;
+        unsigned char *dst = stage + t * SLOT + 16 * k;
+        if (lo >= A && lo + 16 <= Aend) {
+            cp_async16(smem_u32(dst), lo);
         } else {
-            const int64_t u = static_cast<int64_t>(r0) - (W - 1) + t;
-            row = qinv_of(P, mod_M(u - j0, P.M));
+#pragma unroll
+            for (int q = 0; q < 16; q += EB)
+                if (lo + q >= A && lo + q < Aend) cp_async_small<EB>(smem_u32(dst + q), lo + q);
         }
-        ridx[t] = row;
     }
-    __syncthreads();
 
-    // ---- phase 2: load the (skewed) band of the tile into shared memory ------------
-    const int32_t nel = nslots << lw;
-    for (int32_t e = threadIdx.x; e < nel; e += blockDim.x) {
-        const int32_t t = e >> lw, w = e & (W - 1);
-        if (w < Wt) {
-            const T *g = reinterpret_cast<const T *>(A) + static_cast<int64_t>(ridx[t]) * P.N + j0 + w;
-            slot[e] = *g;
-        }
+    // ---- C2R: destination rows of the band, while the loads are in flight ------------
+    if (MODE == COL_C2R_SHUF) {
+        for (int32_t kk = threadIdx.x; kk < nrows; kk += blockDim.x)
+            ridx[kk] = qinv_of(P, mod_M(r0 + kk - j0m, kshM, P.fd_M));
     }
+    cp_async_wait_all();
 
     // In-place hazard barrier: the whole tile has been read before anyone writes it.
     if (P.K > 1) cluster_barrier(); else __syncthreads();
 
-    // ---- phase 3: destination rows of the C2R scatter form -----------------------------
-    if (MODE == COL_C2R_SHUF) {
-        // reuse ridx[0..nrows) for destinations (ridx for sources is no longer needed)
-        for (int32_t kk = threadIdx.x; kk < nrows; kk += blockDim.x)
-            ridx[kk] = qinv_of(P, mod_M(static_cast<int64_t>(r0) + kk - j0, P.M));
-        __syncthreads();
+    // ---- write ---------------------------------------------------------------------------
+    const int32_t w = threadIdx.x & (W - 1);  // blockDim is a multiple of W: fixed per thread
+    if (w >= Wt) return;
+    int32_t dw = 0;
+    if (MODE == COL_ROT) {
+        const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + w), P.fd_b));
+        dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
+    } else if (MODE == COL_C2R_SHUF) {
+        dw = w;
+    } else {
+        dw = W - 1 - w;
     }
-
-    // ---- phase 4: write ----------------------------------------------------------------
-    const int32_t nout = nrows << lw;
-    for (int32_t e = threadIdx.x; e < nout; e += blockDim.x) {
-        const int32_t kk = e >> lw, w = e & (W - 1);
-        if (w >= Wt) continue;
-        T v;
-        int64_t orow;
-        if (MODE == COL_ROT) {
-            const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + w), P.fd_b));
-            const int32_t dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
-            v = slot[((kk + dw) << lw) + w];
-            orow = r0 + kk;
-        } else if (MODE == COL_C2R_SHUF) {
-            v = slot[((kk + w) << lw) + w];
-            orow = ridx[kk];
-        } else {
-            v = slot[((kk - w + W - 1) << lw) + w];
-            orow = r0 + kk;
-        }
-        reinterpret_cast<T *>(A)[orow * P.N + j0 + w] = v;
+    T *out = reinterpret_cast<T *>(A) + j0 + w;
+    for (int32_t kk = threadIdx.x >> LW; kk < nrows; kk += blockDim.x >> LW) {
+        const int32_t t = kk + dw;
+        const T v = *reinterpret_cast<const T *>(stage + t * SLOT + dlt[t] + w * EB);
+        const int64_t orow = MODE == COL_C2R_SHUF ? ridx[kk] : r0 + kk;
+        out[orow * P.N] = v;
     }
 }
 
-template <int EB, int MODE>
-void *col_kernel_ptr() {
-    return reinterpret_cast<void *>(col_tile_kernel<EB, MODE>);
+template <int EB, int MODE, int TWB>
+void *kptr() {
+    return reinterpret_cast<void *>(col_tile_kernel<EB, MODE, TWB>);
 }
 
-void *col_kernel(int mode, int eb) {
-    switch (eb * 4 + mode) {
-        case 4 * 4 + COL_ROT: return col_kernel_ptr<4, COL_ROT>();
-        case 4 * 4 + COL_C2R_SHUF: return col_kernel_ptr<4, COL_C2R_SHUF>();
-        case 4 * 4 + COL_R2C_SHUF: return col_kernel_ptr<4, COL_R2C_SHUF>();
-        case 8 * 4 + COL_ROT: return col_kernel_ptr<8, COL_ROT>();
-        case 8 * 4 + COL_C2R_SHUF: return col_kernel_ptr<8, COL_C2R_SHUF>();
-        case 8 * 4 + COL_R2C_SHUF: return col_kernel_ptr<8, COL_R2C_SHUF>();
-        case 16 * 4 + COL_ROT: return col_kernel_ptr<16, COL_ROT>();
-        case 16 * 4 + COL_C2R_SHUF: return col_kernel_ptr<16, COL_C2R_SHUF>();
-        case 16 * 4 + COL_R2C_SHUF: return col_kernel_ptr<16, COL_R2C_SHUF>();
+template <int EB, int TWB>
+void *col_kernel_w(int mode) {
+    switch (mode) {
+        case COL_ROT: return kptr<EB, COL_ROT, TWB>();
+        case COL_C2R_SHUF: return kptr<EB, COL_C2R_SHUF, TWB>();
+        case COL_R2C_SHUF: return kptr<EB, COL_R2C_SHUF, TWB>();
         default: return nullptr;
     }
 }
 
-cudaError_t prepare(void *kern, int K, size_t smem) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
-    if (e != cudaSuccess) return e;
-    if (K > 8) {
-        e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-        if (e != cudaSuccess) return e;
+template <int EB>
+void *col_kernel_e(int mode, int twb) {
+    switch (twb) {
+        case 32: return col_kernel_w<EB, 32>(mode);
+        case 64: return col_kernel_w<EB, 64>(mode);
+        case 128: return col_kernel_w<EB, 128>(mode);
+        default: return nullptr;
     }
-    return cudaSuccess;
 }
+
+void *col_kernel(int mode, int eb, int twb) {
+    switch (eb) {
+        case 4: return col_kernel_e<4>(mode, twb);
+        case 8: return col_kernel_e<8>(mode, twb);
+        case 16: return col_kernel_e<16>(mode, twb);
+        default: return nullptr;
+    }
+}
+
+cudaError_t prepare(void *kern, int K, size_t smem) { return ensure_kernel_attrs(kern, smem, K > 8); }
 
 }  // namespace
 
 size_t col_smem_bytes(int64_t B, int64_t W, int eb) {
+    const int64_t twb = W * eb;
     const int64_t nslots = B + W - 1;
-    return static_cast<size_t>(nslots * W * eb + nslots * 4);
+    const int64_t slot = twb + 16;
+    return static_cast<size_t>(((nslots * (slot + 1) + 3) & ~int64_t(3)) + nslots * 4);
 }
 
 int col_block_threads() { return kColThreads; }
 
-int col_max_active_clusters(int mode, int eb, int K, size_t smem) {
-    void *kern = col_kernel(mode, eb);
-    if (!kern || prepare(kern, K, smem) != cudaSuccess) return 0;
+int col_max_active_clusters(int mode, int eb, int twb, int K, size_t smem) {
+    void *kern = col_kernel(mode, eb, twb);
+    if (!kern || prepare(kern, K, smem) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
     cudaLaunchConfig_t cfg = {};
     cudaLaunchAttribute attr[1];
     cfg.gridDim = dim3(static_cast<unsigned>(K) * 64);
@@ -206,7 +258,7 @@ int col_max_active_clusters(int mode, int eb, int K, size_t smem) {
 }
 
 cudaError_t launch_col(const ColParams &P, int mode, int eb, cudaStream_t st, size_t smem) {
-    void *kern = col_kernel(mode, eb);
+    void *kern = col_kernel(mode, eb, P.W * eb);
     if (!kern) return cudaErrorInvalidValue;
     cudaError_t e = prepare(kern, P.K, smem);
     if (e != cudaSuccess) return e;

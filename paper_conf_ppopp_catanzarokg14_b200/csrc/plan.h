@@ -59,6 +59,12 @@ struct ColParams {
     int32_t wide_a;     // a >= 2^16
 };
 
+// Kernel attribute / occupancy caches (api.cu): set the dynamic shared-memory limit (and
+// the non-portable cluster flag) once per (kernel, device), and memoise occupancy, so
+// that no device query sits between the launches of a call.
+cudaError_t ensure_kernel_attrs(const void *kern, size_t smem, bool nonportable_cluster);
+int cached_resident_blocks(const void *kern, int threads, size_t smem);  // SMs x blocks per SM
+
 // Launchers (col_tile.cu / row_shuffle.cu).  They return the CUDA error of the launch.
 size_t row_smem_bytes(int64_t N, int eb);
 int row_block_threads();
@@ -67,6 +73,6 @@ cudaError_t launch_row(const RowParams &p, int dir, int eb, cudaStream_t st);
 size_t col_smem_bytes(int64_t B, int64_t W, int eb);
 int col_block_threads();
 cudaError_t launch_col(const ColParams &p, int mode, int eb, cudaStream_t st, size_t smem);
-int col_max_active_clusters(int mode, int eb, int K, size_t smem);
+int col_max_active_clusters(int mode, int eb, int twb, int K, size_t smem);
 
 }  // namespace ipt
