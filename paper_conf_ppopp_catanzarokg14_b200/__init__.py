@@ -28,7 +28,7 @@ STATUS = {0: "IPT_OK", 1: "IPT_ERR_INVALID_ARGUMENT", 2: "IPT_ERR_UNSUPPORTED",
 # Every symbol declared in include/ipt.h.
 EXPORTS = ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_status_string", "ipt_plan_info",
-           "ipt_launch_count", "ipt_profile_enable", "ipt_profile_read")
+           "ipt_launch_count", "ipt_profile_enable", "ipt_profile_read", "ipt_debug_tile_copy")
 PROFILE_KINDS = 8
 KERNEL_KINDS = ("row_shuffle", "col_shuffle", "col_rotate", "skinny")
 
@@ -62,6 +62,8 @@ _lib.ipt_profile_enable.restype = None
 _lib.ipt_profile_read.argtypes = [ctypes.POINTER(_i64), ctypes.POINTER(ctypes.c_double),
                                   ctypes.POINTER(ctypes.c_double)]
 _lib.ipt_profile_read.restype = _i64
+_lib.ipt_debug_tile_copy.argtypes = [_vp, _i64, _i64, _int, _int, _int, _int, _vp]
+_lib.ipt_debug_tile_copy.restype = _int
 for _f in ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_plan_info"):
     getattr(_lib, _f).restype = _int
@@ -170,6 +172,15 @@ def profile_read():
         raise IptError(4, "ipt_profile_read")
     return {KERNEL_KINDS[k]: (int(n[k]), float(ms[k]), float(by[k]))
             for k in range(len(KERNEL_KINDS)) if n[k]}
+
+
+def debug_tile_copy(buf, M: int, N: int, elem_bytes: int, tile_bytes: int, cluster: int, barrier: bool,
+                    stream=None):
+    """Identity pass of the column-tile kernel (include/ipt_debug.h): measurement only."""
+    p, eb, st = _ptr_eb_stream(buf, elem_bytes, stream)
+    _check(_lib.ipt_debug_tile_copy(p, M, N, eb, tile_bytes, cluster, 1 if barrier else 0, st),
+           "ipt_debug_tile_copy")
+    return buf
 
 
 def status_string(s: int) -> str:

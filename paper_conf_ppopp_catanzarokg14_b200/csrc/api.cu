@@ -19,6 +19,7 @@
 #include <unordered_map>
 
 #include "ipt.h"
+#include "ipt_debug.h"
 #include "plan.h"
 
 namespace ipt {
@@ -180,9 +181,21 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     rp.b = static_cast<int32_t>(pl.b);
     rp.ainv = static_cast<int32_t>(mmi64(pl.a, pl.b));
     rp.amodb = static_cast<int32_t>(pl.a % pl.b);
+    rp.Mn = static_cast<int32_t>(pl.M % pl.N);
     rp.fd_c = make_fastdiv(static_cast<uint32_t>(pl.c));
     rp.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
+    rp.fd_N = make_fastdiv(static_cast<uint32_t>(pl.N));
     rp.wide = pl.b >= 65536 ? 1 : 0;
+    rp.wideN = pl.N >= 65536 ? 1 : 0;
+    {
+        const int64_t D = 32;  // lane stride of the row walk
+        rp.w_dl = static_cast<int32_t>(D % pl.c);
+        rp.w_dlb = static_cast<int32_t>((D % pl.c) * pl.b);
+        rp.w_dhc = static_cast<int32_t>((static_cast<int64_t>(rp.ainv) * (D / pl.c)) % pl.b);
+        rp.w_dh = static_cast<int32_t>(D % pl.b);
+        rp.w_dl2 = static_cast<int32_t>(D / pl.b);
+        rp.w_ds = static_cast<int32_t>((D / pl.b + ((D % pl.b) * (pl.M % pl.N)) % pl.N) % pl.N);
+    }
     pl.row_dir = engine == ENG_C2R ? ROW_C2R : ROW_R2C;
 
     ipt_status_t s = plan_col(dev, pl, engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.shuf);
@@ -346,6 +359,7 @@ ipt_status_t run_perm(void *ptr, int64_t batch, int64_t stride, int64_t x, int64
     if (elems == 0 || batch == 0) return IPT_OK;
     if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % static_cast<uintptr_t>(eb) != 0)
         return IPT_ERR_INVALID_ARGUMENT;
+    if (x <= 1 || y <= 1) return IPT_OK;  // P_{1,y} and P_{x,1} are the identity
     Plan pl;
     ipt_status_t s = cached_plan(x, y, eb, pl);
     if (s != IPT_OK) return s;
@@ -479,6 +493,37 @@ ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t la
 }
 
 uint64_t ipt_launch_count(void) { return g_launches.load(); }
+
+ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes, int tile_bytes, int cluster,
+                                 int barrier, void *stream) {
+    if (!valid_eb(elem_bytes) || M < 1 || N < 1 || M >= (1 << 29) || N >= (1 << 29) || cluster < 1 ||
+        cluster > 16 || (tile_bytes != 32 && tile_bytes != 64 && tile_bytes != 128) || tile_bytes < elem_bytes ||
+        !ptr || reinterpret_cast<uintptr_t>(ptr) % elem_bytes)
+        return IPT_ERR_INVALID_ARGUMENT;
+    const DevInfo dev = device_info();
+    if (!dev.ok) return IPT_ERR_CUDA;
+    ColParams p;
+    std::memset(&p, 0, sizeof(p));
+    p.base = static_cast<char *>(ptr);
+    p.batch = 1;
+    p.mat_stride_bytes = M * N * elem_bytes;
+    p.M = static_cast<int32_t>(M);
+    p.N = static_cast<int32_t>(N);
+    p.c = p.a = p.b = 1;
+    p.fd_c = p.fd_a = p.fd_b = make_fastdiv(1);
+    p.fd_M = make_fastdiv(static_cast<uint32_t>(M));
+    p.W = tile_bytes / elem_bytes;
+    p.log2W = ilog2(p.W);
+    p.ntiles = static_cast<int32_t>((N + p.W - 1) / p.W);
+    p.K = cluster;
+    p.B = static_cast<int32_t>((M + cluster - 1) / cluster);
+    p.rot_sign = barrier ? 1 : 0;
+    const size_t smem = col_smem_bytes(p.B, p.W, elem_bytes);
+    if (smem > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
+    if (cluster > 1 && col_max_active_clusters(COL_COPY, elem_bytes, tile_bytes, cluster, smem) < 1)
+        return IPT_ERR_UNSUPPORTED;
+    return check(launch_col(p, COL_COPY, elem_bytes, static_cast<cudaStream_t>(stream), smem));
+}
 
 void ipt_profile_enable(int on) { g_prof_on.store(on ? 1 : 0); }
 

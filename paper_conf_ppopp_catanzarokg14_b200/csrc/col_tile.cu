@@ -113,6 +113,8 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
         if (hi_q == 0) return;
         ext = hi_q - lo_q;
         base_off = P.rot_sign > 0 ? lo_q : -hi_q;  // smallest rotation amount in the tile
+    } else if (MODE == COL_COPY) {
+        ext = 0;
     } else {
         ext = W - 1;
     }
@@ -131,26 +133,34 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     }
 
     // ---- load: cp.async of every staged row's 16-byte hull ------------------------------
+    // Source row of slot t: contiguous (rowbase + t) mod M for ROT / C2R, ridx[t] for R2C.
+    const int32_t rowbase = MODE == COL_ROT ? mod_M(r0 + base_off, kshM, P.fd_M) : r0;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    const char *Aj = A + static_cast<int64_t>(j0) * EB;
+    const uint32_t sst = smem_u32(stage);
     const int32_t nch = nslots * CH;
     for (int32_t e = threadIdx.x; e < nch; e += blockDim.x) {
         const int32_t t = e / CH, k = e - t * CH;
         int32_t row;
-        if (MODE == COL_ROT) row = mod_M(r0 + base_off + t, kshM, P.fd_M);
-        else if (MODE == COL_C2R_SHUF) row = mod_M(r0 + t, kshM, P.fd_M);
-        else row = ridx[t];
-        const char *ra = A + (static_cast<int64_t>(row) * P.N + j0) * EB;
+        if (MODE == COL_R2C_SHUF) {
+            row = ridx[t];
+        } else {
+            row = rowbase + t;
+            if (row >= P.M) row = row - P.M < P.M ? row - P.M : mod_M(row, kshM, P.fd_M);
+        }
+        const char *ra = Aj + row * pitch;
         const int d = static_cast<int>(reinterpret_cast<uintptr_t>(ra) & 15);
         if (k == 0) dlt[t] = static_cast<uint8_t>(d);
         const char *lo = ra - d + 16 * k;
-        const char *vend = ra + Wt * EB;
-        if (lo >= vend) continue;
-        unsigned char *dst = stage + t * SLOT + 16 * k;
-        if (lo >= A && lo + 16 <= Aend) {
-            cp_async16(smem_u32(dst), lo);
+        if (16 * k >= d + Wt * EB) continue;  // past the end of this row's tile
+        const uint32_t dst = sst + t * SLOT + 16 * k;
+        // Only row 0's head and row M-1's tail can leave the matrix.
+        if ((row != 0 && row != P.M - 1) || (lo >= A && lo + 16 <= Aend)) {
+            cp_async16(dst, lo);
         } else {
 #pragma unroll
             for (int q = 0; q < 16; q += EB)
-                if (lo + q >= A && lo + q < Aend) cp_async_small<EB>(smem_u32(dst + q), lo + q);
+                if (lo + q >= A && lo + q < Aend) cp_async_small<EB>(dst + q, lo + q);
         }
     }
 
@@ -162,13 +172,15 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     cp_async_wait_all();
 
     // In-place hazard barrier: the whole tile has been read before anyone writes it.
-    if (P.K > 1) cluster_barrier(); else __syncthreads();
+    if (P.K > 1 && !(MODE == COL_COPY && P.rot_sign == 0)) cluster_barrier(); else __syncthreads();
 
     // ---- write ---------------------------------------------------------------------------
     const int32_t w = threadIdx.x & (W - 1);  // blockDim is a multiple of W: fixed per thread
     if (w >= Wt) return;
     int32_t dw = 0;
-    if (MODE == COL_ROT) {
+    if (MODE == COL_COPY) {
+        dw = 0;
+    } else if (MODE == COL_ROT) {
         const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + w), P.fd_b));
         dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
     } else if (MODE == COL_C2R_SHUF) {
@@ -177,9 +189,12 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
         dw = W - 1 - w;
     }
     T *out = reinterpret_cast<T *>(A) + j0 + w;
-    for (int32_t kk = threadIdx.x >> LW; kk < nrows; kk += blockDim.x >> LW) {
-        const int32_t t = kk + dw;
-        const T v = *reinterpret_cast<const T *>(stage + t * SLOT + dlt[t] + w * EB);
+    const unsigned char *sw = stage + dw * SLOT + w * EB;
+    const uint8_t *dl = dlt + dw;
+    const int32_t kstep = blockDim.x >> LW;
+#pragma unroll 4
+    for (int32_t kk = threadIdx.x >> LW; kk < nrows; kk += kstep) {
+        const T v = *reinterpret_cast<const T *>(sw + kk * SLOT + dl[kk]);
         const int64_t orow = MODE == COL_C2R_SHUF ? ridx[kk] : r0 + kk;
         out[orow * P.N] = v;
     }
@@ -196,6 +211,7 @@ void *col_kernel_w(int mode) {
         case COL_ROT: return kptr<EB, COL_ROT, TWB>();
         case COL_C2R_SHUF: return kptr<EB, COL_C2R_SHUF, TWB>();
         case COL_R2C_SHUF: return kptr<EB, COL_R2C_SHUF, TWB>();
+        case COL_COPY: return kptr<EB, COL_COPY, TWB>();
         default: return nullptr;
     }
 }

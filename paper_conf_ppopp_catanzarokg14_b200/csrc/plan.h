@@ -25,6 +25,8 @@ enum ColMode : int {
     COL_ROT = 0,       // out[i][j] = in[(i + sign*floor(j/b)) mod M][j]   (Eq. 23 / Eq. 36)
     COL_C2R_SHUF = 1,  // out[i][j] = in[(j + q(i)) mod M][j]              (Eq. 26 = p_j o q)
     COL_R2C_SHUF = 2,  // out[i][j] = in[q^{-1}((i - j) mod M)][j]         (Eqs. 34, 35)
+    COL_COPY = 3,      // out[i][j] = in[i][j]: measurement of the tile access pattern only
+                       // (ipt_debug_tile_copy); rot_sign = 0 also drops the cluster barrier
 };
 
 // Row-shuffle directions.
@@ -40,8 +42,17 @@ struct RowParams {
     int32_t M, N, c, a, b;
     int32_t ainv;   // mmi(a, b)
     int32_t amodb;  // a mod b
-    FastDiv fd_c, fd_b;
+    int32_t Mn;     // M mod N
+    FastDiv fd_c, fd_b, fd_N;
     int32_t wide;   // b >= 2^16: products need 64 bits
+    int32_t wideN;  // N >= 2^16
+    // Per-plan constants of a 32-element stride along the row (row_shuffle.cu walks):
+    int32_t w_dl;   // 32 mod c
+    int32_t w_dlb;  // (32 mod c) * b
+    int32_t w_dhc;  // a^{-1} floor(32 / c) mod b
+    int32_t w_dh;   // 32 mod b
+    int32_t w_dl2;  // floor(32 / b)
+    int32_t w_ds;   // (floor(32 / b) + (32 mod b) M) mod N
 };
 
 struct ColParams {

@@ -4,20 +4,21 @@
 // (Theorem 3: d'_i is a bijection for every i).  B200 realisation of the paper's
 // "on-chip row shuffle" (:751): the whole row is staged in shared memory with cp.async
 // (16-byte LDGSTS for the aligned interior, element copies for the ragged head/tail --
-// rows are 16-byte aligned only when N*eb % 16 == 0), then each thread gathers the
-// outputs of one 16-byte chunk from shared memory and writes them back with one vector
-// store.  Global traffic: one read and one write of every element.
+// rows are 16-byte aligned only when N*eb % 16 == 0), then every warp gathers a
+// contiguous segment of the output row from shared memory, lane L writing outputs
+// L, L+32, L+64, ... (coalesced stores).  Global traffic: one read and one write of every
+// element.
 //
-// Gather indices (derived from Eq. 24 by splitting j = l*b + h, l < c, h < b; the parity
-// tests check them against the oracle's Eq. 31 / Eq. 24):
-//   d'_i(l b + h)   = c * ((E_l + (h a mod b)) mod b) + (i + l) mod c
-//   E_l             = (floor(i/c) + [l >= c - i mod c] - a [i + l >= M]) mod b
-// and its inverse for output position p = col * c + rho:
-//   l = (rho - i) mod c,  h = a^{-1} (col - E_l) mod b,  d'^{-1}_i(p) = l b + h,
-// where a^{-1} E_l = a^{-1} floor(i/c) + a^{-1} [rho < i mod c] - [i + l >= M]  (mod b).
-// Along consecutive outputs both are evaluated incrementally (§4.4's strength reduction
-// taken one step further): one strength-reduced division per 16-byte chunk, then adds
-// and compares.
+// Index forms (Eq. 24 rewritten; derivation in DESIGN.md §"Row shuffle", checked against
+// the oracle's Eq. 24 and Eq. 31 by the parity tests).  With j = l b + h (l < c, h < b)
+// and f2 = [i + l >= M]:
+//   R2C gather  d'_i(j)       = (i + l + h M - M f2) mod N
+//   C2R gather  d'^{-1}_i(p)  = l b + (a^{-1} floor(q / c) + f2) mod b,
+//               q = (p - i) mod N,  l = q mod c.
+// Walking p (or j) in steps of 32 changes the state by per-plan constants plus one carry,
+// so a lane spends a handful of integer adds per element (§4.4's strength reduction
+// taken one step further); f2 can only be 1 in the last c - 1 rows, which take a
+// slower walk that tracks l.
 #include "plan.h"
 
 namespace ipt {
@@ -41,197 +42,209 @@ __device__ __forceinline__ void cp_async_wait_all() {
     asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
 }
 
-struct RowConst {
-    int32_t Ri, Qb, Gi, Mi;
-    __device__ __forceinline__ RowConst(const RowParams &P, int32_t i) {
-        const uint32_t Qi = fdiv(static_cast<uint32_t>(i), P.fd_c);
-        Ri = i - static_cast<int32_t>(Qi) * P.c;
-        const uint32_t Qbm = fmod_(Qi, P.fd_b);
-        Qb = static_cast<int32_t>(Qbm);
-        Gi = static_cast<int32_t>(mulmod(static_cast<uint32_t>(P.ainv), Qbm, P.fd_b, P.wide));
-        Mi = P.M - i;  // [i + l >= M]  <=>  l >= M - i
+// C2R walk: src = lb + (hc + f2) mod b with lb = l*b, hc = a^{-1} floor(q/c) mod b.
+template <bool TAIL>
+struct C2RWalk {
+    int32_t lb, hc, l;
+    __device__ __forceinline__ C2RWalk(const RowParams &P, int32_t im, int32_t p) {
+        int32_t q = p - im;
+        q += q < 0 ? P.N : 0;
+        const uint32_t col = fdiv(static_cast<uint32_t>(q), P.fd_c);
+        l = q - static_cast<int32_t>(col) * P.c;
+        lb = l * P.b;
+        hc = static_cast<int32_t>(mulmod(static_cast<uint32_t>(P.ainv), col, P.fd_b, P.wide));
     }
-};
-
-// C2R: source of output position p, d'^{-1}_i(p) (Eq. 31), walked along p.
-struct C2RIter {
-    int32_t rho, l, H;
-    __device__ __forceinline__ C2RIter(const RowParams &P, const RowConst &R, int32_t p) {
-        const uint32_t col = fdiv(static_cast<uint32_t>(p), P.fd_c);
-        rho = p - static_cast<int32_t>(col) * P.c;
-        l = rho - R.Ri;
-        l += l < 0 ? P.c : 0;
-        H = static_cast<int32_t>(mulmod(static_cast<uint32_t>(P.ainv), col, P.fd_b, P.wide));
-    }
-    __device__ __forceinline__ int32_t src(const RowParams &P, const RowConst &R) const {
-        int32_t h = H + (l >= R.Mi ? 1 : 0) - R.Gi;
-        h += h < 0 ? P.b : 0;
-        h -= h >= P.b ? P.b : 0;
-        if (rho < R.Ri) {
-            h -= P.ainv;
-            h += h < 0 ? P.b : 0;
-        }
-        return l * P.b + h;
+    __device__ __forceinline__ int32_t src(const RowParams &P, int32_t Mi) const {
+        if (!TAIL) return lb + hc;
+        int32_t h = hc + (l >= Mi ? 1 : 0);
+        h -= h == P.b ? P.b : 0;
+        return lb + h;
     }
     __device__ __forceinline__ void next(const RowParams &P) {
-        ++rho;
-        ++l;
-        l = l == P.c ? 0 : l;
-        if (rho == P.c) {
-            rho = 0;
-            H += P.ainv;
-            H -= H >= P.b ? P.b : 0;
+        lb += P.w_dlb;
+        const bool carry = lb >= P.N;
+        lb -= carry ? P.N : 0;
+        hc += P.w_dhc + (carry ? P.ainv : 0);
+        hc -= hc >= P.b ? P.b : 0;
+        hc -= hc >= P.b ? P.b : 0;
+        if (TAIL) {
+            l += P.w_dl;
+            l -= l >= P.c ? P.c : 0;
         }
     }
 };
 
-// R2C: source of output position j, d'_i(j) (Eq. 24 used as a gather, §4.3 :717).
-struct R2CIter {
-    int32_t l, h, ha, E, rl;
-    __device__ __forceinline__ int32_t E_of(const RowParams &P, const RowConst &R, int32_t ll) const {
-        int32_t e = R.Qb + (ll >= P.c - R.Ri ? 1 : 0) - (ll >= R.Mi ? P.amodb : 0);
-        e += e < 0 ? P.b : 0;
-        e -= e >= P.b ? P.b : 0;
-        return e;
-    }
-    __device__ __forceinline__ R2CIter(const RowParams &P, const RowConst &R, int32_t j) {
+// R2C walk: src = (i + l + h M) mod N  [- M mod N if f2].
+template <bool TAIL>
+struct R2CWalk {
+    int32_t s, h, l;
+    __device__ __forceinline__ R2CWalk(const RowParams &P, int32_t im, int32_t j) {
         l = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j), P.fd_b));
         h = j - l * P.b;
-        ha = static_cast<int32_t>(mulmod(static_cast<uint32_t>(h), static_cast<uint32_t>(P.amodb), P.fd_b, P.wide));
-        E = E_of(P, R, l);
-        rl = R.Ri + l;
-        rl -= rl >= P.c ? P.c : 0;
+        int32_t t = im + l;
+        t -= t >= P.N ? P.N : 0;
+        t += static_cast<int32_t>(mulmod(static_cast<uint32_t>(h), static_cast<uint32_t>(P.Mn), P.fd_N, P.wideN));
+        t -= t >= P.N ? P.N : 0;
+        s = t;
     }
-    __device__ __forceinline__ int32_t src(const RowParams &P, const RowConst &) const {
-        int32_t col = E + ha;
-        col -= col >= P.b ? P.b : 0;
-        return P.c * col + rl;
+    __device__ __forceinline__ int32_t src(const RowParams &P, int32_t Mi) const {
+        if (!TAIL) return s;
+        int32_t t = s - (l >= Mi ? P.Mn : 0);
+        return t + (t < 0 ? P.N : 0);
     }
-    __device__ __forceinline__ void next(const RowParams &P, const RowConst &R) {
-        ++h;
-        ha += P.amodb;
-        ha -= ha >= P.b ? P.b : 0;
-        if (h == P.b) {
-            h = 0;
-            ha = 0;
-            ++l;
-            E = E_of(P, R, l);
-            ++rl;
-            rl = rl == P.c ? 0 : rl;
-        }
+    __device__ __forceinline__ void next(const RowParams &P) {
+        h += P.w_dh;
+        const bool carry = h >= P.b;
+        h -= carry ? P.b : 0;
+        s += P.w_ds + (carry ? 1 : 0);
+        s -= s >= P.N ? P.N : 0;
+        if (TAIL) l += P.w_dl2 + (carry ? 1 : 0);
     }
 };
 
-template <int EB, int DIR>
-__global__ void __launch_bounds__(kRowThreadsMax) row_shuffle_kernel(RowParams P) {
+template <int EB, int DIR, bool TAIL>
+__device__ __forceinline__ void gather_row(const RowParams &P, char *row, const unsigned char *stage, int32_t i) {
     using T = typename Word<EB>::T;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    const int32_t seg = ((P.N + nwarps - 1) / nwarps + 31) & ~31;  // whole warps' worth
+    const int32_t p_begin = warp * seg, p_end = min(P.N, p_begin + seg);
+    const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
+    const int32_t Mi = P.M - i;
+    const T *src = reinterpret_cast<const T *>(stage);
+    T *out = reinterpret_cast<T *>(row);
+    int32_t p = p_begin + lane;
+    if (p >= p_end) return;
+    if (DIR == ROW_C2R) {
+        C2RWalk<TAIL> w(P, im, p);
+#pragma unroll 4
+        for (; p < p_end; p += 32) {
+            out[p] = src[w.src(P, Mi)];
+            w.next(P);
+        }
+    } else {
+        R2CWalk<TAIL> w(P, im, p);
+#pragma unroll 4
+        for (; p < p_end; p += 32) {
+            out[p] = src[w.src(P, Mi)];
+            w.next(P);
+        }
+    }
+}
+
+// Stage one row with cp.async: smem byte (off + k) holds row byte k.  Not waited.
+template <int EB>
+__device__ __forceinline__ void stage_row(const char *row, int32_t nbytes, uint32_t sbase) {
+    constexpr int PER = 16 / EB;
+    const int off = static_cast<int>(reinterpret_cast<uintptr_t>(row) & 15);  // multiple of EB
+    const char *row0 = row - off;
+    const int nch = (off + nbytes + 15) >> 4;
+    for (int k = threadIdx.x; k < nch; k += blockDim.x) {
+        const int lo = k * 16 - off;
+        if (lo >= 0 && lo + 16 <= nbytes) {
+            cp_async<16>(sbase + 16 * k, row0 + 16 * k);
+        } else {
+#pragma unroll
+            for (int e = 0; e < PER; ++e) {
+                const int q = lo + e * EB;
+                if (q >= 0 && q < nbytes) cp_async<EB>(sbase + off + q, row + q);
+            }
+        }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+// Grid-stride over the M * batch rows.  NBUF = 2: while row r is gathered from one
+// buffer, row r + gridDim.x is already streaming into the other (cp.async groups), so
+// every CTA keeps a row's worth of loads in flight at all times.
+template <int EB, int DIR, int NBUF>
+__global__ void __launch_bounds__(kRowThreadsMax) row_shuffle_kernel(RowParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
-    constexpr int PER = 16 / EB;  // elements per 16-byte chunk
     const int64_t rows_total = static_cast<int64_t>(P.M) * P.batch;
     const int32_t nbytes = P.N * EB;
+    const uint32_t bufbytes = (static_cast<uint32_t>(nbytes) + 31) & ~15u;
+    const uint32_t sbase = smem_u32(smem);
 
+    int64_t mat = blockIdx.x / P.M;
+    int32_t i = static_cast<int32_t>(blockIdx.x - mat * P.M);
+    const int32_t step_i = static_cast<int32_t>(gridDim.x % P.M);
+    const int64_t step_m = gridDim.x / P.M;
+    auto row_ptr = [&](int64_t mm, int32_t ii) {
+        return P.base + mm * P.mat_stride_bytes + static_cast<int64_t>(ii) * nbytes;
+    };
+    if (NBUF == 2 && blockIdx.x < rows_total) stage_row<EB>(row_ptr(mat, i), nbytes, sbase);
+    int buf = 0;
     for (int64_t r = blockIdx.x; r < rows_total; r += gridDim.x) {
-        const int64_t mat = r / P.M;
-        const int32_t i = static_cast<int32_t>(r - mat * P.M);
-        char *row = P.base + mat * P.mat_stride_bytes + static_cast<int64_t>(i) * nbytes;
-        const int off = static_cast<int>(reinterpret_cast<uintptr_t>(row) & 15);  // multiple of EB
-        char *row0 = row - off;
-        const int nch = (off + nbytes + 15) >> 4;
-
-        // ---- stage the row: smem byte (off + k) holds row byte k --------------------
-        const uint32_t sbase = smem_u32(smem);
-        for (int k = threadIdx.x; k < nch; k += blockDim.x) {
-            const int lo = k * 16 - off;
-            if (lo >= 0 && lo + 16 <= nbytes) {
-                cp_async<16>(sbase + 16 * k, row0 + 16 * k);
-            } else {
-#pragma unroll
-                for (int e = 0; e < PER; ++e) {
-                    const int q = lo + e * EB;
-                    if (q >= 0 && q < nbytes) cp_async<EB>(sbase + off + q, row + q);
-                }
-            }
+        char *row = row_ptr(mat, i);
+        int32_t ni = i + step_i;
+        int64_t nmat = mat + step_m;
+        if (ni >= P.M) {
+            ni -= P.M;
+            ++nmat;
         }
-        cp_async_wait_all();
+        if (NBUF == 2) {
+            if (r + gridDim.x < rows_total) {
+                stage_row<EB>(row_ptr(nmat, ni), nbytes, sbase + (buf ^ 1) * bufbytes);
+                asm volatile("cp.async.wait_group 1;" ::: "memory");
+            } else {
+                asm volatile("cp.async.wait_group 0;" ::: "memory");
+            }
+        } else {
+            stage_row<EB>(row, nbytes, sbase);
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+        }
         __syncthreads();
 
-        // ---- gather + write back, one 16-byte chunk per thread ----------------------
-        const RowConst R(P, i);
-        const T *src = reinterpret_cast<const T *>(smem + off);
-        for (int k = threadIdx.x; k < nch; k += blockDim.x) {
-            const int lo = k * 16 - off;
-            const int p0 = lo / EB;  // negative in a misaligned head chunk
-            const int pb = p0 < 0 ? 0 : p0;
-            if (lo >= 0 && lo + 16 <= nbytes) {
-                union { uint4 u; T t[PER]; } v;
-                if (DIR == ROW_C2R) {
-                    C2RIter it(P, R, pb);
-#pragma unroll
-                    for (int e = 0; e < PER; ++e) {
-                        v.t[e] = src[it.src(P, R)];
-                        if (e + 1 < PER) it.next(P);
-                    }
-                } else {
-                    R2CIter it(P, R, pb);
-#pragma unroll
-                    for (int e = 0; e < PER; ++e) {
-                        v.t[e] = src[it.src(P, R)];
-                        if (e + 1 < PER) it.next(P, R);
-                    }
-                }
-                stg16(row0 + 16 * k, v.u);
-            } else {
-                const int pe = min(p0 + PER, P.N);
-                if (DIR == ROW_C2R) {
-                    C2RIter it(P, R, pb);
-                    for (int p = pb; p < pe; ++p) {
-                        reinterpret_cast<T *>(row)[p] = src[it.src(P, R)];
-                        it.next(P);
-                    }
-                } else {
-                    R2CIter it(P, R, pb);
-                    for (int p = pb; p < pe; ++p) {
-                        reinterpret_cast<T *>(row)[p] = src[it.src(P, R)];
-                        it.next(P, R);
-                    }
-                }
-            }
-        }
-        __syncthreads();  // smem is reused by the next row
+        // ---- gather + write back (the last c - 1 rows may have f2 = 1) --------------
+        const unsigned char *stage = smem + buf * bufbytes + (reinterpret_cast<uintptr_t>(row) & 15);
+        if (i >= P.M - P.c + 1) gather_row<EB, DIR, true>(P, row, stage, i);
+        else gather_row<EB, DIR, false>(P, row, stage, i);
+        __syncthreads();  // this buffer is refilled two rows later
+
+        if (NBUF == 2) buf ^= 1;
+        i = ni;
+        mat = nmat;
     }
 }
 
 int row_threads(int64_t N, int eb) { return N * eb >= 48 * 1024 ? 512 : 256; }
 
-template <int EB, int DIR>
+// Double buffering while two row buffers stay within ~110 KB (two CTAs per SM or more).
+int row_nbuf(int64_t N, int eb) { return 2 * row_smem_bytes(N, eb) <= 112 * 1024 ? 2 : 1; }
+
+template <int EB, int DIR, int NBUF>
 cudaError_t launch_row_t(const RowParams &P, cudaStream_t st) {
-    const size_t smem = row_smem_bytes(P.N, EB);
+    const size_t smem = NBUF * row_smem_bytes(P.N, EB);
     const int threads = row_threads(P.N, EB);
-    auto kern = row_shuffle_kernel<EB, DIR>;
+    auto kern = row_shuffle_kernel<EB, DIR, NBUF>;
     cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
     if (e != cudaSuccess) return e;
-    const int per_sm_sms = cached_resident_blocks(reinterpret_cast<const void *>(kern), threads, smem);
-    if (per_sm_sms < 1) return cudaErrorInvalidConfiguration;
+    const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), threads, smem);
+    if (resident < 1) return cudaErrorInvalidConfiguration;
     const int64_t rows = static_cast<int64_t>(P.M) * P.batch;
-    int64_t grid = per_sm_sms;
+    int64_t grid = resident;
     if (grid > rows) grid = rows;
     kern<<<static_cast<unsigned>(grid), threads, smem, st>>>(P);
     return cudaGetLastError();
 }
 
+template <int EB, int DIR>
+cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
+    return row_nbuf(P.N, EB) == 2 ? launch_row_t<EB, DIR, 2>(P, st) : launch_row_t<EB, DIR, 1>(P, st);
+}
+
 }  // namespace
 
-size_t row_smem_bytes(int64_t N, int eb) { return static_cast<size_t>(N) * eb + 16; }
+size_t row_smem_bytes(int64_t N, int eb) { return (static_cast<size_t>(N) * eb + 31) & ~size_t(15); }
 int row_block_threads() { return kRowThreadsMax; }
 
 cudaError_t launch_row(const RowParams &P, int dir, int eb, cudaStream_t st) {
     switch (eb * 2 + dir) {
-        case 4 * 2 + ROW_C2R: return launch_row_t<4, ROW_C2R>(P, st);
-        case 4 * 2 + ROW_R2C: return launch_row_t<4, ROW_R2C>(P, st);
-        case 8 * 2 + ROW_C2R: return launch_row_t<8, ROW_C2R>(P, st);
-        case 8 * 2 + ROW_R2C: return launch_row_t<8, ROW_R2C>(P, st);
-        case 16 * 2 + ROW_C2R: return launch_row_t<16, ROW_C2R>(P, st);
-        case 16 * 2 + ROW_R2C: return launch_row_t<16, ROW_R2C>(P, st);
+        case 4 * 2 + ROW_C2R: return launch_row_d<4, ROW_C2R>(P, st);
+        case 4 * 2 + ROW_R2C: return launch_row_d<4, ROW_R2C>(P, st);
+        case 8 * 2 + ROW_C2R: return launch_row_d<8, ROW_C2R>(P, st);
+        case 8 * 2 + ROW_R2C: return launch_row_d<8, ROW_R2C>(P, st);
+        case 16 * 2 + ROW_C2R: return launch_row_d<16, ROW_C2R>(P, st);
+        case 16 * 2 + ROW_R2C: return launch_row_d<16, ROW_R2C>(P, st);
         default: return cudaErrorInvalidValue;
     }
 }

@@ -8,13 +8,16 @@ import pytest
 
 from conftest import ROOT
 
-HEADER = os.path.join(ROOT, "include", "ipt.h")
+INCLUDE = os.path.join(ROOT, "include")
 
 
 def declared_symbols():
-    text = open(HEADER).read()
-    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
-    return sorted(set(re.findall(r"\b(ipt_[a-z0-9_]+)\s*\(", text)))
+    syms = set()
+    for f in os.listdir(INCLUDE):
+        if f.endswith(".h"):
+            text = re.sub(r"/\*.*?\*/", "", open(os.path.join(INCLUDE, f)).read(), flags=re.S)
+            syms |= set(re.findall(r"\b(ipt_[a-z0-9_]+)\s*\(", text))
+    return sorted(syms)
 
 
 @pytest.fixture(scope="module")
