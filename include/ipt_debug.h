@@ -3,11 +3,12 @@
  *
  * ipt_debug_tile_copy: run the column-tile kernel in identity mode on an M x N row-major
  * array (out[i][j] = in[i][j]): every M x (tile_bytes / elem_bytes) column tile is staged
- * on chip by a cluster of `cluster` CTAs and written back unchanged.  barrier = 1 keeps
- * the cluster barrier of the real column passes, barrier = 0 drops it.  It isolates the
+ * on chip by a group of `cluster` CTAs (bands of ceil(M / cluster) rows) and written back
+ * unchanged.  barrier = 1 keeps the group barrier of the real column passes, barrier = 0
+ * drops it.  It isolates the
  * cost of the tile access pattern (strided tile_bytes-wide sub-rows) and of the cluster
  * synchronisation from the index arithmetic of the permutations (column
- * kernel roofline).  tile_bytes in {32, 64, 128}; cluster in 1..16.  Asynchronous on
+ * kernel roofline).  tile_bytes in {32, 64, 128}; 1 <= cluster <= co-resident CTAs.  Asynchronous on
  * `stream`; the buffer content is unchanged on success.
  */
 #ifndef IPT_DEBUG_H_

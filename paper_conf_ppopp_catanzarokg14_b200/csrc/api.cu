@@ -8,7 +8,7 @@
 //    the row length N = min(x, y) is the dimension staged on chip;
 //  * constants c = gcd, a, b (:275-277), a^{-1} = mmi(a, b), b^{-1} = mmi(b, a)
 //    (:673-685, :719), strength-reduced divisors (§4.4, :745-749);
-//  * pass list and launch geometry (row kernel, column-tile cluster size K and width W).
+//  * pass list and launch geometry (row kernel; column-tile width W, band B, group size G).
 #include <atomic>
 #include <cstdlib>
 #include <cstring>
@@ -103,49 +103,67 @@ int ilog2(int v) {
     return l;
 }
 
-// Column-tile geometry.  Tile width TWB = IPT_TILE_BYTES (32, 64 or 128; default 64 B =
-// two L2 sectors, the best of the three in the round-1 width study, profiles/).  Cluster size: the smallest K <= 16 whose per-CTA band fits the per-CTA
-// shared-memory target IPT_COL_SMEM (default 100 KiB, so that two CTAs -- one loading,
-// one storing -- share an SM), else the smallest K whose band fits the opt-in maximum.
+// Column-tile geometry.  Tile width TWB = IPT_TILE_BYTES (32, 64 or 128; default 128 B =
+// one cache line).  Band: the rows per CTA that fit the per-CTA shared-memory target
+// IPT_COL_SMEM (default 40 KiB: several CTAs per SM in different load/store phases --
+// the regime in which the strided tile pattern reaches copy bandwidth, tools/
+// pattern_probe.cu).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
+// the co-resident CTAs, the band grows (up to the opt-in shared-memory maximum).
 ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp) {
-    int twb = env_int("IPT_TILE_BYTES", 64);
-    if (twb != 32 && twb != 64 && twb != 128) twb = 64;
+    int twb = env_int("IPT_TILE_BYTES", 128);
+    if (twb != 32 && twb != 64 && twb != 128) twb = 128;
+    if (twb < pl.eb) twb = pl.eb;
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
-    const size_t target = static_cast<size_t>(env_int("IPT_COL_SMEM", 100 * 1024));
-    const int W = twb / pl.eb;
-    for (int pass = 0; pass < 2; ++pass) {
-        const size_t limit = pass == 0 ? (target < static_cast<size_t>(dev.smem_optin) ? target : dev.smem_optin)
-                                       : static_cast<size_t>(dev.smem_optin);
-        for (int K = 1; K <= 16; ++K) {
-            const int64_t B = (pl.M + K - 1) / K;
-            const size_t smem = col_smem_bytes(B, W, pl.eb);
-            if (smem > limit) continue;
-            if (K > 1 && col_max_active_clusters(mode, pl.eb, twb, K, smem) < 1) continue;
-            ColParams &p = cp.p;
-            std::memset(&p, 0, sizeof(p));
-            p.M = static_cast<int32_t>(pl.M);
-            p.N = static_cast<int32_t>(pl.N);
-            p.c = static_cast<int32_t>(pl.c);
-            p.a = static_cast<int32_t>(pl.a);
-            p.b = static_cast<int32_t>(pl.b);
-            p.binv = static_cast<int32_t>(mmi64(pl.b, pl.a));
-            p.fd_c = make_fastdiv(static_cast<uint32_t>(pl.c));
-            p.fd_a = make_fastdiv(static_cast<uint32_t>(pl.a));
-            p.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
-            p.fd_M = make_fastdiv(static_cast<uint32_t>(pl.M));
-            p.W = W;
-            p.log2W = ilog2(W);
-            p.ntiles = static_cast<int32_t>((pl.N + W - 1) / W);
-            p.K = K;
-            p.B = static_cast<int32_t>(B);
-            p.rot_sign = 1;
-            p.wide_a = pl.a >= 65536 ? 1 : 0;
-            cp.smem = smem;
-            cp.mode = mode;
-            return IPT_OK;
+    const int64_t target = env_int("IPT_COL_SMEM", 40 * 1024);
+    const int64_t W = twb / pl.eb;
+    const int64_t per_row = twb + 16 + 1 + 4;  // col_smem_bytes: hull + offset + row index
+    int64_t B = target / per_row - (W - 1);
+    if (B < 32) B = 32;
+    if (B > pl.M) B = pl.M;
+    for (;;) {
+        const size_t smem = col_smem_bytes(B, W, pl.eb);
+        if (smem > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
+        const int64_t G = (pl.M + B - 1) / B;
+        const int resident = col_resident_ctas(mode, pl.eb, twb, smem);
+        if (resident < 1) return IPT_ERR_UNSUPPORTED;
+        if (G > resident) {  // a whole group must be co-resident
+            B = (pl.M + resident - 1) / resident;
+            continue;
         }
+        ColParams &p = cp.p;
+        std::memset(&p, 0, sizeof(p));
+        p.M = static_cast<int32_t>(pl.M);
+        p.N = static_cast<int32_t>(pl.N);
+        p.c = static_cast<int32_t>(pl.c);
+        p.a = static_cast<int32_t>(pl.a);
+        p.b = static_cast<int32_t>(pl.b);
+        p.binv = static_cast<int32_t>(mmi64(pl.b, pl.a));
+        p.fd_c = make_fastdiv(static_cast<uint32_t>(pl.c));
+        p.fd_a = make_fastdiv(static_cast<uint32_t>(pl.a));
+        p.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
+        p.fd_M = make_fastdiv(static_cast<uint32_t>(pl.M));
+        p.W = static_cast<int32_t>(W);
+        p.log2W = ilog2(static_cast<int>(W));
+        p.ntiles = static_cast<int32_t>((pl.N + W - 1) / W);
+        p.G = static_cast<int32_t>(G);
+        p.B = static_cast<int32_t>(B);
+        p.resident = resident;
+        p.rot_sign = 1;
+        p.wide_a = pl.a >= 65536 ? 1 : 0;
+        cp.smem = smem;
+        cp.mode = mode;
+        return IPT_OK;
     }
-    return IPT_ERR_UNSUPPORTED;
+}
+
+// Persistent grid of a column pass over `batch` matrices: as many whole groups as are
+// co-resident, never more than there are tiles.
+void finish_col(ColParams &p, int64_t batch) {
+    p.total_tiles = static_cast<int64_t>(p.ntiles) * batch;
+    int64_t ng = p.resident / p.G;
+    if (ng > p.total_tiles) ng = p.total_tiles;
+    if (ng < 1) ng = 1;
+    p.ngroups = static_cast<int32_t>(ng);
 }
 
 // P_{x,y} on `batch` matrices.
@@ -311,6 +329,7 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
         cp->p.base = base;
         cp->p.batch = batch;
         cp->p.mat_stride_bytes = stride_bytes;
+        finish_col(cp->p, batch);
     }
     // IPT_DEBUG_PASSES=k (tests only): stop after the first k passes, so that each pass
     // can be compared with the oracle's snapshot of the same step.
@@ -486,7 +505,7 @@ ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t la
     out[2] = pl.N;
     out[3] = pl.c;
     out[4] = pl.nlaunch;
-    out[5] = pl.engine ? pl.shuf.p.K : 0;
+    out[5] = pl.engine ? pl.shuf.p.G : 0;
     out[6] = pl.engine ? pl.shuf.p.W : 0;
     out[7] = static_cast<int64_t>(pl.onchip);
     return IPT_OK;
@@ -497,7 +516,7 @@ uint64_t ipt_launch_count(void) { return g_launches.load(); }
 ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes, int tile_bytes, int cluster,
                                  int barrier, void *stream) {
     if (!valid_eb(elem_bytes) || M < 1 || N < 1 || M >= (1 << 29) || N >= (1 << 29) || cluster < 1 ||
-        cluster > 16 || (tile_bytes != 32 && tile_bytes != 64 && tile_bytes != 128) || tile_bytes < elem_bytes ||
+        (tile_bytes != 32 && tile_bytes != 64 && tile_bytes != 128) || tile_bytes < elem_bytes ||
         !ptr || reinterpret_cast<uintptr_t>(ptr) % elem_bytes)
         return IPT_ERR_INVALID_ARGUMENT;
     const DevInfo dev = device_info();
@@ -515,13 +534,14 @@ ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes
     p.W = tile_bytes / elem_bytes;
     p.log2W = ilog2(p.W);
     p.ntiles = static_cast<int32_t>((N + p.W - 1) / p.W);
-    p.K = cluster;
     p.B = static_cast<int32_t>((M + cluster - 1) / cluster);
+    p.G = static_cast<int32_t>((M + p.B - 1) / p.B);
     p.rot_sign = barrier ? 1 : 0;
     const size_t smem = col_smem_bytes(p.B, p.W, elem_bytes);
     if (smem > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
-    if (cluster > 1 && col_max_active_clusters(COL_COPY, elem_bytes, tile_bytes, cluster, smem) < 1)
-        return IPT_ERR_UNSUPPORTED;
+    p.resident = col_resident_ctas(COL_COPY, elem_bytes, tile_bytes, smem);
+    if (p.resident < p.G) return IPT_ERR_UNSUPPORTED;
+    finish_col(p, 1);
     return check(launch_col(p, COL_COPY, elem_bytes, static_cast<cudaStream_t>(stream), smem));
 }
 

@@ -3,28 +3,36 @@
 //
 // A column operation permutes every column independently.  The B200 realisation stages a
 // whole column tile -- all M rows x W adjacent columns (TWB = W * eb bytes wide) -- on
-// chip, spread over the shared memory of a thread-block cluster of K CTAs (each CTA holds
-// a band of B = ceil(M/K) rows plus a halo), and makes the operation a single read +
-// write pass.  In-place safety: every CTA finishes reading its part of the tile before
-// ANY CTA of the cluster writes (cluster barrier with release/acquire); tiles are
-// disjoint byte ranges owned by exactly one cluster.  This replaces the paper's
-// multi-pass cache-aware rotate (coarse cycle following + fine on-chip rotation, §4.6)
-// and cycle-following row permute (§4.7) -- prior art for a K20c without clusters.
+// chip, spread over the shared memory of a GROUP of G CTAs (member r holds the band of
+// B rows [r B, r B + B) plus a halo), and makes the operation a single read + write
+// pass.  In-place safety: every member finishes reading its part of the tile before ANY
+// member writes (a per-group barrier in global memory: release-add on a counter, acquire
+// spin until all G members arrived); tiles are disjoint byte ranges owned by exactly one
+// group.  This replaces the paper's multi-pass cache-aware rotate (coarse cycle following
+// + fine on-chip rotation, §4.6) and cycle-following row permute (§4.7) -- prior art for
+// a K20c.
+//
+// Why software groups rather than hardware clusters: the strided tile access reaches
+// copy bandwidth only when each CTA stages a small band (16-64 KB, several CTAs per SM in
+// different phases; tools/pattern_probe.cu, profiles/), which needs groups far larger
+// than the 16-CTA cluster limit (a 17226-row tile of 128 B is ~2.6 MB).  The kernel is
+// persistent and launched cooperatively (every CTA co-resident, so the spin cannot
+// deadlock); group g walks the tiles g, g + ngroups, ...
 //
 // Tile-local forms (w = j - j0 is the column inside the tile [j0, j0 + W)):
 //  * COL_ROT, gather rotation rho_j = sign * floor(j/b) (Eq. 23 for sign = +1 as the C2R
 //    pre-rotation, Eq. 36 for sign = -1 as the R2C post-rotation):
 //        out[i][w] = in[(i + rho_{j0+w}) mod M][w]
-//    The CTA writing band [r0, r1) reads rows [r0 + min rho, r1 + max rho) -- a contiguous
-//    cyclic range (rho varies by < W inside a tile, :767-773 residual bound).
+//    The member writing band [r0, r1) reads rows [r0 + min rho, r1 + max rho) -- a
+//    contiguous cyclic range (rho varies by < W inside a tile, :767-773 residual bound).
 //  * COL_C2R_SHUF, s'_j(i) = (j + q(i)) mod M (Eq. 26 = p_j o q, Eqs. 32-33):
 //        out[i][w] = in[(k + w) mod M][w],  k = (j0 + q(i)) mod M.
-//    Scatter form: the CTA reads rows [r0, r1 + W - 1) (band + halo, contiguous), builds
-//    the skewed row T_k[w] = in[k + w][w] for each k of its band and writes it to output
-//    row i = q^{-1}((k - j0) mod M) (Eq. 34).
+//    Scatter form: the member reads rows [r0, r1 + W - 1) (band + halo, contiguous),
+//    builds the skewed row T_k[w] = in[k + w][w] for each k of its band and writes it to
+//    output row i = q^{-1}((k - j0) mod M) (Eq. 34).
 //  * COL_R2C_SHUF, (s')^{-1}_j(i) = q^{-1}((i - j) mod M) (Eqs. 34-35):
 //        out[i][w] = in[q^{-1}((i - w - j0) mod M)][w].
-//    The CTA writing band [r0, r1) reads the rows q^{-1}((u - j0) mod M) for
+//    The member writing band [r0, r1) reads the rows q^{-1}((u - j0) mod M) for
 //    u in [r0 - W + 1, r1) (scattered whole sub-rows) and writes its band contiguously.
 //
 // Memory access: each staged row is fetched as its 16-byte-aligned hull (TWB/16 + 1
@@ -40,7 +48,7 @@ namespace ipt {
 
 namespace {
 
-constexpr int kColThreads = 512;
+constexpr int kColThreads = 256;
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -70,9 +78,24 @@ __device__ __forceinline__ int32_t qinv_of(const ColParams &P, int32_t i) {
     return static_cast<int32_t>(u + cm * static_cast<uint32_t>(P.a));
 }
 
-// v mod M for v >= -kshift*M (kshift = 2 + W/M covers every caller; M < 2^30).
+// v mod M for v >= -kshift*M (kshift = 2 + W/M covers every caller; M < 2^29).
 __device__ __forceinline__ int32_t mod_M(int32_t v, uint32_t kshiftM, const FastDiv &fdM) {
     return static_cast<int32_t>(fmod_(static_cast<uint32_t>(v) + kshiftM, fdM));
+}
+
+// Group barrier in global memory: counter ctr counts arrivals of all tiles so far.
+__device__ __forceinline__ void group_barrier(unsigned int *ctr, unsigned int target) {
+    __syncthreads();  // every thread's cp.async data has landed in shared memory
+    if (threadIdx.x == 0) {
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
+        unsigned int v;
+        while (true) {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+            if (v >= target) break;
+            __nanosleep(64);
+        }
+    }
+    __syncthreads();
 }
 
 template <int TWB>
@@ -90,113 +113,121 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     constexpr int CH = TileGeom<TWB>::CH;
     extern __shared__ __align__(16) unsigned char smem[];
 
-    const int64_t cid = blockIdx.x / P.K;  // cluster id
-    const int32_t r = blockIdx.x - static_cast<int32_t>(cid * P.K);
-    const int32_t tile = static_cast<int32_t>(cid % P.ntiles);
-    const int64_t mat = cid / P.ntiles;
-    char *A = P.base + mat * P.mat_stride_bytes;
-    const int32_t j0 = tile * W;
-    const int32_t Wt = min(W, P.N - j0);
+    const int32_t g = blockIdx.x / P.G;          // group
+    const int32_t r = blockIdx.x - g * P.G;      // member = band index
+    if (g >= P.ngroups) return;
+    unsigned int *ctr = P.ctr + g;
     const int32_t r0 = r * P.B;
     const int32_t r1 = min(P.M, r0 + P.B);
     const int32_t nrows = max(0, r1 - r0);
-    const char *Aend = A + static_cast<int64_t>(P.M) * P.N * EB;
     const uint32_t kshM = static_cast<uint32_t>(2 + W / P.M) * static_cast<uint32_t>(P.M);
-    const int32_t j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j0), P.fd_M));
-
-    int32_t ext, base_off = 0, lo_q = 0, hi_q = 0;
-    if (MODE == COL_ROT) {
-        lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
-        hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + Wt - 1), P.fd_b));
-        // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.  The
-        // whole cluster shares the tile, so the early exit is cluster-uniform.
-        if (hi_q == 0) return;
-        ext = hi_q - lo_q;
-        base_off = P.rot_sign > 0 ? lo_q : -hi_q;  // smallest rotation amount in the tile
-    } else if (MODE == COL_COPY) {
-        ext = 0;
-    } else {
-        ext = W - 1;
-    }
-    const int32_t nslots = nrows > 0 ? nrows + ext : 0;
-
-    unsigned char *stage = smem;                                  // [nslots][SLOT]
-    uint8_t *dlt = smem + static_cast<size_t>(nslots) * SLOT;    // [nslots] hull offsets
-    int32_t *ridx = reinterpret_cast<int32_t *>(smem + ((static_cast<size_t>(nslots) * (SLOT + 1) + 3) & ~size_t(3)));
-
-    // ---- R2C: the scattered source rows of every slot ---------------------------------
-    if (MODE == COL_R2C_SHUF) {
-        for (int32_t t = threadIdx.x; t < nslots; t += blockDim.x) {
-            ridx[t] = qinv_of(P, mod_M(r0 - (W - 1) + t - j0m, kshM, P.fd_M));
-        }
-        __syncthreads();
-    }
-
-    // ---- load: cp.async of every staged row's 16-byte hull ------------------------------
-    // Source row of slot t: contiguous (rowbase + t) mod M for ROT / C2R, ridx[t] for R2C.
-    const int32_t rowbase = MODE == COL_ROT ? mod_M(r0 + base_off, kshM, P.fd_M) : r0;
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
-    const char *Aj = A + static_cast<int64_t>(j0) * EB;
-    const uint32_t sst = smem_u32(stage);
-    const int32_t nch = nslots * CH;
-    for (int32_t e = threadIdx.x; e < nch; e += blockDim.x) {
-        const int32_t t = e / CH, k = e - t * CH;
-        int32_t row;
+    const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
+    unsigned int nbar = 0;
+
+    for (int64_t tt = g; tt < P.total_tiles; tt += P.ngroups) {
+        const int32_t tile = static_cast<int32_t>(tt % P.ntiles);
+        const int64_t mat = tt / P.ntiles;
+        char *A = P.base + mat * P.mat_stride_bytes;
+        const char *Aend = A + static_cast<int64_t>(P.M) * pitch;
+        const int32_t j0 = tile * W;
+        const int32_t Wt = min(W, P.N - j0);
+        const int32_t j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j0), P.fd_M));
+
+        int32_t ext, base_off = 0, lo_q = 0, hi_q = 0;
+        if (MODE == COL_ROT) {
+            lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
+            hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + Wt - 1), P.fd_b));
+            // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.
+            // Every member sees the same tile, so the skip is group-uniform.
+            if (hi_q == 0) continue;
+            ext = hi_q - lo_q;
+            base_off = P.rot_sign > 0 ? lo_q : -hi_q;  // smallest rotation amount in the tile
+        } else if (MODE == COL_COPY) {
+            ext = 0;
+        } else {
+            ext = W - 1;
+        }
+        const int32_t nslots = nrows > 0 ? nrows + ext : 0;
+
+        unsigned char *stage = smem;                                  // [nslots][SLOT]
+        uint8_t *dlt = smem + static_cast<size_t>(nslots) * SLOT;    // [nslots] hull offsets
+        int32_t *ridx = reinterpret_cast<int32_t *>(smem + ((static_cast<size_t>(nslots) * (SLOT + 1) + 3) & ~size_t(3)));
+
+        // ---- R2C: the scattered source rows of every slot -----------------------------
         if (MODE == COL_R2C_SHUF) {
-            row = ridx[t];
-        } else {
-            row = rowbase + t;
-            if (row >= P.M) row = row - P.M < P.M ? row - P.M : mod_M(row, kshM, P.fd_M);
+            for (int32_t t = threadIdx.x; t < nslots; t += blockDim.x)
+                ridx[t] = qinv_of(P, mod_M(r0 - (W - 1) + t - j0m, kshM, P.fd_M));
+            __syncthreads();
         }
-        const char *ra = Aj + row * pitch;
-        const int d = static_cast<int>(reinterpret_cast<uintptr_t>(ra) & 15);
-        if (k == 0) dlt[t] = static_cast<uint8_t>(d);
-        const char *lo = ra - d + 16 * k;
-        if (16 * k >= d + Wt * EB) continue;  // past the end of this row's tile
-        const uint32_t dst = sst + t * SLOT + 16 * k;
-        // Only row 0's head and row M-1's tail can leave the matrix.
-        if ((row != 0 && row != P.M - 1) || (lo >= A && lo + 16 <= Aend)) {
-            cp_async16(dst, lo);
-        } else {
+
+        // ---- load: cp.async of every staged row's 16-byte hull --------------------------
+        // Source row of slot t: contiguous (rowbase + t) mod M for ROT / C2R / COPY,
+        // ridx[t] for R2C.
+        const int32_t rowbase = MODE == COL_ROT ? mod_M(r0 + base_off, kshM, P.fd_M) : r0;
+        const char *Aj = A + static_cast<int64_t>(j0) * EB;
+        const uint32_t sst = smem_u32(stage);
+        const int32_t nch = nslots * CH;
+        for (int32_t e = threadIdx.x; e < nch; e += blockDim.x) {
+            const int32_t t = e / CH, k = e - t * CH;
+            int32_t row;
+            if (MODE == COL_R2C_SHUF) {
+                row = ridx[t];
+            } else {
+                row = rowbase + t;
+                if (row >= P.M) row = row - P.M < P.M ? row - P.M : mod_M(row, kshM, P.fd_M);
+            }
+            const char *ra = Aj + row * pitch;
+            const int d = static_cast<int>(reinterpret_cast<uintptr_t>(ra) & 15);
+            if (k == 0) dlt[t] = static_cast<uint8_t>(d);
+            const char *lo = ra - d + 16 * k;
+            if (16 * k >= d + Wt * EB) continue;  // past the end of this row's tile
+            const uint32_t dst = sst + t * SLOT + 16 * k;
+            // Only row 0's head and row M-1's tail can leave the matrix.
+            if ((row != 0 && row != P.M - 1) || (lo >= A && lo + 16 <= Aend)) {
+                cp_async16(dst, lo);
+            } else {
 #pragma unroll
-            for (int q = 0; q < 16; q += EB)
-                if (lo + q >= A && lo + q < Aend) cp_async_small<EB>(dst + q, lo + q);
+                for (int q = 0; q < 16; q += EB)
+                    if (lo + q >= A && lo + q < Aend) cp_async_small<EB>(dst + q, lo + q);
+            }
         }
-    }
 
-    // ---- C2R: destination rows of the band, while the loads are in flight ------------
-    if (MODE == COL_C2R_SHUF) {
-        for (int32_t kk = threadIdx.x; kk < nrows; kk += blockDim.x)
-            ridx[kk] = qinv_of(P, mod_M(r0 + kk - j0m, kshM, P.fd_M));
-    }
-    cp_async_wait_all();
+        // ---- C2R: destination rows of the band, while the loads are in flight --------
+        if (MODE == COL_C2R_SHUF) {
+            for (int32_t kk = threadIdx.x; kk < nrows; kk += blockDim.x)
+                ridx[kk] = qinv_of(P, mod_M(r0 + kk - j0m, kshM, P.fd_M));
+        }
+        cp_async_wait_all();
 
-    // In-place hazard barrier: the whole tile has been read before anyone writes it.
-    if (P.K > 1 && !(MODE == COL_COPY && P.rot_sign == 0)) cluster_barrier(); else __syncthreads();
+        // In-place hazard barrier: the whole tile has been read before anyone writes it.
+        if (use_barrier) group_barrier(ctr, (++nbar) * static_cast<unsigned int>(P.G));
+        else __syncthreads();
 
-    // ---- write ---------------------------------------------------------------------------
-    const int32_t w = threadIdx.x & (W - 1);  // blockDim is a multiple of W: fixed per thread
-    if (w >= Wt) return;
-    int32_t dw = 0;
-    if (MODE == COL_COPY) {
-        dw = 0;
-    } else if (MODE == COL_ROT) {
-        const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + w), P.fd_b));
-        dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
-    } else if (MODE == COL_C2R_SHUF) {
-        dw = w;
-    } else {
-        dw = W - 1 - w;
-    }
-    T *out = reinterpret_cast<T *>(A) + j0 + w;
-    const unsigned char *sw = stage + dw * SLOT + w * EB;
-    const uint8_t *dl = dlt + dw;
-    const int32_t kstep = blockDim.x >> LW;
+        // ---- write -----------------------------------------------------------------------
+        const int32_t w = threadIdx.x & (W - 1);  // blockDim is a multiple of W: fixed per thread
+        if (w < Wt) {
+            int32_t dw = 0;
+            if (MODE == COL_ROT) {
+                const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + w), P.fd_b));
+                dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
+            } else if (MODE == COL_C2R_SHUF) {
+                dw = w;
+            } else if (MODE == COL_R2C_SHUF) {
+                dw = W - 1 - w;
+            }
+            T *out = reinterpret_cast<T *>(A) + j0 + w;
+            const unsigned char *sw = stage + dw * SLOT + w * EB;
+            const uint8_t *dl = dlt + dw;
+            const int32_t kstep = blockDim.x >> LW;
 #pragma unroll 4
-    for (int32_t kk = threadIdx.x >> LW; kk < nrows; kk += kstep) {
-        const T v = *reinterpret_cast<const T *>(sw + kk * SLOT + dl[kk]);
-        const int64_t orow = MODE == COL_C2R_SHUF ? ridx[kk] : r0 + kk;
-        out[orow * P.N] = v;
+            for (int32_t kk = threadIdx.x >> LW; kk < nrows; kk += kstep) {
+                const T v = *reinterpret_cast<const T *>(sw + kk * SLOT + dl[kk]);
+                const int64_t orow = MODE == COL_C2R_SHUF ? ridx[kk] : r0 + kk;
+                out[orow * P.N] = v;
+            }
+        }
+        __syncthreads();  // shared memory is refilled for the next tile
     }
 }
 
@@ -235,8 +266,6 @@ void *col_kernel(int mode, int eb, int twb) {
     }
 }
 
-cudaError_t prepare(void *kern, int K, size_t smem) { return ensure_kernel_attrs(kern, smem, K > 8); }
-
 }  // namespace
 
 size_t col_smem_bytes(int64_t B, int64_t W, int eb) {
@@ -248,52 +277,46 @@ size_t col_smem_bytes(int64_t B, int64_t W, int eb) {
 
 int col_block_threads() { return kColThreads; }
 
-int col_max_active_clusters(int mode, int eb, int twb, int K, size_t smem) {
+int col_resident_ctas(int mode, int eb, int twb, size_t smem) {
     void *kern = col_kernel(mode, eb, twb);
-    if (!kern || prepare(kern, K, smem) != cudaSuccess) {
+    if (!kern || ensure_kernel_attrs(kern, smem, false) != cudaSuccess) {
         cudaGetLastError();
         return 0;
     }
-    cudaLaunchConfig_t cfg = {};
-    cudaLaunchAttribute attr[1];
-    cfg.gridDim = dim3(static_cast<unsigned>(K) * 64);
-    cfg.blockDim = dim3(kColThreads);
-    cfg.dynamicSmemBytes = smem;
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = K;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    int n = 0;
-    if (cudaOccupancyMaxActiveClusters(&n, kern, &cfg) != cudaSuccess) {
-        cudaGetLastError();
-        return 0;
-    }
-    return n;
+    return cached_resident_blocks(kern, kColThreads, smem);
 }
 
-cudaError_t launch_col(const ColParams &P, int mode, int eb, cudaStream_t st, size_t smem) {
-    void *kern = col_kernel(mode, eb, P.W * eb);
+cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, size_t smem) {
+    void *kern = col_kernel(mode, eb, P0.W * eb);
     if (!kern) return cudaErrorInvalidValue;
-    cudaError_t e = prepare(kern, P.K, smem);
+    cudaError_t e = ensure_kernel_attrs(kern, smem, false);
     if (e != cudaSuccess) return e;
-    const int64_t grid = static_cast<int64_t>(P.K) * P.ntiles * P.batch;
-    if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+    ColParams P = P0;
+    const bool need_ctr = P.G > 1;
+    if (need_ctr) {
+        // One arrival counter per group, stream-ordered scratch (freed after the launch).
+        e = cudaMallocAsync(reinterpret_cast<void **>(&P.ctr), sizeof(unsigned int) * P.ngroups, st);
+        if (e != cudaSuccess) return e;
+        e = cudaMemsetAsync(P.ctr, 0, sizeof(unsigned int) * P.ngroups, st);
+        if (e != cudaSuccess) return e;
+    }
     cudaLaunchConfig_t cfg = {};
     cudaLaunchAttribute attr[1];
-    cfg.gridDim = dim3(static_cast<unsigned>(grid));
+    cfg.gridDim = dim3(static_cast<unsigned>(P.ngroups) * static_cast<unsigned>(P.G));
     cfg.blockDim = dim3(kColThreads);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = st;
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = P.K;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
+    attr[0].id = cudaLaunchAttributeCooperative;  // all CTAs co-resident: the group spin is safe
+    attr[0].val.cooperative = need_ctr ? 1 : 0;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    void *args[] = {const_cast<ColParams *>(&P)};
-    return cudaLaunchKernelExC(&cfg, kern, args);
+    void *args[] = {&P};
+    e = cudaLaunchKernelExC(&cfg, kern, args);
+    if (need_ctr) {
+        cudaError_t e2 = cudaFreeAsync(P.ctr, st);
+        if (e == cudaSuccess) e = e2;
+    }
+    return e;
 }
 
 }  // namespace ipt

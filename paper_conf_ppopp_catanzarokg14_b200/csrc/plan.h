@@ -63,9 +63,13 @@ struct ColParams {
     int32_t binv;   // mmi(b, a)
     FastDiv fd_c, fd_a, fd_b, fd_M;
     int32_t W, log2W;   // tile width in elements (power of two)
-    int32_t ntiles;     // ceil(N / W)
-    int32_t K;          // cluster size (CTAs per tile)
-    int32_t B;          // rows per CTA band: ceil(M / K)
+    int32_t ntiles;     // ceil(N / W) tiles per matrix
+    int32_t G;          // CTAs per group = bands per tile: ceil(M / B)
+    int32_t B;          // rows per CTA band
+    int32_t ngroups;    // groups in the persistent grid (grid = ngroups * G)
+    int32_t resident;   // co-resident CTAs of this configuration (SMs x CTAs per SM)
+    int64_t total_tiles;  // ntiles * batch
+    unsigned int *ctr;  // per-group arrival counters (stream-ordered scratch, launch_col)
     int32_t rot_sign;   // COL_ROT: +1 (C2R pre-rotation) or -1 (R2C post-rotation)
     int32_t wide_a;     // a >= 2^16
 };
@@ -84,6 +88,6 @@ cudaError_t launch_row(const RowParams &p, int dir, int eb, cudaStream_t st);
 size_t col_smem_bytes(int64_t B, int64_t W, int eb);
 int col_block_threads();
 cudaError_t launch_col(const ColParams &p, int mode, int eb, cudaStream_t st, size_t smem);
-int col_max_active_clusters(int mode, int eb, int twb, int K, size_t smem);
+int col_resident_ctas(int mode, int eb, int twb, size_t smem);
 
 }  // namespace ipt

@@ -42,8 +42,8 @@ def main():
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     t = timed(lambda: y.copy_(x), flush)
     print(json.dumps({"what": "torch copy_", "GBps": round(2 * nb / t / 1e6, 1)}), flush=True)
-    for twb in (32, 64, 128):
-        for K in (4, 6, 8, 10, 12, 14, 16):
+    for twb in (64, 128):
+        for K in (16, 32, 48, 64, 96, 128):
             for bar in (0, 1):
                 try:
                     t = timed(lambda: ipt.debug_tile_copy(x, a.M, a.N, a.eb, twb, K, bar), flush)
