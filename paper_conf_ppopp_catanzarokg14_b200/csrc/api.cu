@@ -105,20 +105,20 @@ int ilog2(int v) {
 
 // Column-tile geometry.  Tile width TWB = IPT_TILE_BYTES (32, 64 or 128; default 128 B =
 // one cache line).  Band: the rows per CTA that fit the per-CTA shared-memory target
-// IPT_COL_SMEM (default 40 KiB: several CTAs per SM in different load/store phases --
-// the regime in which the strided tile pattern reaches copy bandwidth, tools/
-// pattern_probe.cu).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
+// IPT_COL_SMEM (default 100 KiB, two CTAs per SM: the best of the round-1 sweep over
+// 24-200 KiB, profiles/r01_*).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
 // the co-resident CTAs, the band grows (up to the opt-in shared-memory maximum).
 ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp) {
     int twb = env_int("IPT_TILE_BYTES", 128);
     if (twb != 32 && twb != 64 && twb != 128) twb = 128;
     if (twb < pl.eb) twb = pl.eb;
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
-    const int64_t target = env_int("IPT_COL_SMEM", 40 * 1024);
+    const int64_t target = env_int("IPT_COL_SMEM", 100 * 1024);
     const int64_t W = twb / pl.eb;
-    const int64_t per_row = twb + 16 + 1 + 4;  // col_smem_bytes: hull + offset + row index
+    const int64_t per_row = 2 * (twb + 16 + 1 + 4);  // col_smem_bytes: 2 buffers x (hull + offset + row)
     int64_t B = target / per_row - (W - 1);
     if (B < 32) B = 32;
+    if (B > col_max_band(W)) B = col_max_band(W);
     if (B > pl.M) B = pl.M;
     for (;;) {
         const size_t smem = col_smem_bytes(B, W, pl.eb);
@@ -128,6 +128,7 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
         if (resident < 1) return IPT_ERR_UNSUPPORTED;
         if (G > resident) {  // a whole group must be co-resident
             B = (pl.M + resident - 1) / resident;
+            if (B > col_max_band(W)) return IPT_ERR_UNSUPPORTED;
             continue;
         }
         ColParams &p = cp.p;
@@ -159,6 +160,7 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
 // Persistent grid of a column pass over `batch` matrices: as many whole groups as are
 // co-resident, never more than there are tiles.
 void finish_col(ColParams &p, int64_t batch) {
+    if (p.G < 1) return;  // pass not planned (e.g. no rotation when gcd = 1)
     p.total_tiles = static_cast<int64_t>(p.ntiles) * batch;
     int64_t ng = p.resident / p.G;
     if (ng > p.total_tiles) ng = p.total_tiles;
@@ -176,6 +178,9 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     if (dev.major != 10 || dev.minor != 0) return IPT_ERR_UNSUPPORTED;  // sm_100 only
 
     int engine = x > y ? ENG_C2R : ENG_R2C;
+    // IPT_ENGINE_RULE=1: the opposite choice (rows = the long dimension, column tiles of
+    // the short one) -- the B200 retune study of SURVEY §8 f2.
+    if (env_int("IPT_ENGINE_RULE", 0) == 1) engine = x > y ? ENG_R2C : ENG_C2R;
     const char *force = std::getenv("IPT_FORCE_ENGINE");
     if (force && !std::strcmp(force, "c2r")) engine = ENG_C2R;
     if (force && !std::strcmp(force, "r2c")) engine = ENG_R2C;
@@ -250,7 +255,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_FUSE_ROT"}) {
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_FUSE_ROT", "IPT_ENGINE_RULE"}) {
         const char *v = std::getenv(n);
         s += v ? v : "-";
         s += '|';
@@ -420,6 +425,25 @@ cudaError_t ensure_kernel_attrs(const void *kern, size_t smem, bool nonportable_
     return cudaSuccess;
 }
 
+unsigned int *group_counters(cudaStream_t st, int n) {
+    if (n > kMaxGroups) return nullptr;
+    static std::mutex mu;
+    static std::unordered_map<std::string, unsigned int *> blocks;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const std::string key = std::to_string(dev) + "/" + std::to_string(reinterpret_cast<uintptr_t>(st));
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = blocks.find(key);
+    if (it != blocks.end()) return it->second;
+    unsigned int *p = nullptr;
+    if (cudaMalloc(&p, sizeof(unsigned int) * kMaxGroups) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    blocks[key] = p;
+    return p;
+}
+
 int cached_resident_blocks(const void *kern, int threads, size_t smem) {
     static std::mutex mu;
     static std::unordered_map<std::string, int> cache;
@@ -535,6 +559,7 @@ ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes
     p.log2W = ilog2(p.W);
     p.ntiles = static_cast<int32_t>((N + p.W - 1) / p.W);
     p.B = static_cast<int32_t>((M + cluster - 1) / cluster);
+    if (p.B > col_max_band(p.W)) return IPT_ERR_UNSUPPORTED;
     p.G = static_cast<int32_t>((M + p.B - 1) / p.B);
     p.rot_sign = barrier ? 1 : 0;
     const size_t smem = col_smem_bytes(p.B, p.W, elem_bytes);

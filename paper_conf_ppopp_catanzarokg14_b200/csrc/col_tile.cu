@@ -12,12 +12,12 @@
 // + fine on-chip rotation, §4.6) and cycle-following row permute (§4.7) -- prior art for
 // a K20c.
 //
-// Why software groups rather than hardware clusters: the strided tile access reaches
-// copy bandwidth only when each CTA stages a small band (16-64 KB, several CTAs per SM in
-// different phases; tools/pattern_probe.cu, profiles/), which needs groups far larger
-// than the 16-CTA cluster limit (a 17226-row tile of 128 B is ~2.6 MB).  The kernel is
-// persistent and launched cooperatively (every CTA co-resident, so the spin cannot
-// deadlock); group g walks the tiles g, g + ngroups, ...
+// Why software groups rather than hardware clusters: a group can be any size up to the
+// co-resident CTA count (a 17226-row tile of 128 B is ~2.6 MB, beyond a 16-CTA cluster
+// at 128-byte tiles), and the non-persistent grid lets CTAs drift out of lock-step (a
+// persistent cooperative variant and a two-buffer pipelined variant were both slower:
+// profiles/).  The grid is one CTA per (tile, band); see col_tile_kernel for why the spin
+// barrier cannot deadlock.
 //
 // Tile-local forms (w = j - j0 is the column inside the tile [j0, j0 + W)):
 //  * COL_ROT, gather rotation rho_j = sign * floor(j/b) (Eq. 23 for sign = +1 as the C2R
@@ -40,21 +40,23 @@
 // CTA has its whole band in flight at once; rows are 16-byte aligned only when
 // N*eb % 16 == 0, and the hull's extra bytes (neighbouring tiles of the same row) are
 // never used.  Chunks that would leave the matrix (row 0 head, row M-1 tail) are fetched
-// element by element.  Stores are element-wise (eb bytes per thread, a warp covers
-// 32*eb/TWB whole tile rows).
+// element by element.  (One TMA bulk copy per 144-byte hull was tried and is ~2x slower:
+// the TMA engine does not keep up with that many tiny requests; profiles/.)  Stores: one 16-byte destination
+// chunk per thread, gathered from the staged rows and written with a vector store
+// (element stores only in a row's ragged head/tail chunk).
 #include "plan.h"
 
 namespace ipt {
 
 namespace {
 
-constexpr int kColThreads = 256;
+#ifndef IPT_COL_THREADS
+#define IPT_COL_THREADS 512
+#endif
+constexpr int kColThreads = IPT_COL_THREADS;
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void cp_async16(uint32_t dst, const void *src) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(src) : "memory");
 }
 template <int B>
 __device__ __forceinline__ void cp_async_small(uint32_t dst, const void *src) {
@@ -104,131 +106,221 @@ struct TileGeom {
     static constexpr int CH = TWB / 16 + 1;  // hull chunks per staged row
 };
 
+// Per-tile geometry of one staging buffer.
+struct TileCtx {
+    char *A;            // this matrix
+    const char *Aend;
+    int32_t j0, Wt, j0m;
+    int32_t lo_q, hi_q, base_off, nslots;
+};
+
+// Staging buffer layout (one of two): [dw W*4 | stage nslots_max*SLOT | dlt nslots_max |
+// ridx nslots_max*4], nslots_max = B + W - 1.
+template <int TWB>
+__host__ __device__ constexpr size_t buf_dw_bytes(int W) { return (static_cast<size_t>(W) * 4 + 15) & ~size_t(15); }
+__host__ __device__ inline size_t buf_bytes(int64_t nslots_max, int W, int twb) {
+    const size_t slot = static_cast<size_t>(twb) + 16;
+    return ((static_cast<size_t>(W) * 4 + 15) & ~size_t(15)) + ((static_cast<size_t>(nslots_max) * (slot + 1) + 15) & ~size_t(15)) +
+           ((static_cast<size_t>(nslots_max) * 4 + 15) & ~size_t(15));  // keeps the second buffer 16-B aligned
+}
+
 template <int EB, int MODE, int TWB>
-__global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
-    using T = typename Word<EB>::T;
+__device__ __forceinline__ bool make_ctx(const ColParams &P, int64_t tt, int32_t nrows, TileCtx &c) {
     constexpr int W = TWB / EB;
-    constexpr int LW = W == 1 ? 0 : W == 2 ? 1 : W == 4 ? 2 : W == 8 ? 3 : W == 16 ? 4 : 5;
+    const int32_t tile = static_cast<int32_t>(tt % P.ntiles);
+    const int64_t mat = tt / P.ntiles;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    c.A = P.base + mat * P.mat_stride_bytes;
+    c.Aend = c.A + static_cast<int64_t>(P.M) * pitch;
+    c.j0 = tile * W;
+    c.Wt = min(W, P.N - c.j0);
+    c.j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(c.j0), P.fd_M));
+    int32_t ext = W - 1;
+    c.lo_q = c.hi_q = c.base_off = 0;
+    if (MODE == COL_ROT) {
+        c.lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(c.j0), P.fd_b));
+        c.hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(c.j0 + c.Wt - 1), P.fd_b));
+        // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.
+        // Every member sees the same tile, so the skip is group-uniform.
+        if (c.hi_q == 0) return false;
+        ext = c.hi_q - c.lo_q;
+        c.base_off = P.rot_sign > 0 ? c.lo_q : -c.hi_q;  // smallest rotation amount in the tile
+    } else if (MODE == COL_COPY) {
+        ext = 0;
+    }
+    c.nslots = nrows > 0 ? nrows + ext : 0;
+    return true;
+}
+
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ int64_t next_tile(const ColParams &P, int64_t tt, int32_t nrows, TileCtx &c) {
+    for (; tt < P.total_tiles; tt += P.ngroups)
+        if (make_ctx<EB, MODE, TWB>(P, tt, nrows, c)) return tt;
+    return tt;
+}
+
+// Issue the cp.async loads of one tile band into buffer `buf` (one commit group).
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ void load_tile(const ColParams &P, const TileCtx &c, unsigned char *buf, int32_t r0,
+                                          int32_t nrows, int32_t nslots_max, uint32_t kshM) {
+    constexpr int W = TWB / EB;
     constexpr int SLOT = TileGeom<TWB>::SLOT;
     constexpr int CH = TileGeom<TWB>::CH;
-    extern __shared__ __align__(16) unsigned char smem[];
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    int32_t *dwt = reinterpret_cast<int32_t *>(buf);
+    unsigned char *stage = buf + buf_dw_bytes<TWB>(W);
+    uint8_t *dlt = stage + static_cast<size_t>(nslots_max) * SLOT;
+    int32_t *ridx = reinterpret_cast<int32_t *>(stage + ((static_cast<size_t>(nslots_max) * (SLOT + 1) + 15) & ~size_t(15)));
 
-    const int32_t g = blockIdx.x / P.G;          // group
-    const int32_t r = blockIdx.x - g * P.G;      // member = band index
-    if (g >= P.ngroups) return;
-    unsigned int *ctr = P.ctr + g;
+    // Slot offset of column w: the element of output row kk comes from staged row kk + dw[w].
+    for (int32_t w = threadIdx.x; w < W; w += blockDim.x) {
+        int32_t dw = 0;
+        if (MODE == COL_ROT) {
+            const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(c.j0 + min(w, c.Wt - 1)), P.fd_b));
+            dw = P.rot_sign > 0 ? qw - c.lo_q : c.hi_q - qw;  // rho_w - min rho
+        } else if (MODE == COL_C2R_SHUF) {
+            dw = w;
+        } else if (MODE == COL_R2C_SHUF) {
+            dw = W - 1 - w;
+        }
+        dwt[w] = dw;
+    }
+    // Source row of slot t: contiguous (rowbase + t) mod M for ROT / C2R / COPY,
+    // q^{-1}((r0 - W + 1 + t - j0) mod M) for R2C (ridx, computed first).
+    if (MODE == COL_R2C_SHUF) {
+        for (int32_t t = threadIdx.x; t < c.nslots; t += blockDim.x)
+            ridx[t] = qinv_of(P, mod_M(r0 - (W - 1) + t - c.j0m, kshM, P.fd_M));
+        __syncthreads();
+    }
+    const int32_t rowbase = MODE == COL_ROT ? mod_M(r0 + c.base_off, kshM, P.fd_M) : r0;
+    const char *Aj = c.A + static_cast<int64_t>(c.j0) * EB;
+    const uint32_t sst = smem_u32(stage);
+    const int32_t nch = c.nslots * CH;
+    const int32_t vbytes = c.Wt * EB;
+    for (int32_t e = threadIdx.x; e < nch; e += blockDim.x) {
+        const int32_t t = e / CH, k = e - t * CH;
+        int32_t row;
+        if (MODE == COL_R2C_SHUF) {
+            row = ridx[t];
+        } else {
+            row = rowbase + t;
+            if (row >= P.M) row = row - P.M < P.M ? row - P.M : mod_M(row, kshM, P.fd_M);
+        }
+        const char *ra = Aj + row * pitch;
+        const int d = static_cast<int>(reinterpret_cast<uintptr_t>(ra) & 15);
+        if (k == 0) dlt[t] = static_cast<uint8_t>(d);
+        if (16 * k >= d + vbytes) continue;  // past the end of this row's tile
+        const char *lo = ra - d + 16 * k;
+        const uint32_t dst = sst + t * SLOT + 16 * k;
+        // Only row 0's head and row M-1's tail can leave the matrix.
+        if ((row != 0 && row != P.M - 1) || (lo >= c.A && lo + 16 <= c.Aend)) {
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(lo) : "memory");
+        } else {
+#pragma unroll
+            for (int q = 0; q < 16; q += EB)
+                if (lo + q >= c.A && lo + q < c.Aend) cp_async_small<EB>(dst + q, lo + q);
+        }
+    }
+    // C2R: destination rows of the band, while the loads are in flight.
+    if (MODE == COL_C2R_SHUF) {
+        for (int32_t kk = threadIdx.x; kk < nrows; kk += blockDim.x)
+            ridx[kk] = qinv_of(P, mod_M(r0 + kk - c.j0m, kshM, P.fd_M));
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+// Write one tile band from buffer `buf`: one 16-byte destination chunk per thread.
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ void store_tile(const ColParams &P, const TileCtx &c, const unsigned char *buf, int32_t r0,
+                                           int32_t nrows, int32_t nslots_max) {
+    using T = typename Word<EB>::T;
+    constexpr int W = TWB / EB;
+    constexpr int SLOT = TileGeom<TWB>::SLOT;
+    constexpr int NQ = TWB / 16 + 1;  // 16-byte destination chunks a tile row can touch
+    constexpr int PER = 16 / EB;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    const int32_t *dwt = reinterpret_cast<const int32_t *>(buf);
+    const unsigned char *stage = buf + buf_dw_bytes<TWB>(W);
+    const uint8_t *dlt = stage + static_cast<size_t>(nslots_max) * SLOT;
+    const int32_t *ridx =
+        reinterpret_cast<const int32_t *>(stage + ((static_cast<size_t>(nslots_max) * (SLOT + 1) + 15) & ~size_t(15)));
+    char *Aj = c.A + static_cast<int64_t>(c.j0) * EB;
+    const int32_t Wt = c.Wt;
+    const int32_t nout = nrows * NQ;
+    for (int32_t e = threadIdx.x; e < nout; e += blockDim.x) {
+        const int32_t kk = e / NQ, q = e - kk * NQ;
+        const int64_t orow = MODE == COL_C2R_SHUF ? ridx[kk] : r0 + kk;
+        char *da = Aj + orow * pitch;  // output row's tile start
+        const int dd = static_cast<int>(reinterpret_cast<uintptr_t>(da) & 15);
+        const int w0 = (16 * q - dd) / EB;  // first column of this chunk (may be < 0)
+        if (w0 >= Wt) continue;
+        if (w0 >= 0 && w0 + PER <= Wt) {
+            union { uint4 u; T t[PER]; } v;
+            const int32_t ta = kk + dwt[w0], tb = kk + dwt[w0 + PER - 1];
+            const uint32_t so = ta * SLOT + dlt[ta] + w0 * EB;
+            if (ta == tb && (so & 15) == 0) {  // one staged row, aligned: a single LDS.128
+                v.u = *reinterpret_cast<const uint4 *>(stage + so);
+            } else {
+#pragma unroll
+                for (int x = 0; x < PER; ++x) {
+                    const int32_t t = kk + dwt[w0 + x];
+                    v.t[x] = *reinterpret_cast<const T *>(stage + t * SLOT + dlt[t] + (w0 + x) * EB);
+                }
+            }
+            *reinterpret_cast<uint4 *>(da + w0 * EB) = v.u;
+        } else {
+#pragma unroll
+            for (int x = 0; x < PER; ++x) {
+                const int w = w0 + x;
+                if (w < 0 || w >= Wt) continue;
+                const int32_t t = kk + dwt[w];
+                reinterpret_cast<T *>(da)[w] = *reinterpret_cast<const T *>(stage + t * SLOT + dlt[t] + w * EB);
+            }
+        }
+    }
+}
+
+// One CTA per (tile, band).  The CTA's logical id comes from a ticket counter taken at
+// start (dispatch order), so the G members of a tile are exactly G consecutive tickets:
+// every group whose tickets are all taken is fully resident, hence only the newest group
+// can be waiting for members, and those get scheduled as older groups finish -- the spin
+// barrier cannot deadlock as long as one group fits on the GPU (G <= resident CTAs).
+template <int EB, int MODE, int TWB>
+__global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
+    constexpr int W = TWB / EB;
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ unsigned int s_ticket;
+    if (threadIdx.x == 0) s_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
+    __syncthreads();
+    const unsigned int ticket = s_ticket;
+    const int64_t tt = ticket / static_cast<unsigned int>(P.G);   // tile (of all matrices)
+    const int32_t r = static_cast<int32_t>(ticket - tt * P.G);     // band
     const int32_t r0 = r * P.B;
     const int32_t r1 = min(P.M, r0 + P.B);
     const int32_t nrows = max(0, r1 - r0);
+    const int32_t nslots_max = P.B + W - 1;
     const uint32_t kshM = static_cast<uint32_t>(2 + W / P.M) * static_cast<uint32_t>(P.M);
-    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
     const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
-    unsigned int nbar = 0;
 
-    for (int64_t tt = g; tt < P.total_tiles; tt += P.ngroups) {
-        const int32_t tile = static_cast<int32_t>(tt % P.ntiles);
-        const int64_t mat = tt / P.ntiles;
-        char *A = P.base + mat * P.mat_stride_bytes;
-        const char *Aend = A + static_cast<int64_t>(P.M) * pitch;
-        const int32_t j0 = tile * W;
-        const int32_t Wt = min(W, P.N - j0);
-        const int32_t j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j0), P.fd_M));
-
-        int32_t ext, base_off = 0, lo_q = 0, hi_q = 0;
-        if (MODE == COL_ROT) {
-            lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
-            hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + Wt - 1), P.fd_b));
-            // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.
-            // Every member sees the same tile, so the skip is group-uniform.
-            if (hi_q == 0) continue;
-            ext = hi_q - lo_q;
-            base_off = P.rot_sign > 0 ? lo_q : -hi_q;  // smallest rotation amount in the tile
-        } else if (MODE == COL_COPY) {
-            ext = 0;
-        } else {
-            ext = W - 1;
-        }
-        const int32_t nslots = nrows > 0 ? nrows + ext : 0;
-
-        unsigned char *stage = smem;                                  // [nslots][SLOT]
-        uint8_t *dlt = smem + static_cast<size_t>(nslots) * SLOT;    // [nslots] hull offsets
-        int32_t *ridx = reinterpret_cast<int32_t *>(smem + ((static_cast<size_t>(nslots) * (SLOT + 1) + 3) & ~size_t(3)));
-
-        // ---- R2C: the scattered source rows of every slot -----------------------------
-        if (MODE == COL_R2C_SHUF) {
-            for (int32_t t = threadIdx.x; t < nslots; t += blockDim.x)
-                ridx[t] = qinv_of(P, mod_M(r0 - (W - 1) + t - j0m, kshM, P.fd_M));
-            __syncthreads();
-        }
-
-        // ---- load: cp.async of every staged row's 16-byte hull --------------------------
-        // Source row of slot t: contiguous (rowbase + t) mod M for ROT / C2R / COPY,
-        // ridx[t] for R2C.
-        const int32_t rowbase = MODE == COL_ROT ? mod_M(r0 + base_off, kshM, P.fd_M) : r0;
-        const char *Aj = A + static_cast<int64_t>(j0) * EB;
-        const uint32_t sst = smem_u32(stage);
-        const int32_t nch = nslots * CH;
-        for (int32_t e = threadIdx.x; e < nch; e += blockDim.x) {
-            const int32_t t = e / CH, k = e - t * CH;
-            int32_t row;
-            if (MODE == COL_R2C_SHUF) {
-                row = ridx[t];
-            } else {
-                row = rowbase + t;
-                if (row >= P.M) row = row - P.M < P.M ? row - P.M : mod_M(row, kshM, P.fd_M);
-            }
-            const char *ra = Aj + row * pitch;
-            const int d = static_cast<int>(reinterpret_cast<uintptr_t>(ra) & 15);
-            if (k == 0) dlt[t] = static_cast<uint8_t>(d);
-            const char *lo = ra - d + 16 * k;
-            if (16 * k >= d + Wt * EB) continue;  // past the end of this row's tile
-            const uint32_t dst = sst + t * SLOT + 16 * k;
-            // Only row 0's head and row M-1's tail can leave the matrix.
-            if ((row != 0 && row != P.M - 1) || (lo >= A && lo + 16 <= Aend)) {
-                cp_async16(dst, lo);
-            } else {
-#pragma unroll
-                for (int q = 0; q < 16; q += EB)
-                    if (lo + q >= A && lo + q < Aend) cp_async_small<EB>(dst + q, lo + q);
-            }
-        }
-
-        // ---- C2R: destination rows of the band, while the loads are in flight --------
-        if (MODE == COL_C2R_SHUF) {
-            for (int32_t kk = threadIdx.x; kk < nrows; kk += blockDim.x)
-                ridx[kk] = qinv_of(P, mod_M(r0 + kk - j0m, kshM, P.fd_M));
-        }
-        cp_async_wait_all();
-
-        // In-place hazard barrier: the whole tile has been read before anyone writes it.
-        if (use_barrier) group_barrier(ctr, (++nbar) * static_cast<unsigned int>(P.G));
-        else __syncthreads();
-
-        // ---- write -----------------------------------------------------------------------
-        const int32_t w = threadIdx.x & (W - 1);  // blockDim is a multiple of W: fixed per thread
-        if (w < Wt) {
-            int32_t dw = 0;
-            if (MODE == COL_ROT) {
-                const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + w), P.fd_b));
-                dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
-            } else if (MODE == COL_C2R_SHUF) {
-                dw = w;
-            } else if (MODE == COL_R2C_SHUF) {
-                dw = W - 1 - w;
-            }
-            T *out = reinterpret_cast<T *>(A) + j0 + w;
-            const unsigned char *sw = stage + dw * SLOT + w * EB;
-            const uint8_t *dl = dlt + dw;
-            const int32_t kstep = blockDim.x >> LW;
-#pragma unroll 4
-            for (int32_t kk = threadIdx.x >> LW; kk < nrows; kk += kstep) {
-                const T v = *reinterpret_cast<const T *>(sw + kk * SLOT + dl[kk]);
-                const int64_t orow = MODE == COL_C2R_SHUF ? ridx[kk] : r0 + kk;
-                out[orow * P.N] = v;
-            }
-        }
-        __syncthreads();  // shared memory is refilled for the next tile
+    TileCtx c;
+    if (!make_ctx<EB, MODE, TWB>(P, tt, nrows, c)) {  // group-uniform skip (ROT amount 0)
+        // Still arrive: later tiles sharing this counter slot count these arrivals.
+        if (use_barrier && threadIdx.x == 0)
+            atomicAdd(P.ctr + static_cast<unsigned int>(tt % kCtrSlots), 1u);
+        return;
     }
+    load_tile<EB, MODE, TWB>(P, c, smem, r0, nrows, nslots_max, kshM);
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    // In-place hazard barrier: the whole tile has been read before anyone writes it.
+    // Counter slot tt mod kCtrSlots, monotone over the tiles that share it.
+    if (use_barrier) {
+        const unsigned int slot = static_cast<unsigned int>(tt % kCtrSlots);
+        const unsigned int target = static_cast<unsigned int>(tt / kCtrSlots + 1) * static_cast<unsigned int>(P.G);
+        group_barrier(P.ctr + slot, target);
+    } else {
+        __syncthreads();
+    }
+    store_tile<EB, MODE, TWB>(P, c, smem, r0, nrows, nslots_max);
 }
 
 template <int EB, int MODE, int TWB>
@@ -269,11 +361,10 @@ void *col_kernel(int mode, int eb, int twb) {
 }  // namespace
 
 size_t col_smem_bytes(int64_t B, int64_t W, int eb) {
-    const int64_t twb = W * eb;
-    const int64_t nslots = B + W - 1;
-    const int64_t slot = twb + 16;
-    return static_cast<size_t>(((nslots * (slot + 1) + 3) & ~int64_t(3)) + nslots * 4);
+    return buf_bytes(B + W - 1, static_cast<int>(W), static_cast<int>(W * eb));
 }
+
+int64_t col_max_band(int64_t W) { return (int64_t(1) << 24) - W; }
 
 int col_block_threads() { return kColThreads; }
 
@@ -292,31 +383,17 @@ cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, s
     cudaError_t e = ensure_kernel_attrs(kern, smem, false);
     if (e != cudaSuccess) return e;
     ColParams P = P0;
-    const bool need_ctr = P.G > 1;
-    if (need_ctr) {
-        // One arrival counter per group, stream-ordered scratch (freed after the launch).
-        e = cudaMallocAsync(reinterpret_cast<void **>(&P.ctr), sizeof(unsigned int) * P.ngroups, st);
-        if (e != cudaSuccess) return e;
-        e = cudaMemsetAsync(P.ctr, 0, sizeof(unsigned int) * P.ngroups, st);
-        if (e != cudaSuccess) return e;
-    }
-    cudaLaunchConfig_t cfg = {};
-    cudaLaunchAttribute attr[1];
-    cfg.gridDim = dim3(static_cast<unsigned>(P.ngroups) * static_cast<unsigned>(P.G));
-    cfg.blockDim = dim3(kColThreads);
-    cfg.dynamicSmemBytes = smem;
-    cfg.stream = st;
-    attr[0].id = cudaLaunchAttributeCooperative;  // all CTAs co-resident: the group spin is safe
-    attr[0].val.cooperative = need_ctr ? 1 : 0;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
+    const int64_t grid = P.total_tiles * P.G;
+    if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
+    // Ticket + group counters: the stream's own block, zeroed in stream order.
+    P.ctr = group_counters(st, kCtrSlots + 1);
+    if (!P.ctr) return cudaErrorMemoryAllocation;
+    const int64_t used = P.total_tiles < kCtrSlots ? P.total_tiles : kCtrSlots;
+    e = cudaMemsetAsync(P.ctr, 0, sizeof(unsigned int) * (kTicketSlot + 1), st);
+    if (e != cudaSuccess) return e;
+    (void)used;
     void *args[] = {&P};
-    e = cudaLaunchKernelExC(&cfg, kern, args);
-    if (need_ctr) {
-        cudaError_t e2 = cudaFreeAsync(P.ctr, st);
-        if (e == cudaSuccess) e = e2;
-    }
-    return e;
+    return cudaLaunchKernel(kern, dim3(static_cast<unsigned>(grid)), dim3(kColThreads), args, smem, st);
 }
 
 }  // namespace ipt

@@ -80,6 +80,16 @@ struct ColParams {
 cudaError_t ensure_kernel_attrs(const void *kern, size_t smem, bool nonportable_cluster);
 int cached_resident_blocks(const void *kern, int threads, size_t smem);  // SMs x blocks per SM
 
+// Group-barrier counters of the column passes: one block per (device, stream), allocated
+// on first use and reused by every later launch on that stream (launches on one stream
+// are serialised; different streams never share a block).  Slots [0, kCtrSlots) are the
+// per-tile arrival counters (tile t uses slot t mod kCtrSlots), slot kTicketSlot is the
+// dispatch ticket.
+constexpr int kCtrSlots = 4096;
+constexpr int kTicketSlot = kCtrSlots;
+constexpr int kMaxGroups = kCtrSlots + 1;
+unsigned int *group_counters(cudaStream_t st, int n);
+
 // Launchers (col_tile.cu / row_shuffle.cu).  They return the CUDA error of the launch.
 size_t row_smem_bytes(int64_t N, int eb);
 int row_block_threads();
@@ -87,6 +97,7 @@ cudaError_t launch_row(const RowParams &p, int dir, int eb, cudaStream_t st);
 
 size_t col_smem_bytes(int64_t B, int64_t W, int eb);
 int col_block_threads();
+int64_t col_max_band(int64_t W);  // largest band a CTA may be given
 cudaError_t launch_col(const ColParams &p, int mode, int eb, cudaStream_t st, size_t smem);
 int col_resident_ctas(int mode, int eb, int twb, size_t smem);
 

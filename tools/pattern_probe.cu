@@ -33,12 +33,13 @@ __global__ void copy_tile(const char *__restrict__ a, char *__restrict__ b, int 
 }
 
 template <int TW>
-__global__ void copy_tile_staged(char *a, int M, int R, int band) {
+__global__ void copy_tile_staged(char *a, int M, int R, int band, int tile_major) {
     extern __shared__ __align__(16) unsigned char sm[];
     constexpr int LPR = TW / 16;
     const int ntile = R / TW;
-    const int tile = blockIdx.x % ntile;
-    const int bandi = blockIdx.x / ntile;
+    const int nband = (M + band - 1) / band;
+    const int tile = tile_major ? blockIdx.x / nband : blockIdx.x % ntile;
+    const int bandi = tile_major ? blockIdx.x % nband : blockIdx.x / ntile;
     const int r0 = bandi * band, r1 = min(M, r0 + band);
     const int sub = threadIdx.x % LPR;
     uint32_t s = (uint32_t)__cvta_generic_to_shared(sm);
@@ -86,14 +87,15 @@ template <int TW> void run_tile(void *) {
 }
 template <int TW> void run_tile_staged(void *) {
     int ntile = G.R / TW, nb = (G.M + G.band - 1) / G.band;
-    copy_tile_staged<TW><<<ntile * nb, G.threads, G.band * TW>>>(G.a, G.M, G.R, G.band);
+    copy_tile_staged<TW><<<ntile * nb, G.threads, G.band * TW>>>(G.a, G.M, G.R, G.band, G.grid);
 }
 void run_contig(void *) { copy_contig<<<148 * 8, 512>>>((const uint4 *)G.a, (uint4 *)G.b, (size_t)G.M * G.R / 16); }
 
 int main(int argc, char **argv) {
     int M = argc > 1 ? atoi(argv[1]) : 17226;
     int R = argc > 2 ? atoi(argv[2]) : 6052 * 4;
-    R = R / 128 * 128;  // keep tiles aligned for the probe
+    const int align = argc > 3 ? atoi(argv[3]) : 128;
+    R = R / align * align;  // row pitch alignment (128: line-aligned tiles; 16: misaligned rows)
     size_t bytes = (size_t)M * R;
     cudaMalloc(&G.a, bytes);
     cudaMalloc(&G.b, bytes);
@@ -104,9 +106,10 @@ int main(int argc, char **argv) {
     G.M = M;
     G.R = R;
     G.threads = 512;
+    G.grid = argc > 4 ? atoi(argv[4]) : 0;  // 1: tile-major block order
     float t = timeit(run_contig, nullptr, flush, fl);
     printf("{\"what\":\"contiguous\",\"GBps\":%.1f}\n", 2.0 * bytes / t / 1e6);
-    int bands[] = {256, 1024, 2048, 4096};
+    int bands[] = {128, 256, 512};
     for (int band : bands) {
         G.band = band;
         t = timeit(run_tile<32>, nullptr, flush, fl);
