@@ -105,17 +105,17 @@ int ilog2(int v) {
 
 // Column-tile geometry.  Tile width TWB = IPT_TILE_BYTES (32, 64 or 128; default 128 B =
 // one cache line).  Band: the rows per CTA that fit the per-CTA shared-memory target
-// IPT_COL_SMEM (default 100 KiB, two CTAs per SM: the best of the round-1 sweep over
-// 24-200 KiB, profiles/r01_*).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
+// IPT_COL_SMEM (default 50 KiB, four CTAs per SM: the best of the round-1 sweep over
+// 12-100 KiB, profiles/r01_*).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
 // the co-resident CTAs, the band grows (up to the opt-in shared-memory maximum).
 ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp) {
     int twb = env_int("IPT_TILE_BYTES", 128);
     if (twb != 32 && twb != 64 && twb != 128) twb = 128;
     if (twb < pl.eb) twb = pl.eb;
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
-    const int64_t target = env_int("IPT_COL_SMEM", 100 * 1024);
+    const int64_t target = env_int("IPT_COL_SMEM", 50 * 1024);
     const int64_t W = twb / pl.eb;
-    const int64_t per_row = 2 * (twb + 16 + 1 + 4);  // col_smem_bytes: 2 buffers x (hull + offset + row)
+    const int64_t per_row = twb + 16 + 1 + 4;  // col_smem_bytes: hull + offset + row index
     int64_t B = target / per_row - (W - 1);
     if (B < 32) B = 32;
     if (B > col_max_band(W)) B = col_max_band(W);
