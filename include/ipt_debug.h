@@ -25,6 +25,25 @@ extern "C" {
 ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes, int tile_bytes, int cluster,
                                  int barrier, void *stream);
 
+/*
+ * Consumer kernels of include/ipt/aos.cuh (§6.2, Figs. 8-10; SURVEY §8 row a6,
+ * BASELINE config 4) over `count` structs of `words` 4-byte words (1..32), contiguous:
+ *   ipt_debug_aos_copy: dst[k] = src[k];  ipt_debug_aos_fill: word i of dst[k] = k*words + i.
+ * variant: IPT_AOS_DIRECT (compiler-generated per-lane struct access), IPT_AOS_VECTOR
+ * (widest native vector dividing the struct), IPT_AOS_COALESCED (coalesced_ptr<T>).
+ * ipt_debug_warp_load_dump: per 32-struct chunk, dump[lane*words + k] = register k of lane
+ *   after warp_load_aos (must equal the chunk).  ipt_debug_warp_store: lane l's registers
+ *   taken per lane from regs[l*words + k], stored with warp_store_aos (dst must equal regs).
+ * nchunks counts chunks of 32 structs.
+ */
+#define IPT_AOS_DIRECT 0
+#define IPT_AOS_VECTOR 1
+#define IPT_AOS_COALESCED 2
+ipt_status_t ipt_debug_aos_copy(const void *src, void *dst, int64_t count, int words, int variant, void *stream);
+ipt_status_t ipt_debug_aos_fill(void *dst, int64_t count, int words, int variant, void *stream);
+ipt_status_t ipt_debug_warp_load_dump(const void *src, void *dump, int64_t nchunks, int words, void *stream);
+ipt_status_t ipt_debug_warp_store(const void *regs, void *dst, int64_t nchunks, int words, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

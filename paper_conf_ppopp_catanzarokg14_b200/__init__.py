@@ -28,7 +28,9 @@ STATUS = {0: "IPT_OK", 1: "IPT_ERR_INVALID_ARGUMENT", 2: "IPT_ERR_UNSUPPORTED",
 # Every symbol declared in include/ipt.h.
 EXPORTS = ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_status_string", "ipt_plan_info",
-           "ipt_launch_count", "ipt_profile_enable", "ipt_profile_read", "ipt_debug_tile_copy")
+           "ipt_launch_count", "ipt_profile_enable", "ipt_profile_read", "ipt_debug_tile_copy",
+           "ipt_debug_aos_copy", "ipt_debug_aos_fill", "ipt_debug_warp_load_dump", "ipt_debug_warp_store")
+AOS_DIRECT, AOS_VECTOR, AOS_COALESCED = 0, 1, 2
 PROFILE_KINDS = 8
 KERNEL_KINDS = ("row_shuffle", "col_shuffle", "col_rotate", "skinny")
 
@@ -64,6 +66,12 @@ _lib.ipt_profile_read.argtypes = [ctypes.POINTER(_i64), ctypes.POINTER(ctypes.c_
 _lib.ipt_profile_read.restype = _i64
 _lib.ipt_debug_tile_copy.argtypes = [_vp, _i64, _i64, _int, _int, _int, _int, _vp]
 _lib.ipt_debug_tile_copy.restype = _int
+_lib.ipt_debug_aos_copy.argtypes = [_vp, _vp, _i64, _int, _int, _vp]
+_lib.ipt_debug_aos_fill.argtypes = [_vp, _i64, _int, _int, _vp]
+_lib.ipt_debug_warp_load_dump.argtypes = [_vp, _vp, _i64, _int, _vp]
+_lib.ipt_debug_warp_store.argtypes = [_vp, _vp, _i64, _int, _vp]
+for _f in ("ipt_debug_aos_copy", "ipt_debug_aos_fill", "ipt_debug_warp_load_dump", "ipt_debug_warp_store"):
+    getattr(_lib, _f).restype = _int
 for _f in ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_plan_info"):
     getattr(_lib, _f).restype = _int
@@ -181,6 +189,35 @@ def debug_tile_copy(buf, M: int, N: int, elem_bytes: int, tile_bytes: int, clust
     _check(_lib.ipt_debug_tile_copy(p, M, N, eb, tile_bytes, cluster, 1 if barrier else 0, st),
            "ipt_debug_tile_copy")
     return buf
+
+
+def _dev_stream(t, stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream(t.device).cuda_stream
+    return stream if isinstance(stream, int) else stream.cuda_stream
+
+
+def aos_copy(src, dst, count: int, words: int, variant: int, stream=None):
+    """Consumer kernel dst[k] = src[k] over `count` structs of `words` 4-byte words
+    (variant AOS_DIRECT / AOS_VECTOR / AOS_COALESCED; include/ipt_debug.h)."""
+    _check(_lib.ipt_debug_aos_copy(src.data_ptr(), dst.data_ptr(), count, words, variant,
+                                   _dev_stream(dst, stream)), "ipt_debug_aos_copy")
+
+
+def aos_fill(dst, count: int, words: int, variant: int, stream=None):
+    _check(_lib.ipt_debug_aos_fill(dst.data_ptr(), count, words, variant, _dev_stream(dst, stream)),
+           "ipt_debug_aos_fill")
+
+
+def warp_load_dump(src, dump, nchunks: int, words: int, stream=None):
+    _check(_lib.ipt_debug_warp_load_dump(src.data_ptr(), dump.data_ptr(), nchunks, words,
+                                         _dev_stream(dump, stream)), "ipt_debug_warp_load_dump")
+
+
+def warp_store(regs, dst, nchunks: int, words: int, stream=None):
+    _check(_lib.ipt_debug_warp_store(regs.data_ptr(), dst.data_ptr(), nchunks, words, _dev_stream(dst, stream)),
+           "ipt_debug_warp_store")
 
 
 def status_string(s: int) -> str:

@@ -15,7 +15,7 @@ OBJDIR = os.path.join(PKG, "build")
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O2,-Wall", "-Xptxas", "-v",
+FLAGS = ["-O3", "-std=c++20", "-lineinfo", "-Xcompiler", "-fPIC,-O2,-Wall", "-Xptxas", "-v",
          "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC]
 
 
