@@ -57,6 +57,10 @@ def parse_args():
     p.add_argument("--e2e-shapes", type=int, default=8)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--profile-only", action="store_true", help="one short untimed pass (for ncu)")
+    p.add_argument("--config", choices=("sweep", "batched"), default="sweep",
+                   help="sweep: BASELINE configs[1] (the metric's workload); batched: config 5b")
+    p.add_argument("--batch", type=int, default=4096, help="config 5b total matrices")
+    p.add_argument("--chunk", type=int, default=512, help="config 5b resident matrices per call")
     return p.parse_args()
 
 
@@ -206,6 +210,97 @@ def run_reference(args, rank, world):
     print(json.dumps(out), flush=True)
 
 
+def rank_shapes(rank, S):
+    """Rank r transposes sweep shapes [r*S, (r+1)*S): independent matrices, weak scaling."""
+    return workloads.sweep_shapes(S * (rank + 1))[S * rank:]
+
+
+def shard_batch(batch, rank, world):
+    """Contiguous block of matrix indices [lo, hi) owned by `rank` (config 5b)."""
+    lo = batch * rank // world
+    hi = batch * (rank + 1) // world
+    return lo, hi
+
+
+def reduce_over_ranks(sum_vals, max_vals, world, device):
+    """The bench's only collectives: SUM of sum_vals and MAX of max_vals over ranks
+    (no collective ever touches the data path)."""
+    if world == 1:
+        return list(sum_vals), list(max_vals)
+    import torch
+    import torch.distributed as dist
+    s = torch.tensor(list(sum_vals), dtype=torch.float64, device=device)
+    m = torch.tensor(list(max_vals), dtype=torch.float64, device=device)
+    dist.all_reduce(s, op=dist.ReduceOp.SUM)
+    dist.all_reduce(m, op=dist.ReduceOp.MAX)
+    return [float(v) for v in s], [float(v) for v in m]
+
+
+def run_batched(args, rank, world, local_rank):
+    """Config 5b: `--batch` independent 4096 x 3000 float32 matrices (default 4096, 201 GB)
+    sharded contiguously over the ranks (strong scaling); each rank transposes its shard
+    with ipt_c2r_batched in resident chunks of at most --chunk matrices.  value =
+    total Eq. 37 bytes / max-over-ranks device time."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ppopp_catanzarokg14_b200 as ipt
+
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    m, n, eb = workloads.CONFIG5B["m"], workloads.CONFIG5B["n"], workloads.CONFIG5B["elem_bytes"]
+    lo, hi = shard_batch(args.batch, rank, world)
+    mine = hi - lo
+    chunk = min(args.chunk, mine) if mine else 0
+    buf = torch.randint(0, 255, (max(chunk, 1) * m * n * eb,), dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream(dev)
+    pieces = []
+    k = 0
+    while k < mine:
+        pieces.append(min(chunk, mine - k))
+        k += chunk
+
+    def step(record):
+        for i, cnt in enumerate(pieces):
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            (ipt.c2r_batched if i % 2 == 0 else ipt.r2c_batched)(buf, cnt, m * n, m, n, elem_bytes=eb,
+                                                                 stream=stream.cuda_stream)
+            e1.record(stream)
+            if record is not None:
+                record.append((e0, e1))
+
+    for _ in range(args.warmup):
+        step(None)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches0 = ipt.launch_count()
+    rec = []
+    for _ in range(args.steps):
+        step(rec)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    dev_ms = sum(e0.elapsed_time(e1) for e0, e1 in rec) / args.steps
+    (total_bytes,), (t_max,) = reduce_over_ranks([2.0 * mine * m * n * eb], [dev_ms], world, dev)
+    if rank != 0:
+        return
+    peak, peak_src = hbm_peak()
+    value = total_bytes / (t_max * 1e-3) / 1e9
+    print(json.dumps({
+        "metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(t_max, 3), "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": f"cfg5b: batch of {args.batch} independent {m}x{n} float32 matrices, "
+                               f"contiguous shards per rank, chunks of <= {args.chunk} resident matrices",
+                   "parallelism": f"batch sharding x{world}, no data-path collective",
+                   "l2": "inputs (>= 25 GB per chunk) far larger than L2"},
+        "impl": "ours", "frac_of_hbm_peak_per_gpu": round(value / world / peak, 4),
+        "gpu_launches": ipt.launch_count() - launches0}), flush=True)
+
+
 def run_ours(args, rank, world, local_rank):
     import torch
     import torch.distributed as dist
@@ -215,7 +310,7 @@ def run_ours(args, rank, world, local_rank):
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
     S = args.shapes
-    shapes = workloads.sweep_shapes(S * (rank + 1))[S * rank:]
+    shapes = rank_shapes(rank, S)
     ebs = (4, 8)
     maxel = max(m * n for m, n in shapes)
     bufs = {eb: torch.randint(0, 255, (maxel * eb,), dtype=torch.uint8, device=dev) for eb in ebs}
@@ -311,15 +406,8 @@ def run_ours(args, rank, world, local_rank):
                    f"{len(e2e_shapes)} sweep shapes x fp32/fp64"}
 
     # ---- aggregate over ranks (max time, summed medians) ------------------------------
-    if world > 1:
-        t = torch.tensor([median, ms_step, e2e["value"]], dtype=torch.float64, device=dev)
-        tmax = t.clone()
-        dist.all_reduce(t, op=dist.ReduceOp.SUM)
-        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
-        value, ms_step, e2e_value = float(t[0]), float(tmax[1]), float(t[2])
-        e2e["value"] = round(e2e_value, 2)
-    else:
-        value = median
+    (value, e2e_value), (ms_step,) = reduce_over_ranks([median, e2e["value"]], [ms_step], world, dev)
+    e2e["value"] = round(e2e_value, 2)
     if rank != 0:
         return
 
@@ -376,7 +464,10 @@ def main():
         torch.cuda.set_device(local_rank)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     try:
-        run_ours(args, rank, world, local_rank)
+        if args.config == "batched":
+            run_batched(args, rank, world, local_rank)
+        else:
+            run_ours(args, rank, world, local_rank)
     finally:
         if world > 1:
             import torch.distributed as dist

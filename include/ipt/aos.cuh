@@ -172,8 +172,12 @@ struct coalesced_ptr {
 
     __device__ explicit coalesced_ptr(T *ptr) : p(ptr) {}
 
-    // Warp-uniform: every lane active and p_lane == p_0 + lane, p_0 4-byte aligned.
+    // Warp-uniform: every lane active and p_lane == p_0 + lane, p_0 4-byte aligned.  Structs
+    // of at most 16 bytes take the per-lane path: B200's coalescer already merges a warp's
+    // <= 512 contiguous bytes, and the round-1 Fig. 8 measurement (profiles/r01_aos_config4)
+    // shows the transposition only pays from 20-byte structs on.
     __device__ __forceinline__ bool cooperative() const {
+        if constexpr (S <= 4) return false;
         if (__activemask() != 0xffffffffu) return false;
         const unsigned long long u = reinterpret_cast<unsigned long long>(p);
         const unsigned long long u0 = __shfl_sync(0xffffffffu, u, 0);

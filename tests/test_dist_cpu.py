@@ -1,0 +1,64 @@
+"""Multi-process (world_size 2, gloo, CPU) coverage of the N>1 bench path.
+
+The data path has no collective: ranks own disjoint, contiguous shards of independent
+matrices; the only collectives are the timing/throughput reductions (SUM, MAX).  These
+tests run the bench's own sharding and reduction helpers in two real processes.
+"""
+import os
+import socket
+
+import pytest
+import torch.multiprocessing as mp
+
+from conftest import ROOT
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _worker(rank, world, port, out):
+    import sys
+    sys.path.insert(0, ROOT)
+    import torch.distributed as dist
+    import bench
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        sums, maxs = bench.reduce_over_ranks([rank + 1.0, 10.0 * rank], [rank * 3.0 + 1], world, "cpu")
+        shapes = bench.rank_shapes(rank, 4)
+        lo, hi = bench.shard_batch(4096, rank, world)
+        out[rank] = (sums, maxs, shapes, (lo, hi))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2])
+def test_two_rank_sharding_and_reductions(world):
+    port = _free_port()
+    mgr = mp.Manager()
+    out = mgr.dict()
+    mp.spawn(_worker, args=(world, port, out), nprocs=world, join=True)
+    r0, r1 = out[0], out[1]
+    # reductions: SUM and MAX of the per-rank values, identical on every rank
+    assert r0[0] == r1[0] == [3.0, 10.0]
+    assert r0[1] == r1[1] == [4.0]
+    # independent shapes per rank (no rank repeats another's matrices)
+    assert len(r0[2]) == len(r1[2]) == 4 and not set(r0[2]) & set(r1[2])
+    # config 5b: contiguous shards covering [0, 4096) exactly once
+    assert r0[3] == (0, 2048) and r1[3] == (2048, 4096)
+
+
+def test_shard_batch_partitions_exactly():
+    import bench
+    for batch in (1, 7, 4096, 4097):
+        for world in (1, 2, 3, 4, 8):
+            seen = []
+            for r in range(world):
+                lo, hi = bench.shard_batch(batch, r, world)
+                seen.extend(range(lo, hi))
+            assert seen == list(range(batch))

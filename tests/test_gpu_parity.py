@@ -212,3 +212,19 @@ def test_sweep_shapes_full_size(eb):
             _sampled_check(got, host, m, n, 20000, rng)
         ipt.r2c(x, m, n, elem_bytes=eb)
         assert torch.equal(x, to_dev(host)), (m, n)
+
+
+def test_config5b_batch_shape_sampled():
+    """Config 5b matrices (4096 x 3000 float32, gcd 8) in a batch: whole-matrix comparison
+    of the first, sampled one-by-one checks (oracle Eqs. 7-8) of the others."""
+    m, n, batch = 4096, 3000, 6
+    host = workloads.random_words(batch * m * n, 4, seed=55)
+    x = to_dev(host)
+    ipt.c2r_batched(x, batch, m * n, m, n, elem_bytes=4)
+    got = x.cpu().numpy().view(np.uint32)
+    assert got[:m * n].tobytes() == oracle.transpose(host[:m * n], m, n).tobytes()
+    rng = random.Random(5)
+    for k in range(1, batch):
+        _sampled_check(got[k * m * n:(k + 1) * m * n], host[k * m * n:(k + 1) * m * n], m, n, 5000, rng)
+    ipt.r2c_batched(x, batch, m * n, m, n, elem_bytes=4)
+    assert torch.equal(x, to_dev(host))
