@@ -105,7 +105,7 @@ int ilog2(int v) {
 
 // Column-tile geometry.  Tile width TWB = IPT_TILE_BYTES (32, 64 or 128; default 128 B =
 // one cache line).  Band: the rows per CTA that fit the per-CTA shared-memory target
-// IPT_COL_SMEM (default 50 KiB, four CTAs per SM: the best of the round-1 sweep over
+// IPT_COL_SMEM (default 46 KiB, four CTAs per SM: the best of the round-1 sweep over
 // 12-100 KiB, profiles/r01_*).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
 // the co-resident CTAs, the band grows (up to the opt-in shared-memory maximum).
 ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp) {
@@ -113,9 +113,9 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
     if (twb != 32 && twb != 64 && twb != 128) twb = 128;
     if (twb < pl.eb) twb = pl.eb;
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
-    const int64_t target = env_int("IPT_COL_SMEM", 50 * 1024);
+    const int64_t target = env_int("IPT_COL_SMEM", 46 * 1024);
     const int64_t W = twb / pl.eb;
-    const int64_t per_row = twb + 16 + 1 + 4;  // col_smem_bytes: hull + offset + row index
+    const int64_t per_row = twb + 8;  // col_smem_bytes: staged row + two row indices
     int64_t B = target / per_row - (W - 1);
     if (B < 32) B = 32;
     if (B > col_max_band(W)) B = col_max_band(W);
@@ -161,6 +161,9 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
 // co-resident, never more than there are tiles.
 void finish_col(ColParams &p, int64_t batch) {
     if (p.G < 1) return;  // pass not planned (e.g. no rotation when gcd = 1)
+    p.fd_G = make_fastdiv(static_cast<uint32_t>(p.G));
+    p.fd_nt = make_fastdiv(static_cast<uint32_t>(p.ntiles));
+    p.kshM = static_cast<uint32_t>(2 + p.W / p.M) * static_cast<uint32_t>(p.M);
     p.total_tiles = static_cast<int64_t>(p.ntiles) * batch;
     int64_t ng = p.resident / p.G;
     if (ng > p.total_tiles) ng = p.total_tiles;

@@ -2,48 +2,45 @@
 // §4.6-4.7).
 //
 // A column operation permutes every column independently.  The B200 realisation stages a
-// whole column tile -- all M rows x W adjacent columns (TWB = W * eb bytes wide) -- on
-// chip, spread over the shared memory of a GROUP of G CTAs (member r holds the band of
-// B rows [r B, r B + B) plus a halo), and makes the operation a single read + write
-// pass.  In-place safety: every member finishes reading its part of the tile before ANY
-// member writes (a per-group barrier in global memory: release-add on a counter, acquire
-// spin until all G members arrived); tiles are disjoint byte ranges owned by exactly one
-// group.  This replaces the paper's multi-pass cache-aware rotate (coarse cycle following
-// + fine on-chip rotation, §4.6) and cycle-following row permute (§4.7) -- prior art for
-// a K20c.
+// whole column tile -- all M rows x W adjacent columns (TWB = W * eb = 128 bytes wide) --
+// on chip, spread over the shared memory of a GROUP of G CTAs (member r owns the output
+// band [r B, r B + B)), and makes the operation a single read + write pass.  In-place
+// safety: every member finishes reading its part of the tile before ANY member writes (a
+// per-tile barrier in global memory: release-add on a counter, acquire spin until all G
+// members arrived); tiles are disjoint byte ranges owned by exactly one group.  This
+// replaces the paper's multi-pass cache-aware rotate (coarse cycle following + fine
+// on-chip rotation, §4.6) and cycle-following row permute (§4.7) -- prior art for a K20c.
+//
+// Tile-local forms (w = j - j0 is the column inside the tile [j0, j0 + W); "slot" t is the
+// t-th input row a member reads; output row k of the band is written to global row o(k)):
+//  * COL_ROT, gather rotation rho_j = sign * floor(j/b) (Eq. 23, sign = +1: the C2R
+//    pre-rotation; Eq. 36, sign = -1: the R2C post-rotation):
+//        out[i][w] = in[(i + rho_{j0+w}) mod M][w]
+//    slots = input rows r0 + min rho + t (contiguous, cyclic); slot t, column w feeds
+//    band row k = t - (rho_w - min rho); o(k) = r0 + k.  rho varies by < W in a tile
+//    (the residual bound of :767-773).
+//  * COL_C2R_SHUF, s'_j(i) = (j + q(i)) mod M (Eq. 26 = p_j o q, Eqs. 32-33):
+//        out[i][w] = in[(k + w) mod M][w],  k = (j0 + q(i)) mod M,
+//    scatter form: slots = rows r0 + t (band + W-1 halo rows), slot t column w feeds the
+//    skewed row k = t - w, which is output row o(k) = q^{-1}((r0 + k - j0) mod M) (Eq. 34).
+//  * COL_R2C_SHUF, (s')^{-1}_j(i) = q^{-1}((i - j) mod M) (Eqs. 34-35):
+//        out[i][w] = in[q^{-1}((i - w - j0) mod M)][w],
+//    slots = rows q^{-1}((r0 - W + 1 + t - j0) mod M) (scattered), slot t column w feeds
+//    k = t - (W - 1) + w; o(k) = r0 + k.
+//  * COL_COPY: identity (measurement hook).
+//
+// Data path (lane = tile column, see col_tile_kernel): element-granular cp.async from each
+// 128-byte tile row straight into the element's OUTPUT row in shared memory -- the skew /
+// rotation / permutation is the copy's destination address -- then whole output rows
+// written back with coalesced element stores.  Earlier variants, all slower and kept in
+// the round-1 notes (profiles/): 16-byte cp.async hulls + per-element skewed gathers
+// (54 instr/element), 128-bit register loads + shared-memory scatter, TMA bulk copies.
 //
 // Why software groups rather than hardware clusters: a group can be any size up to the
-// co-resident CTA count (a 17226-row tile of 128 B is ~2.6 MB, beyond a 16-CTA cluster
-// at 128-byte tiles), and the non-persistent grid lets CTAs drift out of lock-step (a
-// persistent cooperative variant and a two-buffer pipelined variant were both slower:
-// profiles/).  The grid is one CTA per (tile, band); see col_tile_kernel for why the spin
-// barrier cannot deadlock.
-//
-// Tile-local forms (w = j - j0 is the column inside the tile [j0, j0 + W)):
-//  * COL_ROT, gather rotation rho_j = sign * floor(j/b) (Eq. 23 for sign = +1 as the C2R
-//    pre-rotation, Eq. 36 for sign = -1 as the R2C post-rotation):
-//        out[i][w] = in[(i + rho_{j0+w}) mod M][w]
-//    The member writing band [r0, r1) reads rows [r0 + min rho, r1 + max rho) -- a
-//    contiguous cyclic range (rho varies by < W inside a tile, :767-773 residual bound).
-//  * COL_C2R_SHUF, s'_j(i) = (j + q(i)) mod M (Eq. 26 = p_j o q, Eqs. 32-33):
-//        out[i][w] = in[(k + w) mod M][w],  k = (j0 + q(i)) mod M.
-//    Scatter form: the member reads rows [r0, r1 + W - 1) (band + halo, contiguous),
-//    builds the skewed row T_k[w] = in[k + w][w] for each k of its band and writes it to
-//    output row i = q^{-1}((k - j0) mod M) (Eq. 34).
-//  * COL_R2C_SHUF, (s')^{-1}_j(i) = q^{-1}((i - j) mod M) (Eqs. 34-35):
-//        out[i][w] = in[q^{-1}((i - w - j0) mod M)][w].
-//    The member writing band [r0, r1) reads the rows q^{-1}((u - j0) mod M) for
-//    u in [r0 - W + 1, r1) (scattered whole sub-rows) and writes its band contiguously.
-//
-// Memory access: each staged row is fetched as its 16-byte-aligned hull (TWB/16 + 1
-// chunks) with cp.async (LDGSTS, global -> shared without a register round trip), so a
-// CTA has its whole band in flight at once; rows are 16-byte aligned only when
-// N*eb % 16 == 0, and the hull's extra bytes (neighbouring tiles of the same row) are
-// never used.  Chunks that would leave the matrix (row 0 head, row M-1 tail) are fetched
-// element by element.  (One TMA bulk copy per 144-byte hull was tried and is ~2x slower:
-// the TMA engine does not keep up with that many tiny requests; profiles/.)  Stores: one 16-byte destination
-// chunk per thread, gathered from the staged rows and written with a vector store
-// (element stores only in a row's ragged head/tail chunk).
+// co-resident CTA count (a 17226-row tile of 128 B is ~2.2 MB, beyond a 16-CTA cluster),
+// and the non-persistent grid lets CTAs drift out of lock-step (a persistent cooperative
+// variant and a two-buffer pipelined variant were both slower: profiles/).  The grid is one
+// CTA per (tile, band); see col_tile_kernel for why the spin barrier cannot deadlock.
 #include "plan.h"
 
 namespace ipt {
@@ -54,21 +51,6 @@ namespace {
 #define IPT_COL_THREADS 512
 #endif
 constexpr int kColThreads = IPT_COL_THREADS;
-
-__device__ __forceinline__ uint32_t smem_u32(const void *p) {
-    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-template <int B>
-__device__ __forceinline__ void cp_async_small(uint32_t dst, const void *src) {
-    if constexpr (B == 16) {
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(src) : "memory");
-    } else {
-        asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" :: "r"(dst), "l"(src), "n"(B) : "memory");
-    }
-}
-__device__ __forceinline__ void cp_async_wait_all() {
-    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
-}
 
 // q^{-1}(i) = (floor((c-1+i)/c) b^{-1}) mod a + (((c-1) i) mod c) a  (Eq. 34).
 __device__ __forceinline__ int32_t qinv_of(const ColParams &P, int32_t i) {
@@ -85,199 +67,38 @@ __device__ __forceinline__ int32_t mod_M(int32_t v, uint32_t kshiftM, const Fast
     return static_cast<int32_t>(fmod_(static_cast<uint32_t>(v) + kshiftM, fdM));
 }
 
-// Group barrier in global memory: counter ctr counts arrivals of all tiles so far.
+// Group barrier in global memory: counter ctr counts arrivals of all tiles sharing it.
 __device__ __forceinline__ void group_barrier(unsigned int *ctr, unsigned int target) {
-    __syncthreads();  // every thread's cp.async data has landed in shared memory
+    __syncthreads();  // every thread's staged data is in shared memory
     if (threadIdx.x == 0) {
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
         unsigned int v;
         while (true) {
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
             if (v >= target) break;
-            __nanosleep(64);
+            __nanosleep(128);
         }
     }
     __syncthreads();
 }
 
-template <int TWB>
-struct TileGeom {
-    static constexpr int SLOT = TWB + 16;  // hull bytes per staged row
-    static constexpr int CH = TWB / 16 + 1;  // hull chunks per staged row
-};
-
-// Per-tile geometry of one staging buffer.
-struct TileCtx {
-    char *A;            // this matrix
-    const char *Aend;
-    int32_t j0, Wt, j0m;
-    int32_t lo_q, hi_q, base_off, nslots;
-};
-
-// Staging buffer layout (one of two): [dw W*4 | stage nslots_max*SLOT | dlt nslots_max |
-// ridx nslots_max*4], nslots_max = B + W - 1.
-template <int TWB>
-__host__ __device__ constexpr size_t buf_dw_bytes(int W) { return (static_cast<size_t>(W) * 4 + 15) & ~size_t(15); }
-__host__ __device__ inline size_t buf_bytes(int64_t nslots_max, int W, int twb) {
-    const size_t slot = static_cast<size_t>(twb) + 16;
-    return ((static_cast<size_t>(W) * 4 + 15) & ~size_t(15)) + ((static_cast<size_t>(nslots_max) * (slot + 1) + 15) & ~size_t(15)) +
-           ((static_cast<size_t>(nslots_max) * 4 + 15) & ~size_t(15));  // keeps the second buffer 16-B aligned
+// Shared-memory layout: [orow B*4 | srow nslots*4 | rows B*TWB].
+__host__ __device__ inline size_t al16(size_t x) { return (x + 15) & ~size_t(15); }
+__host__ __device__ inline size_t smem_layout(int64_t B, int W, int twb, size_t *off_srow, size_t *off_rows) {
+    const size_t nslots = static_cast<size_t>(B) + W - 1;
+    size_t o = al16(static_cast<size_t>(B) * 4);
+    *off_srow = o;
+    o += al16(nslots * 4);
+    *off_rows = o;
+    return o + static_cast<size_t>(B) * twb;
 }
 
-template <int EB, int MODE, int TWB>
-__device__ __forceinline__ bool make_ctx(const ColParams &P, int64_t tt, int32_t nrows, TileCtx &c) {
-    constexpr int W = TWB / EB;
-    const int32_t tile = static_cast<int32_t>(tt % P.ntiles);
-    const int64_t mat = tt / P.ntiles;
-    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
-    c.A = P.base + mat * P.mat_stride_bytes;
-    c.Aend = c.A + static_cast<int64_t>(P.M) * pitch;
-    c.j0 = tile * W;
-    c.Wt = min(W, P.N - c.j0);
-    c.j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(c.j0), P.fd_M));
-    int32_t ext = W - 1;
-    c.lo_q = c.hi_q = c.base_off = 0;
-    if (MODE == COL_ROT) {
-        c.lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(c.j0), P.fd_b));
-        c.hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(c.j0 + c.Wt - 1), P.fd_b));
-        // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.
-        // Every member sees the same tile, so the skip is group-uniform.
-        if (c.hi_q == 0) return false;
-        ext = c.hi_q - c.lo_q;
-        c.base_off = P.rot_sign > 0 ? c.lo_q : -c.hi_q;  // smallest rotation amount in the tile
-    } else if (MODE == COL_COPY) {
-        ext = 0;
-    }
-    c.nslots = nrows > 0 ? nrows + ext : 0;
-    return true;
-}
-
-template <int EB, int MODE, int TWB>
-__device__ __forceinline__ int64_t next_tile(const ColParams &P, int64_t tt, int32_t nrows, TileCtx &c) {
-    for (; tt < P.total_tiles; tt += P.ngroups)
-        if (make_ctx<EB, MODE, TWB>(P, tt, nrows, c)) return tt;
-    return tt;
-}
-
-// Issue the cp.async loads of one tile band into buffer `buf` (one commit group).
-template <int EB, int MODE, int TWB>
-__device__ __forceinline__ void load_tile(const ColParams &P, const TileCtx &c, unsigned char *buf, int32_t r0,
-                                          int32_t nrows, int32_t nslots_max, uint32_t kshM) {
-    constexpr int W = TWB / EB;
-    constexpr int SLOT = TileGeom<TWB>::SLOT;
-    constexpr int CH = TileGeom<TWB>::CH;
-    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
-    int32_t *dwt = reinterpret_cast<int32_t *>(buf);
-    unsigned char *stage = buf + buf_dw_bytes<TWB>(W);
-    uint8_t *dlt = stage + static_cast<size_t>(nslots_max) * SLOT;
-    int32_t *ridx = reinterpret_cast<int32_t *>(stage + ((static_cast<size_t>(nslots_max) * (SLOT + 1) + 15) & ~size_t(15)));
-
-    // Slot offset of column w: the element of output row kk comes from staged row kk + dw[w].
-    for (int32_t w = threadIdx.x; w < W; w += blockDim.x) {
-        int32_t dw = 0;
-        if (MODE == COL_ROT) {
-            const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(c.j0 + min(w, c.Wt - 1)), P.fd_b));
-            dw = P.rot_sign > 0 ? qw - c.lo_q : c.hi_q - qw;  // rho_w - min rho
-        } else if (MODE == COL_C2R_SHUF) {
-            dw = w;
-        } else if (MODE == COL_R2C_SHUF) {
-            dw = W - 1 - w;
-        }
-        dwt[w] = dw;
-    }
-    // Source row of slot t: contiguous (rowbase + t) mod M for ROT / C2R / COPY,
-    // q^{-1}((r0 - W + 1 + t - j0) mod M) for R2C (ridx, computed first).
-    if (MODE == COL_R2C_SHUF) {
-        for (int32_t t = threadIdx.x; t < c.nslots; t += blockDim.x)
-            ridx[t] = qinv_of(P, mod_M(r0 - (W - 1) + t - c.j0m, kshM, P.fd_M));
-        __syncthreads();
-    }
-    const int32_t rowbase = MODE == COL_ROT ? mod_M(r0 + c.base_off, kshM, P.fd_M) : r0;
-    const char *Aj = c.A + static_cast<int64_t>(c.j0) * EB;
-    const uint32_t sst = smem_u32(stage);
-    const int32_t nch = c.nslots * CH;
-    const int32_t vbytes = c.Wt * EB;
-    for (int32_t e = threadIdx.x; e < nch; e += blockDim.x) {
-        const int32_t t = e / CH, k = e - t * CH;
-        int32_t row;
-        if (MODE == COL_R2C_SHUF) {
-            row = ridx[t];
-        } else {
-            row = rowbase + t;
-            if (row >= P.M) row = row - P.M < P.M ? row - P.M : mod_M(row, kshM, P.fd_M);
-        }
-        const char *ra = Aj + row * pitch;
-        const int d = static_cast<int>(reinterpret_cast<uintptr_t>(ra) & 15);
-        if (k == 0) dlt[t] = static_cast<uint8_t>(d);
-        if (16 * k >= d + vbytes) continue;  // past the end of this row's tile
-        const char *lo = ra - d + 16 * k;
-        const uint32_t dst = sst + t * SLOT + 16 * k;
-        // Only row 0's head and row M-1's tail can leave the matrix.
-        if ((row != 0 && row != P.M - 1) || (lo >= c.A && lo + 16 <= c.Aend)) {
-            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(lo) : "memory");
-        } else {
-#pragma unroll
-            for (int q = 0; q < 16; q += EB)
-                if (lo + q >= c.A && lo + q < c.Aend) cp_async_small<EB>(dst + q, lo + q);
-        }
-    }
-    // C2R: destination rows of the band, while the loads are in flight.
-    if (MODE == COL_C2R_SHUF) {
-        for (int32_t kk = threadIdx.x; kk < nrows; kk += blockDim.x)
-            ridx[kk] = qinv_of(P, mod_M(r0 + kk - c.j0m, kshM, P.fd_M));
-    }
-    asm volatile("cp.async.commit_group;" ::: "memory");
-}
-
-// Write one tile band from buffer `buf`: one 16-byte destination chunk per thread.
-template <int EB, int MODE, int TWB>
-__device__ __forceinline__ void store_tile(const ColParams &P, const TileCtx &c, const unsigned char *buf, int32_t r0,
-                                           int32_t nrows, int32_t nslots_max) {
-    using T = typename Word<EB>::T;
-    constexpr int W = TWB / EB;
-    constexpr int SLOT = TileGeom<TWB>::SLOT;
-    constexpr int NQ = TWB / 16 + 1;  // 16-byte destination chunks a tile row can touch
-    constexpr int PER = 16 / EB;
-    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
-    const int32_t *dwt = reinterpret_cast<const int32_t *>(buf);
-    const unsigned char *stage = buf + buf_dw_bytes<TWB>(W);
-    const uint8_t *dlt = stage + static_cast<size_t>(nslots_max) * SLOT;
-    const int32_t *ridx =
-        reinterpret_cast<const int32_t *>(stage + ((static_cast<size_t>(nslots_max) * (SLOT + 1) + 15) & ~size_t(15)));
-    char *Aj = c.A + static_cast<int64_t>(c.j0) * EB;
-    const int32_t Wt = c.Wt;
-    const int32_t nout = nrows * NQ;
-    for (int32_t e = threadIdx.x; e < nout; e += blockDim.x) {
-        const int32_t kk = e / NQ, q = e - kk * NQ;
-        const int64_t orow = MODE == COL_C2R_SHUF ? ridx[kk] : r0 + kk;
-        char *da = Aj + orow * pitch;  // output row's tile start
-        const int dd = static_cast<int>(reinterpret_cast<uintptr_t>(da) & 15);
-        const int w0 = (16 * q - dd) / EB;  // first column of this chunk (may be < 0)
-        if (w0 >= Wt) continue;
-        if (w0 >= 0 && w0 + PER <= Wt) {
-            union { uint4 u; T t[PER]; } v;
-            const int32_t ta = kk + dwt[w0], tb = kk + dwt[w0 + PER - 1];
-            const uint32_t so = ta * SLOT + dlt[ta] + w0 * EB;
-            if (ta == tb && (so & 15) == 0) {  // one staged row, aligned: a single LDS.128
-                v.u = *reinterpret_cast<const uint4 *>(stage + so);
-            } else {
-#pragma unroll
-                for (int x = 0; x < PER; ++x) {
-                    const int32_t t = kk + dwt[w0 + x];
-                    v.t[x] = *reinterpret_cast<const T *>(stage + t * SLOT + dlt[t] + (w0 + x) * EB);
-                }
-            }
-            *reinterpret_cast<uint4 *>(da + w0 * EB) = v.u;
-        } else {
-#pragma unroll
-            for (int x = 0; x < PER; ++x) {
-                const int w = w0 + x;
-                if (w < 0 || w >= Wt) continue;
-                const int32_t t = kk + dwt[w];
-                reinterpret_cast<T *>(da)[w] = *reinterpret_cast<const T *>(stage + t * SLOT + dlt[t] + w * EB);
-            }
-        }
-    }
+template <int EB>
+__device__ __forceinline__ void cp_async_elem(uint32_t dst, const void *src) {
+    if constexpr (EB == 16)
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(src) : "memory");
+    else
+        asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" :: "r"(dst), "l"(src), "n"(EB) : "memory");
 }
 
 // One CTA per (tile, band).  The CTA's logical id comes from a ticket counter taken at
@@ -285,42 +106,150 @@ __device__ __forceinline__ void store_tile(const ColParams &P, const TileCtx &c,
 // every group whose tickets are all taken is fully resident, hence only the newest group
 // can be waiting for members, and those get scheduled as older groups finish -- the spin
 // barrier cannot deadlock as long as one group fits on the GPU (G <= resident CTAs).
+//
+// Thread mapping: lane = tile column w (W = TWB/eb lanes per tile row, 32/W rows per warp
+// instruction).  A load instruction copies whole tile rows (128 contiguous bytes) with
+// element-granular cp.async, each element landing directly in its OUTPUT row of the band in
+// shared memory (row k = t - dw[w]): the skew / rotation is done by the copy's
+// destination address, and the bank of every element is its column (conflict-free).  A
+// store instruction writes whole output rows (128 contiguous bytes).  No 16-byte alignment
+// is needed anywhere: element accesses work at every row phase and never leave the tile.
 template <int EB, int MODE, int TWB>
 __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
+    using T = typename Word<EB>::T;
     constexpr int W = TWB / EB;
+    constexpr int RPW = 32 / W;  // tile rows per warp instruction
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ unsigned int s_ticket;
     if (threadIdx.x == 0) s_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
     __syncthreads();
     const unsigned int ticket = s_ticket;
-    const int64_t tt = ticket / static_cast<unsigned int>(P.G);   // tile (of all matrices)
-    const int32_t r = static_cast<int32_t>(ticket - tt * P.G);     // band
+    const uint32_t tt = fdiv(ticket, P.fd_G);                    // tile (of all matrices)
+    const int32_t r = static_cast<int32_t>(ticket - tt * P.G);    // band
     const int32_t r0 = r * P.B;
-    const int32_t r1 = min(P.M, r0 + P.B);
-    const int32_t nrows = max(0, r1 - r0);
-    const int32_t nslots_max = P.B + W - 1;
-    const uint32_t kshM = static_cast<uint32_t>(2 + W / P.M) * static_cast<uint32_t>(P.M);
+    const int32_t nrows = max(0, min(P.M, r0 + P.B) - r0);
     const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
+    const uint32_t kshM = P.kshM;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
 
-    TileCtx c;
-    if (!make_ctx<EB, MODE, TWB>(P, tt, nrows, c)) {  // group-uniform skip (ROT amount 0)
-        // Still arrive: later tiles sharing this counter slot count these arrivals.
-        if (use_barrier && threadIdx.x == 0)
-            atomicAdd(P.ctr + static_cast<unsigned int>(tt % kCtrSlots), 1u);
-        return;
+    // ---- tile geometry --------------------------------------------------------------
+    const uint32_t mat = fdiv(tt, P.fd_nt);
+    const int32_t tile = static_cast<int32_t>(tt - mat * static_cast<uint32_t>(P.ntiles));
+    char *A = P.base + static_cast<int64_t>(mat) * P.mat_stride_bytes;
+    const int32_t j0 = tile * W;
+    const int32_t Wt = min(W, P.N - j0);
+    const int32_t j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j0), P.fd_M));
+    int32_t ext = W - 1, lo_q = 0, hi_q = 0, base_off = 0;
+    if (MODE == COL_ROT) {
+        lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
+        hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + Wt - 1), P.fd_b));
+        ext = hi_q - lo_q;
+        base_off = P.rot_sign > 0 ? lo_q : -hi_q;  // smallest rotation amount in the tile
+        // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.  The
+        // skip is group-uniform; still arrive, later tiles sharing the counter count it.
+        if (hi_q == 0) {
+            if (use_barrier && threadIdx.x == 0) atomicAdd(P.ctr + (tt % kCtrSlots), 1u);
+            return;
+        }
+    } else if (MODE == COL_COPY) {
+        ext = 0;
     }
-    load_tile<EB, MODE, TWB>(P, c, smem, r0, nrows, nslots_max, kshM);
-    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    const int32_t nslots = nrows > 0 ? nrows + ext : 0;
+
+    size_t o_srow, o_rows;
+    smem_layout(P.B, W, TWB, &o_srow, &o_rows);
+    int32_t *orow = reinterpret_cast<int32_t *>(smem);
+    int32_t *srow = reinterpret_cast<int32_t *>(smem + o_srow);
+    unsigned char *rows = smem + o_rows;
+    char *Aj = A + static_cast<int64_t>(j0) * EB;
+
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    const int w = lane % W, sub = lane / W;
+    int32_t dw = 0;  // slot t, column w feeds band row k = t - dw
+    if (MODE == COL_ROT) {
+        const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + min(w, Wt - 1)), P.fd_b));
+        dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
+    } else if (MODE == COL_C2R_SHUF) {
+        dw = w;
+    } else if (MODE == COL_R2C_SHUF) {
+        dw = W - 1 - w;
+    }
+
+    // ---- pre-pass: scattered row indices (C2R destinations, R2C sources) --------------
+    if (MODE == COL_C2R_SHUF) {
+        for (int32_t k = threadIdx.x; k < nrows; k += blockDim.x)
+            orow[k] = qinv_of(P, mod_M(r0 + k - j0m, kshM, P.fd_M));
+    }
+    if (MODE == COL_R2C_SHUF) {
+        for (int32_t t = threadIdx.x; t < nslots; t += blockDim.x)
+            srow[t] = qinv_of(P, mod_M(r0 - (W - 1) + t - j0m, kshM, P.fd_M));
+        __syncthreads();
+    }
+
+    // ---- load: every element straight to its output row -------------------------------
+    const int32_t rowbase = MODE == COL_ROT ? mod_M(r0 + base_off, kshM, P.fd_M) : r0;
+    const uint32_t srows = static_cast<uint32_t>(__cvta_generic_to_shared(rows)) + w * EB;
+    char *colp = Aj + w * EB;
+    const int32_t step = nwarps * RPW;  // slots between a lane's consecutive rows
+    const int32_t t0 = warp * RPW + sub;
+    if (w < Wt) {
+        // This lane's slots t with 0 <= k = t - dw < nrows (the others are halo elements no
+        // band row needs): a branch-free walk with incremental shared and global addresses.
+        int32_t t = t0;
+        if (t < dw) t += ((dw - t + step - 1) / step) * step;
+        const int32_t tend = dw + nrows;
+        uint32_t sa = srows + (t - dw) * TWB;
+        const uint32_t sa_inc = step * TWB;
+        if (MODE == COL_R2C_SHUF) {
+#pragma unroll 4
+            for (; t < tend; t += step, sa += sa_inc) cp_async_elem<EB>(sa, colp + srow[t] * pitch);
+        } else if (step <= P.M) {
+            int32_t s = mod_M(rowbase + t, kshM, P.fd_M);
+            const char *g = colp + s * pitch;
+            const int64_t g_inc = step * pitch, g_wrap = static_cast<int64_t>(P.M) * pitch;
+#pragma unroll 4
+            for (; t < tend; t += step, sa += sa_inc) {
+                cp_async_elem<EB>(sa, g);
+                s += step;
+                g += g_inc;
+                if (s >= P.M) {
+                    s -= P.M;
+                    g -= g_wrap;
+                }
+            }
+        } else {  // tiny M: fewer rows than one step
+            for (; t < tend; t += step, sa += sa_inc)
+                cp_async_elem<EB>(sa, colp + mod_M(rowbase + t, kshM, P.fd_M) * pitch);
+        }
+    }
+    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+
     // In-place hazard barrier: the whole tile has been read before anyone writes it.
     // Counter slot tt mod kCtrSlots, monotone over the tiles that share it.
     if (use_barrier) {
-        const unsigned int slot = static_cast<unsigned int>(tt % kCtrSlots);
-        const unsigned int target = static_cast<unsigned int>(tt / kCtrSlots + 1) * static_cast<unsigned int>(P.G);
+        const unsigned int slot = tt % kCtrSlots;  // power of two
+        const unsigned int target = (tt / kCtrSlots + 1) * static_cast<unsigned int>(P.G);
         group_barrier(P.ctr + slot, target);
     } else {
         __syncthreads();
     }
-    store_tile<EB, MODE, TWB>(P, c, smem, r0, nrows, nslots_max);
+
+    // ---- store: whole output rows -------------------------------------------------------
+    if (w < Wt) {
+        const unsigned char *sr = rows + w * EB;
+        int32_t k = t0;
+        if (MODE == COL_C2R_SHUF) {
+#pragma unroll 4
+            for (; k < nrows; k += step)
+                *reinterpret_cast<T *>(colp + static_cast<int64_t>(orow[k]) * pitch) =
+                    *reinterpret_cast<const T *>(sr + k * TWB);
+        } else {
+            char *g = colp + static_cast<int64_t>(r0 + k) * pitch;
+            const int64_t g_inc = step * pitch;
+#pragma unroll 4
+            for (; k < nrows; k += step, g += g_inc) *reinterpret_cast<T *>(g) = *reinterpret_cast<const T *>(sr + k * TWB);
+        }
+    }
 }
 
 template <int EB, int MODE, int TWB>
@@ -361,7 +290,8 @@ void *col_kernel(int mode, int eb, int twb) {
 }  // namespace
 
 size_t col_smem_bytes(int64_t B, int64_t W, int eb) {
-    return buf_bytes(B + W - 1, static_cast<int>(W), static_cast<int>(W * eb));
+    size_t a, b;
+    return smem_layout(B, static_cast<int>(W), static_cast<int>(W * eb), &a, &b);
 }
 
 int64_t col_max_band(int64_t W) { return (int64_t(1) << 24) - W; }
@@ -388,10 +318,8 @@ cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, s
     // Ticket + group counters: the stream's own block, zeroed in stream order.
     P.ctr = group_counters(st, kCtrSlots + 1);
     if (!P.ctr) return cudaErrorMemoryAllocation;
-    const int64_t used = P.total_tiles < kCtrSlots ? P.total_tiles : kCtrSlots;
     e = cudaMemsetAsync(P.ctr, 0, sizeof(unsigned int) * (kTicketSlot + 1), st);
     if (e != cudaSuccess) return e;
-    (void)used;
     void *args[] = {&P};
     return cudaLaunchKernel(kern, dim3(static_cast<unsigned>(grid)), dim3(kColThreads), args, smem, st);
 }

@@ -72,6 +72,8 @@ struct ColParams {
     unsigned int *ctr;  // per-group arrival counters (stream-ordered scratch, launch_col)
     int32_t rot_sign;   // COL_ROT: +1 (C2R pre-rotation) or -1 (R2C post-rotation)
     int32_t wide_a;     // a >= 2^16
+    FastDiv fd_G, fd_nt;  // ticket -> (tile, band), tile -> (matrix, column tile)
+    uint32_t kshM;      // (2 + W / M) * M: shift making every mod_M argument non-negative
 };
 
 // Kernel attribute / occupancy caches (api.cu): set the dynamic shared-memory limit (and
@@ -85,7 +87,7 @@ int cached_resident_blocks(const void *kern, int threads, size_t smem);  // SMs 
 // are serialised; different streams never share a block).  Slots [0, kCtrSlots) are the
 // per-tile arrival counters (tile t uses slot t mod kCtrSlots), slot kTicketSlot is the
 // dispatch ticket.
-constexpr int kCtrSlots = 4096;
+constexpr int kCtrSlots = 4096;  // a power of two
 constexpr int kTicketSlot = kCtrSlots;
 constexpr int kMaxGroups = kCtrSlots + 1;
 unsigned int *group_counters(cudaStream_t st, int n);
