@@ -57,8 +57,10 @@ def parse_args():
     p.add_argument("--e2e-shapes", type=int, default=8)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--profile-only", action="store_true", help="one short untimed pass (for ncu)")
-    p.add_argument("--config", choices=("sweep", "batched"), default="sweep",
-                   help="sweep: BASELINE configs[1] (the metric's workload); batched: config 5b")
+    p.add_argument("--config", choices=("sweep", "batched", "skinny"), default="sweep",
+                   help="sweep: BASELINE configs[1] (the metric's workload); batched: config 5b; "
+                        "skinny: config 3")
+    p.add_argument("--count", type=int, default=1 << 26, help="config 3 structs")
     p.add_argument("--batch", type=int, default=4096, help="config 5b total matrices")
     p.add_argument("--chunk", type=int, default=512, help="config 5b resident matrices per call")
     return p.parse_args()
@@ -301,6 +303,82 @@ def run_batched(args, rank, world, local_rank):
         "gpu_launches": ipt.launch_count() - launches0}), flush=True)
 
 
+def run_skinny(args, rank, world, local_rank):
+    """Config 3: AoS -> SoA and SoA -> AoS of 2**26 structs x n 4-byte fields, n = 2..32
+    (ipt_aos_to_soa / ipt_soa_to_aos, the skinny engine).  value = median over all calls of
+    Eq. 37 GB/s (2 * count * n * 4 / t); per-n numbers in `per_n`."""
+    import torch
+
+    import paper_conf_ppopp_catanzarokg14_b200 as ipt
+
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    count = args.count
+    ns = workloads.skinny_field_counts()
+    buf = torch.randint(0, 255, (count * max(ns) * 4,), dtype=torch.uint8, device=dev)
+    flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    def one(n, op, rec):
+        flush.zero_()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        op(buf, count, n, field_bytes=4, stream=stream.cuda_stream)
+        e1.record(stream)
+        if rec is not None:
+            rec.append((n, op.__name__, e0, e1))
+
+    for _ in range(args.warmup):
+        for n in ns:
+            one(n, ipt.aos_to_soa, None)
+            one(n, ipt.soa_to_aos, None)
+    torch.cuda.synchronize()
+    launches0 = ipt.launch_count()
+    ipt.profile_enable(True)
+    ipt.profile_read()
+    rec = []
+    for _ in range(args.steps):
+        for n in ns:
+            one(n, ipt.aos_to_soa, rec)
+            one(n, ipt.soa_to_aos, rec)
+    torch.cuda.synchronize()
+    ipt.profile_enable(False)
+    kern = ipt.profile_read()
+    rates, per_n, dev_ms = [], {}, 0.0
+    for n, name, e0, e1 in rec:
+        ms = e0.elapsed_time(e1)
+        dev_ms += ms
+        g = 2.0 * count * n * 4 / (ms * 1e-3) / 1e9
+        rates.append(g)
+        per_n.setdefault(f"{name}_n{n}", []).append(g)
+    peak, peak_src = hbm_peak()
+    value = statistics.median(rates)
+    dom = max(kern.items(), key=lambda kv: kv[1][1]) if kern else None
+    roof = None
+    if dom:
+        name, (nl, ms, by) = dom
+        achieved = by / (ms * 1e-3) / 1e9
+        roof = {"bound": "hbm", "kernel": name, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "peak_source": peak_src, "traffic": None,
+                "share_of_device_time": round(ms / sum(v[1] for v in kern.values()), 3)}
+    if rank == 0:
+        print(json.dumps({
+            "metric": "median in-place AoS<->SoA GB/s (Eq. 37) over n = 2..32 fields", "value": round(value, 2),
+            "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(dev_ms / args.steps, 3), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"cfg3 skinny: {count} structs x n 4-byte fields, n = 2..32, "
+                                   "ipt_aos_to_soa then ipt_soa_to_aos", "l2": "flushed before every timed call"},
+            "impl": "ours", "frac_of_hbm_peak": round(value / peak, 4), "max_GBps": round(max(rates), 2),
+            "per_n": {k: round(statistics.median(v), 1) for k, v in per_n.items()},
+            "paper_context": {"K20c_skinny_median_GBps": 34.3, "K20c_skinny_max_GBps": 51,
+                              "source": "PAPER.md:1069 (64-bit fields, other hardware)"},
+            "roofline": roof,
+            "kernels": {k: {"launches": v[0], "ms": round(v[1], 3), "GBps": round(v[2] / (v[1] * 1e-3) / 1e9, 1)}
+                        for k, v in kern.items()},
+            "gpu_launches": ipt.launch_count() - launches0}), flush=True)
+
+
 def run_ours(args, rank, world, local_rank):
     import torch
     import torch.distributed as dist
@@ -466,6 +544,8 @@ def main():
     try:
         if args.config == "batched":
             run_batched(args, rank, world, local_rank)
+        elif args.config == "skinny":
+            run_skinny(args, rank, world, local_rank)
         else:
             run_ours(args, rank, world, local_rank)
     finally:

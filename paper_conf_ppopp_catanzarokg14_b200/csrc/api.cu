@@ -95,6 +95,9 @@ struct Plan {
     bool has_rot = false;
     int nlaunch = 0;
     size_t onchip = 0;
+    size_t scratch = 0;         // global scratch bytes (skinny: one row of the long dimension)
+    SkinnyRowParams srow{};     // skinny engine long-row shuffle
+    int skinny_dir = 0;         // ROW_R2C (P_{count,n}, AoS -> SoA) or ROW_C2R (P_{n,count})
 };
 
 int ilog2(int v) {
@@ -165,10 +168,86 @@ void finish_col(ColParams &p, int64_t batch) {
     p.fd_nt = make_fastdiv(static_cast<uint32_t>(p.ntiles));
     p.kshM = static_cast<uint32_t>(2 + p.W / p.M) * static_cast<uint32_t>(p.M);
     p.total_tiles = static_cast<int64_t>(p.ntiles) * batch;
+    // One-CTA tiles: enough tiles per CTA for ~4 waves of resident CTAs.
+    p.tpc = 1;
+    if (p.G == 1) {
+        const int64_t want = 4 * static_cast<int64_t>(p.resident);
+        p.tpc = static_cast<int32_t>(std::max<int64_t>(1, (p.total_tiles + want - 1) / want));
+    }
     int64_t ng = p.resident / p.G;
     if (ng > p.total_tiles) ng = p.total_tiles;
     if (ng < 1) ng = 1;
     p.ngroups = static_cast<int32_t>(ng);
+}
+
+// Stream-ordered scratch (the skinny engine's tmp row) from a library-owned pool that keeps
+// its memory between calls (release threshold = max), one pool per device.
+cudaMemPool_t scratch_pool() {
+    static std::mutex mu;
+    static std::unordered_map<int, cudaMemPool_t> pools;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return nullptr;
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = pools.find(dev);
+    if (it != pools.end()) return it->second;
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t pool = nullptr;
+    if (cudaMemPoolCreate(&pool, &props) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    pools[dev] = pool;
+    return pool;
+}
+
+// Skinny engine (§6.1): P_{x,y} with min(x, y) = n <= 32 fields
+// and a long dimension.  Engine view: n rows x N = max(x, y).  P_{count,n} (AoS -> SoA)
+// = R2C(M = n, N = count); P_{n,count} (SoA -> AoS) = C2R(M = n, N = count) (Theorem 2).
+ipt_status_t make_skinny_plan(const DevInfo &dev, int64_t x, int64_t y, int eb, Plan &pl) {
+    pl.engine = ENG_SKINNY;
+    pl.skinny_dir = y < x ? ROW_R2C : ROW_C2R;
+    pl.M = y < x ? y : x;
+    pl.N = y < x ? x : y;
+    if (pl.N >= (int64_t(1) << 31)) return IPT_ERR_UNSUPPORTED;
+    pl.c = gcd64(pl.M, pl.N);
+    pl.a = pl.M / pl.c;
+    pl.b = pl.N / pl.c;
+    const int n = static_cast<int>(pl.M);
+    // Column passes on n-row tiles: one CTA per tile.
+    ipt_status_t s = plan_col(dev, pl, pl.skinny_dir == ROW_R2C ? COL_R2C_SHUF : COL_C2R_SHUF, pl.shuf);
+    if (s != IPT_OK) return s;
+    pl.onchip = pl.shuf.smem;
+    if (pl.c > 1) {
+        s = plan_col(dev, pl, COL_ROT, pl.rot);
+        if (s != IPT_OK) return s;
+        pl.rot.p.rot_sign = pl.skinny_dir == ROW_C2R ? 1 : -1;  // Eq. 23 before / Eq. 36 after
+        pl.has_rot = true;
+        if (pl.rot.smem > pl.onchip) pl.onchip = pl.rot.smem;
+    }
+    // Long-row shuffle windows of n * T elements, T a power of two, ~32 KiB of staging.
+    SkinnyRowParams &r = pl.srow;
+    std::memset(&r, 0, sizeof(r));
+    int T = 32;
+    while (static_cast<int64_t>(n) * (2 * T) * eb <= 32 * 1024 && 2 * T <= pl.b) T *= 2;
+    r.N = pl.N;
+    r.n = n;
+    r.c = static_cast<int32_t>(pl.c);
+    r.b = static_cast<int32_t>(pl.b);
+    r.ainv = mmi64(pl.a, pl.b);
+    r.T = T;
+    r.Tp = T + (32 % n == 0 ? 32 / n : 1);  // residue classes spread over the banks
+    r.fd_n = make_fastdiv(static_cast<uint32_t>(n));
+    const size_t rs = skinny_row_smem(n, r.Tp, eb);
+    if (rs > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
+    if (rs > pl.onchip) pl.onchip = rs;
+    pl.scratch = static_cast<size_t>(pl.N) * eb;  // one row of the long dimension
+    pl.nlaunch = n + 1 + (pl.has_rot ? 1 : 0);
+    return IPT_OK;
 }
 
 // P_{x,y} on `batch` matrices.
@@ -179,6 +258,10 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     const DevInfo dev = device_info();
     if (!dev.ok) return IPT_ERR_CUDA;
     if (dev.major != 10 || dev.minor != 0) return IPT_ERR_UNSUPPORTED;  // sm_100 only
+
+    // Skinny shapes (a dimension <= 32, the other long): the specialised engine (§6.1).
+    if (std::min(x, y) <= 32 && std::max(x, y) >= env_int("IPT_SKINNY_MIN", 65536))
+        return make_skinny_plan(dev, x, y, eb, pl);
 
     int engine = x > y ? ENG_C2R : ENG_R2C;
     // IPT_ENGINE_RULE=1: the opposite choice (rows = the long dimension, column tiles of
@@ -258,7 +341,8 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_FUSE_ROT", "IPT_ENGINE_RULE"}) {
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+                          "IPT_SKINNY_MIN"}) {
         const char *v = std::getenv(n);
         s += v ? v : "-";
         s += '|';
@@ -357,6 +441,61 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
     auto rot = [&] { return launch_col(pl.rot.p, COL_ROT, pl.eb, st, pl.rot.smem); };
     auto row = [&] { return launch_row(pl.row, pl.row_dir, pl.eb, st); };
     ipt_status_t s;
+    if (pl.engine == ENG_SKINNY) {
+        // Rolling rows (§6.1; DESIGN.md §"Skinny"): engine view n rows x N, one
+        // tmp row of N elements.  R2C: column pass writing row r to location r+1 (row n-1 to
+        // tmp); row i then reads location i+1 (tmp for n-1) and writes location i.  C2R:
+        // row i reads location i, writes location i-1 (tmp for 0); the column pass reads the
+        // shifted rows back.  A destination row is never its own source row.
+        const int n = static_cast<int>(pl.M);
+        const int64_t pitch = pl.N * pl.eb;
+        const double rowb = 2.0 * static_cast<double>(pl.N) * pl.eb;
+        char *tmp = nullptr;
+        cudaMemPool_t pool = scratch_pool();
+        if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&tmp), pl.scratch, pool, st) != cudaSuccess) {
+            cudaGetLastError();
+            return IPT_ERR_OUT_OF_MEMORY;
+        }
+        s = IPT_OK;
+        for (int64_t mat = 0; mat < batch; ++mat) {
+            char *A = base + mat * stride_bytes;
+            ColPlan shuf = pl.shuf, rot = pl.rot;
+            for (ColPlan *cp : {&shuf, &rot}) {
+                cp->p.base = A;
+                cp->p.batch = 1;
+                cp->p.tmp = tmp;
+                finish_col(cp->p, 1);
+            }
+            shuf.p.remap = pl.skinny_dir == ROW_R2C ? 1 : -1;
+            auto rot_l = [&] { return launch_col(rot.p, COL_ROT, pl.eb, st, rot.smem); };
+            auto row_l = [&](int i) {
+                SkinnyRowParams rp = pl.srow;
+                rp.i = i;
+                if (pl.skinny_dir == ROW_R2C) {
+                    rp.src = i == n - 1 ? tmp : A + (i + 1) * pitch;
+                    rp.dst = A + i * pitch;
+                } else {
+                    rp.src = A + i * pitch;
+                    rp.dst = i == 0 ? tmp : A + (i - 1) * pitch;
+                }
+                return [rp, &pl, st] { return launch_skinny_row(rp, pl.skinny_dir, pl.eb, st); };
+            };
+            if (pl.skinny_dir == ROW_R2C) {
+                auto shuf_l = [&] { return launch_col(shuf.p, COL_R2C_SHUF, pl.eb, st, shuf.smem); };
+                if ((s = run(PK_COL, rowb * n, shuf_l)) != IPT_OK) break;
+                for (int i = 0; i < n && s == IPT_OK; ++i) s = run(PK_SKINNY, rowb, row_l(i));
+                if (s == IPT_OK && pl.has_rot) s = run(PK_ROT, rowb * n, rot_l);
+            } else {
+                auto shuf_l = [&] { return launch_col(shuf.p, COL_C2R_SHUF, pl.eb, st, shuf.smem); };
+                if (pl.has_rot && (s = run(PK_ROT, rowb * n, rot_l)) != IPT_OK) break;
+                for (int i = 0; i < n && s == IPT_OK; ++i) s = run(PK_SKINNY, rowb, row_l(i));
+                if (s == IPT_OK) s = run(PK_COL, rowb * n, shuf_l);
+            }
+            if (s != IPT_OK) break;
+        }
+        cudaFreeAsync(tmp, st);
+        return s;
+    }
     if (pl.engine == ENG_C2R) {
         auto shuf = [&] { return launch_col(pl.shuf.p, COL_C2R_SHUF, pl.eb, st, pl.shuf.smem); };
         if (pl.has_rot && (s = run(PK_ROT, rot_bytes, rot)) != IPT_OK) return s;  // Eq. 23
@@ -515,7 +654,7 @@ ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *glo
     Plan pl;
     ipt_status_t s = make_plan(m, n, elem_bytes, pl);
     if (s != IPT_OK) return s;
-    if (global_bytes) *global_bytes = 0;
+    if (global_bytes) *global_bytes = pl.scratch;
     if (onchip_per_cta) *onchip_per_cta = pl.onchip;
     return IPT_OK;
 }

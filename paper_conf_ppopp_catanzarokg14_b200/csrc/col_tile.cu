@@ -115,17 +115,10 @@ __device__ __forceinline__ void cp_async_elem(uint32_t dst, const void *src) {
 // store instruction writes whole output rows (128 contiguous bytes).  No 16-byte alignment
 // is needed anywhere: element accesses work at every row phase and never leave the tile.
 template <int EB, int MODE, int TWB>
-__global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
+__device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *smem, uint32_t tt, int32_t r) {
     using T = typename Word<EB>::T;
     constexpr int W = TWB / EB;
     constexpr int RPW = 32 / W;  // tile rows per warp instruction
-    extern __shared__ __align__(16) unsigned char smem[];
-    __shared__ unsigned int s_ticket;
-    if (threadIdx.x == 0) s_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
-    __syncthreads();
-    const unsigned int ticket = s_ticket;
-    const uint32_t tt = fdiv(ticket, P.fd_G);                    // tile (of all matrices)
-    const int32_t r = static_cast<int32_t>(ticket - tt * P.G);    // band
     const int32_t r0 = r * P.B;
     const int32_t nrows = max(0, min(P.M, r0 + P.B) - r0);
     const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
@@ -190,9 +183,17 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     const int32_t rowbase = MODE == COL_ROT ? mod_M(r0 + base_off, kshM, P.fd_M) : r0;
     const uint32_t srows = static_cast<uint32_t>(__cvta_generic_to_shared(rows)) + w * EB;
     char *colp = Aj + w * EB;
+    char *tmpw = P.tmp + static_cast<int64_t>(j0 + w) * EB;  // skinny engine only
     const int32_t step = nwarps * RPW;  // slots between a lane's consecutive rows
     const int32_t t0 = warp * RPW + sub;
-    if (w < Wt) {
+    if (w < Wt && P.remap < 0) {  // skinny: row s is stored at s-1, row 0 in tmp
+        int32_t t = t0;
+        if (t < dw) t += ((dw - t + step - 1) / step) * step;
+        for (; t < dw + nrows; t += step) {
+            const int32_t s = MODE == COL_R2C_SHUF ? srow[t] : mod_M(rowbase + t, kshM, P.fd_M);
+            cp_async_elem<EB>(srows + (t - dw) * TWB, s == 0 ? tmpw : colp + (s - 1) * pitch);
+        }
+    } else if (w < Wt) {
         // This lane's slots t with 0 <= k = t - dw < nrows (the others are halo elements no
         // band row needs): a branch-free walk with incremental shared and global addresses.
         int32_t t = t0;
@@ -238,7 +239,13 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     if (w < Wt) {
         const unsigned char *sr = rows + w * EB;
         int32_t k = t0;
-        if (MODE == COL_C2R_SHUF) {
+        if (P.remap > 0) {  // skinny: output row o is stored at o+1, row M-1 in tmp
+            for (; k < nrows; k += step) {
+                const int32_t o = MODE == COL_C2R_SHUF ? orow[k] : r0 + k;
+                *reinterpret_cast<T *>(o == P.M - 1 ? tmpw : colp + static_cast<int64_t>(o + 1) * pitch) =
+                    *reinterpret_cast<const T *>(sr + k * TWB);
+            }
+        } else if (MODE == COL_C2R_SHUF) {
 #pragma unroll 4
             for (; k < nrows; k += step)
                 *reinterpret_cast<T *>(colp + static_cast<int64_t>(orow[k]) * pitch) =
@@ -250,6 +257,26 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
             for (; k < nrows; k += step, g += g_inc) *reinterpret_cast<T *>(g) = *reinterpret_cast<const T *>(sr + k * TWB);
         }
     }
+}
+
+template <int EB, int MODE, int TWB>
+__global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ unsigned int s_ticket;
+    if (threadIdx.x == 0) s_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
+    __syncthreads();
+    const unsigned int ticket = s_ticket;
+    if (P.G == 1) {  // a tile fits one CTA: no barrier, P.tpc consecutive tiles per CTA
+        const uint64_t t_end = min(static_cast<uint64_t>(P.total_tiles), (static_cast<uint64_t>(ticket) + 1) * P.tpc);
+        for (uint64_t tt = static_cast<uint64_t>(ticket) * P.tpc; tt < t_end; ++tt) {
+            col_tile_one<EB, MODE, TWB>(P, smem, static_cast<uint32_t>(tt), 0);
+            __syncthreads();  // shared memory is reused by the next tile
+        }
+        return;
+    }
+    const uint32_t tt = fdiv(ticket, P.fd_G);                  // tile (of all matrices)
+    const int32_t r = static_cast<int32_t>(ticket - tt * P.G);  // band
+    col_tile_one<EB, MODE, TWB>(P, smem, tt, r);
 }
 
 template <int EB, int MODE, int TWB>
@@ -313,7 +340,7 @@ cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, s
     cudaError_t e = ensure_kernel_attrs(kern, smem, false);
     if (e != cudaSuccess) return e;
     ColParams P = P0;
-    const int64_t grid = P.total_tiles * P.G;
+    const int64_t grid = P.G == 1 ? (P.total_tiles + P.tpc - 1) / P.tpc : P.total_tiles * P.G;
     if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     // Ticket + group counters: the stream's own block, zeroed in stream order.
     P.ctr = group_counters(st, kCtrSlots + 1);

@@ -74,6 +74,24 @@ struct ColParams {
     int32_t wide_a;     // a >= 2^16
     FastDiv fd_G, fd_nt;  // ticket -> (tile, band), tile -> (matrix, column tile)
     uint32_t kshM;      // (2 + W / M) * M: shift making every mod_M argument non-negative
+    // Skinny engine (rolling rows, skinny.cu): row x of the engine view is stored at
+    // location x+remap, the row that falls off the end lives in the one-row buffer `tmp`.
+    //   remap = +1: outputs are written shifted (row M-1 -> tmp); remap = -1: inputs are
+    //   read shifted (row 0 <- tmp).  Only with batch == 1.
+    char *tmp;
+    int32_t remap;
+    int32_t tpc;        // tiles per CTA when G == 1 (each tile fits one CTA)
+};
+
+struct SkinnyRowParams {
+    const char *src;    // source row (N elements)
+    char *dst;          // destination row (N elements), never the source
+    int64_t N;          // row length (the long dimension, count)
+    int32_t n, c, b;    // engine rows M = n (fields), c = gcd(n, N), b = N / c
+    int64_t ainv;       // a^{-1} mod b, a = n / c
+    int32_t i;          // row index
+    int32_t T, Tp;      // run length per residue class; shared-memory row pitch (odd)
+    FastDiv fd_n;
 };
 
 // Kernel attribute / occupancy caches (api.cu): set the dynamic shared-memory limit (and
@@ -102,5 +120,10 @@ int col_block_threads();
 int64_t col_max_band(int64_t W);  // largest band a CTA may be given
 cudaError_t launch_col(const ColParams &p, int mode, int eb, cudaStream_t st, size_t smem);
 int col_resident_ctas(int mode, int eb, int twb, size_t smem);
+
+// Skinny long-row shuffle (skinny.cu): dir ROW_R2C -- dst[d'^{-1}_i(k)] = src[k] driven by
+// source windows; dir ROW_C2R -- dst[j] = src[d'^{-1}_i(j)] driven by output windows.
+size_t skinny_row_smem(int n, int T, int eb);
+cudaError_t launch_skinny_row(const SkinnyRowParams &p, int dir, int eb, cudaStream_t st);
 
 }  // namespace ipt
