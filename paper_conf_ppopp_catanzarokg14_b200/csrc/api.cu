@@ -97,6 +97,7 @@ struct Plan {
     size_t onchip = 0;
     size_t scratch = 0;         // global scratch bytes (skinny: one row of the long dimension)
     SkinnyRowParams srow{};     // skinny engine long-row shuffle
+    SkinnyColParams scol{}, srot{};  // skinny engine column passes (shuffle, rotation)
     int skinny_dir = 0;         // ROW_R2C (P_{count,n}, AoS -> SoA) or ROW_C2R (P_{n,count})
 };
 
@@ -218,16 +219,31 @@ ipt_status_t make_skinny_plan(const DevInfo &dev, int64_t x, int64_t y, int eb, 
     pl.a = pl.M / pl.c;
     pl.b = pl.N / pl.c;
     const int n = static_cast<int>(pl.M);
-    // Column passes on n-row tiles: one CTA per tile.
-    ipt_status_t s = plan_col(dev, pl, pl.skinny_dir == ROW_R2C ? COL_R2C_SHUF : COL_C2R_SHUF, pl.shuf);
-    if (s != IPT_OK) return s;
-    pl.onchip = pl.shuf.smem;
+    // Column passes: all n rows x C columns per CTA (skinny.cu).
+    SkinnyColParams &sc = pl.scol;
+    std::memset(&sc, 0, sizeof(sc));
+    sc.N = pl.N;
+    sc.n = n;
+    sc.c = static_cast<int32_t>(pl.c);
+    sc.b = static_cast<int32_t>(pl.b);
+    sc.fd_n = make_fastdiv(static_cast<uint32_t>(n));
+    sc.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
+    sc.C = std::max(32, static_cast<int>((40 * 1024) / (n * eb)) / 32 * 32);
+    for (int i = 0; i < n; ++i) {  // Eq. 33: q(i) = (i N - floor(i/a)) mod n; q^{-1} its inverse
+        const int64_t q = ((static_cast<int64_t>(i) * (pl.N % n) - i / pl.a) % n + n) % n;
+        sc.q[i] = static_cast<int32_t>(q);
+        sc.qinv[q] = i;
+    }
+    sc.mode = pl.skinny_dir == ROW_R2C ? COL_R2C_SHUF : COL_C2R_SHUF;
+    sc.remap = pl.skinny_dir == ROW_R2C ? 1 : -1;
+    pl.onchip = skinny_col_smem(n, sc.C, eb);
+    if (pl.onchip > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
     if (pl.c > 1) {
-        s = plan_col(dev, pl, COL_ROT, pl.rot);
-        if (s != IPT_OK) return s;
-        pl.rot.p.rot_sign = pl.skinny_dir == ROW_C2R ? 1 : -1;  // Eq. 23 before / Eq. 36 after
+        pl.srot = sc;
+        pl.srot.mode = COL_ROT;
+        pl.srot.remap = 0;
+        pl.srot.rot_sign = pl.skinny_dir == ROW_C2R ? 1 : -1;  // Eq. 23 before / Eq. 36 after
         pl.has_rot = true;
-        if (pl.rot.smem > pl.onchip) pl.onchip = pl.rot.smem;
     }
     // Long-row shuffle windows of n * T elements, T a power of two, ~32 KiB of staging.
     SkinnyRowParams &r = pl.srow;
@@ -459,15 +475,11 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
         s = IPT_OK;
         for (int64_t mat = 0; mat < batch; ++mat) {
             char *A = base + mat * stride_bytes;
-            ColPlan shuf = pl.shuf, rot = pl.rot;
-            for (ColPlan *cp : {&shuf, &rot}) {
-                cp->p.base = A;
-                cp->p.batch = 1;
-                cp->p.tmp = tmp;
-                finish_col(cp->p, 1);
-            }
-            shuf.p.remap = pl.skinny_dir == ROW_R2C ? 1 : -1;
-            auto rot_l = [&] { return launch_col(rot.p, COL_ROT, pl.eb, st, rot.smem); };
+            SkinnyColParams shuf = pl.scol, rotp = pl.srot;
+            shuf.A = rotp.A = A;
+            shuf.tmp = rotp.tmp = tmp;
+            auto rot_l = [&] { return launch_skinny_col(rotp, pl.eb, st); };
+            auto shuf_l = [&] { return launch_skinny_col(shuf, pl.eb, st); };
             auto row_l = [&](int i) {
                 SkinnyRowParams rp = pl.srow;
                 rp.i = i;
@@ -481,12 +493,10 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
                 return [rp, &pl, st] { return launch_skinny_row(rp, pl.skinny_dir, pl.eb, st); };
             };
             if (pl.skinny_dir == ROW_R2C) {
-                auto shuf_l = [&] { return launch_col(shuf.p, COL_R2C_SHUF, pl.eb, st, shuf.smem); };
                 if ((s = run(PK_COL, rowb * n, shuf_l)) != IPT_OK) break;
                 for (int i = 0; i < n && s == IPT_OK; ++i) s = run(PK_SKINNY, rowb, row_l(i));
                 if (s == IPT_OK && pl.has_rot) s = run(PK_ROT, rowb * n, rot_l);
             } else {
-                auto shuf_l = [&] { return launch_col(shuf.p, COL_C2R_SHUF, pl.eb, st, shuf.smem); };
                 if (pl.has_rot && (s = run(PK_ROT, rowb * n, rot_l)) != IPT_OK) break;
                 for (int i = 0; i < n && s == IPT_OK; ++i) s = run(PK_SKINNY, rowb, row_l(i));
                 if (s == IPT_OK) s = run(PK_COL, rowb * n, shuf_l);

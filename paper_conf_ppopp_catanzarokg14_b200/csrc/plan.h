@@ -121,6 +121,23 @@ int64_t col_max_band(int64_t W);  // largest band a CTA may be given
 cudaError_t launch_col(const ColParams &p, int mode, int eb, cudaStream_t st, size_t smem);
 int col_resident_ctas(int mode, int eb, int twb, size_t smem);
 
+// Skinny column pass (skinny.cu): all n rows x C consecutive columns per CTA, the column
+// permutation sigma_j among the n rows applied in shared memory.
+struct SkinnyColParams {
+    char *A;            // the n x N engine view
+    char *tmp;          // the one-row buffer of the rolling scheme
+    int64_t N;
+    int32_t n, c, b;
+    int32_t mode;       // COL_ROT, COL_C2R_SHUF, COL_R2C_SHUF
+    int32_t remap;      // +1: output row o stored at o+1 (n-1 in tmp); -1: input row s at s-1 (0 in tmp)
+    int32_t rot_sign;
+    int32_t C;          // columns per CTA (multiple of 32)
+    int32_t q[32], qinv[32];  // Eq. 33 / Eq. 34 on the n rows
+    FastDiv fd_n, fd_b;
+};
+size_t skinny_col_smem(int n, int C, int eb);
+cudaError_t launch_skinny_col(const SkinnyColParams &p, int eb, cudaStream_t st);
+
 // Skinny long-row shuffle (skinny.cu): dir ROW_R2C -- dst[d'^{-1}_i(k)] = src[k] driven by
 // source windows; dir ROW_C2R -- dst[j] = src[d'^{-1}_i(j)] driven by output windows.
 size_t skinny_row_smem(int n, int T, int eb);

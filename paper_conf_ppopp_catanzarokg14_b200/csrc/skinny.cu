@@ -112,6 +112,88 @@ __global__ void __launch_bounds__(kSkThreads) skinny_row_kernel(SkinnyRowParams 
     }
 }
 
+// Skinny column pass: columns of only n <= 32 elements, so one CTA stages ALL n rows of C
+// consecutive columns (n coalesced row segments), then writes out[i][j] = in[sigma_j(i)][j]:
+//   ROT       sigma_j(i) = (i + sign floor(j/b)) mod n            (Eq. 23 / Eq. 36)
+//   C2R_SHUF  sigma_j(i) = (j + q(i)) mod n                       (Eq. 26 = p_j o q)
+//   R2C_SHUF  sigma_j(i) = q^{-1}((i - j) mod n)                  (Eqs. 34-35)
+// with the rolling-row remaps of the skinny engine on the input or output side.  A CTA
+// reads its columns completely before writing them and CTAs own disjoint columns.
+template <int EB, int MODE>
+__global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams P) {
+    using T = typename Word<EB>::T;
+    extern __shared__ __align__(16) unsigned char smem[];
+    int32_t *qinv_s = reinterpret_cast<int32_t *>(smem);  // 32 entries
+    T *buf = reinterpret_cast<T *>(smem + 128);            // [n][C]
+    const uint32_t sbuf = static_cast<uint32_t>(__cvta_generic_to_shared(buf));
+    const int n = P.n, C = P.C;
+    const int64_t pitch = P.N;  // in elements
+    T *A = reinterpret_cast<T *>(P.A);
+    T *tmp = reinterpret_cast<T *>(P.tmp);
+    if (threadIdx.x < 32) qinv_s[threadIdx.x] = P.qinv[threadIdx.x];
+    for (int64_t j0 = static_cast<int64_t>(blockIdx.x) * C; j0 < P.N; j0 += static_cast<int64_t>(gridDim.x) * C) {
+        const int32_t cols = static_cast<int32_t>(min(static_cast<int64_t>(C), P.N - j0));
+        // stage: row s of the view (remap -1: stored at s-1, row 0 in tmp)
+        for (int s = 0; s < n; ++s) {
+            const T *row = P.remap < 0 ? (s == 0 ? tmp : A + (s - 1) * pitch) : A + s * pitch;
+            for (int32_t x = threadIdx.x; x < cols; x += blockDim.x)
+                cp_async_e<EB>(sbuf + (s * C + x) * EB, row + j0 + x);
+        }
+        asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+        __syncthreads();
+        for (int32_t x = threadIdx.x; x < cols; x += blockDim.x) {
+            const int64_t j = j0 + x;  // < N < 2^31
+            const uint32_t jm = fmod_(static_cast<uint32_t>(j), P.fd_n);
+            int32_t shift = 0;
+            if (MODE == COL_ROT) {  // floor(j/b) < c <= n
+                const int32_t qd = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j), P.fd_b));
+                shift = P.rot_sign > 0 ? qd : (qd == 0 ? 0 : n - qd);
+            }
+            for (int i = 0; i < n; ++i) {
+                int32_t s;
+                if (MODE == COL_ROT) {
+                    s = i + shift;
+                    s -= s >= n ? n : 0;
+                } else if (MODE == COL_C2R_SHUF) {
+                    s = static_cast<int32_t>(jm) + P.q[i];
+                    s -= s >= n ? n : 0;
+                } else {
+                    int32_t u = i - static_cast<int32_t>(jm);
+                    u += u < 0 ? n : 0;
+                    s = qinv_s[u];
+                }
+                T *orow = P.remap > 0 ? (i == n - 1 ? tmp : A + (i + 1) * pitch) : A + i * pitch;
+                orow[j] = buf[s * C + x];
+            }
+        }
+        __syncthreads();  // the buffer is refilled by the next column block
+    }
+}
+
+template <int EB, int MODE>
+cudaError_t launch_col_t(const SkinnyColParams &P, cudaStream_t st) {
+    const size_t smem = skinny_col_smem(P.n, P.C, EB);
+    auto kern = skinny_col_kernel<EB, MODE>;
+    cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
+    if (e != cudaSuccess) return e;
+    const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), kSkThreads, smem);
+    if (resident < 1) return cudaErrorInvalidConfiguration;
+    const int64_t blocks = (P.N + P.C - 1) / P.C;
+    const int64_t grid = blocks < 4 * static_cast<int64_t>(resident) ? blocks : 4 * static_cast<int64_t>(resident);
+    kern<<<static_cast<unsigned>(grid), kSkThreads, smem, st>>>(P);
+    return cudaGetLastError();
+}
+
+template <int EB>
+cudaError_t launch_col_e(const SkinnyColParams &P, cudaStream_t st) {
+    switch (P.mode) {
+        case COL_ROT: return launch_col_t<EB, COL_ROT>(P, st);
+        case COL_C2R_SHUF: return launch_col_t<EB, COL_C2R_SHUF>(P, st);
+        case COL_R2C_SHUF: return launch_col_t<EB, COL_R2C_SHUF>(P, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
 template <int EB, int DIR>
 cudaError_t launch_t(const SkinnyRowParams &P, cudaStream_t st) {
     const size_t smem = skinny_row_smem(P.n, P.Tp, EB);
@@ -130,6 +212,16 @@ cudaError_t launch_t(const SkinnyRowParams &P, cudaStream_t st) {
 }  // namespace
 
 size_t skinny_row_smem(int n, int Tp, int eb) { return 512 + static_cast<size_t>(n) * Tp * eb; }
+size_t skinny_col_smem(int n, int C, int eb) { return 128 + static_cast<size_t>(n) * C * eb; }
+
+cudaError_t launch_skinny_col(const SkinnyColParams &P, int eb, cudaStream_t st) {
+    switch (eb) {
+        case 4: return launch_col_e<4>(P, st);
+        case 8: return launch_col_e<8>(P, st);
+        case 16: return launch_col_e<16>(P, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
 
 cudaError_t launch_skinny_row(const SkinnyRowParams &P, int dir, int eb, cudaStream_t st) {
     switch (eb * 2 + dir) {
