@@ -110,11 +110,14 @@ const char *ipt_status_string(ipt_status_t s);
  * the library would run for ipt_c2r(m, n, elem_bytes, layout): out[0] engine (0 none,
  * 1 C2R, 2 R2C, 3 skinny), out[1] M (engine rows), out[2] N (engine columns), out[3] c =
  * gcd(M, N), out[4] number of kernel launches, out[5] column-tile cluster size, out[6]
- * column-tile width in elements, out[7] largest on-chip staging bytes per CTA.  Returns
- * IPT_ERR_UNSUPPORTED for shapes beyond limits.
+ * column-tile width in elements, out[7] largest on-chip staging bytes per CTA, out[8]
+ * CTAs per row of the row pass (0: one CTA per row; K > 0: a K-CTA cluster sharing the
+ * row through distributed shared memory, for rows longer than one CTA's shared memory),
+ * out[9] global scratch bytes.  Returns IPT_ERR_UNSUPPORTED for shapes beyond limits.
  */
+#define IPT_PLAN_INFO_FIELDS 10
 ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
-                           int64_t out[8]);
+                           int64_t out[IPT_PLAN_INFO_FIELDS]);
 
 /* Number of kernel launches this library has enqueued since load (all threads). */
 uint64_t ipt_launch_count(void);

@@ -154,9 +154,10 @@ def scratch_bytes(m: int, n: int, elem_bytes: int):
 
 
 def plan_info(m: int, n: int, elem_bytes: int, layout="row"):
-    out = (_i64 * 8)()
+    out = (_i64 * 10)()
     _check(_lib.ipt_plan_info(m, n, elem_bytes, _LAYOUTS[layout], out), "ipt_plan_info")
-    keys = ("engine", "M", "N", "c", "launches", "cluster", "tile_w", "onchip_bytes")
+    keys = ("engine", "M", "N", "c", "launches", "cluster", "tile_w", "onchip_bytes", "row_cluster",
+            "scratch_bytes")
     d = dict(zip(keys, (int(v) for v in out)))
     d["engine"] = {0: "none", 1: "c2r", 2: "r2c", 3: "skinny"}[d["engine"]]
     return d

@@ -294,9 +294,11 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     pl.a = pl.M / pl.c;
     pl.b = pl.N / pl.c;
 
-    // Row pass: the whole row must fit one CTA's shared memory.
-    const size_t rsm = row_smem_bytes(pl.N, eb);
-    if (rsm > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
+    // Row pass: one CTA per row while the row fits its shared memory, else (or from
+    // IPT_ROW_CLUSTER_MIN row bytes on) a cluster of K CTAs per row.
+    size_t rsm = row_smem_bytes(pl.N, eb);
+    const int64_t cl_min = env_int("IPT_ROW_CLUSTER_MIN", 0);
+    const bool use_cluster = rsm > static_cast<size_t>(dev.smem_optin) || (cl_min > 0 && pl.N * eb >= cl_min);
     RowParams &rp = pl.row;
     std::memset(&rp, 0, sizeof(rp));
     rp.M = static_cast<int32_t>(pl.M);
@@ -322,6 +324,27 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         rp.w_ds = static_cast<int32_t>((D / pl.b + ((D % pl.b) * (pl.M % pl.N)) % pl.N) % pl.N);
     }
     pl.row_dir = engine == ENG_C2R ? ROW_C2R : ROW_R2C;
+    if (use_cluster) {
+        // K CTAs per row; the K with the most co-resident CTAs (ties: the smaller K).
+        const int forced = env_int("IPT_ROW_CLUSTER_K", 0);
+        int best_ctas = 0;
+        for (int K : {2, 4, 8, 16}) {
+            if (forced && K != forced) continue;
+            const int64_t seg = ((pl.N + K - 1) / K + 31) / 32 * 32;
+            const size_t sm = row_cluster_smem(static_cast<int32_t>(seg), eb);
+            if (sm > static_cast<size_t>(dev.smem_optin)) continue;
+            const int ctas = row_cluster_active(K, static_cast<int32_t>(seg), eb, pl.row_dir) * K;
+            if (ctas > best_ctas) {
+                best_ctas = ctas;
+                rp.cl_K = K;
+                rp.cl_seg = static_cast<int32_t>(seg);
+                rsm = sm;
+            }
+        }
+        if (best_ctas == 0) return IPT_ERR_UNSUPPORTED;
+        rp.fd_seg = make_fastdiv(static_cast<uint32_t>(rp.cl_seg));
+        rp.cl_sync = env_int("IPT_ROW_CLUSTER_SYNC", 1);
+    }
 
     ipt_status_t s = plan_col(dev, pl, engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.shuf);
     if (s != IPT_OK) return s;
@@ -358,7 +381,8 @@ struct PlanKeyHash {
 std::string tunables_key() {
     std::string s;
     for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
-                          "IPT_SKINNY_MIN"}) {
+                          "IPT_SKINNY_MIN", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
+                          "IPT_ROW_CLUSTER_SYNC"}) {
         const char *v = std::getenv(n);
         s += v ? v : "-";
         s += '|';
@@ -455,7 +479,9 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
     // The rotation moves only the columns with a non-zero amount: (c - 1) / c of them.
     const double rot_bytes = full * static_cast<double>(pl.c - 1) / static_cast<double>(pl.c);
     auto rot = [&] { return launch_col(pl.rot.p, COL_ROT, pl.eb, st, pl.rot.smem); };
-    auto row = [&] { return launch_row(pl.row, pl.row_dir, pl.eb, st); };
+    auto row = [&] {
+        return pl.row.cl_K ? launch_row_cluster(pl.row, pl.row_dir, pl.eb, st) : launch_row(pl.row, pl.row_dir, pl.eb, st);
+    };
     ipt_status_t s;
     if (pl.engine == ENG_SKINNY) {
         // Rolling rows (§6.1; DESIGN.md §"Skinny"): engine view n rows x N, one
@@ -669,7 +695,8 @@ ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *glo
     return IPT_OK;
 }
 
-ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout, int64_t out[8]) {
+ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
+                           int64_t out[IPT_PLAN_INFO_FIELDS]) {
     int64_t x, y;
     if (!out || !valid_eb(elem_bytes) || m < 0 || n < 0 || !perm_of(true, m, n, layout, x, y))
         return IPT_ERR_INVALID_ARGUMENT;
@@ -684,6 +711,8 @@ ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t la
     out[5] = pl.engine ? pl.shuf.p.G : 0;
     out[6] = pl.engine ? pl.shuf.p.W : 0;
     out[7] = static_cast<int64_t>(pl.onchip);
+    out[8] = pl.engine ? pl.row.cl_K : 0;
+    out[9] = static_cast<int64_t>(pl.scratch);
     return IPT_OK;
 }
 

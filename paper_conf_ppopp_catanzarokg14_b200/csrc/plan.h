@@ -53,6 +53,12 @@ struct RowParams {
     int32_t w_dh;   // 32 mod b
     int32_t w_dl2;  // floor(32 / b)
     int32_t w_ds;   // (floor(32 / b) + (32 mod b) M) mod N
+    // Cluster row pass (rows too long for one CTA): the row is split
+    // into cl_K segments of cl_seg elements (a multiple of 32), one per CTA of a cluster.
+    int32_t cl_K, cl_seg;
+    int32_t cl_sync;  // 0: release/acquire cluster barriers; 1: CTA fence before the WAR
+                      // barrier; 2: CTA fences on both (IPT_ROW_CLUSTER_SYNC)
+    FastDiv fd_seg;
 };
 
 struct ColParams {
@@ -114,6 +120,11 @@ unsigned int *group_counters(cudaStream_t st, int n);
 size_t row_smem_bytes(int64_t N, int eb);
 int row_block_threads();
 cudaError_t launch_row(const RowParams &p, int dir, int eb, cudaStream_t st);
+// Cluster row pass: p.cl_K CTAs per row, each staging cl_seg elements in shared memory,
+// gathering through distributed shared memory (row_shuffle.cu).
+size_t row_cluster_smem(int32_t seg, int eb);
+int row_cluster_active(int K, int32_t seg, int eb, int dir);  // co-resident clusters (0: none)
+cudaError_t launch_row_cluster(const RowParams &p, int dir, int eb, cudaStream_t st);
 
 size_t col_smem_bytes(int64_t B, int64_t W, int eb);
 int col_block_threads();

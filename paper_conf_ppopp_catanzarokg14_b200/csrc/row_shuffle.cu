@@ -19,6 +19,10 @@
 // so a lane spends a handful of integer adds per element (§4.4's strength reduction
 // taken one step further); f2 can only be 1 in the last c - 1 rows, which take a
 // slower walk that tracks l.
+#include <array>
+#include <map>
+#include <mutex>
+
 #include "plan.h"
 
 namespace ipt {
@@ -206,6 +210,171 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_shuffle_kernel(RowParams P
     }
 }
 
+// ---- Cluster row pass (rows longer than one CTA's shared memory) -----
+// A cluster of K CTAs owns one row at a time.  CTA k stages row elements
+// [k seg, (k+1) seg) in its shared memory; after a cluster barrier every CTA gathers its
+// own output segment, reading each source element from the shared memory of the CTA that
+// holds it (ld.shared::cluster, distributed shared memory), and writes it coalesced.  A
+// second barrier (the loop's) keeps a CTA's buffer alive until every peer has read it.
+// In place: all global reads of a row precede the barrier, all its writes follow it.
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t a, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+// cluster_barrier() (arrive.release / wait.acquire) compiles to MEMBAR.ALL.GPU, which
+// waits for every outstanding global store of the thread.  This form orders the thread's
+// prior accesses at CTA scope only (MEMBAR.ALL.CTA) -- IPT_ROW_CLUSTER_SYNC selects it.
+__device__ __forceinline__ void cluster_barrier_cta_fence() {
+    asm volatile("fence.acq_rel.cta;\n"
+                 "barrier.cluster.arrive.relaxed.aligned;\n"
+                 "barrier.cluster.wait.acquire.aligned;\n" ::: "memory");
+}
+template <int EB>
+__device__ __forceinline__ typename Word<EB>::T ld_cluster(uint32_t a) {
+    typename Word<EB>::T v;
+    // volatile keeps these loads between the cluster barriers; no "memory" clobber, so
+    // the global stores of the gather may be scheduled after a batch of loads
+    if constexpr (EB == 4) {
+        asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    } else if constexpr (EB == 8) {
+        asm volatile("ld.shared::cluster.u64 %0, [%1];" : "=l"(v) : "r"(a));
+    } else {
+        asm volatile("ld.shared::cluster.v4.u32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    }
+    return v;
+}
+
+template <int EB, int DIR, bool TAIL>
+__device__ __forceinline__ void gather_seg(const RowParams &P, char *row, uint32_t rb, int32_t p0, int32_t p1,
+                                           int32_t i) {
+    using T = typename Word<EB>::T;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    const int32_t len = p1 - p0;
+    const int32_t per = ((len + nwarps - 1) / nwarps + 31) & ~31;
+    const int32_t p_end = min(p1, p0 + warp * per + per);
+    const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
+    const int32_t Mi = P.M - i;
+    T *out = reinterpret_cast<T *>(row);
+    int32_t p = p0 + warp * per + lane;
+    if (p - lane >= p_end) return;  // warp-uniform
+    // lane k < K holds the cluster address of CTA k's staged segment (rb)
+    auto fetch = [&](int32_t s) {
+        const uint32_t owner = fdiv(static_cast<uint32_t>(s), P.fd_seg);
+        const uint32_t base = __shfl_sync(0xffffffffu, rb, static_cast<int>(owner));
+        return ld_cluster<EB>(base + static_cast<uint32_t>(s - static_cast<int32_t>(owner) * P.cl_seg) * EB);
+    };
+    // __shfl_sync needs the whole warp: lanes past the end keep walking without storing.
+    // Batches of U remote loads are issued before their stores (memory-level parallelism:
+    // a distributed-shared-memory load costs a round trip through the cluster network).
+    constexpr int U = 8;
+    auto run = [&](auto w) {
+        for (; p - lane < p_end; p += 32 * U) {
+            T v[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                v[u] = fetch(w.src(P, Mi));
+                w.next(P);
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (p + 32 * u < p_end) out[p + 32 * u] = v[u];
+        }
+    };
+    if (DIR == ROW_C2R) run(C2RWalk<TAIL>(P, im, min(p, P.N - 1)));
+    else run(R2CWalk<TAIL>(P, im, min(p, P.N - 1)));
+}
+
+template <int EB, int DIR>
+__global__ void __launch_bounds__(kRowThreadsMax) row_cluster_kernel(RowParams P) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    const uint32_t K = static_cast<uint32_t>(P.cl_K);
+    const uint32_t rank = cluster_rank();
+    const int64_t cid = blockIdx.x / K, ncl = gridDim.x / K;
+    const int64_t rows_total = static_cast<int64_t>(P.M) * P.batch;
+    const int32_t nbytes = P.N * EB;
+    const uint32_t sbase = smem_u32(smem);
+    const int lane = threadIdx.x & 31;
+    const uint32_t rb0 = lane < static_cast<int>(K) ? mapa_u32(sbase, static_cast<uint32_t>(lane)) : 0;
+    const int32_t p0 = static_cast<int32_t>(rank) * P.cl_seg;
+    const int32_t p1 = min(P.N, p0 + P.cl_seg);
+    for (int64_t r = cid; r < rows_total; r += ncl) {
+        const int64_t mat = r / P.M;
+        const int32_t i = static_cast<int32_t>(r - mat * P.M);
+        char *row = P.base + mat * P.mat_stride_bytes + static_cast<int64_t>(i) * nbytes;
+        if (p1 > p0) {
+            stage_row<EB>(row + static_cast<int64_t>(p0) * EB, (p1 - p0) * EB, sbase);
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+        }
+        // every segment of the row is staged and visible cluster-wide
+        if (P.cl_sync >= 2) cluster_barrier_cta_fence();
+        else cluster_barrier();
+        // seg * EB is a multiple of 16: all segments share the row's 16-byte misalignment
+        const uint32_t rb = rb0 + static_cast<uint32_t>(reinterpret_cast<uintptr_t>(row) & 15);
+        if (p1 > p0) {
+            if (i >= P.M - P.c + 1) gather_seg<EB, DIR, true>(P, row, rb, p0, p1, i);
+            else gather_seg<EB, DIR, false>(P, row, rb, p0, p1, i);
+        }
+        // peers are done reading this CTA's buffer (a WAR hazard only: the reads have
+        // returned -- their values feed the stores issued before the arrive)
+        if (P.cl_sync >= 1) cluster_barrier_cta_fence();
+        else cluster_barrier();
+    }
+}
+
+template <int EB, int DIR>
+cudaError_t launch_row_cluster_t(const RowParams &P, cudaStream_t st, int active_only, int *active) {
+    const size_t smem = row_cluster_smem(P.cl_seg, EB);
+    auto kern = row_cluster_kernel<EB, DIR>;
+    cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, P.cl_K > 8);
+    if (e != cudaSuccess) return e;
+    cudaLaunchConfig_t cfg{};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = static_cast<unsigned>(P.cl_K);
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cfg.blockDim = dim3(kRowThreadsMax);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    if (active_only) {
+        int sms = 0, dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cfg.gridDim = dim3(static_cast<unsigned>(sms / P.cl_K * P.cl_K));
+        return cudaOccupancyMaxActiveClusters(active, reinterpret_cast<const void *>(kern), &cfg);
+    }
+    const int64_t rows = static_cast<int64_t>(P.M) * P.batch;
+    int64_t ncl = *active;
+    if (ncl > rows) ncl = rows;
+    cfg.gridDim = dim3(static_cast<unsigned>(ncl * P.cl_K));
+    e = cudaLaunchKernelEx(&cfg, kern, P);
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
+template <int EB>
+cudaError_t launch_row_cluster_e(const RowParams &P, int dir, cudaStream_t st, int active_only, int *active) {
+    return dir == ROW_C2R ? launch_row_cluster_t<EB, ROW_C2R>(P, st, active_only, active)
+                          : launch_row_cluster_t<EB, ROW_R2C>(P, st, active_only, active);
+}
+
+cudaError_t row_cluster_dispatch(const RowParams &P, int dir, int eb, cudaStream_t st, int active_only, int *active) {
+    switch (eb) {
+        case 4: return launch_row_cluster_e<4>(P, dir, st, active_only, active);
+        case 8: return launch_row_cluster_e<8>(P, dir, st, active_only, active);
+        case 16: return launch_row_cluster_e<16>(P, dir, st, active_only, active);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
 int row_threads(int64_t N, int eb) { return N * eb >= 48 * 1024 ? 512 : 256; }
 
 // Double buffering while two row buffers stay within ~110 KB (two CTAs per SM or more).
@@ -236,6 +405,38 @@ cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
 
 size_t row_smem_bytes(int64_t N, int eb) { return (static_cast<size_t>(N) * eb + 31) & ~size_t(15); }
 int row_block_threads() { return kRowThreadsMax; }
+
+size_t row_cluster_smem(int32_t seg, int eb) { return static_cast<size_t>(seg) * eb + 32; }
+
+int row_cluster_active(int K, int32_t seg, int eb, int dir) {
+    static std::mutex mu;
+    static std::map<std::array<int, 5>, int> cache;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const std::array<int, 5> key{K, seg, eb, dir, dev};
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) return it->second;
+    }
+    RowParams P{};
+    P.cl_K = K;
+    P.cl_seg = seg;
+    int active = 0;
+    if (row_cluster_dispatch(P, dir, eb, nullptr, 1, &active) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    std::lock_guard<std::mutex> lk(mu);
+    cache[key] = active;
+    return active;
+}
+
+cudaError_t launch_row_cluster(const RowParams &P, int dir, int eb, cudaStream_t st) {
+    int active = row_cluster_active(P.cl_K, P.cl_seg, eb, dir);
+    if (active < 1) return cudaErrorInvalidConfiguration;
+    return row_cluster_dispatch(P, dir, eb, st, 0, &active);
+}
 
 cudaError_t launch_row(const RowParams &P, int dir, int eb, cudaStream_t st) {
     switch (eb * 2 + dir) {
