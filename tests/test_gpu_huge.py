@@ -107,14 +107,18 @@ def test_cluster_barrier_variants(sync):
         assert x.cpu().numpy().tobytes() == oracle.transpose(host, m, n).tobytes()
 
 
-def index_tensor(total, eb):
-    """Element k carries k (8-byte words; 16-byte words carry (k, ~k)); 4-byte words k mod 2^32."""
-    if eb == 8:
-        return torch.arange(total, dtype=torch.int64, device=DEV)
-    if eb == 4:
-        return torch.arange(total, dtype=torch.int64, device=DEV).to(torch.int32)
-    k = torch.arange(total, dtype=torch.int64, device=DEV)
-    return torch.stack([k, ~k], dim=1).reshape(-1)
+def index_tensor(total, eb, chunk=1 << 28):
+    """Element k carries k (8-byte words; 16-byte words carry (k, ~k)); 4-byte words k mod 2^32.
+    Filled in chunks: one torch.arange over more than 2^32 elements leaves the tail zero."""
+    x = torch.empty(total * (2 if eb == 16 else 1), dtype=torch.int32 if eb == 4 else torch.int64, device=DEV)
+    for s in range(0, total, chunk):
+        e = min(total, s + chunk)
+        k = torch.arange(s, e, dtype=torch.int64, device=DEV)
+        if eb == 16:
+            x.view(-1, 2)[s:e] = torch.stack([k, ~k], dim=1)
+        else:
+            x[s:e] = k.to(x.dtype)
+    return x
 
 
 def check_index_transpose(x, m, n, eb, samples, seed):
@@ -144,13 +148,11 @@ def check_identity_chunked(x, total, eb, chunk=1 << 28):
     flat = x.view(-1)
     for s in range(0, total, chunk):
         e = min(total, s + chunk)
-        want = index_tensor(e - s, eb)
+        k = torch.arange(s, e, dtype=torch.int64, device=DEV)
         if eb == 16:
-            want = (want.view(-1, 2) + torch.tensor([s, -s], dtype=torch.int64, device=DEV)).reshape(-1)
-        elif eb == 8:
-            want += s
+            want = torch.stack([k, ~k], dim=1).reshape(-1)
         else:
-            want = (torch.arange(s, e, dtype=torch.int64, device=DEV)).to(torch.int32)
+            want = k.to(flat.dtype)
         assert torch.equal(flat[s * per:e * per], want), (s, e)
 
 
