@@ -327,13 +327,14 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     if (use_cluster) {
         // K CTAs per row; the K with the most co-resident CTAs (ties: the smaller K).
         const int forced = env_int("IPT_ROW_CLUSTER_K", 0);
+        rp.cl_mode = env_int("IPT_ROW_CLUSTER_MODE", 1);
         int best_ctas = 0;
         for (int K : {2, 4, 8, 16}) {
             if (forced && K != forced) continue;
             const int64_t seg = ((pl.N + K - 1) / K + 31) / 32 * 32;
             const size_t sm = row_cluster_smem(static_cast<int32_t>(seg), eb);
             if (sm > static_cast<size_t>(dev.smem_optin)) continue;
-            const int ctas = row_cluster_active(K, static_cast<int32_t>(seg), eb, pl.row_dir) * K;
+            const int ctas = row_cluster_active(K, static_cast<int32_t>(seg), eb, pl.row_dir, rp.cl_mode) * K;
             if (ctas > best_ctas) {
                 best_ctas = ctas;
                 rp.cl_K = K;
@@ -382,7 +383,7 @@ std::string tunables_key() {
     std::string s;
     for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
-                          "IPT_ROW_CLUSTER_SYNC"}) {
+                          "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
         s += v ? v : "-";
         s += '|';

@@ -58,6 +58,9 @@ struct RowParams {
     int32_t cl_K, cl_seg;
     int32_t cl_sync;  // 0: release/acquire cluster barriers; 1: CTA fence before the WAR
                       // barrier; 2: CTA fences on both (IPT_ROW_CLUSTER_SYNC)
+    int32_t cl_mode;  // 0: stage the row across the cluster, gather through DSMEM;
+                      // 1: gather from the row in L2 into private shared memory
+                      // (IPT_ROW_CLUSTER_MODE)
     FastDiv fd_seg;
 };
 
@@ -123,7 +126,7 @@ cudaError_t launch_row(const RowParams &p, int dir, int eb, cudaStream_t st);
 // Cluster row pass: p.cl_K CTAs per row, each staging cl_seg elements in shared memory,
 // gathering through distributed shared memory (row_shuffle.cu).
 size_t row_cluster_smem(int32_t seg, int eb);
-int row_cluster_active(int K, int32_t seg, int eb, int dir);  // co-resident clusters (0: none)
+int row_cluster_active(int K, int32_t seg, int eb, int dir, int mode);  // co-resident clusters (0: none)
 cudaError_t launch_row_cluster(const RowParams &p, int dir, int eb, cudaStream_t st);
 
 size_t col_smem_bytes(int64_t B, int64_t W, int eb);

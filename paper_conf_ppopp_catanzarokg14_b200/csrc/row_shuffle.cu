@@ -328,10 +328,92 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_cluster_kernel(RowParams P
     }
 }
 
+// L2 variant (cl_mode 1): CTA k gathers its output segment [k seg, (k+1) seg) straight from
+// the row in global memory (random reads served by L2; the row is prefetched into L2 one
+// row ahead with bulk prefetches) into its shared memory; one cluster barrier (every read
+// of the row is done) and the segment is written back coalesced.  Shared memory is private
+// to the CTA, so one barrier per row suffices.
+template <int EB, int DIR, bool TAIL>
+__device__ __forceinline__ void gather_l2(const RowParams &P, const char *row, unsigned char *buf, int32_t p0,
+                                          int32_t p1, int32_t i) {
+    using T = typename Word<EB>::T;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    const int32_t len = p1 - p0;
+    const int32_t per = ((len + nwarps - 1) / nwarps + 31) & ~31;
+    const int32_t p_end = min(p1, p0 + warp * per + per);
+    const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
+    const int32_t Mi = P.M - i;
+    const T *src = reinterpret_cast<const T *>(row);
+    T *out = reinterpret_cast<T *>(buf) - p0;
+    int32_t p = p0 + warp * per + lane;
+    if (p >= p_end) return;
+    constexpr int U = 8;
+    auto run = [&](auto w) {
+        for (; p < p_end; p += 32 * U) {
+            T v[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int32_t s = w.src(P, Mi);
+                if (p + 32 * u < p_end) v[u] = __ldcg(src + s);
+                w.next(P);
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (p + 32 * u < p_end) out[p + 32 * u] = v[u];
+        }
+    };
+    if (DIR == ROW_C2R) run(C2RWalk<TAIL>(P, im, p));
+    else run(R2CWalk<TAIL>(P, im, p));
+}
+
+__device__ __forceinline__ void prefetch_l2(const char *p, int64_t bytes) {
+    // cp.async.bulk.prefetch.L2: 16-byte aligned address and size
+    const uintptr_t a0 = (reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15);
+    const uintptr_t a1 = (reinterpret_cast<uintptr_t>(p) + bytes) & ~uintptr_t(15);
+    for (uintptr_t a = a0 + static_cast<uintptr_t>(threadIdx.x) * 4096; a < a1; a += blockDim.x * 4096ull) {
+        const uint32_t sz = a1 - a < 4096 ? static_cast<uint32_t>(a1 - a) : 4096u;
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(a), "r"(sz) : "memory");
+    }
+}
+
+template <int EB, int DIR>
+__global__ void __launch_bounds__(kRowThreadsMax) row_cluster_l2_kernel(RowParams P) {
+    using T = typename Word<EB>::T;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const uint32_t K = static_cast<uint32_t>(P.cl_K);
+    const uint32_t rank = cluster_rank();
+    const int64_t cid = blockIdx.x / K, ncl = gridDim.x / K;
+    const int64_t rows_total = static_cast<int64_t>(P.M) * P.batch;
+    const int32_t nbytes = P.N * EB;
+    const int32_t p0 = static_cast<int32_t>(rank) * P.cl_seg;
+    const int32_t p1 = min(P.N, p0 + P.cl_seg);
+    auto row_of = [&](int64_t r) {
+        const int64_t mat = r / P.M;
+        return P.base + mat * P.mat_stride_bytes + static_cast<int64_t>(r - mat * P.M) * nbytes;
+    };
+    if (cid < rows_total && p1 > p0) prefetch_l2(row_of(cid) + static_cast<int64_t>(p0) * EB, (p1 - p0) * EB);
+    for (int64_t r = cid; r < rows_total; r += ncl) {
+        const int32_t i = static_cast<int32_t>(r % P.M);
+        char *row = row_of(r);
+        if (r + ncl < rows_total && p1 > p0)
+            prefetch_l2(row_of(r + ncl) + static_cast<int64_t>(p0) * EB, (p1 - p0) * EB);
+        if (p1 > p0) {
+            if (i >= P.M - P.c + 1) gather_l2<EB, DIR, true>(P, row, smem, p0, p1, i);
+            else gather_l2<EB, DIR, false>(P, row, smem, p0, p1, i);
+        }
+        // every CTA of the cluster has read the whole row (its loads have returned)
+        cluster_barrier_cta_fence();
+        const T *buf = reinterpret_cast<const T *>(smem);
+        T *dst = reinterpret_cast<T *>(row) + p0;
+        for (int32_t k = threadIdx.x; k < p1 - p0; k += blockDim.x) dst[k] = buf[k];
+        __syncthreads();  // the buffer is refilled by the next row
+    }
+}
+
 template <int EB, int DIR>
 cudaError_t launch_row_cluster_t(const RowParams &P, cudaStream_t st, int active_only, int *active) {
     const size_t smem = row_cluster_smem(P.cl_seg, EB);
-    auto kern = row_cluster_kernel<EB, DIR>;
+    auto kern = P.cl_mode == 1 ? row_cluster_l2_kernel<EB, DIR> : row_cluster_kernel<EB, DIR>;
     cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, P.cl_K > 8);
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg{};
@@ -408,12 +490,12 @@ int row_block_threads() { return kRowThreadsMax; }
 
 size_t row_cluster_smem(int32_t seg, int eb) { return static_cast<size_t>(seg) * eb + 32; }
 
-int row_cluster_active(int K, int32_t seg, int eb, int dir) {
+int row_cluster_active(int K, int32_t seg, int eb, int dir, int mode) {
     static std::mutex mu;
-    static std::map<std::array<int, 5>, int> cache;
+    static std::map<std::array<int, 6>, int> cache;
     int dev = 0;
     cudaGetDevice(&dev);
-    const std::array<int, 5> key{K, seg, eb, dir, dev};
+    const std::array<int, 6> key{K, seg, eb, dir, dev, mode};
     {
         std::lock_guard<std::mutex> lk(mu);
         auto it = cache.find(key);
@@ -422,6 +504,7 @@ int row_cluster_active(int K, int32_t seg, int eb, int dir) {
     RowParams P{};
     P.cl_K = K;
     P.cl_seg = seg;
+    P.cl_mode = mode;
     int active = 0;
     if (row_cluster_dispatch(P, dir, eb, nullptr, 1, &active) != cudaSuccess) {
         cudaGetLastError();
@@ -433,7 +516,7 @@ int row_cluster_active(int K, int32_t seg, int eb, int dir) {
 }
 
 cudaError_t launch_row_cluster(const RowParams &P, int dir, int eb, cudaStream_t st) {
-    int active = row_cluster_active(P.cl_K, P.cl_seg, eb, dir);
+    int active = row_cluster_active(P.cl_K, P.cl_seg, eb, dir, P.cl_mode);
     if (active < 1) return cudaErrorInvalidConfiguration;
     return row_cluster_dispatch(P, dir, eb, st, 0, &active);
 }

@@ -93,18 +93,23 @@ def test_cluster_rows_forced_medium(K, engine):
             assert x.cpu().numpy().tobytes() == np.ascontiguousarray(host).tobytes()
 
 
-@pytest.mark.parametrize("sync", [0, 1, 2])
-def test_cluster_barrier_variants(sync):
-    """IPT_ROW_CLUSTER_SYNC: release/acquire barriers or CTA-scope fences."""
-    m, n, eb = 3001, 4099, 4
-    host = workloads.random_words(m * n, eb, seed=sync)
-    with env(IPT_ROW_CLUSTER_MIN=1, IPT_ROW_CLUSTER_SYNC=sync):
-        x = to_dev(host)
-        for _ in range(3):
-            ipt.c2r(x, m, n, elem_bytes=eb)
-            ipt.r2c(x, m, n, elem_bytes=eb)
-        ipt.c2r(x, m, n, elem_bytes=eb)
-        assert x.cpu().numpy().tobytes() == oracle.transpose(host, m, n).tobytes()
+@pytest.mark.parametrize("mode,sync", [(0, 0), (0, 1), (0, 2), (1, 1)])
+def test_cluster_variants(mode, sync):
+    """IPT_ROW_CLUSTER_MODE (0: DSMEM gather, 1: L2 gather) and IPT_ROW_CLUSTER_SYNC
+    (release/acquire barriers or CTA-scope fences), every K, both engines."""
+    for (m, n), eb in [((3001, 4099), 4), ((1200, 1800), 8), ((517, 300), 16)]:
+        host = workloads.random_words(m * n, eb, seed=sync + 3 * mode)
+        for K in (2, 4, 8, 16):
+            for engine in ("c2r", "r2c"):
+                with env(IPT_ROW_CLUSTER_MIN=1, IPT_ROW_CLUSTER_SYNC=sync, IPT_ROW_CLUSTER_MODE=mode,
+                         IPT_ROW_CLUSTER_K=K, IPT_FORCE_ENGINE=engine):
+                    x = to_dev(host)
+                    for _ in range(2):
+                        ipt.c2r(x, m, n, elem_bytes=eb)
+                        ipt.r2c(x, m, n, elem_bytes=eb)
+                    ipt.c2r(x, m, n, elem_bytes=eb)
+                    got = vwords(x.cpu().numpy(), eb)
+                    assert got.tobytes() == oracle.transpose(vwords(host, eb), m, n).tobytes(), (m, n, K, engine)
 
 
 def index_tensor(total, eb, chunk=1 << 28):
