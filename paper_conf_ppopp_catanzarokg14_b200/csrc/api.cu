@@ -117,6 +117,10 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
     if (twb != 32 && twb != 64 && twb != 128) twb = 128;
     if (twb < pl.eb) twb = pl.eb;
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
+    // IPT_COL_PIPE (default 1): persistent pipelined kernel with IPT_COL_NBUF unit buffers
+    // per CTA; the shared-memory target is per buffer.
+    const bool pipe = env_int("IPT_COL_PIPE", 1) != 0;
+    const int nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
     const int64_t target = env_int("IPT_COL_SMEM", 46 * 1024);
     const int64_t W = twb / pl.eb;
     const int64_t per_row = twb + 8;  // col_smem_bytes: staged row + two row indices
@@ -125,10 +129,10 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
     if (B > col_max_band(W)) B = col_max_band(W);
     if (B > pl.M) B = pl.M;
     for (;;) {
-        const size_t smem = col_smem_bytes(B, W, pl.eb);
+        const size_t smem = col_smem_bytes(B, W, pl.eb, nbuf);
         if (smem > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
         const int64_t G = (pl.M + B - 1) / B;
-        const int resident = col_resident_ctas(mode, pl.eb, twb, smem);
+        const int resident = col_resident_ctas(mode, pl.eb, twb, smem, pipe);
         if (resident < 1) return IPT_ERR_UNSUPPORTED;
         if (G > resident) {  // a whole group must be co-resident
             B = (pl.M + resident - 1) / resident;
@@ -153,6 +157,8 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
         p.G = static_cast<int32_t>(G);
         p.B = static_cast<int32_t>(B);
         p.resident = resident;
+        p.pipe = pipe ? 1 : 0;
+        p.nbuf = nbuf;
         p.rot_sign = 1;
         p.wide_a = pl.a >= 65536 ? 1 : 0;
         cp.smem = smem;
@@ -381,7 +387,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -744,9 +750,12 @@ ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes
     if (p.B > col_max_band(p.W)) return IPT_ERR_UNSUPPORTED;
     p.G = static_cast<int32_t>((M + p.B - 1) / p.B);
     p.rot_sign = barrier ? 1 : 0;
-    const size_t smem = col_smem_bytes(p.B, p.W, elem_bytes);
+    const bool pipe = env_int("IPT_COL_PIPE", 1) != 0;
+    p.pipe = pipe ? 1 : 0;
+    p.nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
+    const size_t smem = col_smem_bytes(p.B, p.W, elem_bytes, p.nbuf);
     if (smem > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
-    p.resident = col_resident_ctas(COL_COPY, elem_bytes, tile_bytes, smem);
+    p.resident = col_resident_ctas(COL_COPY, elem_bytes, tile_bytes, smem, pipe);
     if (p.resident < p.G) return IPT_ERR_UNSUPPORTED;
     finish_col(p, 1);
     return check(launch_col(p, COL_COPY, elem_bytes, static_cast<cudaStream_t>(stream), smem));

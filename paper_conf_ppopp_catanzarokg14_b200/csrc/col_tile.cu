@@ -41,6 +41,8 @@
 // and the non-persistent grid lets CTAs drift out of lock-step (a persistent cooperative
 // variant and a two-buffer pipelined variant were both slower: profiles/).  The grid is one
 // CTA per (tile, band); see col_tile_kernel for why the spin barrier cannot deadlock.
+#include <algorithm>
+
 #include "plan.h"
 
 namespace ipt {
@@ -51,6 +53,7 @@ namespace {
 #define IPT_COL_THREADS 512
 #endif
 constexpr int kColThreads = IPT_COL_THREADS;
+constexpr int kMaxColBufs = 4;  // unit buffers per CTA of the pipelined kernel
 
 // q^{-1}(i) = (floor((c-1+i)/c) b^{-1}) mod a + (((c-1) i) mod c) a  (Eq. 34).
 __device__ __forceinline__ int32_t qinv_of(const ColParams &P, int32_t i) {
@@ -101,130 +104,174 @@ __device__ __forceinline__ void cp_async_elem(uint32_t dst, const void *src) {
         asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" :: "r"(dst), "l"(src), "n"(EB) : "memory");
 }
 
-// One CTA per (tile, band).  The CTA's logical id comes from a ticket counter taken at
-// start (dispatch order), so the G members of a tile are exactly G consecutive tickets:
-// every group whose tickets are all taken is fully resident, hence only the newest group
-// can be waiting for members, and those get scheduled as older groups finish -- the spin
-// barrier cannot deadlock as long as one group fits on the GPU (G <= resident CTAs).
-//
-// Thread mapping: lane = tile column w (W = TWB/eb lanes per tile row, 32/W rows per warp
-// instruction).  A load instruction copies whole tile rows (128 contiguous bytes) with
-// element-granular cp.async, each element landing directly in its OUTPUT row of the band in
-// shared memory (row k = t - dw[w]): the skew / rotation is done by the copy's
-// destination address, and the bank of every element is its column (conflict-free).  A
-// store instruction writes whole output rows (128 contiguous bytes).  No 16-byte alignment
-// is needed anywhere: element accesses work at every row phase and never leave the tile.
-template <int EB, int MODE, int TWB>
-__device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *smem, uint32_t tt, int32_t r) {
-    using T = typename Word<EB>::T;
-    constexpr int W = TWB / EB;
-    constexpr int RPW = 32 / W;  // tile rows per warp instruction
-    const int32_t r0 = r * P.B;
-    const int32_t nrows = max(0, min(P.M, r0 + P.B) - r0);
-    const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
-    const uint32_t kshM = P.kshM;
-    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+// One column-tile work unit: band r of tile tt (of all matrices).
+struct Unit {
+    char *colp;        // this lane's column in row 0 of the matrix
+    int32_t r0, nrows;  // output band [r0, r0 + nrows)
+    int32_t j0m;        // j0 mod M
+    int32_t rowbase;    // first input row (ROT / C2R)
+    int32_t dw;         // slot t, lane column w feeds band row k = t - dw
+    int32_t nslots;     // input rows read: band + halo
+    int32_t wt;         // columns of this tile (W, or fewer at the ragged right edge)
+    bool skip;          // ROT tile made only of columns rotating by 0
+};
 
-    // ---- tile geometry --------------------------------------------------------------
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ Unit unit_make(const ColParams &P, uint32_t tt, int32_t r) {
+    constexpr int W = TWB / EB;
+    Unit U;
+    U.r0 = r * P.B;
+    U.nrows = max(0, min(P.M, U.r0 + P.B) - U.r0);
     const uint32_t mat = fdiv(tt, P.fd_nt);
     const int32_t tile = static_cast<int32_t>(tt - mat * static_cast<uint32_t>(P.ntiles));
-    char *A = P.base + static_cast<int64_t>(mat) * P.mat_stride_bytes;
     const int32_t j0 = tile * W;
-    const int32_t Wt = min(W, P.N - j0);
-    const int32_t j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j0), P.fd_M));
-    int32_t ext = W - 1, lo_q = 0, hi_q = 0, base_off = 0;
+    U.wt = min(W, P.N - j0);
+    U.j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j0), P.fd_M));
+    U.skip = false;
+    const int w = (threadIdx.x & 31) % W;
+    int32_t ext = W - 1, base_off = 0;
+    U.dw = 0;
     if (MODE == COL_ROT) {
-        lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
-        hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + Wt - 1), P.fd_b));
+        const int32_t lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
+        const int32_t hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + U.wt - 1), P.fd_b));
         ext = hi_q - lo_q;
         base_off = P.rot_sign > 0 ? lo_q : -hi_q;  // smallest rotation amount in the tile
-        // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.  The
-        // skip is group-uniform; still arrive, later tiles sharing the counter count it.
-        if (hi_q == 0) {
-            if (use_barrier && threadIdx.x == 0) atomicAdd(P.ctr + (tt % kCtrSlots), 1u);
-            return;
-        }
+        // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.
+        U.skip = hi_q == 0;
+        const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + min(w, U.wt - 1)), P.fd_b));
+        U.dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
     } else if (MODE == COL_COPY) {
         ext = 0;
+    } else if (MODE == COL_C2R_SHUF) {
+        U.dw = w;
+    } else {
+        U.dw = W - 1 - w;
     }
-    const int32_t nslots = nrows > 0 ? nrows + ext : 0;
+    U.nslots = U.nrows > 0 ? U.nrows + ext : 0;
+    U.rowbase = MODE == COL_ROT ? mod_M(U.r0 + base_off, P.kshM, P.fd_M) : U.r0;
+    U.colp = P.base + static_cast<int64_t>(mat) * P.mat_stride_bytes + static_cast<int64_t>(j0 + w) * EB;
+    return U;
+}
 
+// Scattered row indices of a unit, computed by the whole CTA into shared memory:
+// C2R destinations orow[k] = q^{-1}((r0 + k - j0) mod M) (Eq. 34), R2C sources
+// srow[t] = q^{-1}((r0 - W + 1 + t - j0) mod M).  R2C needs a __syncthreads before the load.
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ void unit_prepass(const ColParams &P, const Unit &U, int32_t *orow, int32_t *srow,
+                                             int nthr) {
+    constexpr int W = TWB / EB;
+    if (MODE == COL_C2R_SHUF) {
+        for (int32_t k = threadIdx.x; k < U.nrows; k += nthr)
+            orow[k] = qinv_of(P, mod_M(U.r0 + k - U.j0m, P.kshM, P.fd_M));
+    }
+    if (MODE == COL_R2C_SHUF) {
+        for (int32_t t = threadIdx.x; t < U.nslots; t += nthr)
+            srow[t] = qinv_of(P, mod_M(U.r0 - (W - 1) + t - U.j0m, P.kshM, P.fd_M));
+    }
+}
+
+// Load: element-granular cp.async from each tile row straight into the element's OUTPUT
+// row of the band in shared memory (row k = t - dw).  Thread mapping: lane = tile column
+// w (W = TWB/eb lanes per tile row, 32/W rows per warp instruction); a load instruction
+// copies whole tile rows (128 contiguous bytes), the bank of every element is its column
+// (conflict-free).  No 16-byte alignment is needed anywhere.  Not committed here.
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ void unit_load(const ColParams &P, const Unit &U, const int32_t *srow, uint32_t rows_s,
+                                          int nthr) {
+    constexpr int W = TWB / EB;
+    constexpr int RPW = 32 / W;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = nthr >> 5;
+    const int w = lane % W, sub = lane / W;
+    if (w >= U.wt || U.skip) return;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    const int32_t step = nwarps * RPW;  // slots between a lane's consecutive rows
+    const int32_t dw = U.dw;
+    // This lane's slots t with 0 <= k = t - dw < nrows (the others are halo elements no
+    // band row needs): a branch-free walk with incremental shared and global addresses.
+    int32_t t = warp * RPW + sub;
+    if (t < dw) t += ((dw - t + step - 1) / step) * step;
+    const int32_t tend = dw + U.nrows;
+    uint32_t sa = rows_s + w * EB + (t - dw) * TWB;
+    const uint32_t sa_inc = step * TWB;
+    const char *colp = U.colp;
+    if (MODE == COL_R2C_SHUF) {
+#pragma unroll 4
+        for (; t < tend; t += step, sa += sa_inc) cp_async_elem<EB>(sa, colp + srow[t] * pitch);
+    } else if (step <= P.M) {
+        int32_t s = mod_M(U.rowbase + t, P.kshM, P.fd_M);
+        const char *g = colp + s * pitch;
+        const int64_t g_inc = step * pitch, g_wrap = static_cast<int64_t>(P.M) * pitch;
+#pragma unroll 4
+        for (; t < tend; t += step, sa += sa_inc) {
+            cp_async_elem<EB>(sa, g);
+            s += step;
+            g += g_inc;
+            if (s >= P.M) {
+                s -= P.M;
+                g -= g_wrap;
+            }
+        }
+    } else {  // tiny M: fewer rows than one step
+        for (; t < tend; t += step, sa += sa_inc)
+            cp_async_elem<EB>(sa, colp + mod_M(U.rowbase + t, P.kshM, P.fd_M) * pitch);
+    }
+}
+
+// Store: whole output rows (128 contiguous bytes per warp instruction).
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, const int32_t *orow,
+                                           const unsigned char *rows, int nthr) {
+    using T = typename Word<EB>::T;
+    constexpr int W = TWB / EB;
+    constexpr int RPW = 32 / W;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = nthr >> 5;
+    const int w = lane % W, sub = lane / W;
+    if (w >= U.wt || U.skip) return;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    const int32_t step = nwarps * RPW;
+    const unsigned char *sr = rows + w * EB;
+    int32_t k = warp * RPW + sub;
+    char *colp = U.colp;
+    if (MODE == COL_C2R_SHUF) {
+#pragma unroll 4
+        for (; k < U.nrows; k += step)
+            *reinterpret_cast<T *>(colp + static_cast<int64_t>(orow[k]) * pitch) =
+                *reinterpret_cast<const T *>(sr + k * TWB);
+    } else {
+        char *g = colp + static_cast<int64_t>(U.r0 + k) * pitch;
+        const int64_t g_inc = step * pitch;
+#pragma unroll 4
+        for (; k < U.nrows; k += step, g += g_inc) *reinterpret_cast<T *>(g) = *reinterpret_cast<const T *>(sr + k * TWB);
+    }
+}
+
+__device__ __forceinline__ void group_arrive(unsigned int *ctr) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
+}
+
+// Non-persistent variant: one CTA per (tile, band).  The CTA's logical id comes from a
+// ticket counter taken at start (dispatch order), so the G members of a tile are exactly
+// G consecutive tickets: every group whose tickets are all taken is fully resident, hence
+// only the newest group can be waiting for members, and those get scheduled as older
+// groups finish -- the spin barrier cannot deadlock as long as one group fits on the GPU
+// (G <= resident CTAs).  G == 1: no barrier, P.tpc consecutive tiles per CTA.
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *smem, uint32_t tt, int32_t r) {
     size_t o_srow, o_rows;
-    smem_layout(P.B, W, TWB, &o_srow, &o_rows);
+    smem_layout(P.B, TWB / EB, TWB, &o_srow, &o_rows);
     int32_t *orow = reinterpret_cast<int32_t *>(smem);
     int32_t *srow = reinterpret_cast<int32_t *>(smem + o_srow);
     unsigned char *rows = smem + o_rows;
-    char *Aj = A + static_cast<int64_t>(j0) * EB;
-
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-    const int w = lane % W, sub = lane / W;
-    int32_t dw = 0;  // slot t, column w feeds band row k = t - dw
-    if (MODE == COL_ROT) {
-        const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + min(w, Wt - 1)), P.fd_b));
-        dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
-    } else if (MODE == COL_C2R_SHUF) {
-        dw = w;
-    } else if (MODE == COL_R2C_SHUF) {
-        dw = W - 1 - w;
+    const Unit U = unit_make<EB, MODE, TWB>(P, tt, r);
+    const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
+    if (U.skip) {  // group-uniform; still arrive, later tiles sharing the counter count it
+        if (use_barrier && threadIdx.x == 0) atomicAdd(P.ctr + (tt % kCtrSlots), 1u);
+        return;
     }
-
-    // ---- pre-pass: scattered row indices (C2R destinations, R2C sources) --------------
-    if (MODE == COL_C2R_SHUF) {
-        for (int32_t k = threadIdx.x; k < nrows; k += blockDim.x)
-            orow[k] = qinv_of(P, mod_M(r0 + k - j0m, kshM, P.fd_M));
-    }
-    if (MODE == COL_R2C_SHUF) {
-        for (int32_t t = threadIdx.x; t < nslots; t += blockDim.x)
-            srow[t] = qinv_of(P, mod_M(r0 - (W - 1) + t - j0m, kshM, P.fd_M));
-        __syncthreads();
-    }
-
-    // ---- load: every element straight to its output row -------------------------------
-    const int32_t rowbase = MODE == COL_ROT ? mod_M(r0 + base_off, kshM, P.fd_M) : r0;
-    const uint32_t srows = static_cast<uint32_t>(__cvta_generic_to_shared(rows)) + w * EB;
-    char *colp = Aj + w * EB;
-    char *tmpw = P.tmp + static_cast<int64_t>(j0 + w) * EB;  // skinny engine only
-    const int32_t step = nwarps * RPW;  // slots between a lane's consecutive rows
-    const int32_t t0 = warp * RPW + sub;
-    if (w < Wt && P.remap < 0) {  // skinny: row s is stored at s-1, row 0 in tmp
-        int32_t t = t0;
-        if (t < dw) t += ((dw - t + step - 1) / step) * step;
-        for (; t < dw + nrows; t += step) {
-            const int32_t s = MODE == COL_R2C_SHUF ? srow[t] : mod_M(rowbase + t, kshM, P.fd_M);
-            cp_async_elem<EB>(srows + (t - dw) * TWB, s == 0 ? tmpw : colp + (s - 1) * pitch);
-        }
-    } else if (w < Wt) {
-        // This lane's slots t with 0 <= k = t - dw < nrows (the others are halo elements no
-        // band row needs): a branch-free walk with incremental shared and global addresses.
-        int32_t t = t0;
-        if (t < dw) t += ((dw - t + step - 1) / step) * step;
-        const int32_t tend = dw + nrows;
-        uint32_t sa = srows + (t - dw) * TWB;
-        const uint32_t sa_inc = step * TWB;
-        if (MODE == COL_R2C_SHUF) {
-#pragma unroll 4
-            for (; t < tend; t += step, sa += sa_inc) cp_async_elem<EB>(sa, colp + srow[t] * pitch);
-        } else if (step <= P.M) {
-            int32_t s = mod_M(rowbase + t, kshM, P.fd_M);
-            const char *g = colp + s * pitch;
-            const int64_t g_inc = step * pitch, g_wrap = static_cast<int64_t>(P.M) * pitch;
-#pragma unroll 4
-            for (; t < tend; t += step, sa += sa_inc) {
-                cp_async_elem<EB>(sa, g);
-                s += step;
-                g += g_inc;
-                if (s >= P.M) {
-                    s -= P.M;
-                    g -= g_wrap;
-                }
-            }
-        } else {  // tiny M: fewer rows than one step
-            for (; t < tend; t += step, sa += sa_inc)
-                cp_async_elem<EB>(sa, colp + mod_M(rowbase + t, kshM, P.fd_M) * pitch);
-        }
-    }
+    unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
+    if (MODE == COL_R2C_SHUF) __syncthreads();
+    unit_load<EB, MODE, TWB>(P, U, srow, static_cast<uint32_t>(__cvta_generic_to_shared(rows)), blockDim.x);
     asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
-
     // In-place hazard barrier: the whole tile has been read before anyone writes it.
     // Counter slot tt mod kCtrSlots, monotone over the tiles that share it.
     if (use_barrier) {
@@ -234,29 +281,7 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     } else {
         __syncthreads();
     }
-
-    // ---- store: whole output rows -------------------------------------------------------
-    if (w < Wt) {
-        const unsigned char *sr = rows + w * EB;
-        int32_t k = t0;
-        if (P.remap > 0) {  // skinny: output row o is stored at o+1, row M-1 in tmp
-            for (; k < nrows; k += step) {
-                const int32_t o = MODE == COL_C2R_SHUF ? orow[k] : r0 + k;
-                *reinterpret_cast<T *>(o == P.M - 1 ? tmpw : colp + static_cast<int64_t>(o + 1) * pitch) =
-                    *reinterpret_cast<const T *>(sr + k * TWB);
-            }
-        } else if (MODE == COL_C2R_SHUF) {
-#pragma unroll 4
-            for (; k < nrows; k += step)
-                *reinterpret_cast<T *>(colp + static_cast<int64_t>(orow[k]) * pitch) =
-                    *reinterpret_cast<const T *>(sr + k * TWB);
-        } else {
-            char *g = colp + static_cast<int64_t>(r0 + k) * pitch;
-            const int64_t g_inc = step * pitch;
-#pragma unroll 4
-            for (; k < nrows; k += step, g += g_inc) *reinterpret_cast<T *>(g) = *reinterpret_cast<const T *>(sr + k * TWB);
-        }
-    }
+    unit_store<EB, MODE, TWB>(P, U, orow, rows, blockDim.x);
 }
 
 template <int EB, int MODE, int TWB>
@@ -266,7 +291,7 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     if (threadIdx.x == 0) s_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
     __syncthreads();
     const unsigned int ticket = s_ticket;
-    if (P.G == 1) {  // a tile fits one CTA: no barrier, P.tpc consecutive tiles per CTA
+    if (P.G == 1) {
         const uint64_t t_end = min(static_cast<uint64_t>(P.total_tiles), (static_cast<uint64_t>(ticket) + 1) * P.tpc);
         for (uint64_t tt = static_cast<uint64_t>(ticket) * P.tpc; tt < t_end; ++tt) {
             col_tile_one<EB, MODE, TWB>(P, smem, static_cast<uint32_t>(tt), 0);
@@ -279,54 +304,223 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     col_tile_one<EB, MODE, TWB>(P, smem, tt, r);
 }
 
+// mbarrier helpers (shared::cta).
+__device__ __forceinline__ void mbar_init(uint64_t *bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))),
+                 "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];"
+                 :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))) : "memory");
+}
+// Arrive once every cp.async this thread issued so far has landed (counted in the init).
+__device__ __forceinline__ void mbar_arrive_cpasync(uint64_t *bar) {
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];"
+                 :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))) : "memory");
+}
+__device__ __forceinline__ bool mbar_test(uint64_t *bar, unsigned parity) {
+    uint32_t ok;
+    asm volatile("{\n .reg .pred p;\n mbarrier.test_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n"
+                 " selp.u32 %0, 1, 0, p;\n}"
+                 : "=r"(ok) : "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))), "r"(parity) : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
+    const uint32_t a = static_cast<uint32_t>(__cvta_generic_to_shared(bar));
+    asm volatile("{\n .reg .pred p;\n WAIT_%=:\n"
+                 " mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%0], %1;\n"
+                 " @!p bra WAIT_%=;\n}" :: "r"(a), "r"(parity) : "memory");
+}
+
+// Persistent, warp-specialised, two-buffer variant (P.pipe).  The last two warps are the
+// TICKET warp and the CONTROL warp (one thread each), the others are workers.  Unit i of
+// a CTA lives in buffer i & 1.  Ticket thread: as soon as unit i-2 is released it takes
+// ticket t_i (units in ticket order: tile-major, the G bands of a tile consecutive; the
+// atomic's latency overlaps the workers' stores of unit i-2) and publishes it once the
+// buffer is free.  Control thread: as soon as the workers' loads of unit i have landed (an
+// mbarrier fed by cp.async.mbarrier.arrive) it arrives on the tile's counter --
+// independently of how far the older unit has got -- and when the whole group has
+// arrived it releases unit i to the workers.  Workers: load unit i, then store unit i-1
+// once released.  So the loads of one unit are in flight while the CTA waits for the
+// group of the other and stores it, and no group's arrival waits for another group's
+// barrier (no lock-step chain).
+//
+// Deadlock freedom (G <= grid): a unit's arrival needs only its own loads.  Take the
+// oldest incomplete group g: its taken tickets all arrive.  If some are untaken, g is the
+// newest group (tickets are taken in order); a CTA can take a ticket once a buffer frees,
+// and every buffer holding an older unit frees (those groups complete).  Only a CTA whose
+// two buffers both hold units of g cannot take more; all CTAs in that state would mean
+// >= 2 grid >= G taken tickets of g, i.e. none untaken.  By induction every group completes.
 template <int EB, int MODE, int TWB>
-void *kptr() {
-    return reinterpret_cast<void *>(col_tile_kernel<EB, MODE, TWB>);
+__global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ unsigned int s_ticket[kMaxColBufs];
+    __shared__ int s_release;  // units released so far (control -> ticket warp)
+    __shared__ __align__(8) uint64_t bar_tk[kMaxColBufs], bar_full[kMaxColBufs], bar_go[kMaxColBufs],
+        bar_empty[kMaxColBufs];
+    constexpr int W = TWB / EB;
+    const int nwt = static_cast<int>(blockDim.x) - 64;  // worker threads
+    const int NB = P.nbuf;
+    size_t o_srow, o_rows;
+    const size_t bufsz = smem_layout(P.B, W, TWB, &o_srow, &o_rows);
+    const uint32_t total = static_cast<uint32_t>(P.total_tiles) * static_cast<uint32_t>(P.G);
+    const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
+    if (threadIdx.x == 0) {
+        for (int b = 0; b < NB; ++b) {
+            mbar_init(&bar_tk[b], 1);
+            mbar_init(&bar_full[b], nwt);
+            mbar_init(&bar_go[b], 1);
+            mbar_init(&bar_empty[b], nwt);
+        }
+        s_release = 0;
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    // Unit u lives in buffer u mod NB and uses phase (u / NB) & 1 of that buffer's mbarriers.
+
+    if (threadIdx.x >= nwt) {
+        if (threadIdx.x == nwt) {  // ---- ticket warp: take and publish tickets ----------
+            int b = 0, k = 0;
+            for (int u = 0;; ++u) {
+                if (k > 0) {  // take unit u's ticket once unit u-NB is released: its buffer then
+                    // frees unconditionally (the workers only have to store it)
+                    while (*reinterpret_cast<volatile int *>(&s_release) < u - NB + 1) __nanosleep(32);
+                }
+                const uint32_t t = atomicAdd(P.ctr + kTicketSlot, 1u);
+                if (k > 0) mbar_wait(&bar_empty[b], (k - 1) & 1);
+                s_ticket[b] = t;
+                mbar_arrive(&bar_tk[b]);
+                if (t >= total) break;
+                if (++b == NB) b = 0, ++k;
+            }
+        } else if (threadIdx.x == nwt + 32) {  // ---- control warp: arrive and release ----
+            int arrive = 0, release = 0;  // next unit to arrive / release
+            int ab = 0, ak = 0, rb = 0;
+            while (true) {
+                bool progress = false;
+                if (mbar_test(&bar_tk[ab], ak & 1)) {  // unit `arrive` published
+                    const uint32_t t = s_ticket[ab];
+                    if (t >= total) {
+                        if (release == arrive) break;  // every real unit released
+                    } else if (mbar_test(&bar_full[ab], ak & 1)) {
+                        if (use_barrier) group_arrive(P.ctr + (fdiv(t, P.fd_G) % kCtrSlots));
+                        ++arrive;
+                        if (++ab == NB) ab = 0, ++ak;
+                        progress = true;
+                    }
+                }
+                if (release < arrive) {
+                    const uint32_t tt = fdiv(s_ticket[rb], P.fd_G);
+                    bool done = !use_barrier;
+                    if (!done) {
+                        unsigned int v;
+                        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.ctr + (tt % kCtrSlots)) : "memory");
+                        done = v >= (tt / kCtrSlots + 1) * static_cast<unsigned int>(P.G);
+                    }
+                    if (done) {
+                        mbar_arrive(&bar_go[rb]);
+                        ++release;
+                        if (++rb == NB) rb = 0;
+                        *reinterpret_cast<volatile int *>(&s_release) = release;
+                        progress = true;
+                    }
+                }
+                if (!progress) __nanosleep(32);
+            }
+        }
+        return;
+    }
+
+    // ---- workers: load unit i, then store unit i - NB + 1 once released ----------------
+    auto store_unit = [&](int sb, int sk) {
+        mbar_wait(&bar_go[sb], sk & 1);
+        const uint32_t st = s_ticket[sb];
+        const uint32_t stt = fdiv(st, P.fd_G);
+        const Unit Us = unit_make<EB, MODE, TWB>(P, stt, static_cast<int32_t>(st - stt * P.G));
+        unsigned char *sbuf = smem + sb * bufsz;
+        unit_store<EB, MODE, TWB>(P, Us, reinterpret_cast<const int32_t *>(sbuf), sbuf + o_rows, nwt);
+    };
+    int b = 0, k = 0;    // buffer / round of unit i
+    int sb = 0, sk = 0;  // buffer / round of the oldest unit not yet stored
+    for (int i = 0;; ++i) {
+        unsigned char *buf = smem + b * bufsz;
+        mbar_wait(&bar_tk[b], k & 1);
+        const uint32_t t = s_ticket[b];
+        if (t >= total) {  // drain: store the units still held, oldest first
+            for (int j = max(0, i - NB + 1); j < i; ++j) {
+                store_unit(sb, sk);
+                if (++sb == NB) sb = 0, ++sk;
+            }
+            break;
+        }
+        const uint32_t tt = fdiv(t, P.fd_G);
+        const Unit U = unit_make<EB, MODE, TWB>(P, tt, static_cast<int32_t>(t - tt * P.G));
+        int32_t *orow = reinterpret_cast<int32_t *>(buf);
+        int32_t *srow = reinterpret_cast<int32_t *>(buf + o_srow);
+        if (!U.skip) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, nwt);
+        asm volatile("bar.sync 1, %0;" :: "r"(nwt) : "memory");  // srow / orow visible
+        unit_load<EB, MODE, TWB>(P, U, srow, static_cast<uint32_t>(__cvta_generic_to_shared(buf + o_rows)), nwt);
+        mbar_arrive_cpasync(&bar_full[b]);
+        if (i - NB + 1 >= 0) {
+            store_unit(sb, sk);
+            mbar_arrive(&bar_empty[sb]);
+            if (++sb == NB) sb = 0, ++sk;
+        }
+        if (++b == NB) b = 0, ++k;
+    }
+}
+
+template <int EB, int MODE, int TWB>
+void *kptr(bool pipe) {
+    return pipe ? reinterpret_cast<void *>(col_pipe_kernel<EB, MODE, TWB>)
+                : reinterpret_cast<void *>(col_tile_kernel<EB, MODE, TWB>);
 }
 
 template <int EB, int TWB>
-void *col_kernel_w(int mode) {
+void *col_kernel_w(int mode, bool pipe) {
     switch (mode) {
-        case COL_ROT: return kptr<EB, COL_ROT, TWB>();
-        case COL_C2R_SHUF: return kptr<EB, COL_C2R_SHUF, TWB>();
-        case COL_R2C_SHUF: return kptr<EB, COL_R2C_SHUF, TWB>();
-        case COL_COPY: return kptr<EB, COL_COPY, TWB>();
+        case COL_ROT: return kptr<EB, COL_ROT, TWB>(pipe);
+        case COL_C2R_SHUF: return kptr<EB, COL_C2R_SHUF, TWB>(pipe);
+        case COL_R2C_SHUF: return kptr<EB, COL_R2C_SHUF, TWB>(pipe);
+        case COL_COPY: return kptr<EB, COL_COPY, TWB>(pipe);
         default: return nullptr;
     }
 }
 
 template <int EB>
-void *col_kernel_e(int mode, int twb) {
+void *col_kernel_e(int mode, int twb, bool pipe) {
     switch (twb) {
-        case 32: return col_kernel_w<EB, 32>(mode);
-        case 64: return col_kernel_w<EB, 64>(mode);
-        case 128: return col_kernel_w<EB, 128>(mode);
+        case 32: return col_kernel_w<EB, 32>(mode, pipe);
+        case 64: return col_kernel_w<EB, 64>(mode, pipe);
+        case 128: return col_kernel_w<EB, 128>(mode, pipe);
         default: return nullptr;
     }
 }
 
-void *col_kernel(int mode, int eb, int twb) {
+void *col_kernel(int mode, int eb, int twb, bool pipe) {
     switch (eb) {
-        case 4: return col_kernel_e<4>(mode, twb);
-        case 8: return col_kernel_e<8>(mode, twb);
-        case 16: return col_kernel_e<16>(mode, twb);
+        case 4: return col_kernel_e<4>(mode, twb, pipe);
+        case 8: return col_kernel_e<8>(mode, twb, pipe);
+        case 16: return col_kernel_e<16>(mode, twb, pipe);
         default: return nullptr;
     }
 }
 
 }  // namespace
 
-size_t col_smem_bytes(int64_t B, int64_t W, int eb) {
+size_t col_smem_bytes(int64_t B, int64_t W, int eb, int nbuf) {
     size_t a, b;
-    return smem_layout(B, static_cast<int>(W), static_cast<int>(W * eb), &a, &b);
+    return smem_layout(B, static_cast<int>(W), static_cast<int>(W * eb), &a, &b) * (nbuf > 0 ? nbuf : 1);
 }
+
+int col_max_bufs() { return kMaxColBufs; }
 
 int64_t col_max_band(int64_t W) { return (int64_t(1) << 24) - W; }
 
 int col_block_threads() { return kColThreads; }
 
-int col_resident_ctas(int mode, int eb, int twb, size_t smem) {
-    void *kern = col_kernel(mode, eb, twb);
+int col_resident_ctas(int mode, int eb, int twb, size_t smem, bool pipe) {
+    void *kern = col_kernel(mode, eb, twb, pipe);
     if (!kern || ensure_kernel_attrs(kern, smem, false) != cudaSuccess) {
         cudaGetLastError();
         return 0;
@@ -335,12 +529,15 @@ int col_resident_ctas(int mode, int eb, int twb, size_t smem) {
 }
 
 cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, size_t smem) {
-    void *kern = col_kernel(mode, eb, P0.W * eb);
+    void *kern = col_kernel(mode, eb, P0.W * eb, P0.pipe != 0);
     if (!kern) return cudaErrorInvalidValue;
     cudaError_t e = ensure_kernel_attrs(kern, smem, false);
     if (e != cudaSuccess) return e;
     ColParams P = P0;
-    const int64_t grid = P.G == 1 ? (P.total_tiles + P.tpc - 1) / P.tpc : P.total_tiles * P.G;
+    const int64_t units = P.total_tiles * P.G;
+    if (units > 0xfffffff0LL) return cudaErrorInvalidConfiguration;
+    const int64_t grid = P.pipe ? std::min<int64_t>(P.resident, units)
+                                : P.G == 1 ? (P.total_tiles + P.tpc - 1) / P.tpc : units;
     if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     // Ticket + group counters: the stream's own block, zeroed in stream order.
     P.ctr = group_counters(st, kCtrSlots + 1);

@@ -83,13 +83,9 @@ struct ColParams {
     int32_t wide_a;     // a >= 2^16
     FastDiv fd_G, fd_nt;  // ticket -> (tile, band), tile -> (matrix, column tile)
     uint32_t kshM;      // (2 + W / M) * M: shift making every mod_M argument non-negative
-    // Skinny engine (rolling rows, skinny.cu): row x of the engine view is stored at
-    // location x+remap, the row that falls off the end lives in the one-row buffer `tmp`.
-    //   remap = +1: outputs are written shifted (row M-1 -> tmp); remap = -1: inputs are
-    //   read shifted (row 0 <- tmp).  Only with batch == 1.
-    char *tmp;
-    int32_t remap;
     int32_t tpc;        // tiles per CTA when G == 1 (each tile fits one CTA)
+    int32_t pipe;       // 1: persistent pipelined kernel (col_pipe_kernel) with nbuf unit buffers
+    int32_t nbuf;
 };
 
 struct SkinnyRowParams {
@@ -129,11 +125,13 @@ size_t row_cluster_smem(int32_t seg, int eb);
 int row_cluster_active(int K, int32_t seg, int eb, int dir, int mode);  // co-resident clusters (0: none)
 cudaError_t launch_row_cluster(const RowParams &p, int dir, int eb, cudaStream_t st);
 
-size_t col_smem_bytes(int64_t B, int64_t W, int eb);
+// Shared memory of a column-pass CTA: nbuf unit buffers (0 or 1: the non-pipelined kernel).
+size_t col_smem_bytes(int64_t B, int64_t W, int eb, int nbuf);
+int col_max_bufs();
 int col_block_threads();
 int64_t col_max_band(int64_t W);  // largest band a CTA may be given
 cudaError_t launch_col(const ColParams &p, int mode, int eb, cudaStream_t st, size_t smem);
-int col_resident_ctas(int mode, int eb, int twb, size_t smem);
+int col_resident_ctas(int mode, int eb, int twb, size_t smem, bool pipe);
 
 // Skinny column pass (skinny.cu): all n rows x C consecutive columns per CTA, the column
 // permutation sigma_j among the n rows applied in shared memory.

@@ -1,0 +1,124 @@
+// DRAM access-pattern probe for the column pass (measurement tool, not product code).
+// An M x R-byte array is processed in column tiles of TW bytes x all M rows, bands of
+// `band` rows per CTA, CTAs in tile-major order (the column pass's order).  Each CTA
+// stages its band (16-B cp.async), __syncthreads, then writes it back to row
+//   identity : r
+//   scatter  : (r * K) mod M   (K coprime with M: rows spread over the whole column)
+// Variants: rw (read + write), ro (read only), wo (write only).  GB/s = bytes moved / t.
+// nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -o tile_probe tools/tile_probe.cu
+#include <cstdio>
+#include <cstdint>
+#include <cstdlib>
+#include <cuda_runtime.h>
+
+__global__ void copy_contig(const uint4 *__restrict__ a, uint4 *__restrict__ b, size_t n) {
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
+        b[i] = a[i];
+}
+
+template <int TW>
+__global__ void staged(char *a, int M, long R, int band, int scatter, int K, int what) {
+    extern __shared__ __align__(16) unsigned char sm[];
+    constexpr int LPR = TW / 16;
+    const int nband = (M + band - 1) / band;
+    const int tile = blockIdx.x / nband;
+    const int bandi = blockIdx.x % nband;
+    const int r0 = bandi * band, r1 = min(M, r0 + band);
+    const int sub = threadIdx.x % LPR;
+    const int rstep = blockDim.x / LPR;
+    uint32_t s = (uint32_t)__cvta_generic_to_shared(sm);
+    if (what != 2) {
+        for (int r = r0 + threadIdx.x / LPR; r < r1; r += rstep) {
+            size_t off = (size_t)r * R + (size_t)tile * TW + sub * 16;
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s + (uint32_t)((r - r0) * TW + sub * 16)),
+                         "l"(a + off));
+        }
+        asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+    }
+    __syncthreads();
+    if (what == 1) {
+        if (threadIdx.x == 0 && *(volatile int *)sm == 0x7fffffff) a[0] = 1;  // keep loads
+        return;
+    }
+    for (int r = r0 + threadIdx.x / LPR; r < r1; r += rstep) {
+        const int o = scatter ? (int)(((long long)r * K) % M) : r;
+        size_t off = (size_t)o * R + (size_t)tile * TW + sub * 16;
+        *(uint4 *)(a + off) = *(const uint4 *)(sm + (r - r0) * TW + sub * 16);
+    }
+}
+
+static float timeit(void (*f)(), char *flush, size_t fl) {
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    float best = 1e9;
+    for (int k = 0; k < 5; ++k) {
+        cudaMemset(flush, k, fl);
+        cudaEventRecord(e0);
+        f();
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms;
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (k > 0 && ms < best) best = ms;
+    }
+    return best;
+}
+
+struct Args {
+    char *a, *b;
+    int M, band, scatter, K, what, threads;
+    long R;
+};
+static Args G;
+
+template <int TW> void run() {
+    const int ntile = (int)(G.R / TW), nb = (G.M + G.band - 1) / G.band;
+    staged<TW><<<ntile * nb, G.threads, (size_t)G.band * TW>>>(G.a, G.M, G.R, G.band, G.scatter, G.K, G.what);
+}
+void run_contig() { copy_contig<<<148 * 8, 512>>>((const uint4 *)G.a, (uint4 *)G.b, (size_t)G.M * G.R / 32); }
+
+template <int TW> void sweep(size_t bytes, char *flush, size_t fl) {
+    cudaFuncSetAttribute(staged<TW>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    for (int smem_kb : {24, 46, 96}) {
+        G.band = smem_kb * 1024 / TW;
+        for (int what = 0; what < 3; ++what) {
+            for (int sc = 0; sc < 2; ++sc) {
+                if (what == 1 && sc) continue;
+                G.what = what;
+                G.scatter = sc;
+                float t = timeit(run<TW>, flush, fl);
+                const double moved = what == 0 ? 2.0 * bytes : (double)bytes;
+                printf("{\"TW\":%d,\"smem_kb\":%d,\"op\":\"%s\",\"scatter\":%d,\"GBps\":%.1f}\n", TW, smem_kb,
+                       what == 0 ? "rw" : what == 1 ? "ro" : "wo", sc, moved / t / 1e6);
+            }
+        }
+    }
+}
+
+int main(int argc, char **argv) {
+    int M = argc > 1 ? atoi(argv[1]) : 14414;
+    long R = argc > 2 ? atol(argv[2]) : 6565L * 8;
+    R = R / 1024 * 1024;
+    size_t bytes = (size_t)M * R;
+    cudaMalloc(&G.a, bytes);
+    cudaMalloc(&G.b, bytes);
+    cudaMemset(G.a, 1, bytes);
+    char *flush;
+    size_t fl = 256u << 20;
+    cudaMalloc(&flush, fl);
+    G.M = M;
+    G.R = R;
+    G.threads = 512;
+    G.K = 7919;  // prime, coprime with M unless M is a multiple
+    if (M % G.K == 0) G.K = 7907;
+    float t = timeit(run_contig, flush, fl);
+    printf("{\"what\":\"contiguous copy\",\"M\":%d,\"R\":%ld,\"GBps\":%.1f}\n", M, R, bytes / t / 1e6);
+    sweep<128>(bytes, flush, fl);
+    sweep<256>(bytes, flush, fl);
+    sweep<512>(bytes, flush, fl);
+    sweep<1024>(bytes, flush, fl);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) printf("err %s\n", cudaGetErrorString(e));
+    return 0;
+}
