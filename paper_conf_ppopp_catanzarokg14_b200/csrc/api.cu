@@ -123,8 +123,9 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
     const int nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
     const int64_t target = env_int("IPT_COL_SMEM", 46 * 1024);
     const int64_t W = twb / pl.eb;
-    const int64_t per_row = twb + 8;  // col_smem_bytes: staged row + two row indices
-    int64_t B = target / per_row - (W - 1);
+    // Largest band whose buffer fits the target (col_smem_bytes: staged rows + row indices).
+    int64_t B = target / (twb + 8);
+    while (B > 32 && col_smem_bytes(B, W, pl.eb, 1) > static_cast<size_t>(target)) B -= 8;
     if (B < 32) B = 32;
     if (B > col_max_band(W)) B = col_max_band(W);
     if (B > pl.M) B = pl.M;

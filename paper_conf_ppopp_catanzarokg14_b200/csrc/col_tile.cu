@@ -85,15 +85,27 @@ __device__ __forceinline__ void group_barrier(unsigned int *ctr, unsigned int ta
     __syncthreads();
 }
 
-// Shared-memory layout: [orow B*4 | srow nslots*4 | rows B*TWB].
+// Shared-memory layout of one unit buffer:
+//   [orow B*4 | srow nslots*4 | sbase nslots*4 | rows]
+// rows: element path (eb = 8, 16) -- B output rows of TWB bytes; hull path (eb = 4) --
+// nslots input rows ("slots") of HS = TWB + 16 bytes, each the 16-byte-aligned hull of the
+// tile row, sbase[t] = shared address of slot t's first tile element.
 __host__ __device__ inline size_t al16(size_t x) { return (x + 15) & ~size_t(15); }
-__host__ __device__ inline size_t smem_layout(int64_t B, int W, int twb, size_t *off_srow, size_t *off_rows) {
+struct SmemLayout {
+    size_t srow, sbase, rows, total;
+};
+__host__ __device__ constexpr bool hull_path(int eb) { return eb == 4; }
+__host__ __device__ inline SmemLayout smem_layout(int64_t B, int W, int twb, int eb) {
     const size_t nslots = static_cast<size_t>(B) + W - 1;
+    SmemLayout L;
     size_t o = al16(static_cast<size_t>(B) * 4);
-    *off_srow = o;
+    L.srow = o;
     o += al16(nslots * 4);
-    *off_rows = o;
-    return o + static_cast<size_t>(B) * twb;
+    L.sbase = o;
+    if (hull_path(eb)) o += al16(nslots * 4);
+    L.rows = o;
+    L.total = o + (hull_path(eb) ? nslots * static_cast<size_t>(twb + 16) : static_cast<size_t>(B) * twb);
+    return L;
 }
 
 template <int EB>
@@ -170,20 +182,53 @@ __device__ __forceinline__ void unit_prepass(const ColParams &P, const Unit &U, 
     }
 }
 
-// Load: element-granular cp.async from each tile row straight into the element's OUTPUT
-// row of the band in shared memory (row k = t - dw).  Thread mapping: lane = tile column
-// w (W = TWB/eb lanes per tile row, 32/W rows per warp instruction); a load instruction
-// copies whole tile rows (128 contiguous bytes), the bank of every element is its column
-// (conflict-free).  No 16-byte alignment is needed anywhere.  Not committed here.
+// Load.  Element path (eb = 8, 16): element-granular cp.async from each tile row straight
+// into the element's OUTPUT row of the band in shared memory (row k = t - dw); lane = tile
+// column w, a load instruction copies whole tile rows, the bank of every element is its
+// column (conflict-free).  Hull path (eb = 4; 4-byte cp.async runs at ~75% of the
+// 16-byte rate on B200, tools/tile_probe.cu): every input row ("slot" t) is staged as the
+// 16-byte-aligned hull of its tile row (TWB/16 + 1 chunks, the last one only when the
+// row is misaligned) and sbase[t] records where its first element landed; the skew is
+// applied when the store phase reads shared memory.  Not committed here.
 template <int EB, int MODE, int TWB>
-__device__ __forceinline__ void unit_load(const ColParams &P, const Unit &U, const int32_t *srow, uint32_t rows_s,
-                                          int nthr) {
+__device__ __forceinline__ void unit_load(const ColParams &P, const Unit &U, const int32_t *srow, uint32_t *sbase,
+                                          uint32_t rows_s, int nthr) {
     constexpr int W = TWB / EB;
+    if (U.skip) return;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    if constexpr (hull_path(EB)) {
+        constexpr int CPR = TWB / 16 + 1;  // chunks per slot
+        constexpr int HS = TWB + 16;       // slot pitch in shared memory
+        const char *tilep = U.colp - ((threadIdx.x & 31) % W) * EB;  // column j0 of row 0
+        const int32_t nchunk = U.nslots * CPR;
+        const int32_t wbytes = U.wt * EB;
+        for (int32_t f = threadIdx.x; f < nchunk; f += nthr) {
+            const int32_t t = f / CPR, c = f - t * CPR;
+            int32_t g;
+            if (MODE == COL_R2C_SHUF) {
+                g = srow[t];
+            } else {
+                g = U.rowbase + t;
+                while (g >= P.M) g -= P.M;  // t < nslots <= M + W
+            }
+            const char *rp = tilep + static_cast<int64_t>(g) * pitch;
+            const uint32_t off = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(rp)) & 15u;
+            const char *cp = rp - off + c * 16;
+            const uint32_t dst = rows_s + t * HS + c * 16;
+            if (c == 0) sbase[t] = dst + off;
+            const int32_t rem = static_cast<int32_t>(off) + wbytes - c * 16;  // bytes of the hull from cp on
+            if (rem >= 16) {
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(cp) : "memory");
+            } else if (rem > 0) {  // row end: read only the tile's bytes (never past the buffer)
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(dst), "l"(cp), "r"(rem) : "memory");
+            }
+        }
+        return;
+    }
     constexpr int RPW = 32 / W;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = nthr >> 5;
     const int w = lane % W, sub = lane / W;
-    if (w >= U.wt || U.skip) return;
-    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    if (w >= U.wt) return;
     const int32_t step = nwarps * RPW;  // slots between a lane's consecutive rows
     const int32_t dw = U.dw;
     // This lane's slots t with 0 <= k = t - dw < nrows (the others are halo elements no
@@ -217,10 +262,11 @@ __device__ __forceinline__ void unit_load(const ColParams &P, const Unit &U, con
     }
 }
 
-// Store: whole output rows (128 contiguous bytes per warp instruction).
+// Store: whole output rows (a warp instruction writes TWB... contiguous bytes of one or
+// more rows).  Hull path: output row k, column w is slot k + dw(w), read at sbase + w eb.
 template <int EB, int MODE, int TWB>
 __device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, const int32_t *orow,
-                                           const unsigned char *rows, int nthr) {
+                                           const uint32_t *sbase, const unsigned char *rows, int nthr) {
     using T = typename Word<EB>::T;
     constexpr int W = TWB / EB;
     constexpr int RPW = 32 / W;
@@ -229,9 +275,39 @@ __device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, co
     if (w >= U.wt || U.skip) return;
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
     const int32_t step = nwarps * RPW;
-    const unsigned char *sr = rows + w * EB;
     int32_t k = warp * RPW + sub;
     char *colp = U.colp;
+    if constexpr (hull_path(EB)) {
+        const uint32_t *sb = sbase + U.dw;
+        const uint32_t wo = w * EB;
+        if (MODE == COL_C2R_SHUF) {
+#pragma unroll 4
+            for (; k < U.nrows; k += step) {
+                T v;
+                const uint32_t a = sb[k] + wo;
+                if constexpr (EB == 4)
+                    asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a));
+                else
+                    asm volatile("ld.shared.b64 %0, [%1];" : "=l"(v) : "r"(a));
+                *reinterpret_cast<T *>(colp + static_cast<int64_t>(orow[k]) * pitch) = v;
+            }
+        } else {
+            char *g = colp + static_cast<int64_t>(U.r0 + k) * pitch;
+            const int64_t g_inc = step * pitch;
+#pragma unroll 4
+            for (; k < U.nrows; k += step, g += g_inc) {
+                T v;
+                const uint32_t a = sb[k] + wo;
+                if constexpr (EB == 4)
+                    asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a));
+                else
+                    asm volatile("ld.shared.b64 %0, [%1];" : "=l"(v) : "r"(a));
+                *reinterpret_cast<T *>(g) = v;
+            }
+        }
+        return;
+    }
+    const unsigned char *sr = rows + w * EB;
     if (MODE == COL_C2R_SHUF) {
 #pragma unroll 4
         for (; k < U.nrows; k += step)
@@ -257,11 +333,11 @@ __device__ __forceinline__ void group_arrive(unsigned int *ctr) {
 // (G <= resident CTAs).  G == 1: no barrier, P.tpc consecutive tiles per CTA.
 template <int EB, int MODE, int TWB>
 __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *smem, uint32_t tt, int32_t r) {
-    size_t o_srow, o_rows;
-    smem_layout(P.B, TWB / EB, TWB, &o_srow, &o_rows);
+    const SmemLayout L = smem_layout(P.B, TWB / EB, TWB, EB);
     int32_t *orow = reinterpret_cast<int32_t *>(smem);
-    int32_t *srow = reinterpret_cast<int32_t *>(smem + o_srow);
-    unsigned char *rows = smem + o_rows;
+    int32_t *srow = reinterpret_cast<int32_t *>(smem + L.srow);
+    uint32_t *sbase = reinterpret_cast<uint32_t *>(smem + L.sbase);
+    unsigned char *rows = smem + L.rows;
     const Unit U = unit_make<EB, MODE, TWB>(P, tt, r);
     const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
     if (U.skip) {  // group-uniform; still arrive, later tiles sharing the counter count it
@@ -270,7 +346,7 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     }
     unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
     if (MODE == COL_R2C_SHUF) __syncthreads();
-    unit_load<EB, MODE, TWB>(P, U, srow, static_cast<uint32_t>(__cvta_generic_to_shared(rows)), blockDim.x);
+    unit_load<EB, MODE, TWB>(P, U, srow, sbase, static_cast<uint32_t>(__cvta_generic_to_shared(rows)), blockDim.x);
     asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
     // In-place hazard barrier: the whole tile has been read before anyone writes it.
     // Counter slot tt mod kCtrSlots, monotone over the tiles that share it.
@@ -281,7 +357,7 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     } else {
         __syncthreads();
     }
-    unit_store<EB, MODE, TWB>(P, U, orow, rows, blockDim.x);
+    unit_store<EB, MODE, TWB>(P, U, orow, sbase, rows, blockDim.x);
 }
 
 template <int EB, int MODE, int TWB>
@@ -361,8 +437,8 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
     constexpr int W = TWB / EB;
     const int nwt = static_cast<int>(blockDim.x) - 64;  // worker threads
     const int NB = P.nbuf;
-    size_t o_srow, o_rows;
-    const size_t bufsz = smem_layout(P.B, W, TWB, &o_srow, &o_rows);
+    const SmemLayout L = smem_layout(P.B, W, TWB, EB);
+    const size_t bufsz = L.total;
     const uint32_t total = static_cast<uint32_t>(P.total_tiles) * static_cast<uint32_t>(P.G);
     const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
     if (threadIdx.x == 0) {
@@ -438,7 +514,8 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
         const uint32_t stt = fdiv(st, P.fd_G);
         const Unit Us = unit_make<EB, MODE, TWB>(P, stt, static_cast<int32_t>(st - stt * P.G));
         unsigned char *sbuf = smem + sb * bufsz;
-        unit_store<EB, MODE, TWB>(P, Us, reinterpret_cast<const int32_t *>(sbuf), sbuf + o_rows, nwt);
+        unit_store<EB, MODE, TWB>(P, Us, reinterpret_cast<const int32_t *>(sbuf),
+                                  reinterpret_cast<const uint32_t *>(sbuf + L.sbase), sbuf + L.rows, nwt);
     };
     int b = 0, k = 0;    // buffer / round of unit i
     int sb = 0, sk = 0;  // buffer / round of the oldest unit not yet stored
@@ -456,10 +533,11 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
         const uint32_t tt = fdiv(t, P.fd_G);
         const Unit U = unit_make<EB, MODE, TWB>(P, tt, static_cast<int32_t>(t - tt * P.G));
         int32_t *orow = reinterpret_cast<int32_t *>(buf);
-        int32_t *srow = reinterpret_cast<int32_t *>(buf + o_srow);
+        int32_t *srow = reinterpret_cast<int32_t *>(buf + L.srow);
         if (!U.skip) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, nwt);
         asm volatile("bar.sync 1, %0;" :: "r"(nwt) : "memory");  // srow / orow visible
-        unit_load<EB, MODE, TWB>(P, U, srow, static_cast<uint32_t>(__cvta_generic_to_shared(buf + o_rows)), nwt);
+        unit_load<EB, MODE, TWB>(P, U, srow, reinterpret_cast<uint32_t *>(buf + L.sbase),
+                                 static_cast<uint32_t>(__cvta_generic_to_shared(buf + L.rows)), nwt);
         mbar_arrive_cpasync(&bar_full[b]);
         if (i - NB + 1 >= 0) {
             store_unit(sb, sk);
@@ -509,8 +587,7 @@ void *col_kernel(int mode, int eb, int twb, bool pipe) {
 }  // namespace
 
 size_t col_smem_bytes(int64_t B, int64_t W, int eb, int nbuf) {
-    size_t a, b;
-    return smem_layout(B, static_cast<int>(W), static_cast<int>(W * eb), &a, &b) * (nbuf > 0 ? nbuf : 1);
+    return smem_layout(B, static_cast<int>(W), static_cast<int>(W * eb), eb).total * (nbuf > 0 ? nbuf : 1);
 }
 
 int col_max_bufs() { return kMaxColBufs; }

@@ -16,10 +16,10 @@ __global__ void copy_contig(const uint4 *__restrict__ a, uint4 *__restrict__ b, 
         b[i] = a[i];
 }
 
-template <int TW>
+template <int TW, int EB = 16>
 __global__ void staged(char *a, int M, long R, int band, int scatter, int K, int what) {
     extern __shared__ __align__(16) unsigned char sm[];
-    constexpr int LPR = TW / 16;
+    constexpr int LPR = TW / EB;
     const int nband = (M + band - 1) / band;
     const int tile = blockIdx.x / nband;
     const int bandi = blockIdx.x % nband;
@@ -29,9 +29,13 @@ __global__ void staged(char *a, int M, long R, int band, int scatter, int K, int
     uint32_t s = (uint32_t)__cvta_generic_to_shared(sm);
     if (what != 2) {
         for (int r = r0 + threadIdx.x / LPR; r < r1; r += rstep) {
-            size_t off = (size_t)r * R + (size_t)tile * TW + sub * 16;
-            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s + (uint32_t)((r - r0) * TW + sub * 16)),
-                         "l"(a + off));
+            size_t off = (size_t)r * R + (size_t)tile * TW + sub * EB;
+            if (EB == 16)
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s + (uint32_t)((r - r0) * TW + sub * 16)),
+                             "l"(a + off));
+            else
+                asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(s + (uint32_t)((r - r0) * TW + sub * EB)),
+                             "l"(a + off), "n"(EB));
         }
         asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
     }
@@ -42,8 +46,10 @@ __global__ void staged(char *a, int M, long R, int band, int scatter, int K, int
     }
     for (int r = r0 + threadIdx.x / LPR; r < r1; r += rstep) {
         const int o = scatter ? (int)(((long long)r * K) % M) : r;
-        size_t off = (size_t)o * R + (size_t)tile * TW + sub * 16;
-        *(uint4 *)(a + off) = *(const uint4 *)(sm + (r - r0) * TW + sub * 16);
+        size_t off = (size_t)o * R + (size_t)tile * TW + sub * EB;
+        if (EB == 16) *(uint4 *)(a + off) = *(const uint4 *)(sm + (r - r0) * TW + sub * 16);
+        else if (EB == 8) *(uint2 *)(a + off) = *(const uint2 *)(sm + (r - r0) * TW + sub * 8);
+        else *(uint32_t *)(a + off) = *(const uint32_t *)(sm + (r - r0) * TW + sub * 4);
     }
 }
 
@@ -72,14 +78,14 @@ struct Args {
 };
 static Args G;
 
-template <int TW> void run() {
+template <int TW, int EB = 16> void run() {
     const int ntile = (int)(G.R / TW), nb = (G.M + G.band - 1) / G.band;
-    staged<TW><<<ntile * nb, G.threads, (size_t)G.band * TW>>>(G.a, G.M, G.R, G.band, G.scatter, G.K, G.what);
+    staged<TW, EB><<<ntile * nb, G.threads, (size_t)G.band * TW>>>(G.a, G.M, G.R, G.band, G.scatter, G.K, G.what);
 }
 void run_contig() { copy_contig<<<148 * 8, 512>>>((const uint4 *)G.a, (uint4 *)G.b, (size_t)G.M * G.R / 32); }
 
-template <int TW> void sweep(size_t bytes, char *flush, size_t fl) {
-    cudaFuncSetAttribute(staged<TW>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+template <int TW, int EB = 16> void sweep(size_t bytes, char *flush, size_t fl) {
+    cudaFuncSetAttribute(staged<TW, EB>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     for (int smem_kb : {24, 46, 96}) {
         G.band = smem_kb * 1024 / TW;
         for (int what = 0; what < 3; ++what) {
@@ -87,9 +93,9 @@ template <int TW> void sweep(size_t bytes, char *flush, size_t fl) {
                 if (what == 1 && sc) continue;
                 G.what = what;
                 G.scatter = sc;
-                float t = timeit(run<TW>, flush, fl);
+                float t = timeit(run<TW, EB>, flush, fl);
                 const double moved = what == 0 ? 2.0 * bytes : (double)bytes;
-                printf("{\"TW\":%d,\"smem_kb\":%d,\"op\":\"%s\",\"scatter\":%d,\"GBps\":%.1f}\n", TW, smem_kb,
+                printf("{\"TW\":%d,\"EB\":%d,\"smem_kb\":%d,\"op\":\"%s\",\"scatter\":%d,\"GBps\":%.1f}\n", TW, EB, smem_kb,
                        what == 0 ? "rw" : what == 1 ? "ro" : "wo", sc, moved / t / 1e6);
             }
         }
@@ -114,10 +120,17 @@ int main(int argc, char **argv) {
     if (M % G.K == 0) G.K = 7907;
     float t = timeit(run_contig, flush, fl);
     printf("{\"what\":\"contiguous copy\",\"M\":%d,\"R\":%ld,\"GBps\":%.1f}\n", M, R, bytes / t / 1e6);
-    sweep<128>(bytes, flush, fl);
-    sweep<256>(bytes, flush, fl);
-    sweep<512>(bytes, flush, fl);
-    sweep<1024>(bytes, flush, fl);
+    const int only = argc > 3 ? atoi(argv[3]) : 0;
+    if (only == 0 || only == 1) {
+        sweep<128>(bytes, flush, fl);
+        sweep<128, 8>(bytes, flush, fl);
+        sweep<128, 4>(bytes, flush, fl);
+    }
+    if (only == 0) {
+        sweep<256>(bytes, flush, fl);
+        sweep<512>(bytes, flush, fl);
+        sweep<1024>(bytes, flush, fl);
+    }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) printf("err %s\n", cudaGetErrorString(e));
     return 0;
