@@ -112,14 +112,21 @@ int ilog2(int v) {
 // IPT_COL_SMEM (default 46 KiB, four CTAs per SM: the best of the round-1 sweep over
 // 12-100 KiB, profiles/r01_*).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
 // the co-resident CTAs, the band grows (up to the opt-in shared-memory maximum).
+ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe);
+
+// IPT_COL_PIPE (default 1): the persistent pipelined kernel with IPT_COL_NBUF unit buffers
+// per CTA (the shared-memory target is per buffer); tiles whose group would not fit the
+// co-resident CTAs that way (very tall matrices, config 5a) take the one-unit kernel.
 ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp) {
+    if (env_int("IPT_COL_PIPE", 1) != 0 && plan_col_v(dev, pl, mode, cp, true) == IPT_OK) return IPT_OK;
+    return plan_col_v(dev, pl, mode, cp, false);
+}
+
+ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe) {
     int twb = env_int("IPT_TILE_BYTES", 128);
     if (twb != 32 && twb != 64 && twb != 128) twb = 128;
     if (twb < pl.eb) twb = pl.eb;
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
-    // IPT_COL_PIPE (default 1): persistent pipelined kernel with IPT_COL_NBUF unit buffers
-    // per CTA; the shared-memory target is per buffer.
-    const bool pipe = env_int("IPT_COL_PIPE", 1) != 0;
     const int nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
     const int64_t target = env_int("IPT_COL_SMEM", 46 * 1024);
     const int64_t W = twb / pl.eb;
@@ -354,11 +361,26 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         rp.cl_sync = env_int("IPT_ROW_CLUSTER_SYNC", 1);
     }
 
+    // Small gcd: fold the column rotation into the row pass (row_rot_kernel; IPT_FUSE_ROT=0
+    // keeps the separate rotation pass).  Global scratch: one flag per row, and for C2R a
+    // copy of rows 0..c-2 (the rows the last c-1 staircases wrap onto).
+    if (pl.c > 1 && pl.c <= kMaxFuseC && !use_cluster && env_int("IPT_FUSE_ROT", 1) != 0) {
+        rp.segp = static_cast<int32_t>(((pl.b * eb + 15) & ~int64_t(15)) + 32);
+        rp.fd_cps = make_fastdiv(static_cast<uint32_t>(rp.segp / 16));
+        const size_t fsm = row_fused_smem_bytes(rp, eb, pl.row_dir);
+        if (fsm <= static_cast<size_t>(dev.smem_optin)) {
+            rp.fuse = 1;
+            rsm = fsm;
+            pl.scratch = static_cast<size_t>(pl.M) * 4 +
+                         (engine == ENG_C2R ? static_cast<size_t>(pl.c - 1) * pl.N * eb : 0);
+        }
+    }
+
     ipt_status_t s = plan_col(dev, pl, engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.shuf);
     if (s != IPT_OK) return s;
     pl.onchip = rsm > pl.shuf.smem ? rsm : pl.shuf.smem;
     pl.nlaunch = 2;
-    if (pl.c > 1) {
+    if (pl.c > 1 && !rp.fuse) {
         s = plan_col(dev, pl, COL_ROT, pl.rot);
         if (s != IPT_OK) return s;
         pl.rot.p.rot_sign = engine == ENG_C2R ? 1 : -1;
@@ -540,6 +562,37 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
         cudaFreeAsync(tmp, st);
         return s;
     }
+    // Fused rotation: per-call scratch (row flags, zeroed; C2R: the wrapped rows' copy).
+    char *fscratch = nullptr;
+    if (pl.row.fuse) {
+        const int64_t pitch = pl.N * pl.eb;
+        const size_t flag_bytes = (static_cast<size_t>(pl.M * batch) * 4 + 255) & ~size_t(255);
+        const size_t wrap_row_bytes = static_cast<size_t>(pl.c - 1) * pitch;
+        const size_t wrap_bytes = pl.engine == ENG_C2R ? wrap_row_bytes * batch : 0;
+        cudaMemPool_t pool = scratch_pool();
+        if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&fscratch), flag_bytes + wrap_bytes, pool, st) !=
+                         cudaSuccess) {
+            cudaGetLastError();
+            return IPT_ERR_OUT_OF_MEMORY;
+        }
+        pl.row.flags = reinterpret_cast<unsigned int *>(fscratch);
+        pl.row.wrap = fscratch + flag_bytes;
+        ipt_status_t s0 = check(cudaMemsetAsync(fscratch, 0, flag_bytes, st));
+        if (s0 == IPT_OK && wrap_bytes)
+            s0 = check(cudaMemcpy2DAsync(fscratch + flag_bytes, wrap_row_bytes, base, stride_bytes, wrap_row_bytes,
+                                         batch, cudaMemcpyDeviceToDevice, st));
+        if (s0 != IPT_OK) {
+            cudaFreeAsync(fscratch, st);
+            return s0;
+        }
+    }
+    struct FreeScratch {
+        char *p;
+        cudaStream_t st;
+        ~FreeScratch() {
+            if (p) cudaFreeAsync(p, st);
+        }
+    } free_scratch{fscratch, st};
     if (pl.engine == ENG_C2R) {
         auto shuf = [&] { return launch_col(pl.shuf.p, COL_C2R_SHUF, pl.eb, st, pl.shuf.smem); };
         if (pl.has_rot && (s = run(PK_ROT, rot_bytes, rot)) != IPT_OK) return s;  // Eq. 23

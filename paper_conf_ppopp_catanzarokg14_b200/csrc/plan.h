@@ -62,7 +62,15 @@ struct RowParams {
                       // 1: gather from the row in L2 into private shared memory
                       // (IPT_ROW_CLUSTER_MODE)
     FastDiv fd_seg;
+    // Fused rotation (c > 1, c <= kMaxFuseC; row_rot_kernel): the column rotation of the
+    // engine (C2R pre-rotation Eq. 23 / R2C post-rotation Eq. 36) folded into this pass.
+    int32_t fuse;
+    int32_t segp;            // C2R staircase: shared bytes per source segment (b elements)
+    FastDiv fd_cps;          // segp / 16 (16-byte chunks per segment)
+    unsigned int *flags;     // per-row "read" flags (M * batch, zeroed per call)
+    const char *wrap;        // C2R: copy of rows 0..c-2 of every matrix (batch x (c-1) rows)
 };
+constexpr int kMaxFuseC = 32;
 
 struct ColParams {
     char *base;
@@ -119,6 +127,12 @@ unsigned int *group_counters(cudaStream_t st, int n);
 size_t row_smem_bytes(int64_t N, int eb);
 int row_block_threads();
 cudaError_t launch_row(const RowParams &p, int dir, int eb, cudaStream_t st);
+// Fused rotation + row shuffle (p.fuse): shared bytes of one row buffer -- R2C: the row
+// (as row_smem_bytes); C2R: c staircase segments of segp bytes + the c-entry pad table.
+__host__ __device__ inline size_t row_fused_smem_bytes(const RowParams &p, int eb, int dir) {
+    if (dir == ROW_R2C) return (static_cast<size_t>(p.N) * eb + 31) & ~size_t(15);
+    return static_cast<size_t>(p.c) * static_cast<size_t>(p.segp) + ((static_cast<size_t>(p.c) * 4 + 15) & ~size_t(15));
+}
 // Cluster row pass: p.cl_K CTAs per row, each staging cl_seg elements in shared memory,
 // gathering through distributed shared memory (row_shuffle.cu).
 size_t row_cluster_smem(int32_t seg, int eb);

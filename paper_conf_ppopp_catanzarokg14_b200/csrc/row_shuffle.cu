@@ -210,6 +210,164 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_shuffle_kernel(RowParams P
     }
 }
 
+// ---- Fused rotation + row shuffle (c > 1, c <= kMaxFuseC) --------------------------------
+// The engine's column rotation moves column j by rho_j = floor(j/b) in [0, c) rows; for
+// small c it folds into the row pass, saving a whole read + write of the matrix.
+//  * C2R (Eq. 23 then Eq. 31):  out[i][p] = V_i[d'^{-1}_i(p)],
+//        V_i[l] = A[(i + floor(l/b)) mod M][l]  -- the pre-rotated row i,
+//    staged as a "staircase": segment rho (source columns [rho b, rho b + b)) comes from row
+//    i + rho; rows i + rho >= M come from `wrap`, a copy of rows 0..c-2 taken before the
+//    pass.  Each segment sits in its own 16-byte-aligned region at the source's own
+//    misalignment, so the interior moves with 16-byte cp.async; padl[rho] maps a source
+//    index l to its shared-memory byte (padl[floor(l/b)] + l eb).
+//  * R2C (Eq. 24 then Eq. 36):  out[(i + floor(p/b)) mod M][p] = A[i][d'_i(p)]:
+//    row i is staged whole and its gathered output block rho is written into row i + rho.
+// In place: flags[row] is set (release) once the row's CTA has read everything it needs.
+//  C2R: row i is written after rows i-1 .. i-c+1 (each read a block of row i) are flagged;
+//  R2C: CTA i writes into rows i+1 .. i+c-1 after they are flagged (read by their CTAs).
+// No deadlock with a co-resident grid of > c CTAs: every CTA flags its current row before
+// it waits, and a waited-for row is either some CTA's current row (flagged) or that CTA's
+// later row, which it reaches because its own current row only waits on flagged rows
+// (by induction on the chain, whose rows decrease by at least grid - c per hop).
+template <int EB>
+__device__ __forceinline__ void stage_stair(const RowParams &P, const char *mbase, const char *wrapbase, int32_t i,
+                                            uint32_t sbase, int32_t *padl) {
+    const int32_t Lb = P.b * EB;
+    const int32_t segp = P.segp;
+    const int32_t cps = segp >> 4;
+    const int32_t total = P.c * cps;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    for (int32_t f = threadIdx.x; f < total; f += blockDim.x) {
+        const int32_t rho = static_cast<int32_t>(fdiv(static_cast<uint32_t>(f), P.fd_cps));
+        const int32_t k = f - rho * cps;
+        const int32_t y = i + rho;
+        const char *S = (y < P.M ? mbase + y * pitch : wrapbase + (y - P.M) * pitch) + static_cast<int64_t>(rho) * Lb;
+        const int32_t so = static_cast<int32_t>(reinterpret_cast<uintptr_t>(S) & 15);
+        const uint32_t seg_s = sbase + rho * segp;
+        if (k == 0) padl[rho] = rho * segp + so - rho * Lb;
+        const int32_t lo = 16 * k - so;  // segment byte at the start of this 16-byte chunk
+        if (lo >= Lb || lo + 16 <= 0) continue;
+        if (lo >= 0 && lo + 16 <= Lb) {
+            cp_async<16>(seg_s + 16 * k, S + lo);
+        } else {
+#pragma unroll
+            for (int e = 0; e < 16 / EB; ++e) {
+                const int32_t q = lo + e * EB;
+                if (q >= 0 && q < Lb) cp_async<EB>(seg_s + so + q, S + q);
+            }
+        }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+template <int EB, int DIR>
+__device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, const unsigned char *buf,
+                                               const int32_t *padl, int32_t i) {
+    using T = typename Word<EB>::T;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    const int32_t seg = ((P.N + nwarps - 1) / nwarps + 31) & ~31;
+    const int32_t p_begin = warp * seg, p_end = min(P.N, p_begin + seg);
+    const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
+    const int32_t Mi = P.M - i;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    int32_t p = p_begin + lane;
+    if (p >= p_end) return;
+    if (DIR == ROW_C2R) {
+        T *out = reinterpret_cast<T *>(mbase + static_cast<int64_t>(i) * pitch);
+        C2RWalk<true> w(P, im, p);
+#pragma unroll 4
+        for (; p < p_end; p += 32) {
+            out[p] = *reinterpret_cast<const T *>(buf + padl[w.l] + w.src(P, Mi) * EB);
+            w.next(P);
+        }
+    } else {
+        const T *src = reinterpret_cast<const T *>(buf);
+        R2CWalk<true> w(P, im, p);
+#pragma unroll 4
+        for (; p < p_end; p += 32) {
+            int32_t r = i + w.l;
+            r -= r >= P.M ? P.M : 0;
+            *reinterpret_cast<T *>(mbase + r * pitch + static_cast<int64_t>(p) * EB) = src[w.src(P, Mi)];
+            w.next(P);
+        }
+    }
+}
+
+template <int EB, int DIR, int NBUF>
+__global__ void __launch_bounds__(kRowThreadsMax) row_rot_kernel(RowParams P) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int64_t rows_total = static_cast<int64_t>(P.M) * P.batch;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    const uint32_t bufbytes = static_cast<uint32_t>(row_fused_smem_bytes(P, EB, DIR));
+    const uint32_t padoff = static_cast<uint32_t>(P.c) * static_cast<uint32_t>(P.segp);  // C2R pad table
+    const uint32_t sbase = smem_u32(smem);
+    const int64_t wrap_stride = static_cast<int64_t>(P.c - 1) * pitch;
+
+    int64_t mat = blockIdx.x / P.M;
+    int32_t i = static_cast<int32_t>(blockIdx.x - mat * P.M);
+    const int32_t step_i = static_cast<int32_t>(gridDim.x % P.M);
+    const int64_t step_m = gridDim.x / P.M;
+    auto stage = [&](int64_t mm, int32_t ii, int b) {
+        char *mb = P.base + mm * P.mat_stride_bytes;
+        if (DIR == ROW_C2R)
+            stage_stair<EB>(P, mb, P.wrap + mm * wrap_stride, ii, sbase + b * bufbytes,
+                            reinterpret_cast<int32_t *>(smem + b * bufbytes + padoff));
+        else
+            stage_row<EB>(mb + ii * pitch, P.N * EB, sbase + b * bufbytes);
+    };
+    if (NBUF == 2 && blockIdx.x < rows_total) stage(mat, i, 0);
+    int buf = 0;
+    for (int64_t r = blockIdx.x; r < rows_total; r += gridDim.x) {
+        char *mbase = P.base + mat * P.mat_stride_bytes;
+        int32_t ni = i + step_i;
+        int64_t nmat = mat + step_m;
+        if (ni >= P.M) {
+            ni -= P.M;
+            ++nmat;
+        }
+        if (NBUF == 2) {
+            if (r + gridDim.x < rows_total) {
+                stage(nmat, ni, buf ^ 1);
+                asm volatile("cp.async.wait_group 1;" ::: "memory");
+            } else {
+                asm volatile("cp.async.wait_group 0;" ::: "memory");
+            }
+        } else {
+            stage(mat, i, 0);
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+        }
+        __syncthreads();  // row r's reads are complete
+        unsigned int *fl = P.flags + mat * P.M;
+        if (threadIdx.x == 0) {
+            asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(fl + i), "r"(1u) : "memory");
+        } else if (threadIdx.x < P.c) {
+            int32_t y = DIR == ROW_C2R ? i - static_cast<int32_t>(threadIdx.x) : i + static_cast<int32_t>(threadIdx.x);
+            if (y >= P.M) y -= P.M;
+            if (y >= 0) {
+                unsigned int v;
+                while (true) {
+                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(fl + y) : "memory");
+                    if (v) break;
+                    __nanosleep(64);
+                }
+            }
+        }
+        __syncthreads();  // every row this one overwrites has been read
+
+        const unsigned char *b = smem + buf * bufbytes;
+        if (DIR == ROW_C2R) {
+            gather_row_rot<EB, DIR>(P, mbase, b, reinterpret_cast<const int32_t *>(b + padoff), i);
+        } else {
+            gather_row_rot<EB, DIR>(P, mbase, b + (reinterpret_cast<uintptr_t>(mbase + i * pitch) & 15), nullptr, i);
+        }
+        __syncthreads();  // this buffer is refilled two rows later
+
+        if (NBUF == 2) buf ^= 1;
+        i = ni;
+        mat = nmat;
+    }
+}
+
 // ---- Cluster row pass (rows longer than one CTA's shared memory) -----
 // A cluster of K CTAs owns one row at a time.  CTA k stages row elements
 // [k seg, (k+1) seg) in its shared memory; after a cluster barrier every CTA gathers its
@@ -478,8 +636,27 @@ cudaError_t launch_row_t(const RowParams &P, cudaStream_t st) {
     return cudaGetLastError();
 }
 
+template <int EB, int DIR, int NBUF>
+cudaError_t launch_row_rot_t(const RowParams &P, cudaStream_t st) {
+    const size_t smem = NBUF * row_fused_smem_bytes(P, EB, DIR);
+    const int threads = row_threads(P.N, EB);
+    auto kern = row_rot_kernel<EB, DIR, NBUF>;
+    cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
+    if (e != cudaSuccess) return e;
+    const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), threads, smem);
+    if (resident <= P.c) return cudaErrorInvalidConfiguration;  // the flag waits need > c co-resident CTAs
+    const int64_t rows = static_cast<int64_t>(P.M) * P.batch;
+    int64_t grid = resident;
+    if (grid > rows) grid = rows;
+    kern<<<static_cast<unsigned>(grid), threads, smem, st>>>(P);
+    return cudaGetLastError();
+}
+
 template <int EB, int DIR>
 cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
+    if (P.fuse)
+        return 2 * row_fused_smem_bytes(P, EB, DIR) <= 112 * 1024 ? launch_row_rot_t<EB, DIR, 2>(P, st)
+                                                                   : launch_row_rot_t<EB, DIR, 1>(P, st);
     return row_nbuf(P.N, EB) == 2 ? launch_row_t<EB, DIR, 2>(P, st) : launch_row_t<EB, DIR, 1>(P, st);
 }
 

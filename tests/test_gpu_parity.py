@@ -4,6 +4,7 @@ Tolerance is zero: the transpose moves opaque words (north_star: "bit-exact agai
 oracle for every element type, including floats").  Inputs are random bit patterns from
 workloads.py (NaN payloads, -0.0 and subnormals included when viewed as floats).
 """
+import math
 import os
 import random
 
@@ -93,16 +94,68 @@ def run_packed(shapes, eb, op, layout, engine, seed):
     assert dev_bytes(buf) == np.ascontiguousarray(host).tobytes()
 
 
+class env_var:
+    def __init__(self, name, value):
+        self.name, self.value = name, value
+
+    def __enter__(self):
+        self.old = os.environ.get(self.name)
+        os.environ[self.name] = self.value
+
+    def __exit__(self, *a):
+        if self.old is None:
+            os.environ.pop(self.name, None)
+        else:
+            os.environ[self.name] = self.old
+
+
+@pytest.mark.parametrize("fuse", ["1", "0"])
 @pytest.mark.parametrize("engine", [None, "c2r", "r2c"])
-def test_bruteforce_all_shapes_to_64_fp32(engine):
+def test_bruteforce_all_shapes_to_64_fp32(engine, fuse):
+    """fuse=1: gcd <= 32 takes the fused rotation + row pass; fuse=0: the separate
+    column-rotation pass for every gcd > 1."""
     shapes = workloads.small_shapes(64)
-    run_packed(shapes, 4, ipt.c2r, "row", engine, seed=11)
+    with env_var("IPT_FUSE_ROT", fuse):
+        run_packed(shapes, 4, ipt.c2r, "row", engine, seed=11)
 
 
+@pytest.mark.parametrize("fuse", ["1", "0"])
 @pytest.mark.parametrize("eb", [8, 16])
 @pytest.mark.parametrize("engine", ["c2r", "r2c"])
-def test_bruteforce_shapes_to_40_wide_elements(eb, engine):
-    run_packed(workloads.small_shapes(40), eb, ipt.c2r, "row", engine, seed=eb)
+def test_bruteforce_shapes_to_40_wide_elements(eb, engine, fuse):
+    with env_var("IPT_FUSE_ROT", fuse):
+        run_packed(workloads.small_shapes(40), eb, ipt.c2r, "row", engine, seed=eb)
+
+
+@pytest.mark.parametrize("shape", [(1200, 1816), (1816, 1200), (4096, 3000), (96, 40), (640, 32 * 33)])
+@pytest.mark.parametrize("engine", ["c2r", "r2c"])
+def test_fused_rotation_each_pass(shape, engine):
+    """gcd in 2..32: the rotation folds into the row pass (Eq. 23 + Eq. 31 for
+    C2R, Eq. 24 + Eq. 36 for R2C).  Each of the two passes is compared with the oracle's
+    gather-form snapshot after the same steps."""
+    m, n = shape
+    eb = 4
+    assert 1 < math.gcd(m, n) <= 32
+    host = workloads.random_words(m * n, eb, seed=m ^ n)
+    with forced_engine(engine):
+        x = to_dev(host)
+        ipt.c2r(x, m, n, elem_bytes=eb)
+        assert dev_bytes(x) == oracle.transpose(host, m, n).tobytes()
+        ipt.r2c(x, m, n, elem_bytes=eb)
+        assert dev_bytes(x) == host.tobytes()
+        if engine == "c2r":       # C2R(M=m, N=n): [r_j + d'^{-1}], p_j o q
+            _, snaps = oracle.c2r_gather_forms(host, m, n, snapshots=True)
+            expect = [snaps[1], snaps[3]]
+        else:                     # R2C(M=n, N=m): q^{-1} o p^{-1}, [d' + r^{-1}]
+            _, snaps = oracle.r2c_gather_forms(host, n, m, snapshots=True)
+            expect = [snaps[1], snaps[3]]
+        for k, e in enumerate(expect, start=1):
+            x = to_dev(host)
+            with debug_passes(k):
+                ipt.c2r(x, m, n, elem_bytes=eb)
+            assert dev_bytes(x) == e.tobytes(), f"pass {k}"
+        info = ipt.plan_info(m, n, eb)
+        assert info["launches"] == 2, info
 
 
 @pytest.mark.parametrize("layout", ["row", "col"])
