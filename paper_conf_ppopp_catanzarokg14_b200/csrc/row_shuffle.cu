@@ -315,7 +315,34 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_rot_kernel(RowParams P) {
         else
             stage_row<EB>(mb + ii * pitch, P.N * EB, sbase + b * bufbytes);
     };
-    if (NBUF == 2 && blockIdx.x < rows_total) stage(mat, i, 0);
+    auto set_flag = [&](int64_t r) {  // row r's reads are complete (after a __syncthreads)
+        if (threadIdx.x == 0)
+            asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(P.flags + r), "r"(1u) : "memory");
+    };
+    auto wait_deps = [&](int64_t mm, int32_t ii) {  // every row that row ii overwrites has been read
+        if (threadIdx.x >= 1 && threadIdx.x < P.c) {
+            int32_t y = DIR == ROW_C2R ? ii - static_cast<int32_t>(threadIdx.x) : ii + static_cast<int32_t>(threadIdx.x);
+            if (y >= P.M) y -= P.M;
+            if (y >= 0) {
+                const unsigned int *f = P.flags + mm * P.M + y;
+                unsigned int v;
+                while (true) {
+                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
+                    if (v) break;
+                    __nanosleep(32);
+                }
+            }
+        }
+        __syncthreads();
+    };
+    // NBUF = 2: row r + grid is staged while row r is gathered, and flagged as soon as the
+    // gather of row r is done -- a full row ahead of the moment its neighbours wait for it.
+    if (blockIdx.x < rows_total) {
+        stage(mat, i, 0);
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
+        __syncthreads();
+        set_flag(blockIdx.x);
+    }
     int buf = 0;
     for (int64_t r = blockIdx.x; r < rows_total; r += gridDim.x) {
         char *mbase = P.base + mat * P.mat_stride_bytes;
@@ -325,34 +352,9 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_rot_kernel(RowParams P) {
             ni -= P.M;
             ++nmat;
         }
-        if (NBUF == 2) {
-            if (r + gridDim.x < rows_total) {
-                stage(nmat, ni, buf ^ 1);
-                asm volatile("cp.async.wait_group 1;" ::: "memory");
-            } else {
-                asm volatile("cp.async.wait_group 0;" ::: "memory");
-            }
-        } else {
-            stage(mat, i, 0);
-            asm volatile("cp.async.wait_group 0;" ::: "memory");
-        }
-        __syncthreads();  // row r's reads are complete
-        unsigned int *fl = P.flags + mat * P.M;
-        if (threadIdx.x == 0) {
-            asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(fl + i), "r"(1u) : "memory");
-        } else if (threadIdx.x < P.c) {
-            int32_t y = DIR == ROW_C2R ? i - static_cast<int32_t>(threadIdx.x) : i + static_cast<int32_t>(threadIdx.x);
-            if (y >= P.M) y -= P.M;
-            if (y >= 0) {
-                unsigned int v;
-                while (true) {
-                    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(fl + y) : "memory");
-                    if (v) break;
-                    __nanosleep(64);
-                }
-            }
-        }
-        __syncthreads();  // every row this one overwrites has been read
+        const bool more = r + gridDim.x < rows_total;
+        if (NBUF == 2 && more) stage(nmat, ni, buf ^ 1);
+        wait_deps(mat, i);
 
         const unsigned char *b = smem + buf * bufbytes;
         if (DIR == ROW_C2R) {
@@ -360,8 +362,13 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_rot_kernel(RowParams P) {
         } else {
             gather_row_rot<EB, DIR>(P, mbase, b + (reinterpret_cast<uintptr_t>(mbase + i * pitch) & 15), nullptr, i);
         }
-        __syncthreads();  // this buffer is refilled two rows later
-
+        __syncthreads();  // this buffer is free again
+        if (more) {
+            if (NBUF == 1) stage(nmat, ni, 0);
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
+            __syncthreads();
+            set_flag(r + gridDim.x);
+        }
         if (NBUF == 2) buf ^= 1;
         i = ni;
         mat = nmat;
