@@ -17,9 +17,9 @@ bench)
 ncu)
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$TAG.csv \
       python bench.py --profile-only --no-cpu-baseline > gpurun_out/ncu_launch_$TAG.log 2>&1
-  timeout 900 ncu --set full --clock-control none --import-source on -k regex:col_tile -s 20 -c 2 -f -o gpurun_out/col_$TAG \
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:col_ -s 20 -c 2 -f -o gpurun_out/col_$TAG \
       python bench.py --profile-only --no-cpu-baseline > gpurun_out/ncu_col_$TAG.log 2>&1
-  timeout 900 ncu --set full --clock-control none --import-source on -k regex:row_shuffle -s 20 -c 1 -f -o gpurun_out/row_$TAG \
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:row_ -s 20 -c 1 -f -o gpurun_out/row_$TAG \
       python bench.py --profile-only --no-cpu-baseline > gpurun_out/ncu_row_$TAG.log 2>&1 ;;
 esac
 done
