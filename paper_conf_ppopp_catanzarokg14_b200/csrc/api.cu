@@ -124,7 +124,8 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
 
 ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe) {
     int twb = env_int("IPT_TILE_BYTES", 128);
-    if (twb != 32 && twb != 64 && twb != 128) twb = 128;
+    if (twb != 32 && twb != 64 && twb != 128 && twb != 256) twb = 128;
+    if (twb == 256 && pl.eb < 8) twb = 128;  // lane = tile column: W = twb / eb <= 32
     if (twb < pl.eb) twb = pl.eb;
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
     const int nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
@@ -250,12 +251,17 @@ ipt_status_t make_skinny_plan(const DevInfo &dev, int64_t x, int64_t y, int eb, 
     }
     sc.mode = pl.skinny_dir == ROW_R2C ? COL_R2C_SHUF : COL_C2R_SHUF;
     sc.remap = pl.skinny_dir == ROW_R2C ? 1 : -1;
+    // c > 1: fold the rotation into the rolling locations (no rotation pass), unless
+    // IPT_FUSE_ROT=0.
+    const bool fold = pl.c > 1 && env_int("IPT_FUSE_ROT", 1) != 0;
+    sc.fold = fold ? 1 : 0;
     pl.onchip = skinny_col_smem(n, sc.C, eb);
     if (pl.onchip > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
-    if (pl.c > 1) {
+    if (pl.c > 1 && !fold) {
         pl.srot = sc;
         pl.srot.mode = COL_ROT;
         pl.srot.remap = 0;
+        pl.srot.fold = 0;
         pl.srot.rot_sign = pl.skinny_dir == ROW_C2R ? 1 : -1;  // Eq. 23 before / Eq. 36 after
         pl.has_rot = true;
     }
@@ -272,6 +278,8 @@ ipt_status_t make_skinny_plan(const DevInfo &dev, int64_t x, int64_t y, int eb, 
     r.T = T;
     r.Tp = T + (32 % n == 0 ? 32 / n : 1);  // residue classes spread over the banks
     r.fd_n = make_fastdiv(static_cast<uint32_t>(n));
+    r.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
+    r.fold = fold ? 1 : 0;
     const size_t rs = skinny_row_smem(n, r.Tp, eb);
     if (rs > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
     if (rs > pl.onchip) pl.onchip = rs;
@@ -518,9 +526,10 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
         // tmp row of N elements.  R2C: column pass writing row r to location r+1 (row n-1 to
         // tmp); row i then reads location i+1 (tmp for n-1) and writes location i.  C2R:
         // row i reads location i, writes location i-1 (tmp for 0); the column pass reads the
-        // shifted rows back.  A destination row is never its own source row.
+        // shifted rows back.  A destination row is never its own source row.  With c > 1 the
+        // rotation is folded in: block rho = floor(j/b) of every rolled location is shifted
+        // by another rho rows (plan.h, SkinnyRowParams).
         const int n = static_cast<int>(pl.M);
-        const int64_t pitch = pl.N * pl.eb;
         const double rowb = 2.0 * static_cast<double>(pl.N) * pl.eb;
         char *tmp = nullptr;
         cudaMemPool_t pool = scratch_pool();
@@ -539,13 +548,8 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
             auto row_l = [&](int i) {
                 SkinnyRowParams rp = pl.srow;
                 rp.i = i;
-                if (pl.skinny_dir == ROW_R2C) {
-                    rp.src = i == n - 1 ? tmp : A + (i + 1) * pitch;
-                    rp.dst = A + i * pitch;
-                } else {
-                    rp.src = A + i * pitch;
-                    rp.dst = i == 0 ? tmp : A + (i - 1) * pitch;
-                }
+                rp.A = A;
+                rp.tmp = tmp;
                 return [rp, &pl, st] { return launch_skinny_row(rp, pl.skinny_dir, pl.eb, st); };
             };
             if (pl.skinny_dir == ROW_R2C) {
@@ -782,7 +786,8 @@ uint64_t ipt_launch_count(void) { return g_launches.load(); }
 ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes, int tile_bytes, int cluster,
                                  int barrier, void *stream) {
     if (!valid_eb(elem_bytes) || M < 1 || N < 1 || M >= (1 << 29) || N >= (1 << 29) || cluster < 1 ||
-        (tile_bytes != 32 && tile_bytes != 64 && tile_bytes != 128) || tile_bytes < elem_bytes ||
+        (tile_bytes != 32 && tile_bytes != 64 && tile_bytes != 128 && tile_bytes != 256) ||
+        (tile_bytes == 256 && elem_bytes < 8) || tile_bytes < elem_bytes ||
         !ptr || reinterpret_cast<uintptr_t>(ptr) % elem_bytes)
         return IPT_ERR_INVALID_ARGUMENT;
     const DevInfo dev = device_info();

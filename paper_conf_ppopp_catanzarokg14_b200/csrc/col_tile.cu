@@ -571,6 +571,9 @@ void *col_kernel_e(int mode, int twb, bool pipe) {
         case 32: return col_kernel_w<EB, 32>(mode, pipe);
         case 64: return col_kernel_w<EB, 64>(mode, pipe);
         case 128: return col_kernel_w<EB, 128>(mode, pipe);
+        case 256:
+            if constexpr (EB >= 8) return col_kernel_w<EB, 256>(mode, pipe);  // lane = column needs W <= 32
+            return nullptr;
         default: return nullptr;
     }
 }

@@ -96,15 +96,26 @@ struct ColParams {
     int32_t nbuf;
 };
 
+// Skinny engine storage: "location" L in [0, n] is row L of the n x N view, location n is
+// the one-row buffer tmp.  Logical row r's column block rho = floor(j / b) lives at
+// the location below between the passes (rolling rows with the rotation folded in, DESIGN.md
+// §"Skinny engine"):
+//   R2C (AoS -> SoA): column pass writes (r, rho) to  r == n-1 ? n : (r + 1 + rho) mod n;
+//                     row shuffle i reads there and writes (i, rho) to (i + rho) mod n.
+//   C2R (SoA -> AoS): row shuffle i reads (i, rho) at (i + rho) mod n (the pre-rotation)
+//                     and writes it to                i == 0 ? n : (i - 1 + rho) mod n,
+//                     where the column pass reads it back.
+// Without rotation (c = 1) rho is always 0: the plain rolling scheme.
 struct SkinnyRowParams {
-    const char *src;    // source row (N elements)
-    char *dst;          // destination row (N elements), never the source
+    char *A;            // the n x N engine view
+    char *tmp;          // location n
     int64_t N;          // row length (the long dimension, count)
     int32_t n, c, b;    // engine rows M = n (fields), c = gcd(n, N), b = N / c
     int64_t ainv;       // a^{-1} mod b, a = n / c
     int32_t i;          // row index
     int32_t T, Tp;      // run length per residue class; shared-memory row pitch (odd)
-    FastDiv fd_n;
+    int32_t fold;       // 1: the rotation (Eq. 23 / Eq. 36) is folded into the locations
+    FastDiv fd_n, fd_b;
 };
 
 // Kernel attribute / occupancy caches (api.cu): set the dynamic shared-memory limit (and
@@ -156,6 +167,7 @@ struct SkinnyColParams {
     int32_t n, c, b;
     int32_t mode;       // COL_ROT, COL_C2R_SHUF, COL_R2C_SHUF
     int32_t remap;      // +1: output row o stored at o+1 (n-1 in tmp); -1: input row s at s-1 (0 in tmp)
+    int32_t fold;       // with remap: + floor(j / b) (mod n) on the rolled side (folded rotation)
     int32_t rot_sign;
     int32_t C;          // columns per CTA (multiple of 32)
     int32_t q[32], qinv[32];  // Eq. 33 / Eq. 34 on the n rows

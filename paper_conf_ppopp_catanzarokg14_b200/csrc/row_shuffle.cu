@@ -42,9 +42,6 @@ __device__ __forceinline__ void cp_async(uint32_t dst, const void *src) {
         asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" :: "r"(dst), "l"(src), "n"(B) : "memory");
     }
 }
-__device__ __forceinline__ void cp_async_wait_all() {
-    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
-}
 
 // C2R walk: src = lb + (hc + f2) mod b with lb = l*b, hc = a^{-1} floor(q/c) mod b.
 template <bool TAIL>

@@ -48,24 +48,63 @@ __device__ __forceinline__ void dpinv(const SkinnyRowParams &P, int64_t x, int64
 
 // Shared memory: run tables [n] x (l*b, h) as int64, then the window re-sorted by residue
 // class: element t of class r at row r, column t (row pitch Tp elements).
-template <int EB, int DIR>
+// Storage locations of row shuffle i's source and destination blocks (plan.h).
+__device__ __forceinline__ int32_t sk_src_loc(const SkinnyRowParams &P, int DIR, int32_t rho) {
+    int32_t L;
+    if (DIR == ROW_R2C) {
+        if (P.i == P.n - 1) return P.n;
+        L = P.i + 1 + rho;
+    } else {
+        L = P.i + rho;
+    }
+    return L >= P.n ? L - P.n : L;
+}
+__device__ __forceinline__ int32_t sk_dst_loc(const SkinnyRowParams &P, int DIR, int32_t rho) {
+    int32_t L;
+    if (DIR == ROW_R2C) {
+        L = P.i + rho;
+    } else {
+        if (P.i == 0) return P.n;
+        L = P.i - 1 + rho;
+    }
+    return L >= P.n ? L - P.n : L;
+}
+
+template <int EB, int DIR, bool FOLD>
 __global__ void __launch_bounds__(kSkThreads) skinny_row_kernel(SkinnyRowParams P) {
     using T = typename Word<EB>::T;
     extern __shared__ __align__(16) unsigned char smem[];
     int64_t *run_lb = reinterpret_cast<int64_t *>(smem);
     int64_t *run_h = run_lb + 32;
-    T *buf = reinterpret_cast<T *>(smem + 512);
+    T **src_b = reinterpret_cast<T **>(smem + 512);  // [c] source row base per block
+    T **dst_b = src_b + 32;                          // [c] destination row base per block
+    T *buf = reinterpret_cast<T *>(smem + 1024);
     const uint32_t sbuf = static_cast<uint32_t>(__cvta_generic_to_shared(buf));
     const int n = P.n;
     const int64_t L = static_cast<int64_t>(n) * P.T;
     const int lt = 31 - __clz(P.T);  // T is a power of two
-    const T *src = reinterpret_cast<const T *>(P.src);
-    T *dst = reinterpret_cast<T *>(P.dst);
+    const int nblk = FOLD ? P.c : 1;
+    if (threadIdx.x < nblk) {
+        const int32_t ls = sk_src_loc(P, DIR, FOLD ? threadIdx.x : 0);
+        const int32_t ld = sk_dst_loc(P, DIR, FOLD ? threadIdx.x : 0);
+        src_b[threadIdx.x] = reinterpret_cast<T *>(ls == n ? P.tmp : P.A + ls * P.N * EB);
+        dst_b[threadIdx.x] = reinterpret_cast<T *>(ld == n ? P.tmp : P.A + ld * P.N * EB);
+    }
+    // Without folding one base serves the whole row (kept in registers).
+    const int32_t l0 = sk_src_loc(P, DIR, 0), d0 = sk_dst_loc(P, DIR, 0);
+    T *const src0 = reinterpret_cast<T *>(l0 == n ? P.tmp : P.A + l0 * P.N * EB);
+    T *const dst0 = reinterpret_cast<T *>(d0 == n ? P.tmp : P.A + d0 * P.N * EB);
+    auto srcb = [&](int64_t x) -> T * {
+        return FOLD ? src_b[fdiv(static_cast<uint32_t>(x), P.fd_b)] : src0;
+    };
+    auto dstb = [&](int64_t x) -> T * {
+        return FOLD ? dst_b[fdiv(static_cast<uint32_t>(x), P.fd_b)] : dst0;
+    };
 
     for (int64_t win = blockIdx.x; win * L < P.N; win += gridDim.x) {
         const int64_t x0 = win * L;
         const int32_t len = static_cast<int32_t>(min(L, P.N - x0));
-        // run starts: class r of the window starts at x0 + r
+        // run starts: class r of the window starts at x0 + r; run r lies in block lb / b
         if (threadIdx.x < n) {
             int64_t lb, h;
             dpinv(P, x0 + threadIdx.x, lb, h);
@@ -73,11 +112,13 @@ __global__ void __launch_bounds__(kSkThreads) skinny_row_kernel(SkinnyRowParams 
             run_h[threadIdx.x] = h;
         }
         if (DIR == ROW_R2C) {
+            __syncthreads();  // block bases
             // stage the source window, sorted by residue class
             for (int32_t v = threadIdx.x; v < len; v += blockDim.x) {
                 const uint32_t t = fdiv(static_cast<uint32_t>(v), P.fd_n);
                 const uint32_t r = static_cast<uint32_t>(v) - t * n;
-                cp_async_e<EB>(sbuf + (r * P.Tp + t) * EB, src + x0 + v);
+                const int64_t x = x0 + v;
+                cp_async_e<EB>(sbuf + (r * P.Tp + t) * EB, srcb(x) + x);
             }
             asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
             __syncthreads();
@@ -87,17 +128,18 @@ __global__ void __launch_bounds__(kSkThreads) skinny_row_kernel(SkinnyRowParams 
                 if (t * n + r >= len) continue;
                 int64_t h = run_h[r] + t;
                 if (h >= P.b) h -= P.b;
-                dst[run_lb[r] + h] = buf[r * P.Tp + t];
+                const int64_t y = run_lb[r] + h;
+                dstb(run_lb[r])[y] = buf[r * P.Tp + t];
             }
         } else {
-            __syncthreads();  // run tables
+            __syncthreads();  // run tables, block bases
             // gather the n source runs of the output window
             for (int32_t e = threadIdx.x; e < n * P.T; e += blockDim.x) {
                 const int32_t r = e >> lt, t = e & (P.T - 1);
                 if (t * n + r >= len) continue;
                 int64_t h = run_h[r] + t;
                 if (h >= P.b) h -= P.b;
-                cp_async_e<EB>(sbuf + (r * P.Tp + t) * EB, src + run_lb[r] + h);
+                cp_async_e<EB>(sbuf + (r * P.Tp + t) * EB, srcb(run_lb[r]) + run_lb[r] + h);
             }
             asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
             __syncthreads();
@@ -105,7 +147,8 @@ __global__ void __launch_bounds__(kSkThreads) skinny_row_kernel(SkinnyRowParams 
             for (int32_t v = threadIdx.x; v < len; v += blockDim.x) {
                 const uint32_t t = fdiv(static_cast<uint32_t>(v), P.fd_n);
                 const uint32_t r = static_cast<uint32_t>(v) - t * n;
-                dst[x0 + v] = buf[r * P.Tp + t];
+                const int64_t x = x0 + v;
+                dstb(x)[x] = buf[r * P.Tp + t];
             }
         }
         __syncthreads();  // tables and buffer are reused by the next window
@@ -119,7 +162,7 @@ __global__ void __launch_bounds__(kSkThreads) skinny_row_kernel(SkinnyRowParams 
 //   R2C_SHUF  sigma_j(i) = q^{-1}((i - j) mod n)                  (Eqs. 34-35)
 // with the rolling-row remaps of the skinny engine on the input or output side.  A CTA
 // reads its columns completely before writing them and CTAs own disjoint columns.
-template <int EB, int MODE>
+template <int EB, int MODE, bool FOLD>
 __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams P) {
     using T = typename Word<EB>::T;
     extern __shared__ __align__(16) unsigned char smem[];
@@ -134,10 +177,18 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
     for (int64_t j0 = static_cast<int64_t>(blockIdx.x) * C; j0 < P.N; j0 += static_cast<int64_t>(gridDim.x) * C) {
         const int32_t cols = static_cast<int32_t>(min(static_cast<int64_t>(C), P.N - j0));
         // stage: row s of the view (remap -1: stored at s-1, row 0 in tmp)
+        // (folded: + floor(j/b) mod n on the rolled side; rho is constant within a block)
         for (int s = 0; s < n; ++s) {
-            const T *row = P.remap < 0 ? (s == 0 ? tmp : A + (s - 1) * pitch) : A + s * pitch;
-            for (int32_t x = threadIdx.x; x < cols; x += blockDim.x)
+            const T *row0 = P.remap < 0 ? (s == 0 ? tmp : A + (s - 1) * pitch) : A + s * pitch;
+            for (int32_t x = threadIdx.x; x < cols; x += blockDim.x) {
+                const T *row = row0;
+                if (FOLD && P.remap < 0 && s > 0) {
+                    int32_t L = s - 1 + static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + x), P.fd_b));
+                    L -= L >= n ? n : 0;
+                    row = A + L * pitch;
+                }
                 cp_async_e<EB>(sbuf + (s * C + x) * EB, row + j0 + x);
+            }
         }
         asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
         __syncthreads();
@@ -145,6 +196,7 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
             const int64_t j = j0 + x;  // < N < 2^31
             const uint32_t jm = fmod_(static_cast<uint32_t>(j), P.fd_n);
             int32_t shift = 0;
+            const int32_t rho = FOLD ? static_cast<int32_t>(fdiv(static_cast<uint32_t>(j), P.fd_b)) : 0;
             if (MODE == COL_ROT) {  // floor(j/b) < c <= n
                 const int32_t qd = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j), P.fd_b));
                 shift = P.rot_sign > 0 ? qd : (qd == 0 ? 0 : n - qd);
@@ -163,6 +215,11 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
                     s = qinv_s[u];
                 }
                 T *orow = P.remap > 0 ? (i == n - 1 ? tmp : A + (i + 1) * pitch) : A + i * pitch;
+                if (FOLD && P.remap > 0 && i < n - 1) {
+                    int32_t L = i + 1 + rho;
+                    L -= L >= n ? n : 0;
+                    orow = A + L * pitch;
+                }
                 orow[j] = buf[s * C + x];
             }
         }
@@ -173,7 +230,7 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
 template <int EB, int MODE>
 cudaError_t launch_col_t(const SkinnyColParams &P, cudaStream_t st) {
     const size_t smem = skinny_col_smem(P.n, P.C, EB);
-    auto kern = skinny_col_kernel<EB, MODE>;
+    auto kern = P.fold ? skinny_col_kernel<EB, MODE, true> : skinny_col_kernel<EB, MODE, false>;
     cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
     if (e != cudaSuccess) return e;
     const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), kSkThreads, smem);
@@ -197,7 +254,7 @@ cudaError_t launch_col_e(const SkinnyColParams &P, cudaStream_t st) {
 template <int EB, int DIR>
 cudaError_t launch_t(const SkinnyRowParams &P, cudaStream_t st) {
     const size_t smem = skinny_row_smem(P.n, P.Tp, EB);
-    auto kern = skinny_row_kernel<EB, DIR>;
+    auto kern = P.fold ? skinny_row_kernel<EB, DIR, true> : skinny_row_kernel<EB, DIR, false>;
     cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
     if (e != cudaSuccess) return e;
     const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), kSkThreads, smem);
@@ -211,7 +268,7 @@ cudaError_t launch_t(const SkinnyRowParams &P, cudaStream_t st) {
 
 }  // namespace
 
-size_t skinny_row_smem(int n, int Tp, int eb) { return 512 + static_cast<size_t>(n) * Tp * eb; }
+size_t skinny_row_smem(int n, int Tp, int eb) { return 1024 + static_cast<size_t>(n) * Tp * eb; }
 size_t skinny_col_smem(int n, int C, int eb) { return 128 + static_cast<size_t>(n) * C * eb; }
 
 cudaError_t launch_skinny_col(const SkinnyColParams &P, int eb, cudaStream_t st) {

@@ -38,10 +38,24 @@ class skinny_min:
         os.environ.pop("IPT_SKINNY_MIN", None)
 
 
+class fuse_rot:
+    def __init__(self, v):
+        self.v = v
+
+    def __enter__(self):
+        os.environ["IPT_FUSE_ROT"] = self.v
+
+    def __exit__(self, *a):
+        os.environ.pop("IPT_FUSE_ROT", None)
+
+
+@pytest.mark.parametrize("fold", ["1", "0"])
 @pytest.mark.parametrize("count", [4099, 4096, 6000])
 @pytest.mark.parametrize("eb", [4, 8])
-def test_all_field_counts_both_directions(count, eb):
-    with skinny_min(1000):
+def test_all_field_counts_both_directions(count, eb, fold):
+    """fold=1: for gcd(n, count) > 1 the rotation is folded into the rolling-row locations
+    (no rotation pass); fold=0: the separate rotation pass."""
+    with skinny_min(1000), fuse_rot(fold):
         for n in range(2, 33):
             assert ipt.plan_info(count, n, eb)["engine"] == "skinny"
             host = workloads.random_words(count * n, eb, seed=count + n)
