@@ -280,6 +280,7 @@ ipt_status_t make_skinny_plan(const DevInfo &dev, int64_t x, int64_t y, int eb, 
     r.fd_n = make_fastdiv(static_cast<uint32_t>(n));
     r.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
     r.fold = fold ? 1 : 0;
+    r.reg = eb == 4 && env_int("IPT_SKINNY_REG", 1) != 0 ? 1 : 0;
     const size_t rs = skinny_row_smem(n, r.Tp, eb);
     if (rs > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
     if (rs > pl.onchip) pl.onchip = rs;
@@ -419,7 +420,7 @@ struct PlanKeyHash {
 std::string tunables_key() {
     std::string s;
     for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
-                          "IPT_SKINNY_MIN", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
+                          "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
         s += v ? v : "-";

@@ -115,6 +115,7 @@ struct SkinnyRowParams {
     int32_t i;          // row index
     int32_t T, Tp;      // run length per residue class; shared-memory row pitch (odd)
     int32_t fold;       // 1: the rotation (Eq. 23 / Eq. 36) is folded into the locations
+    int32_t reg;        // 1: in-register SIMD transposition kernel (skinny_reg.cu; 4-byte fields)
     FastDiv fd_n, fd_b;
 };
 
@@ -180,5 +181,6 @@ cudaError_t launch_skinny_col(const SkinnyColParams &p, int eb, cudaStream_t st)
 // source windows; dir ROW_C2R -- dst[j] = src[d'^{-1}_i(j)] driven by output windows.
 size_t skinny_row_smem(int n, int T, int eb);
 cudaError_t launch_skinny_row(const SkinnyRowParams &p, int dir, int eb, cudaStream_t st);
+cudaError_t launch_skinny_row_reg(const SkinnyRowParams &p, int dir, cudaStream_t st);
 
 }  // namespace ipt

@@ -281,6 +281,7 @@ cudaError_t launch_skinny_col(const SkinnyColParams &P, int eb, cudaStream_t st)
 }
 
 cudaError_t launch_skinny_row(const SkinnyRowParams &P, int dir, int eb, cudaStream_t st) {
+    if (P.reg && eb == 4) return launch_skinny_row_reg(P, dir, st);
     switch (eb * 2 + dir) {
         case 4 * 2 + ROW_C2R: return launch_t<4, ROW_C2R>(P, st);
         case 4 * 2 + ROW_R2C: return launch_t<4, ROW_R2C>(P, st);
