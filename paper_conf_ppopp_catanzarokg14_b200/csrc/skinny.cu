@@ -178,16 +178,30 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
         const int32_t cols = static_cast<int32_t>(min(static_cast<int64_t>(C), P.N - j0));
         // stage: row s of the view (remap -1: stored at s-1, row 0 in tmp)
         // (folded: + floor(j/b) mod n on the rolled side; rho is constant within a block)
+        auto row_of = [&](int s, int64_t j) -> const T * {
+            if (P.remap >= 0) return A + s * pitch;
+            if (s == 0) return tmp;
+            int32_t L = s - 1;
+            if (FOLD) {
+                L += static_cast<int32_t>(fdiv(static_cast<uint32_t>(j), P.fd_b));
+                L -= L >= n ? n : 0;
+            }
+            return A + L * pitch;
+        };
         for (int s = 0; s < n; ++s) {
-            const T *row0 = P.remap < 0 ? (s == 0 ? tmp : A + (s - 1) * pitch) : A + s * pitch;
-            for (int32_t x = threadIdx.x; x < cols; x += blockDim.x) {
-                const T *row = row0;
-                if (FOLD && P.remap < 0 && s > 0) {
-                    int32_t L = s - 1 + static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + x), P.fd_b));
-                    L -= L >= n ? n : 0;
-                    row = A + L * pitch;
-                }
-                cp_async_e<EB>(sbuf + (s * C + x) * EB, row + j0 + x);
+            const T *row0 = row_of(s, j0);
+            const bool one_base = !FOLD || row_of(s, j0 + cols - 1) == row0;
+            const T *seg = row0 + j0;
+            if (one_base && (reinterpret_cast<uintptr_t>(seg) & 15) == 0 && (cols * EB) % 16 == 0) {
+                // 16-byte chunks (cp.async.cg): 4-byte cp.async runs at ~75 % of this rate
+                const int nch = cols * EB / 16;
+                for (int ch = threadIdx.x; ch < nch; ch += blockDim.x)
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
+                                 :: "r"(sbuf + s * C * EB + ch * 16), "l"(reinterpret_cast<const char *>(seg) + ch * 16)
+                                 : "memory");
+            } else {
+                for (int32_t x = threadIdx.x; x < cols; x += blockDim.x)
+                    cp_async_e<EB>(sbuf + (s * C + x) * EB, (one_base ? row0 : row_of(s, j0 + x)) + j0 + x);
             }
         }
         asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
