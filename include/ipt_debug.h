@@ -8,7 +8,7 @@
  * drops it.  It isolates the
  * cost of the tile access pattern (strided tile_bytes-wide sub-rows) and of the cluster
  * synchronisation from the index arithmetic of the permutations (column
- * kernel roofline).  tile_bytes in {32, 64, 128}; 1 <= cluster <= co-resident CTAs.  Asynchronous on
+ * kernel roofline).  tile_bytes in {128, 256, 512}; 1 <= cluster <= co-resident CTAs.  Asynchronous on
  * `stream`; the buffer content is unchanged on success.
  */
 #ifndef IPT_DEBUG_H_

@@ -124,9 +124,8 @@ ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp)
 
 ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe) {
     int twb = env_int("IPT_TILE_BYTES", 128);
-    if (twb != 32 && twb != 64 && twb != 128 && twb != 256) twb = 128;
-    if (twb == 256 && pl.eb < 8) twb = 128;  // lane = tile column: W = twb / eb <= 32
-    if (twb < pl.eb) twb = pl.eb;
+    if (twb != 128 && twb != 256 && twb != 512) twb = 128;
+    if (twb > 32 * pl.eb) twb = 32 * pl.eb;  // lane = tile column: W <= 32
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
     const int nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
     const int64_t target = env_int("IPT_COL_SMEM", 46 * 1024);
@@ -141,7 +140,8 @@ ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &c
         const size_t smem = col_smem_bytes(B, W, pl.eb, nbuf);
         if (smem > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
         const int64_t G = (pl.M + B - 1) / B;
-        const int resident = col_resident_ctas(mode, pl.eb, twb, smem, pipe);
+        const int threads = pipe ? col_block_threads() : static_cast<int>(env_int("IPT_COL_THREADS", 256));
+        const int resident = col_resident_ctas(mode, pl.eb, twb, smem, pipe, threads);
         if (resident < 1) return IPT_ERR_UNSUPPORTED;
         if (G > resident) {  // a whole group must be co-resident
             B = (pl.M + resident - 1) / resident;
@@ -168,6 +168,7 @@ ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &c
         p.resident = resident;
         p.pipe = pipe ? 1 : 0;
         p.nbuf = nbuf;
+        p.threads = threads;
         p.rot_sign = 1;
         p.wide_a = pl.a >= 65536 ? 1 : 0;
         cp.smem = smem;
@@ -419,7 +420,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -787,8 +788,7 @@ uint64_t ipt_launch_count(void) { return g_launches.load(); }
 ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes, int tile_bytes, int cluster,
                                  int barrier, void *stream) {
     if (!valid_eb(elem_bytes) || M < 1 || N < 1 || M >= (1 << 29) || N >= (1 << 29) || cluster < 1 ||
-        (tile_bytes != 32 && tile_bytes != 64 && tile_bytes != 128 && tile_bytes != 256) ||
-        (tile_bytes == 256 && elem_bytes < 8) || tile_bytes < elem_bytes ||
+        (tile_bytes != 128 && tile_bytes != 256 && tile_bytes != 512) || tile_bytes > 32 * elem_bytes ||
         !ptr || reinterpret_cast<uintptr_t>(ptr) % elem_bytes)
         return IPT_ERR_INVALID_ARGUMENT;
     const DevInfo dev = device_info();
@@ -815,7 +815,8 @@ ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes
     p.nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
     const size_t smem = col_smem_bytes(p.B, p.W, elem_bytes, p.nbuf);
     if (smem > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
-    p.resident = col_resident_ctas(COL_COPY, elem_bytes, tile_bytes, smem, pipe);
+    p.threads = pipe ? col_block_threads() : static_cast<int>(env_int("IPT_COL_THREADS", 256));
+    p.resident = col_resident_ctas(COL_COPY, elem_bytes, tile_bytes, smem, pipe, p.threads);
     if (p.resident < p.G) return IPT_ERR_UNSUPPORTED;
     finish_col(p, 1);
     return check(launch_col(p, COL_COPY, elem_bytes, static_cast<cudaStream_t>(stream), smem));

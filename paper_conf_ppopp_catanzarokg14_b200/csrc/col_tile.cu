@@ -87,42 +87,34 @@ __device__ __forceinline__ void group_barrier(unsigned int *ctr, unsigned int ta
 
 // Shared-memory layout of one unit buffer:
 //   [orow B*4 | srow nslots*4 | sbase nslots*4 | rows]
-// rows: element path (eb = 8, 16) -- B output rows of TWB bytes; hull path (eb = 4) --
-// nslots input rows ("slots") of HS = TWB + 16 bytes, each the 16-byte-aligned hull of the
-// tile row, sbase[t] = shared address of slot t's first tile element.
+// rows: nslots input rows ("slots") of HS = TWB + 16 bytes, each the 16-byte-aligned hull
+// of its tile row; sbase[t] = shared address of slot t's first tile element.
 __host__ __device__ inline size_t al16(size_t x) { return (x + 15) & ~size_t(15); }
 struct SmemLayout {
     size_t srow, sbase, rows, total;
 };
-__host__ __device__ constexpr bool hull_path(int eb) { return eb == 4; }
+__host__ __device__ constexpr int hull_pitch(int twb) { return twb + 16; }
 __host__ __device__ inline SmemLayout smem_layout(int64_t B, int W, int twb, int eb) {
+    (void)eb;
     const size_t nslots = static_cast<size_t>(B) + W - 1;
     SmemLayout L;
     size_t o = al16(static_cast<size_t>(B) * 4);
     L.srow = o;
     o += al16(nslots * 4);
     L.sbase = o;
-    if (hull_path(eb)) o += al16(nslots * 4);
+    o += al16(nslots * 4);
     L.rows = o;
-    L.total = o + (hull_path(eb) ? nslots * static_cast<size_t>(twb + 16) : static_cast<size_t>(B) * twb);
+    L.total = o + nslots * static_cast<size_t>(hull_pitch(twb));
     return L;
-}
-
-template <int EB>
-__device__ __forceinline__ void cp_async_elem(uint32_t dst, const void *src) {
-    if constexpr (EB == 16)
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(src) : "memory");
-    else
-        asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" :: "r"(dst), "l"(src), "n"(EB) : "memory");
 }
 
 // One column-tile work unit: band r of tile tt (of all matrices).
 struct Unit {
-    char *colp;        // this lane's column in row 0 of the matrix
+    char *tilep;        // column j0 of row 0 of the matrix
     int32_t r0, nrows;  // output band [r0, r0 + nrows)
-    int32_t j0m;        // j0 mod M
+    int32_t j0, j0m;    // first column of the tile, j0 mod M
     int32_t rowbase;    // first input row (ROT / C2R)
-    int32_t dw;         // slot t, lane column w feeds band row k = t - dw
+    int32_t lo_q, hi_q; // ROT: floor(j/b) of the tile's first / last column
     int32_t nslots;     // input rows read: band + halo
     int32_t wt;         // columns of this tile (W, or fewer at the ragged right edge)
     bool skip;          // ROT tile made only of columns rotating by 0
@@ -137,32 +129,37 @@ __device__ __forceinline__ Unit unit_make(const ColParams &P, uint32_t tt, int32
     const uint32_t mat = fdiv(tt, P.fd_nt);
     const int32_t tile = static_cast<int32_t>(tt - mat * static_cast<uint32_t>(P.ntiles));
     const int32_t j0 = tile * W;
+    U.j0 = j0;
     U.wt = min(W, P.N - j0);
     U.j0m = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j0), P.fd_M));
     U.skip = false;
-    const int w = (threadIdx.x & 31) % W;
+    U.lo_q = U.hi_q = 0;
     int32_t ext = W - 1, base_off = 0;
-    U.dw = 0;
     if (MODE == COL_ROT) {
-        const int32_t lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
-        const int32_t hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + U.wt - 1), P.fd_b));
-        ext = hi_q - lo_q;
-        base_off = P.rot_sign > 0 ? lo_q : -hi_q;  // smallest rotation amount in the tile
+        U.lo_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
+        U.hi_q = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + U.wt - 1), P.fd_b));
+        ext = U.hi_q - U.lo_q;
+        base_off = P.rot_sign > 0 ? U.lo_q : -U.hi_q;  // smallest rotation amount in the tile
         // Columns j < b rotate by 0 (Eq. 23): a tile made only of them is left alone.
-        U.skip = hi_q == 0;
-        const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + min(w, U.wt - 1)), P.fd_b));
-        U.dw = P.rot_sign > 0 ? qw - lo_q : hi_q - qw;  // rho_w - min rho
+        U.skip = U.hi_q == 0;
     } else if (MODE == COL_COPY) {
         ext = 0;
-    } else if (MODE == COL_C2R_SHUF) {
-        U.dw = w;
-    } else {
-        U.dw = W - 1 - w;
     }
     U.nslots = U.nrows > 0 ? U.nrows + ext : 0;
     U.rowbase = MODE == COL_ROT ? mod_M(U.r0 + base_off, P.kshM, P.fd_M) : U.r0;
-    U.colp = P.base + static_cast<int64_t>(mat) * P.mat_stride_bytes + static_cast<int64_t>(j0 + w) * EB;
+    U.tilep = P.base + static_cast<int64_t>(mat) * P.mat_stride_bytes + static_cast<int64_t>(j0) * EB;
     return U;
+}
+
+// Slot offset of tile column w: output band row k, column w is slot k + dw(w).
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ int32_t dw_of(const ColParams &P, const Unit &U, int32_t w) {
+    constexpr int W = TWB / EB;
+    if (MODE == COL_C2R_SHUF) return w;
+    if (MODE == COL_R2C_SHUF) return W - 1 - w;
+    if (MODE == COL_COPY) return 0;
+    const int32_t qw = static_cast<int32_t>(fdiv(static_cast<uint32_t>(U.j0 + w), P.fd_b));
+    return P.rot_sign > 0 ? qw - U.lo_q : U.hi_q - qw;  // rho_w - min rho
 }
 
 // Scattered row indices of a unit, computed by the whole CTA into shared memory:
@@ -182,93 +179,79 @@ __device__ __forceinline__ void unit_prepass(const ColParams &P, const Unit &U, 
     }
 }
 
-// Load.  Element path (eb = 8, 16): element-granular cp.async from each tile row straight
-// into the element's OUTPUT row of the band in shared memory (row k = t - dw); lane = tile
-// column w, a load instruction copies whole tile rows, the bank of every element is its
-// column (conflict-free).  Hull path (eb = 4; 4-byte cp.async runs at ~75% of the
-// 16-byte rate on B200, tools/tile_probe.cu): every input row ("slot" t) is staged as the
-// 16-byte-aligned hull of its tile row (TWB/16 + 1 chunks, the last one only when the
-// row is misaligned) and sbase[t] records where its first element landed; the skew is
-// applied when the store phase reads shared memory.  Not committed here.
+// Chunks of 16 bytes per tile row: the 16-byte-aligned hull of a TWB-byte row segment
+// (one more chunk when the segment is misaligned; 16-byte elements never are).
+template <int EB, int TWB> constexpr int chunks_per_row() { return TWB / 16 + (EB < 16 ? 1 : 0); }
+
+// Load: every input row ("slot" t) is staged as the 16-byte-aligned hull of its tile row
+// with 16-byte cp.async (element-granular cp.async runs at ~70% of the 16-byte rate on
+// B200 for 4-byte elements: tools/tile_probe.cu), the last chunk with a src-size so no
+// byte past the tile's row end is read; sbase[t] records where its first element landed.
+// The skew / rotation / permutation is applied when the store phase reads shared memory.
+// Not committed here.
 template <int EB, int MODE, int TWB>
 __device__ __forceinline__ void unit_load(const ColParams &P, const Unit &U, const int32_t *srow, uint32_t *sbase,
                                           uint32_t rows_s, int nthr) {
-    constexpr int W = TWB / EB;
     if (U.skip) return;
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
-    if constexpr (hull_path(EB)) {
-        constexpr int CPR = TWB / 16 + 1;  // chunks per slot
-        constexpr int HS = TWB + 16;       // slot pitch in shared memory
-        const char *tilep = U.colp - ((threadIdx.x & 31) % W) * EB;  // column j0 of row 0
-        const int32_t nchunk = U.nslots * CPR;
-        const int32_t wbytes = U.wt * EB;
-        for (int32_t f = threadIdx.x; f < nchunk; f += nthr) {
-            const int32_t t = f / CPR, c = f - t * CPR;
-            int32_t g;
-            if (MODE == COL_R2C_SHUF) {
-                g = srow[t];
-            } else {
-                g = U.rowbase + t;
-                while (g >= P.M) g -= P.M;  // t < nslots <= M + W
-            }
-            const char *rp = tilep + static_cast<int64_t>(g) * pitch;
-            const uint32_t off = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(rp)) & 15u;
-            const char *cp = rp - off + c * 16;
-            const uint32_t dst = rows_s + t * HS + c * 16;
-            if (c == 0) sbase[t] = dst + off;
-            const int32_t rem = static_cast<int32_t>(off) + wbytes - c * 16;  // bytes of the hull from cp on
-            if (rem >= 16) {
-                asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(cp) : "memory");
-            } else if (rem > 0) {  // row end: read only the tile's bytes (never past the buffer)
-                asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(dst), "l"(cp), "r"(rem) : "memory");
-            }
+    constexpr int CPR = chunks_per_row<EB, TWB>();
+    constexpr int HS = hull_pitch(TWB);
+    const int32_t nchunk = U.nslots * CPR;
+    const int32_t wbytes = U.wt * EB;
+    for (int32_t f = threadIdx.x; f < nchunk; f += nthr) {
+        const int32_t t = f / CPR, c = f - t * CPR;
+        int32_t g;
+        if (MODE == COL_R2C_SHUF) {
+            g = srow[t];
+        } else {
+            g = U.rowbase + t;
+            while (g >= P.M) g -= P.M;  // t < nslots <= M + W
         }
-        return;
-    }
-    constexpr int RPW = 32 / W;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = nthr >> 5;
-    const int w = lane % W, sub = lane / W;
-    if (w >= U.wt) return;
-    const int32_t step = nwarps * RPW;  // slots between a lane's consecutive rows
-    const int32_t dw = U.dw;
-    // This lane's slots t with 0 <= k = t - dw < nrows (the others are halo elements no
-    // band row needs): a branch-free walk with incremental shared and global addresses.
-    int32_t t = warp * RPW + sub;
-    if (t < dw) t += ((dw - t + step - 1) / step) * step;
-    const int32_t tend = dw + U.nrows;
-    uint32_t sa = rows_s + w * EB + (t - dw) * TWB;
-    const uint32_t sa_inc = step * TWB;
-    const char *colp = U.colp;
-    if (MODE == COL_R2C_SHUF) {
-#pragma unroll 4
-        for (; t < tend; t += step, sa += sa_inc) cp_async_elem<EB>(sa, colp + srow[t] * pitch);
-    } else if (step <= P.M) {
-        int32_t s = mod_M(U.rowbase + t, P.kshM, P.fd_M);
-        const char *g = colp + s * pitch;
-        const int64_t g_inc = step * pitch, g_wrap = static_cast<int64_t>(P.M) * pitch;
-#pragma unroll 4
-        for (; t < tend; t += step, sa += sa_inc) {
-            cp_async_elem<EB>(sa, g);
-            s += step;
-            g += g_inc;
-            if (s >= P.M) {
-                s -= P.M;
-                g -= g_wrap;
-            }
+        const char *rp = U.tilep + static_cast<int64_t>(g) * pitch;
+        const uint32_t off = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(rp)) & 15u;
+        const char *cp = rp - off + c * 16;
+        const uint32_t dst = rows_s + t * HS + c * 16;
+        if (c == 0) sbase[t] = dst + off;
+        const int32_t rem = static_cast<int32_t>(off) + wbytes - c * 16;  // bytes of the hull from cp on
+        if (rem >= 16) {
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(cp) : "memory");
+        } else if (rem > 0) {  // row end: read only the tile's bytes (never past the buffer)
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(dst), "l"(cp), "r"(rem) : "memory");
         }
-    } else {  // tiny M: fewer rows than one step
-        for (; t < tend; t += step, sa += sa_inc)
-            cp_async_elem<EB>(sa, colp + mod_M(U.rowbase + t, P.kshM, P.fd_M) * pitch);
     }
 }
 
-// Store: whole output rows (a warp instruction writes TWB... contiguous bytes of one or
-// more rows).  Hull path: output row k, column w is slot k + dw(w), read at sbase + w eb.
+template <int EB>
+__device__ __forceinline__ void lds_elem(uint32_t *v, uint32_t a) {
+    if constexpr (EB == 4) {
+        asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v[0]) : "r"(a));
+    } else if constexpr (EB == 8) {
+        asm volatile("ld.shared.v2.b32 {%0,%1}, [%2];" : "=r"(v[0]), "=r"(v[1]) : "r"(a));
+    } else {
+        asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]) : "r"(a));
+    }
+}
+template <int EB>
+__device__ __forceinline__ void stg_elem(char *p, const uint32_t *v) {
+    if constexpr (EB == 4) {
+        *reinterpret_cast<uint32_t *>(p) = v[0];
+    } else if constexpr (EB == 8) {
+        *reinterpret_cast<uint2 *>(p) = make_uint2(v[0], v[1]);
+    } else {
+        *reinterpret_cast<uint4 *>(p) = make_uint4(v[0], v[1], v[2], v[3]);
+    }
+}
+
+// Store: lane = tile column w (W <= 32; a warp instruction writes 32 / W whole tile rows,
+// TWB contiguous bytes each).  Output band row k goes to global row o(k) (orow[k] for
+// C2R, r0 + k otherwise); its element w is slot k + dw(w), read at sbase[slot] + w eb --
+// for C2R / R2C the lanes of a row read a diagonal of the slot array, conflict-free in
+// the banks (slot pitch TWB + 16 bytes).
 template <int EB, int MODE, int TWB>
 __device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, const int32_t *orow,
-                                           const uint32_t *sbase, const unsigned char *rows, int nthr) {
-    using T = typename Word<EB>::T;
+                                           const uint32_t *sbase, int nthr) {
     constexpr int W = TWB / EB;
+    static_assert(W <= 32, "lane = tile column");
     constexpr int RPW = 32 / W;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = nthr >> 5;
     const int w = lane % W, sub = lane / W;
@@ -276,48 +259,24 @@ __device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, co
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
     const int32_t step = nwarps * RPW;
     int32_t k = warp * RPW + sub;
-    char *colp = U.colp;
-    if constexpr (hull_path(EB)) {
-        const uint32_t *sb = sbase + U.dw;
-        const uint32_t wo = w * EB;
-        if (MODE == COL_C2R_SHUF) {
-#pragma unroll 4
-            for (; k < U.nrows; k += step) {
-                T v;
-                const uint32_t a = sb[k] + wo;
-                if constexpr (EB == 4)
-                    asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a));
-                else
-                    asm volatile("ld.shared.b64 %0, [%1];" : "=l"(v) : "r"(a));
-                *reinterpret_cast<T *>(colp + static_cast<int64_t>(orow[k]) * pitch) = v;
-            }
-        } else {
-            char *g = colp + static_cast<int64_t>(U.r0 + k) * pitch;
-            const int64_t g_inc = step * pitch;
-#pragma unroll 4
-            for (; k < U.nrows; k += step, g += g_inc) {
-                T v;
-                const uint32_t a = sb[k] + wo;
-                if constexpr (EB == 4)
-                    asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a));
-                else
-                    asm volatile("ld.shared.b64 %0, [%1];" : "=l"(v) : "r"(a));
-                *reinterpret_cast<T *>(g) = v;
-            }
-        }
-        return;
-    }
-    const unsigned char *sr = rows + w * EB;
+    char *colp = U.tilep + w * EB;
+    const uint32_t *sb = sbase + dw_of<EB, MODE, TWB>(P, U, w);
+    const uint32_t wo = w * EB;
+    uint32_t v[4];
     if (MODE == COL_C2R_SHUF) {
 #pragma unroll 4
-        for (; k < U.nrows; k += step)
-            *reinterpret_cast<T *>(colp + static_cast<int64_t>(orow[k]) * pitch) =
-                *reinterpret_cast<const T *>(sr + k * TWB);
+        for (; k < U.nrows; k += step) {
+            lds_elem<EB>(v, sb[k] + wo);
+            stg_elem<EB>(colp + static_cast<int64_t>(orow[k]) * pitch, v);
+        }
     } else {
         char *g = colp + static_cast<int64_t>(U.r0 + k) * pitch;
         const int64_t g_inc = step * pitch;
 #pragma unroll 4
-        for (; k < U.nrows; k += step, g += g_inc) *reinterpret_cast<T *>(g) = *reinterpret_cast<const T *>(sr + k * TWB);
+        for (; k < U.nrows; k += step, g += g_inc) {
+            lds_elem<EB>(v, sb[k] + wo);
+            stg_elem<EB>(g, v);
+        }
     }
 }
 
@@ -337,7 +296,6 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     int32_t *orow = reinterpret_cast<int32_t *>(smem);
     int32_t *srow = reinterpret_cast<int32_t *>(smem + L.srow);
     uint32_t *sbase = reinterpret_cast<uint32_t *>(smem + L.sbase);
-    unsigned char *rows = smem + L.rows;
     const Unit U = unit_make<EB, MODE, TWB>(P, tt, r);
     const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
     if (U.skip) {  // group-uniform; still arrive, later tiles sharing the counter count it
@@ -346,7 +304,7 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     }
     unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
     if (MODE == COL_R2C_SHUF) __syncthreads();
-    unit_load<EB, MODE, TWB>(P, U, srow, sbase, static_cast<uint32_t>(__cvta_generic_to_shared(rows)), blockDim.x);
+    unit_load<EB, MODE, TWB>(P, U, srow, sbase, static_cast<uint32_t>(__cvta_generic_to_shared(smem + L.rows)), blockDim.x);
     asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
     // In-place hazard barrier: the whole tile has been read before anyone writes it.
     // Counter slot tt mod kCtrSlots, monotone over the tiles that share it.
@@ -357,7 +315,7 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     } else {
         __syncthreads();
     }
-    unit_store<EB, MODE, TWB>(P, U, orow, sbase, rows, blockDim.x);
+    unit_store<EB, MODE, TWB>(P, U, orow, sbase, blockDim.x);
 }
 
 template <int EB, int MODE, int TWB>
@@ -515,7 +473,7 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
         const Unit Us = unit_make<EB, MODE, TWB>(P, stt, static_cast<int32_t>(st - stt * P.G));
         unsigned char *sbuf = smem + sb * bufsz;
         unit_store<EB, MODE, TWB>(P, Us, reinterpret_cast<const int32_t *>(sbuf),
-                                  reinterpret_cast<const uint32_t *>(sbuf + L.sbase), sbuf + L.rows, nwt);
+                                  reinterpret_cast<const uint32_t *>(sbuf + L.sbase), nwt);
     };
     int b = 0, k = 0;    // buffer / round of unit i
     int sb = 0, sk = 0;  // buffer / round of the oldest unit not yet stored
@@ -567,12 +525,14 @@ void *col_kernel_w(int mode, bool pipe) {
 
 template <int EB>
 void *col_kernel_e(int mode, int twb, bool pipe) {
+    // lane = tile column: W = twb / EB <= 32
     switch (twb) {
-        case 32: return col_kernel_w<EB, 32>(mode, pipe);
-        case 64: return col_kernel_w<EB, 64>(mode, pipe);
         case 128: return col_kernel_w<EB, 128>(mode, pipe);
         case 256:
-            if constexpr (EB >= 8) return col_kernel_w<EB, 256>(mode, pipe);  // lane = column needs W <= 32
+            if constexpr (EB >= 8) return col_kernel_w<EB, 256>(mode, pipe);
+            return nullptr;
+        case 512:
+            if constexpr (EB >= 16) return col_kernel_w<EB, 512>(mode, pipe);
             return nullptr;
         default: return nullptr;
     }
@@ -599,13 +559,13 @@ int64_t col_max_band(int64_t W) { return (int64_t(1) << 24) - W; }
 
 int col_block_threads() { return kColThreads; }
 
-int col_resident_ctas(int mode, int eb, int twb, size_t smem, bool pipe) {
+int col_resident_ctas(int mode, int eb, int twb, size_t smem, bool pipe, int threads) {
     void *kern = col_kernel(mode, eb, twb, pipe);
     if (!kern || ensure_kernel_attrs(kern, smem, false) != cudaSuccess) {
         cudaGetLastError();
         return 0;
     }
-    return cached_resident_blocks(kern, kColThreads, smem);
+    return cached_resident_blocks(kern, threads, smem);
 }
 
 cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, size_t smem) {
@@ -625,7 +585,8 @@ cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, s
     e = cudaMemsetAsync(P.ctr, 0, sizeof(unsigned int) * (kTicketSlot + 1), st);
     if (e != cudaSuccess) return e;
     void *args[] = {&P};
-    return cudaLaunchKernel(kern, dim3(static_cast<unsigned>(grid)), dim3(kColThreads), args, smem, st);
+    const int threads = P.threads > 0 ? P.threads : kColThreads;
+    return cudaLaunchKernel(kern, dim3(static_cast<unsigned>(grid)), dim3(threads), args, smem, st);
 }
 
 }  // namespace ipt

@@ -94,6 +94,7 @@ struct ColParams {
     int32_t tpc;        // tiles per CTA when G == 1 (each tile fits one CTA)
     int32_t pipe;       // 1: persistent pipelined kernel (col_pipe_kernel) with nbuf unit buffers
     int32_t nbuf;
+    int32_t threads;    // threads per CTA (col_block_threads() for the pipelined kernel)
 };
 
 // Skinny engine storage: "location" L in [0, n] is row L of the n x N view, location n is
@@ -157,7 +158,7 @@ int col_max_bufs();
 int col_block_threads();
 int64_t col_max_band(int64_t W);  // largest band a CTA may be given
 cudaError_t launch_col(const ColParams &p, int mode, int eb, cudaStream_t st, size_t smem);
-int col_resident_ctas(int mode, int eb, int twb, size_t smem, bool pipe);
+int col_resident_ctas(int mode, int eb, int twb, size_t smem, bool pipe, int threads);
 
 // Skinny column pass (skinny.cu): all n rows x C consecutive columns per CTA, the column
 // permutation sigma_j among the n rows applied in shared memory.

@@ -281,3 +281,20 @@ def test_config5b_batch_shape_sampled():
         _sampled_check(got[k * m * n:(k + 1) * m * n], host[k * m * n:(k + 1) * m * n], m, n, 5000, rng)
     ipt.r2c_batched(x, batch, m * n, m, n, elem_bytes=4)
     assert torch.equal(x, to_dev(host))
+
+
+@pytest.mark.parametrize("twb", ["128", "256", "512"])
+@pytest.mark.parametrize("pipe", ["1", "0"])
+def test_column_tile_widths_and_small_bands(twb, pipe):
+    """Column-pass geometry: every tile width (16-byte hull staging, 16-byte vector stores
+    with element stores at misaligned segment ends), tiny bands (IPT_COL_SMEM small, so a
+    tile spans many group members and the halo crosses band edges), pipelined and one-unit
+    kernels; the separate rotation pass (IPT_FUSE_ROT=0) exercises COL_ROT.  Shapes mix
+    coprime / gcd > 1, ragged right tiles and rows misaligned to 16 bytes."""
+    shapes = [(1200, 1800), (97, 1031), (1031, 97), (513, 700), (700, 513), (64, 4096), (2003, 129),
+              (384, 640), (129, 2003)]
+    with env_var("IPT_TILE_BYTES", twb), env_var("IPT_COL_PIPE", pipe), env_var("IPT_COL_SMEM", "12000"), \
+            env_var("IPT_FUSE_ROT", "0"):
+        for eb in (4, 8, 16):
+            for engine in ("c2r", "r2c"):
+                run_packed(shapes, eb, ipt.c2r, "row", engine, seed=int(twb) + eb)
