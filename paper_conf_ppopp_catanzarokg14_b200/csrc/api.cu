@@ -96,6 +96,7 @@ struct Plan {
     int nlaunch = 0;
     size_t onchip = 0;
     size_t scratch = 0;         // global scratch bytes (skinny: one row of the long dimension)
+    size_t side_bytes = 0;      // lagged layouts: side block bytes per matrix (M x (D TWB + pad))
     SkinnyRowParams srow{};     // skinny engine long-row shuffle
     SkinnyColParams scol{}, srot{};  // skinny engine column passes (shuffle, rotation)
     int skinny_dir = 0;         // ROW_R2C (P_{count,n}, AoS -> SoA) or ROW_C2R (P_{n,count})
@@ -114,18 +115,17 @@ int ilog2(int v) {
 // the co-resident CTAs, the band grows (up to the opt-in shared-memory maximum).
 ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe);
 
-// IPT_COL_PIPE (default 1): the persistent pipelined kernel with IPT_COL_NBUF unit buffers
+// IPT_COL_PIPE (default 0; 1 selects it): the persistent pipelined kernel with IPT_COL_NBUF unit buffers
 // per CTA (the shared-memory target is per buffer); tiles whose group would not fit the
 // co-resident CTAs that way (very tall matrices, config 5a) take the one-unit kernel.
 ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp) {
-    if (env_int("IPT_COL_PIPE", 1) != 0 && plan_col_v(dev, pl, mode, cp, true) == IPT_OK) return IPT_OK;
+    if (env_int("IPT_COL_PIPE", 0) != 0 && plan_col_v(dev, pl, mode, cp, true) == IPT_OK) return IPT_OK;
     return plan_col_v(dev, pl, mode, cp, false);
 }
 
 ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe) {
     int twb = env_int("IPT_TILE_BYTES", 128);
     if (twb != 128 && twb != 256 && twb != 512) twb = 128;
-    if (twb > 32 * pl.eb) twb = 32 * pl.eb;  // lane = tile column: W <= 32
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
     const int nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
     const int64_t target = env_int("IPT_COL_SMEM", 46 * 1024);
@@ -169,6 +169,7 @@ ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &c
         p.pipe = pipe ? 1 : 0;
         p.nbuf = nbuf;
         p.threads = threads;
+        p.dbg = env_int("IPT_COL_DEBUG", 0);
         p.rot_sign = 1;
         p.wide_a = pl.a >= 65536 ? 1 : 0;
         cp.smem = smem;
@@ -220,6 +221,22 @@ cudaMemPool_t scratch_pool() {
     cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
     pools[dev] = pool;
     return pool;
+}
+
+// Lag of the shuffle pass's tile layout (col_tile.cu "In-place hazard"): D tiles, at most
+// ntiles - 1; sets the side-block geometry shared by the column and row passes.
+void set_lag(Plan &pl, int64_t D) {
+    ColParams &cq = pl.shuf.p;
+    RowParams &rp = pl.row;
+    D = std::max<int64_t>(1, std::min<int64_t>(D, cq.ntiles - 1));
+    const int64_t twb = static_cast<int64_t>(cq.W) * pl.eb;
+    cq.lagD = static_cast<int32_t>(D);
+    cq.spitch = D * twb + (pl.N * pl.eb) % 16;
+    cq.sstride = (pl.M * cq.spitch + 31) & ~int64_t(15);
+    rp.shW = static_cast<int32_t>(D * cq.W);
+    rp.spitch = cq.spitch;
+    rp.sstride = cq.sstride;
+    pl.side_bytes = static_cast<size_t>(cq.sstride);
 }
 
 // Skinny engine (§6.1): P_{x,y} with min(x, y) = n <= 32 fields
@@ -386,8 +403,33 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         }
     }
 
+    // Row groups: R consecutive rows per CTA stage while R rows stay within IPT_ROW_STAGE
+    // bytes (default 16 KiB), so that short rows still keep enough bytes in flight per SM.
+    rp.R = 1;
+    if (!use_cluster) {
+        const size_t rowbuf = rp.fuse ? row_fused_smem_bytes(rp, eb, pl.row_dir) : row_smem_bytes(pl.N, eb);
+        const int nw = row_threads(pl.N, eb) / 32;
+        const size_t target = static_cast<size_t>(env_int("IPT_ROW_STAGE", 16384));
+        while (rp.R * 2 <= nw && rp.R * 2 * rowbuf <= target) rp.R *= 2;
+        rsm = rowbuf * rp.R;
+    }
+
     ipt_status_t s = plan_col(dev, pl, engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.shuf);
     if (s != IPT_OK) return s;
+    // Lagged tile layouts (col_tile.cu "In-place hazard"; IPT_COL_LAG=0 keeps the per-tile
+    // group barrier): the shuffle pass waits only for the previous tile's group, and the
+    // row pass reads (R2C) / writes (C2R) the shifted layout with the side tile S of M x TWB
+    // bytes per matrix (O(max(m, n)) scratch).  Not with the cluster row pass.
+    if (env_int("IPT_COL_LAG", 1) != 0 && !use_cluster && pl.shuf.p.ntiles >= 2) {
+        ColParams &cq = pl.shuf.p;
+        cq.lag = engine == ENG_C2R ? LAG_C2R : LAG_R2C;
+        // D: about twice the co-resident CTAs' worth of groups between a unit and the group
+        // it waits for (IPT_COL_LAGD overrides); at most ntiles - 1.
+        int64_t D = env_int("IPT_COL_LAGD", 0);
+        if (D <= 0) D = (2 * static_cast<int64_t>(cq.resident) + cq.G - 1) / cq.G;
+        set_lag(pl, D);
+        pl.scratch += pl.side_bytes;
+    }
     pl.onchip = rsm > pl.shuf.smem ? rsm : pl.shuf.smem;
     pl.nlaunch = 2;
     if (pl.c > 1 && !rp.fuse) {
@@ -420,7 +462,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_ROW_STAGE", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -568,22 +610,32 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
         cudaFreeAsync(tmp, st);
         return s;
     }
-    // Fused rotation: per-call scratch (row flags, zeroed; C2R: the wrapped rows' copy).
+    // Per-call scratch: fused rotation -- row flags (zeroed) and, for C2R, a copy of the
+    // rows the last staircases wrap onto; lagged layouts -- the side tiles.
     char *fscratch = nullptr;
-    if (pl.row.fuse) {
-        const int64_t pitch = pl.N * pl.eb;
-        const size_t flag_bytes = (static_cast<size_t>(pl.M * batch) * 4 + 255) & ~size_t(255);
-        const size_t wrap_row_bytes = static_cast<size_t>(pl.c - 1) * pitch;
-        const size_t wrap_bytes = pl.engine == ENG_C2R ? wrap_row_bytes * batch : 0;
+    const int64_t pitch = pl.N * pl.eb;
+    const size_t flag_bytes = pl.row.fuse ? (static_cast<size_t>(pl.M * batch) * 4 + 255) & ~size_t(255) : 0;
+    const size_t wrap_row_bytes = pl.row.fuse ? static_cast<size_t>(pl.c - 1) * pitch : 0;
+    const size_t wrap_bytes = pl.engine == ENG_C2R ? (wrap_row_bytes * batch + 255) & ~size_t(255) : 0;
+    if (pl.side_bytes && batch > 1) {
+        // Batches: keep the side blocks within max(256 MiB, 1/32 of the data) -- a smaller D.
+        const double cap = std::max(256.0 * (1 << 20), full / 2.0 / 32.0);
+        const double per_tile = static_cast<double>(pl.M) * pl.shuf.p.W * pl.eb * static_cast<double>(batch);
+        const int64_t dmax = static_cast<int64_t>(cap / per_tile);
+        if (dmax < pl.shuf.p.lagD) set_lag(pl, dmax);
+    }
+    const size_t side_bytes = pl.side_bytes * static_cast<size_t>(batch);
+    if (flag_bytes + wrap_bytes + side_bytes) {
         cudaMemPool_t pool = scratch_pool();
-        if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&fscratch), flag_bytes + wrap_bytes, pool, st) !=
-                         cudaSuccess) {
+        if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&fscratch), flag_bytes + wrap_bytes + side_bytes,
+                                             pool, st) != cudaSuccess) {
             cudaGetLastError();
             return IPT_ERR_OUT_OF_MEMORY;
         }
         pl.row.flags = reinterpret_cast<unsigned int *>(fscratch);
         pl.row.wrap = fscratch + flag_bytes;
-        ipt_status_t s0 = check(cudaMemsetAsync(fscratch, 0, flag_bytes, st));
+        pl.row.side = pl.shuf.p.side = side_bytes ? fscratch + flag_bytes + wrap_bytes : nullptr;
+        ipt_status_t s0 = flag_bytes ? check(cudaMemsetAsync(fscratch, 0, flag_bytes, st)) : IPT_OK;
         if (s0 == IPT_OK && wrap_bytes)
             s0 = check(cudaMemcpy2DAsync(fscratch + flag_bytes, wrap_row_bytes, base, stride_bytes, wrap_row_bytes,
                                          batch, cudaMemcpyDeviceToDevice, st));
@@ -599,6 +651,7 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
             if (p) cudaFreeAsync(p, st);
         }
     } free_scratch{fscratch, st};
+    const int passes = budget;
     if (pl.engine == ENG_C2R) {
         auto shuf = [&] { return launch_col(pl.shuf.p, COL_C2R_SHUF, pl.eb, st, pl.shuf.smem); };
         if (pl.has_rot && (s = run(PK_ROT, rot_bytes, rot)) != IPT_OK) return s;  // Eq. 23
@@ -609,6 +662,30 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
         if ((s = run(PK_COL, full, shuf)) != IPT_OK) return s;                    // Eqs. 34-35
         if ((s = run(PK_ROW, full, row)) != IPT_OK) return s;                     // Eq. 24
         if (pl.has_rot && (s = run(PK_ROT, rot_bytes, rot)) != IPT_OK) return s;  // Eq. 36
+    }
+    // IPT_DEBUG_PASSES stopping between the row and column passes of a lagged plan: put the
+    // logical layout back (side tile -> columns [0, W), A columns [0, N - W) -> [W, N)) so
+    // the snapshot compares with the oracle's.
+    if (pl.side_bytes && passes < (1 << 30)) {
+        const int before_second = pl.engine == ENG_C2R ? (pl.has_rot ? 2 : 1) : 1;  // passes up to the lagged state
+        if (passes == before_second) {
+            const size_t W = static_cast<size_t>(pl.row.shW), sp = static_cast<size_t>(pl.row.spitch);
+            char *tmp = nullptr;
+            if (cudaMallocAsync(reinterpret_cast<void **>(&tmp), static_cast<size_t>(pitch) * pl.M, st) != cudaSuccess)
+                return IPT_ERR_OUT_OF_MEMORY;
+            for (int64_t k = 0; k < batch && s == IPT_OK; ++k) {
+                char *A = base + k * stride_bytes;
+                s = check(cudaMemcpy2DAsync(tmp + W * pl.eb, pitch, A, pitch, pitch - W * pl.eb, pl.M,
+                                            cudaMemcpyDeviceToDevice, st));
+                if (s == IPT_OK)
+                    s = check(cudaMemcpy2DAsync(tmp, pitch, side_matrix(pl.row.side, pl.row.sstride, k, A), sp,
+                                                W * pl.eb, pl.M, cudaMemcpyDeviceToDevice, st));
+                if (s == IPT_OK)
+                    s = check(cudaMemcpyAsync(A, tmp, static_cast<size_t>(pitch) * pl.M, cudaMemcpyDeviceToDevice, st));
+            }
+            cudaFreeAsync(tmp, st);
+            return s;
+        }
     }
     return IPT_OK;
 }
@@ -788,7 +865,7 @@ uint64_t ipt_launch_count(void) { return g_launches.load(); }
 ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes, int tile_bytes, int cluster,
                                  int barrier, void *stream) {
     if (!valid_eb(elem_bytes) || M < 1 || N < 1 || M >= (1 << 29) || N >= (1 << 29) || cluster < 1 ||
-        (tile_bytes != 128 && tile_bytes != 256 && tile_bytes != 512) || tile_bytes > 32 * elem_bytes ||
+        (tile_bytes != 128 && tile_bytes != 256 && tile_bytes != 512) ||
         !ptr || reinterpret_cast<uintptr_t>(ptr) % elem_bytes)
         return IPT_ERR_INVALID_ARGUMENT;
     const DevInfo dev = device_info();

@@ -70,21 +70,6 @@ __device__ __forceinline__ int32_t mod_M(int32_t v, uint32_t kshiftM, const Fast
     return static_cast<int32_t>(fmod_(static_cast<uint32_t>(v) + kshiftM, fdM));
 }
 
-// Group barrier in global memory: counter ctr counts arrivals of all tiles sharing it.
-__device__ __forceinline__ void group_barrier(unsigned int *ctr, unsigned int target) {
-    __syncthreads();  // every thread's staged data is in shared memory
-    if (threadIdx.x == 0) {
-        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
-        unsigned int v;
-        while (true) {
-            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
-            if (v >= target) break;
-            __nanosleep(128);
-        }
-    }
-    __syncthreads();
-}
-
 // Shared-memory layout of one unit buffer:
 //   [orow B*4 | srow nslots*4 | sbase nslots*4 | rows]
 // rows: nslots input rows ("slots") of HS = TWB + 16 bytes, each the 16-byte-aligned hull
@@ -110,7 +95,8 @@ __host__ __device__ inline SmemLayout smem_layout(int64_t B, int W, int twb, int
 
 // One column-tile work unit: band r of tile tt (of all matrices).
 struct Unit {
-    char *tilep;        // column j0 of row 0 of the matrix
+    char *inp, *outp;   // column j0 of row 0 of the tile's input / output location
+    int64_t in_pitch, out_pitch;  // bytes between rows there (N eb, or TWB in the side tile)
     int32_t r0, nrows;  // output band [r0, r0 + nrows)
     int32_t j0, j0m;    // first column of the tile, j0 mod M
     int32_t rowbase;    // first input row (ROT / C2R)
@@ -127,7 +113,8 @@ __device__ __forceinline__ Unit unit_make(const ColParams &P, uint32_t tt, int32
     U.r0 = r * P.B;
     U.nrows = max(0, min(P.M, U.r0 + P.B) - U.r0);
     const uint32_t mat = fdiv(tt, P.fd_nt);
-    const int32_t tile = static_cast<int32_t>(tt - mat * static_cast<uint32_t>(P.ntiles));
+    int32_t tile = static_cast<int32_t>(tt - mat * static_cast<uint32_t>(P.ntiles));
+    if (P.lag == LAG_C2R) tile = P.ntiles - 1 - tile;  // right to left
     const int32_t j0 = tile * W;
     U.j0 = j0;
     U.wt = min(W, P.N - j0);
@@ -147,7 +134,25 @@ __device__ __forceinline__ Unit unit_make(const ColParams &P, uint32_t tt, int32
     }
     U.nslots = U.nrows > 0 ? U.nrows + ext : 0;
     U.rowbase = MODE == COL_ROT ? mod_M(U.r0 + base_off, P.kshM, P.fd_M) : U.r0;
-    U.tilep = P.base + static_cast<int64_t>(mat) * P.mat_stride_bytes + static_cast<int64_t>(j0) * EB;
+    char *A = P.base + static_cast<int64_t>(mat) * P.mat_stride_bytes;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    U.inp = U.outp = A + static_cast<int64_t>(j0) * EB;
+    U.in_pitch = U.out_pitch = pitch;
+    if (P.lag != LAG_NONE) {
+        // Lagged layouts (see "In-place hazard"): tile t >= D lives D tiles to the left,
+        // tiles t < D in the side block (columns [t W, t W + W) of its rows).
+        const int32_t D = P.lagD;
+        char *shifted = tile < D ? side_matrix(P.side, P.sstride, mat, A) + static_cast<int64_t>(tile) * TWB
+                                 : A + static_cast<int64_t>(j0 - D * W) * EB;
+        const int64_t shifted_pitch = tile < D ? P.spitch : pitch;
+        if (P.lag == LAG_R2C) {
+            U.outp = shifted;
+            U.out_pitch = shifted_pitch;
+        } else {
+            U.inp = shifted;
+            U.in_pitch = shifted_pitch;
+        }
+    }
     return U;
 }
 
@@ -193,31 +198,58 @@ template <int EB, int MODE, int TWB>
 __device__ __forceinline__ void unit_load(const ColParams &P, const Unit &U, const int32_t *srow, uint32_t *sbase,
                                           uint32_t rows_s, int nthr) {
     if (U.skip) return;
-    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
     constexpr int CPR = chunks_per_row<EB, TWB>();
+    constexpr int LPS = CPR < 32 ? CPR : 32;  // lanes per slot
+    constexpr int RPI = 32 / LPS;             // slots per warp iteration
+    constexpr int CPL = (CPR + 31) / 32;      // chunks per lane
     constexpr int HS = hull_pitch(TWB);
-    const int32_t nchunk = U.nslots * CPR;
-    const int32_t wbytes = U.wt * EB;
-    for (int32_t f = threadIdx.x; f < nchunk; f += nthr) {
-        const int32_t t = f / CPR, c = f - t * CPR;
-        int32_t g;
-        if (MODE == COL_R2C_SHUF) {
-            g = srow[t];
-        } else {
-            g = U.rowbase + t;
-            while (g >= P.M) g -= P.M;  // t < nslots <= M + W
-        }
-        const char *rp = U.tilep + static_cast<int64_t>(g) * pitch;
-        const uint32_t off = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(rp)) & 15u;
-        const char *cp = rp - off + c * 16;
-        const uint32_t dst = rows_s + t * HS + c * 16;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = nthr >> 5;
+    const int c = lane % LPS, sub = lane / LPS;
+    if (sub >= RPI) return;  // lanes beyond the last whole slot of the warp
+    const int32_t step = nwarps * RPI;
+    int32_t t = warp * RPI + sub;
+    if (t >= U.nslots) return;
+    const int64_t pitch = U.in_pitch;
+    const int32_t c16 = c * 16;
+    const int32_t rem0 = U.wt * EB - c16;  // + off: bytes of the hull from this chunk on
+    uint32_t dst = rows_s + t * HS + c16;
+    const uint32_t dst_inc = step * HS;
+    // Chunks c (+ 32, ...) of slot t's hull; rp = the slot's first tile element in global.
+    auto issue = [&](const char *rp) {
+        const int32_t off = static_cast<int32_t>(reinterpret_cast<uintptr_t>(rp) & 15u);
         if (c == 0) sbase[t] = dst + off;
-        const int32_t rem = static_cast<int32_t>(off) + wbytes - c * 16;  // bytes of the hull from cp on
-        if (rem >= 16) {
-            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(cp) : "memory");
-        } else if (rem > 0) {  // row end: read only the tile's bytes (never past the buffer)
-            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(dst), "l"(cp), "r"(rem) : "memory");
+#pragma unroll
+        for (int k = 0; k < CPL; ++k) {
+            if (CPL > 1 && c + 32 * k >= CPR) break;
+            const char *src = rp - off + c16 + 512 * k;
+            const uint32_t d = dst + 512 * k;
+            const int32_t rem = rem0 + off - 512 * k;
+            if (rem >= 16) {
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(d), "l"(src) : "memory");
+            } else if (rem > 0) {  // row end: read only the tile's bytes (never past the buffer)
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(d), "l"(src), "r"(rem) : "memory");
+            }
         }
+    };
+    if (MODE == COL_R2C_SHUF) {
+        for (; t < U.nslots; t += step, dst += dst_inc) issue(U.inp + static_cast<int64_t>(srow[t]) * pitch);
+    } else if (step <= P.M) {
+        // contiguous (cyclic) input rows rowbase + t: incremental row index and pointer
+        int32_t g = mod_M(U.rowbase + t, P.kshM, P.fd_M);
+        const char *rp = U.inp + static_cast<int64_t>(g) * pitch;
+        const int64_t rp_inc = step * pitch, rp_wrap = static_cast<int64_t>(P.M) * pitch;
+        for (; t < U.nslots; t += step, dst += dst_inc) {
+            issue(rp);
+            g += step;
+            rp += rp_inc;
+            if (g >= P.M) {
+                g -= P.M;
+                rp -= rp_wrap;
+            }
+        }
+    } else {  // tiny M: fewer rows than one step
+        for (; t < U.nslots; t += step, dst += dst_inc)
+            issue(U.inp + static_cast<int64_t>(mod_M(U.rowbase + t, P.kshM, P.fd_M)) * pitch);
     }
 }
 
@@ -242,40 +274,47 @@ __device__ __forceinline__ void stg_elem(char *p, const uint32_t *v) {
     }
 }
 
-// Store: lane = tile column w (W <= 32; a warp instruction writes 32 / W whole tile rows,
-// TWB contiguous bytes each).  Output band row k goes to global row o(k) (orow[k] for
-// C2R, r0 + k otherwise); its element w is slot k + dw(w), read at sbase[slot] + w eb --
-// for C2R / R2C the lanes of a row read a diagonal of the slot array, conflict-free in
-// the banks (slot pitch TWB + 16 bytes).
+// Store: lane = tile column w (mod 32: W > 32 columns take W / 32 passes over the row);
+// a warp instruction writes min(W, 32) eb contiguous bytes of each of max(1, 32 / W) tile
+// rows.  Output band row k goes to global row o(k) (orow[k] for C2R, r0 + k otherwise);
+// its element w is slot k + dw(w), read at sbase[slot] + w eb -- for C2R / R2C the lanes
+// of a row read a diagonal of the slot array, conflict-free in the banks (slot pitch
+// TWB + 16 bytes).
 template <int EB, int MODE, int TWB>
 __device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, const int32_t *orow,
                                            const uint32_t *sbase, int nthr) {
     constexpr int W = TWB / EB;
-    static_assert(W <= 32, "lane = tile column");
-    constexpr int RPW = 32 / W;
+    constexpr int LPR = W < 32 ? W : 32;  // lanes per tile row
+    constexpr int RPW = 32 / LPR;         // tile rows per warp instruction
+    constexpr int CPL = W / LPR;          // columns per lane
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = nthr >> 5;
-    const int w = lane % W, sub = lane / W;
-    if (w >= U.wt || U.skip) return;
-    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    const int w0 = lane % LPR, sub = lane / LPR;
+    if (U.skip) return;
+    const int64_t pitch = U.out_pitch;
     const int32_t step = nwarps * RPW;
-    int32_t k = warp * RPW + sub;
-    char *colp = U.tilep + w * EB;
-    const uint32_t *sb = sbase + dw_of<EB, MODE, TWB>(P, U, w);
-    const uint32_t wo = w * EB;
-    uint32_t v[4];
-    if (MODE == COL_C2R_SHUF) {
+#pragma unroll
+    for (int cc = 0; cc < CPL; ++cc) {
+        const int w = w0 + cc * LPR;
+        if (w >= U.wt) break;
+        int32_t k = warp * RPW + sub;
+        char *colp = U.outp + w * EB;
+        const uint32_t *sb = sbase + dw_of<EB, MODE, TWB>(P, U, w);
+        const uint32_t wo = w * EB;
+        uint32_t v[4];
+        if (MODE == COL_C2R_SHUF) {
 #pragma unroll 4
-        for (; k < U.nrows; k += step) {
-            lds_elem<EB>(v, sb[k] + wo);
-            stg_elem<EB>(colp + static_cast<int64_t>(orow[k]) * pitch, v);
-        }
-    } else {
-        char *g = colp + static_cast<int64_t>(U.r0 + k) * pitch;
-        const int64_t g_inc = step * pitch;
+            for (; k < U.nrows; k += step) {
+                lds_elem<EB>(v, sb[k] + wo);
+                stg_elem<EB>(colp + static_cast<int64_t>(orow[k]) * pitch, v);
+            }
+        } else {
+            char *g = colp + static_cast<int64_t>(U.r0 + k) * pitch;
+            const int64_t g_inc = step * pitch;
 #pragma unroll 4
-        for (; k < U.nrows; k += step, g += g_inc) {
-            lds_elem<EB>(v, sb[k] + wo);
-            stg_elem<EB>(g, v);
+            for (; k < U.nrows; k += step, g += g_inc) {
+                lds_elem<EB>(v, sb[k] + wo);
+                stg_elem<EB>(g, v);
+            }
         }
     }
 }
@@ -284,12 +323,56 @@ __device__ __forceinline__ void group_arrive(unsigned int *ctr) {
     asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
 }
 
+// In-place hazard of a column pass, per tile (unit order = ticket order, tile-major):
+//  * barrier mode (P.lag == 0): every member of a tile's group reads before any member
+//    writes the tile -- each member arrives on the tile's counter once its loads have
+//    landed and waits for all G arrivals;
+//  * lagged layouts (P.lag != 0; the shuffle passes of two-pass engines): the tile's
+//    output location is not its input location.  R2C (LAG_R2C, tiles left to right)
+//    writes tile t D tiles to the left (tiles t < D into the side block), where the input
+//    of tile t - D lived; C2R (LAG_C2R, tiles right to left) reads tile t from D tiles to
+//    the left (tiles t < D from the side block), left there by the lagged row pass, and
+//    writes it to its own location, where the input of tile t + D lived.  Either way a
+//    unit waits only for the group processed D groups before its own (unit-order tile
+//    tt - D; D is chosen so that D groups span about twice the co-resident CTAs, i.e. that
+//    group is normally long complete), and the row pass reads / writes the shifted layout
+//    (row_shuffle.cu).  Ticket order makes both waits deadlock-free: a waited-for group's
+//    members all hold smaller tickets (they are resident or done) and their loads wait on
+//    nothing; barrier mode additionally needs G <= co-resident CTAs.
+// Counter slot x mod kCtrSlots counts the arrivals of every tile x sharing it (monotone).
+__device__ __forceinline__ unsigned int ctr_target(uint32_t x, int G) {
+    return (x / kCtrSlots + 1) * static_cast<unsigned int>(G);
+}
+__device__ __forceinline__ bool ctr_reached(const ColParams &P, uint32_t x) {
+    unsigned int v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.ctr + (x % kCtrSlots)) : "memory");
+    return v >= ctr_target(x, P.G);
+}
+struct Dep {
+    bool arrive;   // arrive on the own tile's counter after the loads
+    bool wait;     // wait for the counter of tile `on`
+    uint32_t on;
+};
+template <int MODE>
+__device__ __forceinline__ Dep unit_dep(const ColParams &P, uint32_t tt) {
+    Dep d;
+    if (P.lag) {
+        const uint32_t tin = tt - fdiv(tt, P.fd_nt) * static_cast<uint32_t>(P.ntiles);  // position in its matrix
+        d.arrive = true;
+        d.wait = tin >= static_cast<uint32_t>(P.lagD);
+        d.on = tt - P.lagD;
+    } else {
+        d.arrive = d.wait = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
+        d.on = tt;
+    }
+    return d;
+}
+
 // Non-persistent variant: one CTA per (tile, band).  The CTA's logical id comes from a
 // ticket counter taken at start (dispatch order), so the G members of a tile are exactly
 // G consecutive tickets: every group whose tickets are all taken is fully resident, hence
 // only the newest group can be waiting for members, and those get scheduled as older
-// groups finish -- the spin barrier cannot deadlock as long as one group fits on the GPU
-// (G <= resident CTAs).  G == 1: no barrier, P.tpc consecutive tiles per CTA.
+// groups finish.  G == 1: P.tpc consecutive tiles per CTA.
 template <int EB, int MODE, int TWB>
 __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *smem, uint32_t tt, int32_t r) {
     const SmemLayout L = smem_layout(P.B, TWB / EB, TWB, EB);
@@ -297,32 +380,32 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     int32_t *srow = reinterpret_cast<int32_t *>(smem + L.srow);
     uint32_t *sbase = reinterpret_cast<uint32_t *>(smem + L.sbase);
     const Unit U = unit_make<EB, MODE, TWB>(P, tt, r);
-    const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
+    const Dep D = unit_dep<MODE>(P, tt);
     if (U.skip) {  // group-uniform; still arrive, later tiles sharing the counter count it
-        if (use_barrier && threadIdx.x == 0) atomicAdd(P.ctr + (tt % kCtrSlots), 1u);
+        if (D.arrive && threadIdx.x == 0) atomicAdd(P.ctr + (tt % kCtrSlots), 1u);
         return;
     }
-    unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
+    if (P.dbg != 4) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
     if (MODE == COL_R2C_SHUF) __syncthreads();
-    unit_load<EB, MODE, TWB>(P, U, srow, sbase, static_cast<uint32_t>(__cvta_generic_to_shared(smem + L.rows)), blockDim.x);
+    if (P.dbg != 2)  // measurement knob: 2 = skip the loads
+        unit_load<EB, MODE, TWB>(P, U, srow, sbase, static_cast<uint32_t>(__cvta_generic_to_shared(smem + L.rows)),
+                                 blockDim.x);
     asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
-    // In-place hazard barrier: the whole tile has been read before anyone writes it.
-    // Counter slot tt mod kCtrSlots, monotone over the tiles that share it.
-    if (use_barrier) {
-        const unsigned int slot = tt % kCtrSlots;  // power of two
-        const unsigned int target = (tt / kCtrSlots + 1) * static_cast<unsigned int>(P.G);
-        group_barrier(P.ctr + slot, target);
-    } else {
-        __syncthreads();
+    __syncthreads();  // every thread's staged data is in shared memory
+    if (threadIdx.x == 0) {
+        if (D.arrive) asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(P.ctr + (tt % kCtrSlots)) : "memory");
+        if (D.wait && P.dbg != 5)
+            while (!ctr_reached(P, D.on)) __nanosleep(64);
     }
-    unit_store<EB, MODE, TWB>(P, U, orow, sbase, blockDim.x);
+    __syncthreads();
+    if (P.dbg == 0) unit_store<EB, MODE, TWB>(P, U, orow, sbase, blockDim.x);  // 1, 3, 4 = loads only
 }
 
 template <int EB, int MODE, int TWB>
 __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ unsigned int s_ticket;
-    if (threadIdx.x == 0) s_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
+    if (threadIdx.x == 0) s_ticket = P.dbg == 3 ? blockIdx.x : atomicAdd(P.ctr + kTicketSlot, 1u);
     __syncthreads();
     const unsigned int ticket = s_ticket;
     if (P.G == 1) {
@@ -398,7 +481,6 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
     const SmemLayout L = smem_layout(P.B, W, TWB, EB);
     const size_t bufsz = L.total;
     const uint32_t total = static_cast<uint32_t>(P.total_tiles) * static_cast<uint32_t>(P.G);
-    const bool use_barrier = P.G > 1 && !(MODE == COL_COPY && P.rot_sign == 0);
     if (threadIdx.x == 0) {
         for (int b = 0; b < NB; ++b) {
             mbar_init(&bar_tk[b], 1);
@@ -437,20 +519,16 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
                     if (t >= total) {
                         if (release == arrive) break;  // every real unit released
                     } else if (mbar_test(&bar_full[ab], ak & 1)) {
-                        if (use_barrier) group_arrive(P.ctr + (fdiv(t, P.fd_G) % kCtrSlots));
+                        const uint32_t tt = fdiv(t, P.fd_G);
+                        if (unit_dep<MODE>(P, tt).arrive) group_arrive(P.ctr + (tt % kCtrSlots));
                         ++arrive;
                         if (++ab == NB) ab = 0, ++ak;
                         progress = true;
                     }
                 }
                 if (release < arrive) {
-                    const uint32_t tt = fdiv(s_ticket[rb], P.fd_G);
-                    bool done = !use_barrier;
-                    if (!done) {
-                        unsigned int v;
-                        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.ctr + (tt % kCtrSlots)) : "memory");
-                        done = v >= (tt / kCtrSlots + 1) * static_cast<unsigned int>(P.G);
-                    }
+                    const Dep d = unit_dep<MODE>(P, fdiv(s_ticket[rb], P.fd_G));
+                    const bool done = !d.wait || ctr_reached(P, d.on);
                     if (done) {
                         mbar_arrive(&bar_go[rb]);
                         ++release;
@@ -525,15 +603,10 @@ void *col_kernel_w(int mode, bool pipe) {
 
 template <int EB>
 void *col_kernel_e(int mode, int twb, bool pipe) {
-    // lane = tile column: W = twb / EB <= 32
     switch (twb) {
         case 128: return col_kernel_w<EB, 128>(mode, pipe);
-        case 256:
-            if constexpr (EB >= 8) return col_kernel_w<EB, 256>(mode, pipe);
-            return nullptr;
-        case 512:
-            if constexpr (EB >= 16) return col_kernel_w<EB, 512>(mode, pipe);
-            return nullptr;
+        case 256: return col_kernel_w<EB, 256>(mode, pipe);
+        case 512: return col_kernel_w<EB, 512>(mode, pipe);
         default: return nullptr;
     }
 }

@@ -29,6 +29,15 @@ enum ColMode : int {
                        // (ipt_debug_tile_copy); rot_sign = 0 also drops the cluster barrier
 };
 
+// Column-shuffle tile layouts (col_tile.cu, "In-place hazard").
+enum ColLag : int { LAG_NONE = 0, LAG_R2C = 1, LAG_C2R = 2 };
+// Side tiles of the lagged layouts: matrix k's M x (D W) side block, rows spitch bytes apart,
+// placed so that side row i has the same address mod 16 as row i of the matrix (spitch =
+// N eb mod 16): the lagged row pass stages side part and row part with 16-byte copies.
+__host__ __device__ inline char *side_matrix(char *side, int64_t sstride, int64_t mat, const char *A_mat) {
+    char *raw = side + mat * sstride;
+    return raw + ((reinterpret_cast<uintptr_t>(A_mat) - reinterpret_cast<uintptr_t>(raw)) & 15);
+}
 // Row-shuffle directions.
 enum RowDir : int {
     ROW_C2R = 0,  // out[i][j] = in[i][d'^{-1}_i(j)]  (Eq. 31)
@@ -65,6 +74,13 @@ struct RowParams {
     // Fused rotation (c > 1, c <= kMaxFuseC; row_rot_kernel): the column rotation of the
     // engine (C2R pre-rotation Eq. 23 / R2C post-rotation Eq. 36) folded into this pass.
     int32_t fuse;
+    int32_t R;               // rows per CTA stage (row groups; a power of two dividing the warps)
+    // Lagged layout shared with the column shuffle (col_tile.cu): logical columns [0, shW)
+    // of row i live in the side tile, side + (mat M + i) spitch; columns [shW, N) at A
+    // columns [0, N - shW).  R2C reads it (the column pass ran first), C2R writes it.
+    int32_t shW;
+    int64_t spitch, sstride;  // as ColParams (side_matrix)
+    char *side;
     int32_t segp;            // C2R staircase: shared bytes per source segment (b elements)
     FastDiv fd_cps;          // segp / 16 (16-byte chunks per segment)
     unsigned int *flags;     // per-row "read" flags (M * batch, zeroed per call)
@@ -95,6 +111,12 @@ struct ColParams {
     int32_t pipe;       // 1: persistent pipelined kernel (col_pipe_kernel) with nbuf unit buffers
     int32_t nbuf;
     int32_t threads;    // threads per CTA (col_block_threads() for the pipelined kernel)
+    int32_t lag;        // LAG_NONE, LAG_R2C or LAG_C2R (col_tile.cu: lagged tile layouts)
+    char *side;         // LAG_*: the side tiles (side_matrix() locates a matrix's)
+    int32_t lagD;       // LAG_*: the lag in tiles (tiles 0..D-1 live in the side tiles)
+    int64_t spitch;     // side row pitch: D TWB + (N eb mod 16) (rows as aligned as A's)
+    int64_t sstride;    // side bytes reserved per matrix
+    int32_t dbg;        // measurement only (IPT_COL_DEBUG): 1 loads only, 3 + no ticket, 4 + no prepass
 };
 
 // Skinny engine storage: "location" L in [0, n] is row L of the n x N view, location n is
@@ -139,6 +161,7 @@ unsigned int *group_counters(cudaStream_t st, int n);
 // Launchers (col_tile.cu / row_shuffle.cu).  They return the CUDA error of the launch.
 size_t row_smem_bytes(int64_t N, int eb);
 int row_block_threads();
+int row_threads(int64_t N, int eb);  // threads per CTA of the one-CTA-per-row-group kernels
 cudaError_t launch_row(const RowParams &p, int dir, int eb, cudaStream_t st);
 // Fused rotation + row shuffle (p.fuse): shared bytes of one row buffer -- R2C: the row
 // (as row_smem_bytes); C2R: c staircase segments of segp bytes + the c-entry pad table.

@@ -27,6 +27,8 @@
 
 namespace ipt {
 
+int row_threads(int64_t N, int eb) { return N * eb >= 48 * 1024 ? 512 : 256; }
+
 namespace {
 
 constexpr int kRowThreadsMax = 512;
@@ -103,38 +105,50 @@ struct R2CWalk {
     }
 };
 
+// Gather one output row: warps [0, wn) of the row's warp team (this warp is number wl)
+// each write a contiguous, 32-aligned segment, lane L writing outputs L, L+32, ...
 template <int EB, int DIR, bool TAIL>
-__device__ __forceinline__ void gather_row(const RowParams &P, char *row, const unsigned char *stage, int32_t i) {
+__device__ __forceinline__ void gather_row(const RowParams &P, char *row, char *srow, const unsigned char *stage,
+                                           int32_t i, int wl, int wn) {
     using T = typename Word<EB>::T;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-    const int32_t seg = ((P.N + nwarps - 1) / nwarps + 31) & ~31;  // whole warps' worth
-    const int32_t p_begin = warp * seg, p_end = min(P.N, p_begin + seg);
+    const int lane = threadIdx.x & 31;
+    const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;  // whole warps' worth
+    const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
     const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
     const int32_t Mi = P.M - i;
     const T *src = reinterpret_cast<const T *>(stage);
-    T *out = reinterpret_cast<T *>(row);
+    // Lagged C2R output (P.shW > 0): logical column p < shW goes to the side tile row srow,
+    // the others to row[p - shW]; only the iterations that start below shW select.
+    T *out = reinterpret_cast<T *>(row) - P.shW;
     int32_t p = p_begin + lane;
     if (p >= p_end) return;
     if (DIR == ROW_C2R) {
         C2RWalk<TAIL> w(P, im, p);
+        for (; p - lane < P.shW && p < p_end; p += 32) {  // iterations that reach below shW
+            const T v = src[w.src(P, Mi)];
+            if (p < P.shW) reinterpret_cast<T *>(srow)[p] = v;
+            else out[p] = v;
+            w.next(P);
+        }
 #pragma unroll 4
         for (; p < p_end; p += 32) {
             out[p] = src[w.src(P, Mi)];
             w.next(P);
         }
     } else {
+        T *o = reinterpret_cast<T *>(row);
         R2CWalk<TAIL> w(P, im, p);
 #pragma unroll 4
         for (; p < p_end; p += 32) {
-            out[p] = src[w.src(P, Mi)];
+            o[p] = src[w.src(P, Mi)];
             w.next(P);
         }
     }
 }
 
-// Stage one row with cp.async: smem byte (off + k) holds row byte k.  Not waited.
+// Stage one row with cp.async (no commit): smem byte (off + k) holds row byte k.
 template <int EB>
-__device__ __forceinline__ void stage_row(const char *row, int32_t nbytes, uint32_t sbase) {
+__device__ __forceinline__ void stage_row_chunks(const char *row, int32_t nbytes, uint32_t sbase) {
     constexpr int PER = 16 / EB;
     const int off = static_cast<int>(reinterpret_cast<uintptr_t>(row) & 15);  // multiple of EB
     const char *row0 = row - off;
@@ -151,59 +165,102 @@ __device__ __forceinline__ void stage_row(const char *row, int32_t nbytes, uint3
             }
         }
     }
+}
+
+// Stage a lagged R2C input row (P.shW > 0): logical columns [0, shW) from the side row
+// `srow`, [shW, N) from row[0, N - shW), so that smem byte (off + k) holds logical byte k,
+// off = row & 15 (as stage_row_chunks for an unlagged row).  The side row has the same
+// address mod 16 as the row (side_matrix), so both parts move with 16-byte copies.  No commit.
+template <int EB>
+__device__ __forceinline__ void stage_row_lagged(const RowParams &P, const char *row, const char *srow,
+                                                 uint32_t sbase) {
+    stage_row_chunks<EB>(srow, P.shW * EB, sbase);
+    stage_row_chunks<EB>(row, (P.N - P.shW) * EB, sbase + P.shW * EB);
+}
+
+template <int EB>
+__device__ __forceinline__ void stage_row(const char *row, int32_t nbytes, uint32_t sbase) {
+    stage_row_chunks<EB>(row, nbytes, sbase);
     asm volatile("cp.async.commit_group;" ::: "memory");
 }
 
-// Grid-stride over the M * batch rows.  NBUF = 2: while row r is gathered from one
-// buffer, row r + gridDim.x is already streaming into the other (cp.async groups), so
-// every CTA keeps a row's worth of loads in flight at all times.
+// Row groups: a CTA stages P.R consecutive rows of one matrix at a time (short rows: one
+// row alone keeps too few bytes in flight per SM), and the CTA's warps split into R teams
+// of nwarps / R warps, team t gathering row i0 + t.  Group g of the batch is rows
+// [i0, i0 + nr) of matrix g / gpm, i0 = (g mod gpm) R, nr = min(R, M - i0).
+struct RowGroup {
+    int64_t mat;
+    int32_t i0, nr;
+};
+__device__ __forceinline__ RowGroup row_group(const RowParams &P, int64_t g, int32_t gpm) {
+    RowGroup G;
+    G.mat = g / gpm;
+    G.i0 = static_cast<int32_t>(g - G.mat * gpm) * P.R;
+    G.nr = min(P.R, P.M - G.i0);
+    return G;
+}
+
+// Grid-stride over the row groups.  NBUF = 2: while group g is gathered from one buffer,
+// group g + grid is already streaming into the other (cp.async groups), so every CTA
+// keeps a group's worth of loads in flight at all times.
 template <int EB, int DIR, int NBUF>
 __global__ void __launch_bounds__(kRowThreadsMax) row_shuffle_kernel(RowParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
-    const int64_t rows_total = static_cast<int64_t>(P.M) * P.batch;
     const int32_t nbytes = P.N * EB;
-    const uint32_t bufbytes = (static_cast<uint32_t>(nbytes) + 31) & ~15u;
+    const uint32_t rowbuf = (static_cast<uint32_t>(nbytes) + 31) & ~15u;
+    const uint32_t bufbytes = rowbuf * static_cast<uint32_t>(P.R);
     const uint32_t sbase = smem_u32(smem);
-
-    int64_t mat = blockIdx.x / P.M;
-    int32_t i = static_cast<int32_t>(blockIdx.x - mat * P.M);
-    const int32_t step_i = static_cast<int32_t>(gridDim.x % P.M);
-    const int64_t step_m = gridDim.x / P.M;
+    const int32_t gpm = (P.M + P.R - 1) / P.R;
+    const int64_t groups_total = static_cast<int64_t>(gpm) * P.batch;
+    const int wn = (blockDim.x >> 5) / P.R;  // warps per row team
+    const int team = (threadIdx.x >> 5) / wn, wl = (threadIdx.x >> 5) - team * wn;
     auto row_ptr = [&](int64_t mm, int32_t ii) {
         return P.base + mm * P.mat_stride_bytes + static_cast<int64_t>(ii) * nbytes;
     };
-    if (NBUF == 2 && blockIdx.x < rows_total) stage_row<EB>(row_ptr(mat, i), nbytes, sbase);
-    int buf = 0;
-    for (int64_t r = blockIdx.x; r < rows_total; r += gridDim.x) {
-        char *row = row_ptr(mat, i);
-        int32_t ni = i + step_i;
-        int64_t nmat = mat + step_m;
-        if (ni >= P.M) {
-            ni -= P.M;
-            ++nmat;
+    auto side_ptr = [&](int64_t mm, int32_t ii) {
+        return side_matrix(P.side, P.sstride, mm, P.base + mm * P.mat_stride_bytes) + ii * P.spitch;
+    };
+    auto stage = [&](const RowGroup &G, int b) {
+        for (int32_t rr = 0; rr < G.nr; ++rr) {
+            const uint32_t sb = sbase + b * bufbytes + rr * rowbuf;
+            if (DIR == ROW_R2C && P.shW) stage_row_lagged<EB>(P, row_ptr(G.mat, G.i0 + rr), side_ptr(G.mat, G.i0 + rr), sb);
+            else stage_row_chunks<EB>(row_ptr(G.mat, G.i0 + rr), nbytes, sb);
         }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    int64_t g = blockIdx.x;
+    RowGroup G = row_group(P, g, gpm);
+    if (NBUF == 2 && g < groups_total) stage(G, 0);
+    int buf = 0;
+    for (; g < groups_total; g += gridDim.x) {
+        const int64_t ng = g + gridDim.x;
+        const RowGroup NG = row_group(P, ng, gpm);
         if (NBUF == 2) {
-            if (r + gridDim.x < rows_total) {
-                stage_row<EB>(row_ptr(nmat, ni), nbytes, sbase + (buf ^ 1) * bufbytes);
+            if (ng < groups_total) {
+                stage(NG, buf ^ 1);
                 asm volatile("cp.async.wait_group 1;" ::: "memory");
             } else {
                 asm volatile("cp.async.wait_group 0;" ::: "memory");
             }
         } else {
-            stage_row<EB>(row, nbytes, sbase);
+            stage(G, 0);
             asm volatile("cp.async.wait_group 0;" ::: "memory");
         }
         __syncthreads();
 
         // ---- gather + write back (the last c - 1 rows may have f2 = 1) --------------
-        const unsigned char *stage = smem + buf * bufbytes + (reinterpret_cast<uintptr_t>(row) & 15);
-        if (i >= P.M - P.c + 1) gather_row<EB, DIR, true>(P, row, stage, i);
-        else gather_row<EB, DIR, false>(P, row, stage, i);
-        __syncthreads();  // this buffer is refilled two rows later
+        if (team < G.nr) {
+            const int32_t i = G.i0 + team;
+            char *row = row_ptr(G.mat, i);
+            const unsigned char *st = smem + buf * bufbytes + team * rowbuf + (reinterpret_cast<uintptr_t>(row) & 15);
+            char *srow = P.shW ? side_ptr(G.mat, i) : nullptr;
+            if (i >= P.M - P.c + 1) gather_row<EB, DIR, true>(P, row, srow, st, i, wl, wn);
+            else gather_row<EB, DIR, false>(P, row, srow, st, i, wl, wn);
+        }
+        __syncthreads();  // this buffer is refilled two groups later
 
         if (NBUF == 2) buf ^= 1;
-        i = ni;
-        mat = nmat;
+        G = NG;
     }
 }
 
@@ -219,13 +276,15 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_shuffle_kernel(RowParams P
 //    index l to its shared-memory byte (padl[floor(l/b)] + l eb).
 //  * R2C (Eq. 24 then Eq. 36):  out[(i + floor(p/b)) mod M][p] = A[i][d'_i(p)]:
 //    row i is staged whole and its gathered output block rho is written into row i + rho.
+// Rows are processed in groups of P.R consecutive rows (as row_shuffle_kernel).
 // In place: flags[row] is set (release) once the row's CTA has read everything it needs.
-//  C2R: row i is written after rows i-1 .. i-c+1 (each read a block of row i) are flagged;
-//  R2C: CTA i writes into rows i+1 .. i+c-1 after they are flagged (read by their CTAs).
-// No deadlock with a co-resident grid of > c CTAs: every CTA flags its current row before
-// it waits, and a waited-for row is either some CTA's current row (flagged) or that CTA's
-// later row, which it reaches because its own current row only waits on flagged rows
-// (by induction on the chain, whose rows decrease by at least grid - c per hop).
+//  C2R: rows i0.. of a group are written after rows i0-1 .. i0-c+1 (each read a block of a
+//  row of the group) are flagged; R2C: a group writes into rows up to i0+nr-1+c-1, after
+//  the ones beyond the group are flagged (read by their CTAs).
+// No deadlock with a co-resident grid of > c CTAs: every CTA flags its current group before
+// it waits, and a waited-for row is either some CTA's current group (flagged) or that CTA's
+// later group, which it reaches because its own current group only waits on flagged rows
+// (by induction on the chain, whose groups decrease by at least grid - c per hop).
 template <int EB>
 __device__ __forceinline__ void stage_stair(const RowParams &P, const char *mbase, const char *wrapbase, int32_t i,
                                             uint32_t sbase, int32_t *padl) {
@@ -254,24 +313,30 @@ __device__ __forceinline__ void stage_stair(const RowParams &P, const char *mbas
             }
         }
     }
-    asm volatile("cp.async.commit_group;" ::: "memory");
 }
 
 template <int EB, int DIR>
-__device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, const unsigned char *buf,
-                                               const int32_t *padl, int32_t i) {
+__device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, char *srow, const unsigned char *buf,
+                                               const int32_t *padl, int32_t i, int wl, int wn) {
     using T = typename Word<EB>::T;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-    const int32_t seg = ((P.N + nwarps - 1) / nwarps + 31) & ~31;
-    const int32_t p_begin = warp * seg, p_end = min(P.N, p_begin + seg);
+    const int lane = threadIdx.x & 31;
+    const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;
+    const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
     const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
     const int32_t Mi = P.M - i;
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
     int32_t p = p_begin + lane;
     if (p >= p_end) return;
     if (DIR == ROW_C2R) {
-        T *out = reinterpret_cast<T *>(mbase + static_cast<int64_t>(i) * pitch);
+        // lagged output as in gather_row: p < shW -> side tile row, else row[p - shW]
+        T *out = reinterpret_cast<T *>(mbase + static_cast<int64_t>(i) * pitch) - P.shW;
         C2RWalk<true> w(P, im, p);
+        for (; p - lane < P.shW && p < p_end; p += 32) {
+            const T v = *reinterpret_cast<const T *>(buf + padl[w.l] + w.src(P, Mi) * EB);
+            if (p < P.shW) reinterpret_cast<T *>(srow)[p] = v;
+            else out[p] = v;
+            w.next(P);
+        }
 #pragma unroll 4
         for (; p < p_end; p += 32) {
             out[p] = *reinterpret_cast<const T *>(buf + padl[w.l] + w.src(P, Mi) * EB);
@@ -293,35 +358,44 @@ __device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, 
 template <int EB, int DIR, int NBUF>
 __global__ void __launch_bounds__(kRowThreadsMax) row_rot_kernel(RowParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
-    const int64_t rows_total = static_cast<int64_t>(P.M) * P.batch;
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
-    const uint32_t bufbytes = static_cast<uint32_t>(row_fused_smem_bytes(P, EB, DIR));
+    const uint32_t rowbuf = static_cast<uint32_t>(row_fused_smem_bytes(P, EB, DIR));
+    const uint32_t bufbytes = rowbuf * static_cast<uint32_t>(P.R);
     const uint32_t padoff = static_cast<uint32_t>(P.c) * static_cast<uint32_t>(P.segp);  // C2R pad table
     const uint32_t sbase = smem_u32(smem);
     const int64_t wrap_stride = static_cast<int64_t>(P.c - 1) * pitch;
+    const int32_t gpm = (P.M + P.R - 1) / P.R;
+    const int64_t groups_total = static_cast<int64_t>(gpm) * P.batch;
+    const int wn = (blockDim.x >> 5) / P.R;
+    const int team = (threadIdx.x >> 5) / wn, wl = (threadIdx.x >> 5) - team * wn;
 
-    int64_t mat = blockIdx.x / P.M;
-    int32_t i = static_cast<int32_t>(blockIdx.x - mat * P.M);
-    const int32_t step_i = static_cast<int32_t>(gridDim.x % P.M);
-    const int64_t step_m = gridDim.x / P.M;
-    auto stage = [&](int64_t mm, int32_t ii, int b) {
-        char *mb = P.base + mm * P.mat_stride_bytes;
-        if (DIR == ROW_C2R)
-            stage_stair<EB>(P, mb, P.wrap + mm * wrap_stride, ii, sbase + b * bufbytes,
-                            reinterpret_cast<int32_t *>(smem + b * bufbytes + padoff));
-        else
-            stage_row<EB>(mb + ii * pitch, P.N * EB, sbase + b * bufbytes);
+    auto stage = [&](const RowGroup &G, int b) {
+        char *mb = P.base + G.mat * P.mat_stride_bytes;
+        for (int32_t rr = 0; rr < G.nr; ++rr) {
+            const uint32_t o = b * bufbytes + rr * rowbuf;
+            if (DIR == ROW_C2R)
+                stage_stair<EB>(P, mb, P.wrap + G.mat * wrap_stride, G.i0 + rr, sbase + o,
+                                reinterpret_cast<int32_t *>(smem + o + padoff));
+            else if (P.shW)
+                stage_row_lagged<EB>(P, mb + (G.i0 + rr) * pitch,
+                                     side_matrix(P.side, P.sstride, G.mat, mb) + (G.i0 + rr) * P.spitch, sbase + o);
+            else
+                stage_row_chunks<EB>(mb + (G.i0 + rr) * pitch, P.N * EB, sbase + o);
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
     };
-    auto set_flag = [&](int64_t r) {  // row r's reads are complete (after a __syncthreads)
-        if (threadIdx.x == 0)
-            asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(P.flags + r), "r"(1u) : "memory");
+    auto set_flags = [&](const RowGroup &G) {  // the group's reads are complete (after a __syncthreads)
+        if (threadIdx.x < G.nr)
+            asm volatile("st.release.gpu.global.u32 [%0], %1;"
+                         :: "l"(P.flags + G.mat * P.M + G.i0 + threadIdx.x), "r"(1u) : "memory");
     };
-    auto wait_deps = [&](int64_t mm, int32_t ii) {  // every row that row ii overwrites has been read
+    auto wait_deps = [&](const RowGroup &G) {  // every row the group overwrites has been read
         if (threadIdx.x >= 1 && threadIdx.x < P.c) {
-            int32_t y = DIR == ROW_C2R ? ii - static_cast<int32_t>(threadIdx.x) : ii + static_cast<int32_t>(threadIdx.x);
+            int32_t y = DIR == ROW_C2R ? G.i0 - static_cast<int32_t>(threadIdx.x)
+                                       : G.i0 + G.nr - 1 + static_cast<int32_t>(threadIdx.x);
             if (y >= P.M) y -= P.M;
             if (y >= 0) {
-                const unsigned int *f = P.flags + mm * P.M + y;
+                const unsigned int *f = P.flags + G.mat * P.M + y;
                 unsigned int v;
                 while (true) {
                     asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
@@ -332,43 +406,45 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_rot_kernel(RowParams P) {
         }
         __syncthreads();
     };
-    // NBUF = 2: row r + grid is staged while row r is gathered, and flagged as soon as the
-    // gather of row r is done -- a full row ahead of the moment its neighbours wait for it.
-    if (blockIdx.x < rows_total) {
-        stage(mat, i, 0);
+    // NBUF = 2: group g + grid is staged while group g is gathered, and flagged as soon as
+    // the gather of group g is done -- a full group ahead of the moment its neighbours wait.
+    int64_t g = blockIdx.x;
+    RowGroup G = row_group(P, g, gpm);
+    if (g < groups_total) {
+        stage(G, 0);
         asm volatile("cp.async.wait_group 0;" ::: "memory");
         __syncthreads();
-        set_flag(blockIdx.x);
+        set_flags(G);
     }
     int buf = 0;
-    for (int64_t r = blockIdx.x; r < rows_total; r += gridDim.x) {
-        char *mbase = P.base + mat * P.mat_stride_bytes;
-        int32_t ni = i + step_i;
-        int64_t nmat = mat + step_m;
-        if (ni >= P.M) {
-            ni -= P.M;
-            ++nmat;
-        }
-        const bool more = r + gridDim.x < rows_total;
-        if (NBUF == 2 && more) stage(nmat, ni, buf ^ 1);
-        wait_deps(mat, i);
+    for (; g < groups_total; g += gridDim.x) {
+        char *mbase = P.base + G.mat * P.mat_stride_bytes;
+        const int64_t ng = g + gridDim.x;
+        const RowGroup NG = row_group(P, ng, gpm);
+        const bool more = ng < groups_total;
+        if (NBUF == 2 && more) stage(NG, buf ^ 1);
+        wait_deps(G);
 
-        const unsigned char *b = smem + buf * bufbytes;
-        if (DIR == ROW_C2R) {
-            gather_row_rot<EB, DIR>(P, mbase, b, reinterpret_cast<const int32_t *>(b + padoff), i);
-        } else {
-            gather_row_rot<EB, DIR>(P, mbase, b + (reinterpret_cast<uintptr_t>(mbase + i * pitch) & 15), nullptr, i);
+        if (team < G.nr) {
+            const int32_t i = G.i0 + team;
+            const unsigned char *b = smem + buf * bufbytes + team * rowbuf;
+            char *srow = P.shW ? side_matrix(P.side, P.sstride, G.mat, mbase) + i * P.spitch : nullptr;
+            if (DIR == ROW_C2R) {
+                gather_row_rot<EB, DIR>(P, mbase, srow, b, reinterpret_cast<const int32_t *>(b + padoff), i, wl, wn);
+            } else {
+                gather_row_rot<EB, DIR>(P, mbase, srow, b + (reinterpret_cast<uintptr_t>(mbase + i * pitch) & 15),
+                                        nullptr, i, wl, wn);
+            }
         }
         __syncthreads();  // this buffer is free again
         if (more) {
-            if (NBUF == 1) stage(nmat, ni, 0);
+            if (NBUF == 1) stage(NG, 0);
             asm volatile("cp.async.wait_group 0;" ::: "memory");
             __syncthreads();
-            set_flag(r + gridDim.x);
+            set_flags(NG);
         }
         if (NBUF == 2) buf ^= 1;
-        i = ni;
-        mat = nmat;
+        G = NG;
     }
 }
 
@@ -619,21 +695,18 @@ cudaError_t row_cluster_dispatch(const RowParams &P, int dir, int eb, cudaStream
     }
 }
 
-int row_threads(int64_t N, int eb) { return N * eb >= 48 * 1024 ? 512 : 256; }
 
-// Double buffering while two row buffers stay within ~110 KB (two CTAs per SM or more).
-int row_nbuf(int64_t N, int eb) { return 2 * row_smem_bytes(N, eb) <= 112 * 1024 ? 2 : 1; }
 
 template <int EB, int DIR, int NBUF>
 cudaError_t launch_row_t(const RowParams &P, cudaStream_t st) {
-    const size_t smem = NBUF * row_smem_bytes(P.N, EB);
+    const size_t smem = NBUF * P.R * row_smem_bytes(P.N, EB);
     const int threads = row_threads(P.N, EB);
     auto kern = row_shuffle_kernel<EB, DIR, NBUF>;
     cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
     if (e != cudaSuccess) return e;
     const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), threads, smem);
     if (resident < 1) return cudaErrorInvalidConfiguration;
-    const int64_t rows = static_cast<int64_t>(P.M) * P.batch;
+    const int64_t rows = static_cast<int64_t>((P.M + P.R - 1) / P.R) * P.batch;
     int64_t grid = resident;
     if (grid > rows) grid = rows;
     kern<<<static_cast<unsigned>(grid), threads, smem, st>>>(P);
@@ -642,14 +715,14 @@ cudaError_t launch_row_t(const RowParams &P, cudaStream_t st) {
 
 template <int EB, int DIR, int NBUF>
 cudaError_t launch_row_rot_t(const RowParams &P, cudaStream_t st) {
-    const size_t smem = NBUF * row_fused_smem_bytes(P, EB, DIR);
+    const size_t smem = NBUF * P.R * row_fused_smem_bytes(P, EB, DIR);
     const int threads = row_threads(P.N, EB);
     auto kern = row_rot_kernel<EB, DIR, NBUF>;
     cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
     if (e != cudaSuccess) return e;
     const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), threads, smem);
     if (resident <= P.c) return cudaErrorInvalidConfiguration;  // the flag waits need > c co-resident CTAs
-    const int64_t rows = static_cast<int64_t>(P.M) * P.batch;
+    const int64_t rows = static_cast<int64_t>((P.M + P.R - 1) / P.R) * P.batch;
     int64_t grid = resident;
     if (grid > rows) grid = rows;
     kern<<<static_cast<unsigned>(grid), threads, smem, st>>>(P);
@@ -659,9 +732,10 @@ cudaError_t launch_row_rot_t(const RowParams &P, cudaStream_t st) {
 template <int EB, int DIR>
 cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
     if (P.fuse)
-        return 2 * row_fused_smem_bytes(P, EB, DIR) <= 112 * 1024 ? launch_row_rot_t<EB, DIR, 2>(P, st)
-                                                                   : launch_row_rot_t<EB, DIR, 1>(P, st);
-    return row_nbuf(P.N, EB) == 2 ? launch_row_t<EB, DIR, 2>(P, st) : launch_row_t<EB, DIR, 1>(P, st);
+        return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= 112 * 1024 ? launch_row_rot_t<EB, DIR, 2>(P, st)
+                                                                         : launch_row_rot_t<EB, DIR, 1>(P, st);
+    return 2 * P.R * row_smem_bytes(P.N, EB) <= 112 * 1024 ? launch_row_t<EB, DIR, 2>(P, st)
+                                                           : launch_row_t<EB, DIR, 1>(P, st);
 }
 
 }  // namespace

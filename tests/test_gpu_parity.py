@@ -298,3 +298,54 @@ def test_column_tile_widths_and_small_bands(twb, pipe):
         for eb in (4, 8, 16):
             for engine in ("c2r", "r2c"):
                 run_packed(shapes, eb, ipt.c2r, "row", engine, seed=int(twb) + eb)
+
+
+@pytest.mark.parametrize("stage", ["1", "16384", "200000"])
+@pytest.mark.parametrize("fuse", ["1", "0"])
+def test_row_groups(stage, fuse):
+    """Row pass in groups of R rows per CTA stage (IPT_ROW_STAGE bytes: R = 1, the default,
+    and the largest R); groups that straddle the last rows (f2 = 1 tails, C2R wrap rows of
+    the fused rotation), partial last groups, M < R, and batches whose groups must not
+    cross matrix boundaries."""
+    shapes = [(1200, 1800), (1114, 5285), (5285, 1114), (1026, 19126 // 7), (333, 999), (7, 300), (300, 7),
+              (64, 96), (96, 64), (130, 2050), (2050, 130)]
+    with env_var("IPT_ROW_STAGE", stage), env_var("IPT_FUSE_ROT", fuse):
+        for eb in (4, 8):
+            for engine in ("c2r", "r2c"):
+                run_packed(shapes, eb, ipt.c2r, "row", engine, seed=len(stage) + eb)
+        m, n, batch = 130, 2050, 3
+        host = workloads.random_words(batch * m * n, 4, seed=9)
+        x = to_dev(host)
+        ipt.c2r_batched(x, batch, m * n, m, n, elem_bytes=4)
+        got = x.cpu().numpy().view(np.uint32)
+        for k in range(batch):
+            assert got[k * m * n:(k + 1) * m * n].tobytes() == oracle.transpose(host[k * m * n:(k + 1) * m * n], m, n).tobytes()
+
+
+@pytest.mark.parametrize("lagd", ["1", "3", "1000"])
+def test_lagged_tile_layouts(lagd):
+    """Shuffle pass with lagged tile layouts (D = IPT_COL_LAGD tiles, clamped to ntiles - 1):
+    tiles t < D go through the side block, the rest D tiles to the left; the row pass reads
+    (R2C) / writes (C2R) that layout.  Both engines, fused and separate rotation, ragged last
+    tiles, rows misaligned to 16 bytes, batches (the side block of each matrix aligned like
+    its rows), and IPT_COL_LAG=0 (per-tile barrier) for comparison."""
+    shapes = [(1200, 1800), (1031, 97), (97, 1031), (513, 700), (700, 513), (2003, 129), (129, 2003), (333, 4099)]
+    for lag in ("1", "0"):
+        with env_var("IPT_COL_LAGD", lagd), env_var("IPT_COL_LAG", lag):
+            for fuse in ("1", "0"):
+                with env_var("IPT_FUSE_ROT", fuse):
+                    for eb in (4, 8, 16):
+                        for engine in ("c2r", "r2c"):
+                            run_packed(shapes, eb, ipt.c2r, "row", engine, seed=eb + len(lagd))
+            m, n, batch = 300, 1001, 4
+            for eb in (4, 8):
+                host = workloads.random_words(1 + batch * (m * n + 5), eb, seed=77)
+                hv = vwords(host, eb)
+                x = to_dev(host)
+                ipt.c2r_batched(x.data_ptr() + eb, batch, m * n + 5, m, n, elem_bytes=eb)
+                got = vwords(x.cpu().numpy(), eb)
+                for k in range(batch):
+                    o = 1 + k * (m * n + 5)
+                    assert got[o:o + m * n].tobytes() == oracle.ipt_c2r(hv[o:o + m * n], m, n).tobytes()
+                ipt.r2c_batched(x.data_ptr() + eb, batch, m * n + 5, m, n, elem_bytes=eb)
+                assert dev_bytes(x) == np.ascontiguousarray(host).tobytes()
