@@ -363,6 +363,8 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         rp.w_dh = static_cast<int32_t>(D % pl.b);
         rp.w_dl2 = static_cast<int32_t>(D / pl.b);
         rp.w_ds = static_cast<int32_t>((D / pl.b + ((D % pl.b) * (pl.M % pl.N)) % pl.N) % pl.N);
+        rp.c1_step = static_cast<int32_t>(engine == ENG_C2R ? ((D % pl.N) * rp.ainv) % pl.N
+                                                            : ((D % pl.N) * (pl.M % pl.N)) % pl.N);
     }
     pl.row_dir = engine == ENG_C2R ? ROW_C2R : ROW_R2C;
     if (use_cluster) {
@@ -413,6 +415,7 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         while (rp.R * 2 <= nw && rp.R * 2 * rowbuf <= target) rp.R *= 2;
         rsm = rowbuf * rp.R;
     }
+    rp.fd_gpm = make_fastdiv(static_cast<uint32_t>((pl.M + rp.R - 1) / rp.R));
 
     ipt_status_t s = plan_col(dev, pl, engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.shuf);
     if (s != IPT_OK) return s;
@@ -423,9 +426,10 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     if (env_int("IPT_COL_LAG", 1) != 0 && !use_cluster && pl.shuf.p.ntiles >= 2) {
         ColParams &cq = pl.shuf.p;
         cq.lag = engine == ENG_C2R ? LAG_C2R : LAG_R2C;
-        // D: about twice the co-resident CTAs' worth of groups between a unit and the group
-        // it waits for (IPT_COL_LAGD overrides); at most ntiles - 1.
-        int64_t D = env_int("IPT_COL_LAGD", 0);
+        // D (IPT_COL_LAGD, default 8 tiles; 0: twice the co-resident CTAs' worth of
+        // groups): the round-1 sweep found 4-8 tiles of slack enough to take the wait off
+        // the critical path (tools/col_sweep.sh), larger D no better; at most ntiles - 1.
+        int64_t D = env_int("IPT_COL_LAGD", 8);
         if (D <= 0) D = (2 * static_cast<int64_t>(cq.resident) + cq.G - 1) / cq.G;
         set_lag(pl, D);
         pl.scratch += pl.side_bytes;
@@ -536,6 +540,9 @@ void profile_end(ProfRec &r, cudaStream_t st) {
 ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_bytes, cudaStream_t st) {
     if (pl0.engine == ENG_NONE || batch == 0) return IPT_OK;
     Plan pl = pl0;
+    // Row groups are numbered in 32 bits (row_shuffle.cu row_group).
+    if (pl.engine != ENG_SKINNY && (pl.M + pl.row.R - 1) / pl.row.R * batch >= (int64_t(1) << 32))
+        return IPT_ERR_UNSUPPORTED;
     pl.row.base = base;
     pl.row.batch = batch;
     pl.row.mat_stride_bytes = stride_bytes;

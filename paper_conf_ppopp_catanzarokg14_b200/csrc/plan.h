@@ -62,6 +62,8 @@ struct RowParams {
     int32_t w_dh;   // 32 mod b
     int32_t w_dl2;  // floor(32 / b)
     int32_t w_ds;   // (floor(32 / b) + (32 mod b) M) mod N
+    int32_t c1_step;  // c = 1: the gather index step of 32 outputs, (32 a^{-1}) mod N (C2R) or
+                      // (32 M) mod N (R2C)
     // Cluster row pass (rows too long for one CTA): the row is split
     // into cl_K segments of cl_seg elements (a multiple of 32), one per CTA of a cluster.
     int32_t cl_K, cl_seg;
@@ -75,6 +77,7 @@ struct RowParams {
     // engine (C2R pre-rotation Eq. 23 / R2C post-rotation Eq. 36) folded into this pass.
     int32_t fuse;
     int32_t R;               // rows per CTA stage (row groups; a power of two dividing the warps)
+    FastDiv fd_gpm;          // ceil(M / R): row groups per matrix
     // Lagged layout shared with the column shuffle (col_tile.cu): logical columns [0, shW)
     // of row i live in the side tile, side + (mat M + i) spitch; columns [shW, N) at A
     // columns [0, N - shW).  R2C reads it (the column pass ran first), C2R writes it.

@@ -109,25 +109,59 @@ struct R2CWalk {
 // each write a contiguous, 32-aligned segment, lane L writing outputs L, L+32, ...
 template <int EB, int DIR, bool TAIL>
 __device__ __forceinline__ void gather_row(const RowParams &P, char *row, char *srow, const unsigned char *stage,
-                                           int32_t i, int wl, int wn) {
+                                           int32_t i, int32_t p_begin, int32_t p_end) {
     using T = typename Word<EB>::T;
     const int lane = threadIdx.x & 31;
-    const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;  // whole warps' worth
-    const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
     const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
     const int32_t Mi = P.M - i;
     const T *src = reinterpret_cast<const T *>(stage);
-    // Lagged C2R output (P.shW > 0): logical column p < shW goes to the side tile row srow,
-    // the others to row[p - shW]; only the iterations that start below shW select.
+    // Lagged C2R output (P.shW > 0): logical column p < shW goes to the side row srow, the
+    // others to row[p - shW].
     T *out = reinterpret_cast<T *>(row) - P.shW;
     int32_t p = p_begin + lane;
     if (p >= p_end) return;
+    if (P.c == 1) {
+        // gcd 1 (Theorem 3 with c = 1): the gather index is an arithmetic progression
+        // mod N -- C2R d'^{-1}_i(p) = a^{-1} (p - i) mod N, R2C d'_i(j) = (i + j M) mod N --
+        // so a lane's next source (32 outputs on) is one add and one conditional subtract.
+        uint32_t sidx;
+        if (DIR == ROW_C2R) {
+            int32_t q = p - im;
+            q += q < 0 ? P.N : 0;
+            sidx = mulmod(static_cast<uint32_t>(P.ainv), static_cast<uint32_t>(q), P.fd_N, P.wideN);
+        } else {
+            sidx = static_cast<uint32_t>(im) + mulmod(static_cast<uint32_t>(p), static_cast<uint32_t>(P.Mn), P.fd_N, P.wideN);
+            sidx -= sidx >= static_cast<uint32_t>(P.N) ? P.N : 0;
+        }
+        const uint32_t d = static_cast<uint32_t>(P.c1_step), n = static_cast<uint32_t>(P.N);
+        T *o = DIR == ROW_C2R ? out : reinterpret_cast<T *>(row);
+        if (DIR == ROW_C2R) {
+            const int32_t p_side = min(p_end, P.shW);
+            T *so = reinterpret_cast<T *>(srow);
+#pragma unroll 4
+            for (; p < p_side; p += 32) {
+                so[p] = src[sidx];
+                sidx += d;
+                sidx -= sidx >= n ? n : 0;
+            }
+        }
+#pragma unroll 8
+        for (; p < p_end; p += 32) {
+            o[p] = src[sidx];
+            sidx += d;
+            sidx -= sidx >= n ? n : 0;
+        }
+        return;
+    }
     if (DIR == ROW_C2R) {
         C2RWalk<TAIL> w(P, im, p);
-        for (; p - lane < P.shW && p < p_end; p += 32) {  // iterations that reach below shW
-            const T v = src[w.src(P, Mi)];
-            if (p < P.shW) reinterpret_cast<T *>(srow)[p] = v;
-            else out[p] = v;
+        // each lane: its outputs below shW to the side row, then the rest (lanes diverge
+        // for at most one iteration; every lane's walk is its own)
+        const int32_t p_side = min(p_end, P.shW);
+        T *so = reinterpret_cast<T *>(srow);
+#pragma unroll 4
+        for (; p < p_side; p += 32) {
+            so[p] = src[w.src(P, Mi)];
             w.next(P);
         }
 #pragma unroll 4
@@ -146,23 +180,27 @@ __device__ __forceinline__ void gather_row(const RowParams &P, char *row, char *
     }
 }
 
-// Stage one row with cp.async (no commit): smem byte (off + k) holds row byte k.
+// Stage one row with cp.async (no commit): smem byte (off + k) holds row byte k, off =
+// row & 15.  Whole 16-byte chunks of the row's aligned hull move with 16-byte copies (a
+// plain strided loop); the at most two partial chunks at the ends element by element
+// (lanes 0.. of warp 0 the head, of warp 1 the tail).
 template <int EB>
 __device__ __forceinline__ void stage_row_chunks(const char *row, int32_t nbytes, uint32_t sbase) {
-    constexpr int PER = 16 / EB;
     const int off = static_cast<int>(reinterpret_cast<uintptr_t>(row) & 15);  // multiple of EB
     const char *row0 = row - off;
-    const int nch = (off + nbytes + 15) >> 4;
-    for (int k = threadIdx.x; k < nch; k += blockDim.x) {
-        const int lo = k * 16 - off;
-        if (lo >= 0 && lo + 16 <= nbytes) {
-            cp_async<16>(sbase + 16 * k, row0 + 16 * k);
-        } else {
-#pragma unroll
-            for (int e = 0; e < PER; ++e) {
-                const int q = lo + e * EB;
-                if (q >= 0 && q < nbytes) cp_async<EB>(sbase + off + q, row + q);
-            }
+    const int k0 = off ? 1 : 0;                 // first whole chunk
+    const int k1 = (off + nbytes) >> 4;         // end of the whole chunks
+    for (int k = k0 + threadIdx.x; k < k1; k += blockDim.x) cp_async<16>(sbase + 16 * k, row0 + 16 * k);
+    if (EB < 16) {
+        const int t = threadIdx.x;
+        if (off && t < (16 - off) / EB) {  // head: bytes [0, 16 - off) of the row
+            const int q = t * EB;
+            if (q < nbytes) cp_async<EB>(sbase + off + q, row + q);
+        }
+        const int tail = k1 * 16 - off;  // first byte of the partial last chunk
+        if (t >= 32 && t - 32 < (nbytes - tail) / EB && tail >= (off ? 16 - off : 0)) {
+            const int q = tail + (t - 32) * EB;
+            cp_async<EB>(sbase + off + q, row + q);
         }
     }
 }
@@ -194,8 +232,9 @@ struct RowGroup {
 };
 __device__ __forceinline__ RowGroup row_group(const RowParams &P, int64_t g, int32_t gpm) {
     RowGroup G;
-    G.mat = g / gpm;
-    G.i0 = static_cast<int32_t>(g - G.mat * gpm) * P.R;
+    const uint32_t m = fdiv(static_cast<uint32_t>(g), P.fd_gpm);  // groups_total < 2^32 (planner)
+    G.mat = m;
+    G.i0 = static_cast<int32_t>(static_cast<uint32_t>(g) - m * static_cast<uint32_t>(gpm)) * P.R;
     G.nr = min(P.R, P.M - G.i0);
     return G;
 }
@@ -204,7 +243,7 @@ __device__ __forceinline__ RowGroup row_group(const RowParams &P, int64_t g, int
 // group g + grid is already streaming into the other (cp.async groups), so every CTA
 // keeps a group's worth of loads in flight at all times.
 template <int EB, int DIR, int NBUF>
-__global__ void __launch_bounds__(kRowThreadsMax) row_shuffle_kernel(RowParams P) {
+__global__ void __launch_bounds__(kRowThreadsMax, 4) row_shuffle_kernel(RowParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
     const int32_t nbytes = P.N * EB;
     const uint32_t rowbuf = (static_cast<uint32_t>(nbytes) + 31) & ~15u;
@@ -214,6 +253,8 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_shuffle_kernel(RowParams P
     const int64_t groups_total = static_cast<int64_t>(gpm) * P.batch;
     const int wn = (blockDim.x >> 5) / P.R;  // warps per row team
     const int team = (threadIdx.x >> 5) / wn, wl = (threadIdx.x >> 5) - team * wn;
+    const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;  // output segment of a warp: whole warps' worth
+    const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
     auto row_ptr = [&](int64_t mm, int32_t ii) {
         return P.base + mm * P.mat_stride_bytes + static_cast<int64_t>(ii) * nbytes;
     };
@@ -254,8 +295,8 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_shuffle_kernel(RowParams P
             char *row = row_ptr(G.mat, i);
             const unsigned char *st = smem + buf * bufbytes + team * rowbuf + (reinterpret_cast<uintptr_t>(row) & 15);
             char *srow = P.shW ? side_ptr(G.mat, i) : nullptr;
-            if (i >= P.M - P.c + 1) gather_row<EB, DIR, true>(P, row, srow, st, i, wl, wn);
-            else gather_row<EB, DIR, false>(P, row, srow, st, i, wl, wn);
+            if (i >= P.M - P.c + 1) gather_row<EB, DIR, true>(P, row, srow, st, i, p_begin, p_end);
+            else gather_row<EB, DIR, false>(P, row, srow, st, i, p_begin, p_end);
         }
         __syncthreads();  // this buffer is refilled two groups later
 
@@ -317,11 +358,9 @@ __device__ __forceinline__ void stage_stair(const RowParams &P, const char *mbas
 
 template <int EB, int DIR>
 __device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, char *srow, const unsigned char *buf,
-                                               const int32_t *padl, int32_t i, int wl, int wn) {
+                                               const int32_t *padl, int32_t i, int32_t p_begin, int32_t p_end) {
     using T = typename Word<EB>::T;
     const int lane = threadIdx.x & 31;
-    const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;
-    const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
     const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
     const int32_t Mi = P.M - i;
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
@@ -331,10 +370,11 @@ __device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, 
         // lagged output as in gather_row: p < shW -> side tile row, else row[p - shW]
         T *out = reinterpret_cast<T *>(mbase + static_cast<int64_t>(i) * pitch) - P.shW;
         C2RWalk<true> w(P, im, p);
-        for (; p - lane < P.shW && p < p_end; p += 32) {
-            const T v = *reinterpret_cast<const T *>(buf + padl[w.l] + w.src(P, Mi) * EB);
-            if (p < P.shW) reinterpret_cast<T *>(srow)[p] = v;
-            else out[p] = v;
+        const int32_t p_side = min(p_end, P.shW);
+        T *so = reinterpret_cast<T *>(srow);
+#pragma unroll 4
+        for (; p < p_side; p += 32) {
+            so[p] = *reinterpret_cast<const T *>(buf + padl[w.l] + w.src(P, Mi) * EB);
             w.next(P);
         }
 #pragma unroll 4
@@ -356,7 +396,7 @@ __device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, 
 }
 
 template <int EB, int DIR, int NBUF>
-__global__ void __launch_bounds__(kRowThreadsMax) row_rot_kernel(RowParams P) {
+__global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
     const uint32_t rowbuf = static_cast<uint32_t>(row_fused_smem_bytes(P, EB, DIR));
@@ -368,6 +408,8 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_rot_kernel(RowParams P) {
     const int64_t groups_total = static_cast<int64_t>(gpm) * P.batch;
     const int wn = (blockDim.x >> 5) / P.R;
     const int team = (threadIdx.x >> 5) / wn, wl = (threadIdx.x >> 5) - team * wn;
+    const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;
+    const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
 
     auto stage = [&](const RowGroup &G, int b) {
         char *mb = P.base + G.mat * P.mat_stride_bytes;
@@ -430,10 +472,10 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_rot_kernel(RowParams P) {
             const unsigned char *b = smem + buf * bufbytes + team * rowbuf;
             char *srow = P.shW ? side_matrix(P.side, P.sstride, G.mat, mbase) + i * P.spitch : nullptr;
             if (DIR == ROW_C2R) {
-                gather_row_rot<EB, DIR>(P, mbase, srow, b, reinterpret_cast<const int32_t *>(b + padoff), i, wl, wn);
+                gather_row_rot<EB, DIR>(P, mbase, srow, b, reinterpret_cast<const int32_t *>(b + padoff), i, p_begin, p_end);
             } else {
                 gather_row_rot<EB, DIR>(P, mbase, srow, b + (reinterpret_cast<uintptr_t>(mbase + i * pitch) & 15),
-                                        nullptr, i, wl, wn);
+                                        nullptr, i, p_begin, p_end);
             }
         }
         __syncthreads();  // this buffer is free again
