@@ -399,6 +399,7 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         const size_t fsm = row_fused_smem_bytes(rp, eb, pl.row_dir);
         if (fsm <= static_cast<size_t>(dev.smem_optin)) {
             rp.fuse = 1;
+            rp.vec = env_int("IPT_ROW_VEC", 1);
             rsm = fsm;
             pl.scratch = static_cast<size_t>(pl.M) * 4 +
                          (engine == ENG_C2R ? static_cast<size_t>(pl.c - 1) * pl.N * eb : 0);
@@ -466,7 +467,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_ROW_STAGE", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);

@@ -76,6 +76,7 @@ struct RowParams {
     // Fused rotation (c > 1, c <= kMaxFuseC; row_rot_kernel): the column rotation of the
     // engine (C2R pre-rotation Eq. 23 / R2C post-rotation Eq. 36) folded into this pass.
     int32_t fuse;
+    int32_t vec;             // fused C2R: vectorised gather for rows with f2 = 0 (IPT_ROW_VEC)
     int32_t R;               // rows per CTA stage (row groups; a power of two dividing the warps)
     FastDiv fd_gpm;          // ceil(M / R): row groups per matrix
     // Lagged layout shared with the column shuffle (col_tile.cu): logical columns [0, shW)

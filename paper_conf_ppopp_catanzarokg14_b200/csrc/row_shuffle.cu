@@ -356,6 +356,87 @@ __device__ __forceinline__ void stage_stair(const RowParams &P, const char *mbas
     }
 }
 
+// Fused C2R gather of a row with f2 = 0 (i < M - c + 1), vectorised: thread tt of the
+// row's team (T threads) writes the 16-byte chunks tt, tt + T, ... of the output row's
+// aligned chunk grid (chunk k = logical outputs [k K - oe, k K - oe + K), K = 16 / eb, oe =
+// the row's misalignment in elements; the lagged split at shW keeps the alignment, side
+// rows being placed like their rows) with one st.global.v4 -- a warp writes 512 contiguous
+// bytes -- and the partial chunks (row ends, a chunk straddling shW) element by element.
+// Sources: Eq. 31 with q = (p - i) mod N, src = (q mod c) b + (a^{-1} floor(q/c)) mod b,
+// stepped by 1 inside a chunk (l += 1; on l == c: l = 0, h += a^{-1}) and by D = T K between
+// a thread's chunks (dl = D mod c, dh = a^{-1} floor(D/c) mod b, one carry) -- a few
+// integer ops per element instead of a full stride-32 walk per element.
+template <int EB>
+__device__ __forceinline__ void gather_row_rot_c2r_vec(const RowParams &P, char *mbase, char *srow,
+                                                       const unsigned char *buf, const int32_t *padl, int32_t i,
+                                                       int32_t tt, int32_t T, int32_t dl, int32_t dh) {
+    constexpr int K = 16 / EB;
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    char *arow = mbase + static_cast<int64_t>(i) * pitch;
+    const int32_t oe = static_cast<int32_t>((reinterpret_cast<uintptr_t>(arow) & 15) / EB);
+    const int32_t nk = (P.N + oe + K - 1) / K;
+    int32_t k = tt;
+    if (k >= nk) return;
+    const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
+    int32_t q = k * K - oe - im;
+    q += q < 0 ? P.N : 0;
+    q += q < 0 ? P.N : 0;
+    const uint32_t col = fdiv(static_cast<uint32_t>(q), P.fd_c);
+    int32_t l = q - static_cast<int32_t>(col) * P.c;
+    int32_t h = static_cast<int32_t>(mulmod(static_cast<uint32_t>(P.ainv), col, P.fd_b, P.wide));
+    char *sbk = srow;                  // side row (logical p < shW)
+    char *abk = arow - P.shW * EB;     // A row (logical p >= shW)
+    for (; k < nk; k += T) {
+        const int32_t p0 = k * K - oe;
+        uint32_t v[4];
+        int32_t ll = l, hh = h;
+#pragma unroll
+        for (int e = 0; e < K; ++e) {
+            const uint32_t a = static_cast<uint32_t>(padl[ll] + (ll * P.b + hh) * EB);
+            if constexpr (EB == 4) {
+                v[e] = *reinterpret_cast<const uint32_t *>(buf + a);
+            } else if constexpr (EB == 8) {
+                const uint2 x = *reinterpret_cast<const uint2 *>(buf + a);
+                v[2 * e] = x.x;
+                v[2 * e + 1] = x.y;
+            } else {
+                const uint4 x = *reinterpret_cast<const uint4 *>(buf + a);
+                v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+            }
+            if (K > 1) {
+                ++ll;
+                if (ll == P.c) {
+                    ll = 0;
+                    hh += P.ainv;
+                    hh -= hh >= P.b ? P.b : 0;
+                }
+            }
+        }
+        const bool full = p0 >= 0 && p0 + K <= P.N && (p0 >= P.shW || p0 + K <= P.shW);
+        if (full) {
+            char *dst = (p0 < P.shW ? sbk : abk) + static_cast<int64_t>(p0) * EB;
+            stg16(dst, make_uint4(v[0], v[1], v[2], v[3]));
+        } else {
+#pragma unroll
+            for (int e = 0; e < K; ++e) {
+                const int32_t p = p0 + e;
+                if (p < 0 || p >= P.N) continue;
+                char *dst = (p < P.shW ? sbk : abk) + static_cast<int64_t>(p) * EB;
+                if constexpr (EB == 4) *reinterpret_cast<uint32_t *>(dst) = v[e];
+                else if constexpr (EB == 8) *reinterpret_cast<uint2 *>(dst) = make_uint2(v[2 * e], v[2 * e + 1]);
+                else *reinterpret_cast<uint4 *>(dst) = make_uint4(v[0], v[1], v[2], v[3]);
+            }
+        }
+        // next chunk of this thread: q += D
+        l += dl;
+        const bool carry = l >= P.c;
+        l -= carry ? P.c : 0;
+        h += dh + (carry ? P.ainv : 0);
+        h -= h >= P.b ? P.b : 0;
+        h -= h >= P.b ? P.b : 0;
+    }
+}
+
 template <int EB, int DIR>
 __device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, char *srow, const unsigned char *buf,
                                                const int32_t *padl, int32_t i, int32_t p_begin, int32_t p_end) {
@@ -410,6 +491,10 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P)
     const int team = (threadIdx.x >> 5) / wn, wl = (threadIdx.x >> 5) - team * wn;
     const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;
     const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
+    // vectorised C2R gather: the walk constants of a thread's chunk stride D = 32 wn 16 / eb
+    const int64_t vD = static_cast<int64_t>(wn) * 32 * (16 / EB);
+    const int32_t vdl = static_cast<int32_t>(vD % P.c);
+    const int32_t vdh = static_cast<int32_t>((static_cast<int64_t>(P.ainv) * ((vD / P.c) % P.b)) % P.b);
 
     auto stage = [&](const RowGroup &G, int b) {
         char *mb = P.base + G.mat * P.mat_stride_bytes;
@@ -472,7 +557,12 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P)
             const unsigned char *b = smem + buf * bufbytes + team * rowbuf;
             char *srow = P.shW ? side_matrix(P.side, P.sstride, G.mat, mbase) + i * P.spitch : nullptr;
             if (DIR == ROW_C2R) {
-                gather_row_rot<EB, DIR>(P, mbase, srow, b, reinterpret_cast<const int32_t *>(b + padoff), i, p_begin, p_end);
+                if (P.vec && i < P.M - P.c + 1)
+                    gather_row_rot_c2r_vec<EB>(P, mbase, srow, b, reinterpret_cast<const int32_t *>(b + padoff), i,
+                                               wl * 32 + (threadIdx.x & 31), wn * 32, vdl, vdh);
+                else
+                    gather_row_rot<EB, DIR>(P, mbase, srow, b, reinterpret_cast<const int32_t *>(b + padoff), i,
+                                            p_begin, p_end);
             } else {
                 gather_row_rot<EB, DIR>(P, mbase, srow, b + (reinterpret_cast<uintptr_t>(mbase + i * pitch) & 15),
                                         nullptr, i, p_begin, p_end);

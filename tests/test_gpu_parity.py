@@ -349,3 +349,18 @@ def test_lagged_tile_layouts(lagd):
                     assert got[o:o + m * n].tobytes() == oracle.ipt_c2r(hv[o:o + m * n], m, n).tobytes()
                 ipt.r2c_batched(x.data_ptr() + eb, batch, m * n + 5, m, n, elem_bytes=eb)
                 assert dev_bytes(x) == np.ascontiguousarray(host).tobytes()
+
+
+@pytest.mark.parametrize("vec", ["1", "0"])
+def test_fused_rotation_vector_gather(vec):
+    """Fused C2R rotation + row pass, rows with f2 = 0 gathered in 16-byte output chunks of
+    the row's aligned chunk grid (IPT_ROW_VEC=1: stepped walk, vector stores, element stores
+    at the row ends and at a chunk straddling the lagged split) vs the per-element walk
+    (IPT_ROW_VEC=0): gcd 2..32, misaligned rows, row groups, every element size, both lag
+    settings."""
+    shapes = [(1200, 1816), (1816, 1200), (96, 40), (640, 32 * 33), (2 * 1009, 2 * 1013), (30 * 37, 30 * 41),
+              (4 * 999, 4 * 250), (2 * 3001, 2 * 2203), (6 * 301, 6 * 77)]
+    for lag in ("1", "0"):
+        with env_var("IPT_ROW_VEC", vec), env_var("IPT_COL_LAG", lag):
+            for eb in (4, 8, 16):
+                run_packed(shapes, eb, ipt.c2r, "row", "c2r", seed=eb * 7 + len(vec))
