@@ -404,10 +404,18 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
 template <int EB, int MODE, int TWB>
 __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
+    // Unit order.  Barrier mode: a dispatch ticket (an atomic), so a tile's G members are G
+    // consecutive dispatches -- the whole group is co-resident.  Lagged layouts only ever wait
+    // for units of smaller index, and CTAs are dispatched in blockIdx order (the premise of
+    // single-pass scans' decoupled look-back), so the block index serves and the ticket's
+    // atomic round trip (~5 % of a loads-only pass, IPT_COL_DEBUG=3) is saved.
     __shared__ unsigned int s_ticket;
-    if (threadIdx.x == 0) s_ticket = P.dbg == 3 ? blockIdx.x : atomicAdd(P.ctr + kTicketSlot, 1u);
-    __syncthreads();
-    const unsigned int ticket = s_ticket;
+    unsigned int ticket = blockIdx.x;
+    if (P.lag == LAG_NONE && P.dbg != 3) {
+        if (threadIdx.x == 0) s_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
+        __syncthreads();
+        ticket = s_ticket;
+    }
     if (P.G == 1) {
         const uint64_t t_end = min(static_cast<uint64_t>(P.total_tiles), (static_cast<uint64_t>(ticket) + 1) * P.tpc);
         for (uint64_t tt = static_cast<uint64_t>(ticket) * P.tpc; tt < t_end; ++tt) {
