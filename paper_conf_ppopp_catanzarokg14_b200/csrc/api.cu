@@ -416,6 +416,7 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         while (rp.R * 2 <= nw && rp.R * 2 * rowbuf <= target) rp.R *= 2;
         rsm = rowbuf * rp.R;
     }
+    rp.db_max = env_int("IPT_ROW_DB_MAX", 112 * 1024);
     rp.fd_gpm = make_fastdiv(static_cast<uint32_t>((pl.M + rp.R - 1) / rp.R));
 
     ipt_status_t s = plan_col(dev, pl, engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.shuf);

@@ -71,7 +71,7 @@ __device__ __forceinline__ int32_t mod_M(int32_t v, uint32_t kshiftM, const Fast
 }
 
 // Shared-memory layout of one unit buffer:
-//   [orow B*4 | srow nslots*4 | sbase nslots*4 | rows]
+//   [orow B*8 | srow nslots*4 | sbase nslots*4 | rows]   (orow: C2R output row byte offsets)
 // rows: nslots input rows ("slots") of HS = TWB + 16 bytes, each the 16-byte-aligned hull
 // of its tile row; sbase[t] = shared address of slot t's first tile element.
 __host__ __device__ inline size_t al16(size_t x) { return (x + 15) & ~size_t(15); }
@@ -83,7 +83,7 @@ __host__ __device__ inline SmemLayout smem_layout(int64_t B, int W, int twb, int
     (void)eb;
     const size_t nslots = static_cast<size_t>(B) + W - 1;
     SmemLayout L;
-    size_t o = al16(static_cast<size_t>(B) * 4);
+    size_t o = al16(static_cast<size_t>(B) * 8);
     L.srow = o;
     o += al16(nslots * 4);
     L.sbase = o;
@@ -168,15 +168,16 @@ __device__ __forceinline__ int32_t dw_of(const ColParams &P, const Unit &U, int3
 }
 
 // Scattered row indices of a unit, computed by the whole CTA into shared memory:
-// C2R destinations orow[k] = q^{-1}((r0 + k - j0) mod M) (Eq. 34), R2C sources
+// C2R destinations orow[k] = q^{-1}((r0 + k - j0) mod M) (Eq. 34; stored as the row's byte
+// offset in the output location, so the store loop adds it to the column pointer), R2C sources
 // srow[t] = q^{-1}((r0 - W + 1 + t - j0) mod M).  R2C needs a __syncthreads before the load.
 template <int EB, int MODE, int TWB>
-__device__ __forceinline__ void unit_prepass(const ColParams &P, const Unit &U, int32_t *orow, int32_t *srow,
+__device__ __forceinline__ void unit_prepass(const ColParams &P, const Unit &U, int64_t *orow, int32_t *srow,
                                              int nthr) {
     constexpr int W = TWB / EB;
     if (MODE == COL_C2R_SHUF) {
         for (int32_t k = threadIdx.x; k < U.nrows; k += nthr)
-            orow[k] = qinv_of(P, mod_M(U.r0 + k - U.j0m, P.kshM, P.fd_M));
+            orow[k] = static_cast<int64_t>(qinv_of(P, mod_M(U.r0 + k - U.j0m, P.kshM, P.fd_M))) * U.out_pitch;
     }
     if (MODE == COL_R2C_SHUF) {
         for (int32_t t = threadIdx.x; t < U.nslots; t += nthr)
@@ -281,7 +282,7 @@ __device__ __forceinline__ void stg_elem(char *p, const uint32_t *v) {
 // of a row read a diagonal of the slot array, conflict-free in the banks (slot pitch
 // TWB + 16 bytes).
 template <int EB, int MODE, int TWB>
-__device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, const int32_t *orow,
+__device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, const int64_t *orow,
                                            const uint32_t *sbase, int nthr) {
     constexpr int W = TWB / EB;
     constexpr int LPR = W < 32 ? W : 32;  // lanes per tile row
@@ -305,7 +306,7 @@ __device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, co
 #pragma unroll 4
             for (; k < U.nrows; k += step) {
                 lds_elem<EB>(v, sb[k] + wo);
-                stg_elem<EB>(colp + static_cast<int64_t>(orow[k]) * pitch, v);
+                stg_elem<EB>(colp + orow[k], v);
             }
         } else {
             char *g = colp + static_cast<int64_t>(U.r0 + k) * pitch;
@@ -376,7 +377,7 @@ __device__ __forceinline__ Dep unit_dep(const ColParams &P, uint32_t tt) {
 template <int EB, int MODE, int TWB>
 __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *smem, uint32_t tt, int32_t r) {
     const SmemLayout L = smem_layout(P.B, TWB / EB, TWB, EB);
-    int32_t *orow = reinterpret_cast<int32_t *>(smem);
+    int64_t *orow = reinterpret_cast<int64_t *>(smem);
     int32_t *srow = reinterpret_cast<int32_t *>(smem + L.srow);
     uint32_t *sbase = reinterpret_cast<uint32_t *>(smem + L.sbase);
     const Unit U = unit_make<EB, MODE, TWB>(P, tt, r);
@@ -393,12 +394,22 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
     __syncthreads();  // every thread's staged data is in shared memory
     if (threadIdx.x == 0) {
-        if (D.arrive) asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(P.ctr + (tt % kCtrSlots)) : "memory");
+        // The arrival only says "this unit's reads of its input are complete" (write-after-
+        // read): every thread's cp.async copies have landed in shared memory (wait_group 0 +
+        // the barrier above) before it is issued, so no later write by a waiter can reach
+        // them, and a relaxed add suffices.  A release add compiles to MEMBAR.ALL.GPU, which
+        // waits on the SM's outstanding stores: 6-8 % of the pass (IPT_COL_DEBUG=7 keeps it).
+        if (D.arrive) {
+            if (P.dbg == 7)
+                asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(P.ctr + (tt % kCtrSlots)) : "memory");
+            else
+                asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" :: "l"(P.ctr + (tt % kCtrSlots)) : "memory");
+        }
         if (D.wait && P.dbg != 5)
             while (!ctr_reached(P, D.on)) __nanosleep(64);
     }
     __syncthreads();
-    if (P.dbg == 0) unit_store<EB, MODE, TWB>(P, U, orow, sbase, blockDim.x);  // 1, 3, 4 = loads only
+    if (P.dbg == 0 || P.dbg == 7) unit_store<EB, MODE, TWB>(P, U, orow, sbase, blockDim.x);  // 1, 3, 4, 5 = loads only
 }
 
 template <int EB, int MODE, int TWB>
@@ -558,7 +569,7 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
         const uint32_t stt = fdiv(st, P.fd_G);
         const Unit Us = unit_make<EB, MODE, TWB>(P, stt, static_cast<int32_t>(st - stt * P.G));
         unsigned char *sbuf = smem + sb * bufsz;
-        unit_store<EB, MODE, TWB>(P, Us, reinterpret_cast<const int32_t *>(sbuf),
+        unit_store<EB, MODE, TWB>(P, Us, reinterpret_cast<const int64_t *>(sbuf),
                                   reinterpret_cast<const uint32_t *>(sbuf + L.sbase), nwt);
     };
     int b = 0, k = 0;    // buffer / round of unit i
@@ -576,7 +587,7 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
         }
         const uint32_t tt = fdiv(t, P.fd_G);
         const Unit U = unit_make<EB, MODE, TWB>(P, tt, static_cast<int32_t>(t - tt * P.G));
-        int32_t *orow = reinterpret_cast<int32_t *>(buf);
+        int64_t *orow = reinterpret_cast<int64_t *>(buf);
         int32_t *srow = reinterpret_cast<int32_t *>(buf + L.srow);
         if (!U.skip) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, nwt);
         asm volatile("bar.sync 1, %0;" :: "r"(nwt) : "memory");  // srow / orow visible

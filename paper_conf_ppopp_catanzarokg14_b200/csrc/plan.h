@@ -78,6 +78,7 @@ struct RowParams {
     int32_t fuse;
     int32_t vec;             // fused C2R: vectorised gather for rows with f2 = 0 (IPT_ROW_VEC)
     int32_t R;               // rows per CTA stage (row groups; a power of two dividing the warps)
+    int32_t db_max;          // double-buffer the row stage while two buffers fit in this many bytes
     FastDiv fd_gpm;          // ceil(M / R): row groups per matrix
     // Lagged layout shared with the column shuffle (col_tile.cu): logical columns [0, shW)
     // of row i live in the side tile, side + (mat M + i) spitch; columns [shW, N) at A
@@ -120,7 +121,8 @@ struct ColParams {
     int32_t lagD;       // LAG_*: the lag in tiles (tiles 0..D-1 live in the side tiles)
     int64_t spitch;     // side row pitch: D TWB + (N eb mod 16) (rows as aligned as A's)
     int64_t sstride;    // side bytes reserved per matrix
-    int32_t dbg;        // measurement only (IPT_COL_DEBUG): 1 loads only, 3 + no ticket, 4 + no prepass
+    int32_t dbg;        // measurement only (IPT_COL_DEBUG): 1 loads only, 3 + no ticket, 4 + no prepass,
+                        // 5 loads only without the wait, 7 release arrivals
 };
 
 // Skinny engine storage: "location" L in [0, n] is row L of the n x N view, location n is

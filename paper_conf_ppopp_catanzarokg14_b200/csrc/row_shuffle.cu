@@ -511,9 +511,13 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P)
         }
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
-    auto set_flags = [&](const RowGroup &G) {  // the group's reads are complete (after a __syncthreads)
+    // The group's reads are complete (after cp.async.wait_group 0 and a __syncthreads): the
+    // flag only orders those completed reads before the neighbours' writes (write-after-
+    // read), so a relaxed store suffices -- a release store is a MEMBAR.ALL.GPU, which waits
+    // on the SM's outstanding stores (as col_tile.cu's arrivals).
+    auto set_flags = [&](const RowGroup &G) {
         if (threadIdx.x < G.nr)
-            asm volatile("st.release.gpu.global.u32 [%0], %1;"
+            asm volatile("st.relaxed.gpu.global.u32 [%0], %1;"
                          :: "l"(P.flags + G.mat * P.M + G.i0 + threadIdx.x), "r"(1u) : "memory");
     };
     auto wait_deps = [&](const RowGroup &G) {  // every row the group overwrites has been read
@@ -864,9 +868,10 @@ cudaError_t launch_row_rot_t(const RowParams &P, cudaStream_t st) {
 template <int EB, int DIR>
 cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
     if (P.fuse)
-        return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= 112 * 1024 ? launch_row_rot_t<EB, DIR, 2>(P, st)
+        return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max)
+                   ? launch_row_rot_t<EB, DIR, 2>(P, st)
                                                                          : launch_row_rot_t<EB, DIR, 1>(P, st);
-    return 2 * P.R * row_smem_bytes(P.N, EB) <= 112 * 1024 ? launch_row_t<EB, DIR, 2>(P, st)
+    return 2 * P.R * row_smem_bytes(P.N, EB) <= static_cast<size_t>(P.db_max) ? launch_row_t<EB, DIR, 2>(P, st)
                                                            : launch_row_t<EB, DIR, 1>(P, st);
 }
 
