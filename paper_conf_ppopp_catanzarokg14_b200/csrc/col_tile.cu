@@ -320,8 +320,9 @@ __device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, co
     }
 }
 
+// Arrival of a unit whose reads have completed (see col_tile_one: relaxed suffices).
 __device__ __forceinline__ void group_arrive(unsigned int *ctr) {
-    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
+    asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" :: "l"(ctr) : "memory");
 }
 
 // In-place hazard of a column pass, per tile (unit order = ticket order, tile-major):

@@ -180,6 +180,17 @@ __device__ __forceinline__ void gather_row(const RowParams &P, char *row, char *
     }
 }
 
+// Bulk prefetch of [p, p + bytes) into L2 (the CTA's threads, 4 KB each).
+__device__ __forceinline__ void prefetch_l2(const char *p, int64_t bytes) {
+    // cp.async.bulk.prefetch.L2: 16-byte aligned address and size
+    const uintptr_t a0 = (reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15);
+    const uintptr_t a1 = (reinterpret_cast<uintptr_t>(p) + bytes) & ~uintptr_t(15);
+    for (uintptr_t a = a0 + static_cast<uintptr_t>(threadIdx.x) * 4096; a < a1; a += blockDim.x * 4096ull) {
+        const uint32_t sz = a1 - a < 4096 ? static_cast<uint32_t>(a1 - a) : 4096u;
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(a), "r"(sz) : "memory");
+    }
+}
+
 // Stage one row with cp.async (no commit): smem byte (off + k) holds row byte k, off =
 // row & 15.  Whole 16-byte chunks of the row's aligned hull move with 16-byte copies (a
 // plain strided loop); the at most two partial chunks at the ends element by element
@@ -285,6 +296,9 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_shuffle_kernel(RowParam
             }
         } else {
             stage(G, 0);
+            // single buffer (rows > 56 KB): the next group streams into L2 meanwhile
+            if (ng < groups_total)
+                prefetch_l2(row_ptr(NG.mat, NG.i0), static_cast<int64_t>(NG.nr) * nbytes);
             asm volatile("cp.async.wait_group 0;" ::: "memory");
         }
         __syncthreads();
@@ -554,6 +568,8 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P)
         const RowGroup NG = row_group(P, ng, gpm);
         const bool more = ng < groups_total;
         if (NBUF == 2 && more) stage(NG, buf ^ 1);
+        if (NBUF == 1 && more)  // single buffer: the next group's rows stream into L2 meanwhile
+            prefetch_l2(P.base + NG.mat * P.mat_stride_bytes + NG.i0 * pitch, static_cast<int64_t>(NG.nr) * pitch);
         wait_deps(G);
 
         if (team < G.nr) {
@@ -740,15 +756,6 @@ __device__ __forceinline__ void gather_l2(const RowParams &P, const char *row, u
     else run(R2CWalk<TAIL>(P, im, p));
 }
 
-__device__ __forceinline__ void prefetch_l2(const char *p, int64_t bytes) {
-    // cp.async.bulk.prefetch.L2: 16-byte aligned address and size
-    const uintptr_t a0 = (reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15);
-    const uintptr_t a1 = (reinterpret_cast<uintptr_t>(p) + bytes) & ~uintptr_t(15);
-    for (uintptr_t a = a0 + static_cast<uintptr_t>(threadIdx.x) * 4096; a < a1; a += blockDim.x * 4096ull) {
-        const uint32_t sz = a1 - a < 4096 ? static_cast<uint32_t>(a1 - a) : 4096u;
-        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(a), "r"(sz) : "memory");
-    }
-}
 
 template <int EB, int DIR>
 __global__ void __launch_bounds__(kRowThreadsMax) row_cluster_l2_kernel(RowParams P) {
