@@ -343,30 +343,16 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_shuffle_kernel(RowParam
 template <int EB>
 __device__ __forceinline__ void stage_stair(const RowParams &P, const char *mbase, const char *wrapbase, int32_t i,
                                             uint32_t sbase, int32_t *padl) {
+    // Segment rho (source columns [rho b, rho b + b)) of the staircase comes from row i + rho
+    // (from `wrap` past the last row); each is staged like a row (stage_row_chunks: 16-byte
+    // copies of its aligned hull) into its own region, its byte k at rho segp + so + k.
     const int32_t Lb = P.b * EB;
-    const int32_t segp = P.segp;
-    const int32_t cps = segp >> 4;
-    const int32_t total = P.c * cps;
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
-    for (int32_t f = threadIdx.x; f < total; f += blockDim.x) {
-        const int32_t rho = static_cast<int32_t>(fdiv(static_cast<uint32_t>(f), P.fd_cps));
-        const int32_t k = f - rho * cps;
+    for (int32_t rho = 0; rho < P.c; ++rho) {
         const int32_t y = i + rho;
         const char *S = (y < P.M ? mbase + y * pitch : wrapbase + (y - P.M) * pitch) + static_cast<int64_t>(rho) * Lb;
-        const int32_t so = static_cast<int32_t>(reinterpret_cast<uintptr_t>(S) & 15);
-        const uint32_t seg_s = sbase + rho * segp;
-        if (k == 0) padl[rho] = rho * segp + so - rho * Lb;
-        const int32_t lo = 16 * k - so;  // segment byte at the start of this 16-byte chunk
-        if (lo >= Lb || lo + 16 <= 0) continue;
-        if (lo >= 0 && lo + 16 <= Lb) {
-            cp_async<16>(seg_s + 16 * k, S + lo);
-        } else {
-#pragma unroll
-            for (int e = 0; e < 16 / EB; ++e) {
-                const int32_t q = lo + e * EB;
-                if (q >= 0 && q < Lb) cp_async<EB>(seg_s + so + q, S + q);
-            }
-        }
+        if (threadIdx.x == 0) padl[rho] = rho * P.segp + static_cast<int32_t>(reinterpret_cast<uintptr_t>(S) & 15) - rho * Lb;
+        stage_row_chunks<EB>(S, Lb, sbase + rho * P.segp);
     }
 }
 
