@@ -574,12 +574,19 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P)
                                         nullptr, i, p_begin, p_end);
             }
         }
-        __syncthreads();  // this buffer is free again
-        if (more) {
-            if (NBUF == 1) stage(NG, 0);
+        if (NBUF == 2) {
+            // one barrier: this buffer is free again AND the prefetched group has landed
             asm volatile("cp.async.wait_group 0;" ::: "memory");
             __syncthreads();
-            set_flags(NG);
+            if (more) set_flags(NG);
+        } else {
+            __syncthreads();  // this buffer is free again
+            if (more) {
+                stage(NG, 0);
+                asm volatile("cp.async.wait_group 0;" ::: "memory");
+                __syncthreads();
+                set_flags(NG);
+            }
         }
         if (NBUF == 2) buf ^= 1;
         G = NG;
