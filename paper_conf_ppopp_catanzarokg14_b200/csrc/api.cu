@@ -110,7 +110,7 @@ int ilog2(int v) {
 
 // Column-tile geometry.  Tile width TWB = IPT_TILE_BYTES (32, 64 or 128; default 128 B =
 // one cache line).  Band: the rows per CTA that fit the per-CTA shared-memory target
-// IPT_COL_SMEM (default 46 KiB, four CTAs per SM: the best of the round-1 sweep over
+// IPT_COL_SMEM (default 54000 B, four CTAs per SM: the best of the round-1 sweeps over
 // 12-100 KiB, profiles/r01_*).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
 // the co-resident CTAs, the band grows (up to the opt-in shared-memory maximum).
 ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe);
@@ -128,7 +128,7 @@ ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &c
     if (twb != 128 && twb != 256 && twb != 512) twb = 128;
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
     const int nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
-    const int64_t target = env_int("IPT_COL_SMEM", 46 * 1024);
+    const int64_t target = env_int("IPT_COL_SMEM", 54000);
     const int64_t W = twb / pl.eb;
     // Largest band whose buffer fits the target (col_smem_bytes: staged rows + row indices).
     int64_t B = target / (twb + 8);
@@ -407,12 +407,12 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     }
 
     // Row groups: R consecutive rows per CTA stage while R rows stay within IPT_ROW_STAGE
-    // bytes (default 16 KiB), so that short rows still keep enough bytes in flight per SM.
+    // bytes (default 32 KiB), so that short rows still keep enough bytes in flight per SM.
     rp.R = 1;
     if (!use_cluster) {
         const size_t rowbuf = rp.fuse ? row_fused_smem_bytes(rp, eb, pl.row_dir) : row_smem_bytes(pl.N, eb);
         const int nw = row_threads(pl.N, eb) / 32;
-        const size_t target = static_cast<size_t>(env_int("IPT_ROW_STAGE", 16384));
+        const size_t target = static_cast<size_t>(env_int("IPT_ROW_STAGE", 32768));
         while (rp.R * 2 <= nw && rp.R * 2 * rowbuf <= target) rp.R *= 2;
         rsm = rowbuf * rp.R;
     }
