@@ -19,6 +19,8 @@
 //                                structs (same pointer in every lane, 4-byte aligned);
 //                                afterwards r[k] = chunk[lane*S + k].
 //   warp_store_aos<S>(chunk, r): inverse: chunk[lane*S + k] = r[k].
+//   warp_gather_aos<S>(base, idx, r) / warp_scatter_aos<S>(base, idx, r): random access,
+//                                lane l's struct base[idx_l*S .. idx_l*S + S) (below).
 //   coalesced_ptr<T>: Fig. 10 interface (:1089-1097): `T v = *cp;` / `*cp = v;`.  Uses the
 //                     cooperative path when the whole warp is converged and the lanes'
 //                     pointers are unit-stride (p_lane == p_0 + lane); otherwise a plain
@@ -161,6 +163,42 @@ __device__ __forceinline__ void warp_store_aos(uint32_t *chunk, uint32_t (&r)[S]
     c2r_registers<S>(r);
 #pragma unroll
     for (int k = 0; k < S; ++k) chunk[k * 32 + j] = r[k];  // S coalesced 128-byte stores
+}
+
+// Random-access AoS gather / scatter (SURVEY §8 row f1; PAPER.md :1087, :1099, Fig. 9):
+// lane l wants struct idx_l (any index, repeats allowed for the gather) of an S-word AoS
+// array.  The 32 structs are treated as one virtual contiguous 32*S-word chunk: virtual
+// word v = k*32 + l is word (v mod S) of lane (v / S)'s struct, whose index the warp
+// exchanges with one __shfl_sync per register ("shuffle indices across lanes"); register k
+// of lane l loads it, so each load instruction fetches whole structs cooperatively (32/S
+// structs, their words contiguous) instead of one word of 32 scattered structs.  The
+// register array is then exactly the unit-stride chunk of warp_load_aos, and R2C(S, 32)
+// hands lane l its struct.  The scatter is the inverse (C2R(S, 32), then the cooperative
+// stores); with repeated indices the stored value is that of one of the lanes.
+//   warp_gather_aos<S>(base, idx, r):  r[k] = base[idx * S + k]   (all 32 lanes)
+//   warp_scatter_aos<S>(base, idx, r): base[idx * S + k] = r[k]
+template <int S>
+__device__ __forceinline__ void warp_gather_aos(const uint32_t *base, uint32_t idx, uint32_t (&r)[S]) {
+    const int j = aos_detail::lane_id();
+#pragma unroll
+    for (int k = 0; k < S; ++k) {
+        const int v = k * 32 + j;  // virtual word: word v % S of the struct of lane v / S
+        const uint32_t owner_idx = __shfl_sync(0xffffffffu, idx, v / S);
+        r[k] = base[static_cast<uint64_t>(owner_idx) * S + (v % S)];
+    }
+    r2c_registers<S>(r);
+}
+
+template <int S>
+__device__ __forceinline__ void warp_scatter_aos(uint32_t *base, uint32_t idx, uint32_t (&r)[S]) {
+    const int j = aos_detail::lane_id();
+    c2r_registers<S>(r);
+#pragma unroll
+    for (int k = 0; k < S; ++k) {
+        const int v = k * 32 + j;
+        const uint32_t owner_idx = __shfl_sync(0xffffffffu, idx, v / S);
+        base[static_cast<uint64_t>(owner_idx) * S + (v % S)] = r[k];
+    }
 }
 
 // Fig. 10: `coalesced_ptr<T> c_ptr(ptr); T v = *c_ptr; *c_ptr = v;`

@@ -42,6 +42,17 @@ ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes
 ipt_status_t ipt_debug_aos_copy(const void *src, void *dst, int64_t count, int words, int variant, void *stream);
 ipt_status_t ipt_debug_aos_fill(void *dst, int64_t count, int words, int variant, void *stream);
 ipt_status_t ipt_debug_warp_load_dump(const void *src, void *dump, int64_t nchunks, int words, void *stream);
+/*
+ * Random-access consumers (SURVEY §8 row f1; PAPER.md :1087, :1099, Fig. 9) of
+ * warp_gather_aos / warp_scatter_aos: ipt_debug_aos_gather: dst[k] = src[idx[k]];
+ * ipt_debug_aos_scatter: dst[idx[k]] = src[k] (idx a permutation for a defined result).
+ * `count` structs of `words` words; idx[k] < number of structs of src (gather) / dst
+ * (scatter); variants as above (COALESCED = the cooperative helpers on whole warps).
+ */
+ipt_status_t ipt_debug_aos_gather(const void *src, const uint32_t *idx, void *dst, int64_t count, int words,
+                                  int variant, void *stream);
+ipt_status_t ipt_debug_aos_scatter(const void *src, const uint32_t *idx, void *dst, int64_t count, int words,
+                                   int variant, void *stream);
 ipt_status_t ipt_debug_warp_store(const void *regs, void *dst, int64_t nchunks, int words, void *stream);
 
 #ifdef __cplusplus

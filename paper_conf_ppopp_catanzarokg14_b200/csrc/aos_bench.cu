@@ -80,6 +80,45 @@ __global__ void __launch_bounds__(256) aos_kernel(const Words<S> *src, Words<S> 
     }
 }
 
+// Random access (Fig. 9): gather dst[k] = src[idx[k]] / scatter
+// dst[idx[k]] = src[k].  DIRECT: per-lane struct access (compiler-generated); COALESCED:
+// warp_gather_aos + warp_store_aos / warp_load_aos + warp_scatter_aos on whole warps, the
+// tail warp per lane.  (VECTOR is treated as DIRECT with native vectors.)
+template <int S, int VARIANT, bool GATHER>
+__global__ void __launch_bounds__(256) aos_random_kernel(const Words<S> *src, const uint32_t *idx, Words<S> *dst,
+                                                         int64_t count) {
+    const int64_t nthreads = static_cast<int64_t>(gridDim.x) * blockDim.x;
+    for (int64_t k = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x; k - (threadIdx.x & 31) < count;
+         k += nthreads) {
+        const int64_t k0 = k - (threadIdx.x & 31);
+        if (VARIANT == IPT_AOS_COALESCED && k0 + 32 <= count) {  // whole warp: cooperative
+            uint32_t r[S];
+            const uint32_t j = idx[k];
+            if (GATHER) {
+                warp_gather_aos<S>(reinterpret_cast<const uint32_t *>(src), j, r);
+                warp_store_aos<S>(reinterpret_cast<uint32_t *>(dst + k0), r);
+            } else {
+                warp_load_aos<S>(reinterpret_cast<const uint32_t *>(src + k0), r);
+                warp_scatter_aos<S>(reinterpret_cast<uint32_t *>(dst), j, r);
+            }
+            continue;
+        }
+        if (k >= count) continue;
+        const uint32_t j = idx[k];
+        if (VARIANT == IPT_AOS_VECTOR) {
+            if (GATHER) vec_copy<S>(src + j, dst + k);
+            else vec_copy<S>(src + k, dst + j);
+        } else {
+            if (GATHER) dst[k] = src[j];
+            else dst[j] = src[k];
+        }
+    }
+}
+
+template <int S>
+cudaError_t run_random(const void *src, const uint32_t *idx, void *dst, int64_t count, int variant, bool gather,
+                       cudaStream_t st);
+
 // warp_load_aos dump: chunk c of 32 structs -> dump[c*32*S + lane*S + k] = r[k].
 template <int S>
 __global__ void warp_load_dump_kernel(const uint32_t *src, uint32_t *dump, int64_t nchunks) {
@@ -146,17 +185,46 @@ cudaError_t run_dump(const void *in, void *out, int64_t nchunks, bool load, cuda
     return cudaGetLastError();
 }
 
+int grid_for(int64_t count);
+
+template <int S>
+cudaError_t run_random(const void *src, const uint32_t *idx, void *dst, int64_t count, int variant, bool gather,
+                       cudaStream_t st) {
+    const auto *s = static_cast<const Words<S> *>(src);
+    auto *d = static_cast<Words<S> *>(dst);
+    const int grid = grid_for(count);
+#define IPT_AOS_RLAUNCH(V, G) aos_random_kernel<S, V, G><<<grid, 256, 0, st>>>(s, idx, d, count)
+    if (gather) {
+        if (variant == IPT_AOS_DIRECT) IPT_AOS_RLAUNCH(IPT_AOS_DIRECT, true);
+        else if (variant == IPT_AOS_VECTOR) IPT_AOS_RLAUNCH(IPT_AOS_VECTOR, true);
+        else IPT_AOS_RLAUNCH(IPT_AOS_COALESCED, true);
+    } else {
+        if (variant == IPT_AOS_DIRECT) IPT_AOS_RLAUNCH(IPT_AOS_DIRECT, false);
+        else if (variant == IPT_AOS_VECTOR) IPT_AOS_RLAUNCH(IPT_AOS_VECTOR, false);
+        else IPT_AOS_RLAUNCH(IPT_AOS_COALESCED, false);
+    }
+#undef IPT_AOS_RLAUNCH
+    return cudaGetLastError();
+}
+
 template <int... Ss>
 struct Dispatch;
 template <>
 struct Dispatch<> {
     static cudaError_t aos(int, const void *, void *, int64_t, int, bool, cudaStream_t) { return cudaErrorInvalidValue; }
+    static cudaError_t random(int, const void *, const uint32_t *, void *, int64_t, int, bool, cudaStream_t) {
+        return cudaErrorInvalidValue;
+    }
     static cudaError_t dump(int, const void *, void *, int64_t, bool, cudaStream_t) { return cudaErrorInvalidValue; }
 };
 template <int S0, int... Ss>
 struct Dispatch<S0, Ss...> {
     static cudaError_t aos(int S, const void *a, void *b, int64_t n, int v, bool c, cudaStream_t st) {
         return S == S0 ? run_aos<S0>(a, b, n, v, c, st) : Dispatch<Ss...>::aos(S, a, b, n, v, c, st);
+    }
+    static cudaError_t random(int S, const void *a, const uint32_t *ix, void *b, int64_t n, int v, bool g,
+                              cudaStream_t st) {
+        return S == S0 ? run_random<S0>(a, ix, b, n, v, g, st) : Dispatch<Ss...>::random(S, a, ix, b, n, v, g, st);
     }
     static cudaError_t dump(int S, const void *a, void *b, int64_t n, bool l, cudaStream_t st) {
         return S == S0 ? run_dump<S0>(a, b, n, l, st) : Dispatch<Ss...>::dump(S, a, b, n, l, st);
@@ -187,6 +255,24 @@ ipt_status_t ipt_debug_aos_fill(void *dst, int64_t count, int words, int variant
     if (!dst || count < 0 || words < 1 || words > 32 || variant < 0 || variant > 2) return IPT_ERR_INVALID_ARGUMENT;
     if (count == 0) return IPT_OK;
     return ipt::to_status(ipt::AllS::aos(words, nullptr, dst, count, variant, false, static_cast<cudaStream_t>(stream)));
+}
+
+ipt_status_t ipt_debug_aos_gather(const void *src, const uint32_t *idx, void *dst, int64_t count, int words,
+                                  int variant, void *stream) {
+    if (!src || !idx || !dst || count < 0 || words < 1 || words > 32 || variant < 0 || variant > 2)
+        return IPT_ERR_INVALID_ARGUMENT;
+    if (count == 0) return IPT_OK;
+    return ipt::to_status(
+        ipt::AllS::random(words, src, idx, dst, count, variant, true, static_cast<cudaStream_t>(stream)));
+}
+
+ipt_status_t ipt_debug_aos_scatter(const void *src, const uint32_t *idx, void *dst, int64_t count, int words,
+                                   int variant, void *stream) {
+    if (!src || !idx || !dst || count < 0 || words < 1 || words > 32 || variant < 0 || variant > 2)
+        return IPT_ERR_INVALID_ARGUMENT;
+    if (count == 0) return IPT_OK;
+    return ipt::to_status(
+        ipt::AllS::random(words, src, idx, dst, count, variant, false, static_cast<cudaStream_t>(stream)));
 }
 
 ipt_status_t ipt_debug_warp_load_dump(const void *src, void *dump, int64_t nchunks, int words, void *stream) {

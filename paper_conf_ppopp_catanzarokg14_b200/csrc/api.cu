@@ -108,7 +108,7 @@ int ilog2(int v) {
     return l;
 }
 
-// Column-tile geometry.  Tile width TWB = IPT_TILE_BYTES (32, 64 or 128; default 128 B =
+// Column-tile geometry.  Tile width TWB = IPT_TILE_BYTES (128, 256 or 512; default 128 B =
 // one cache line).  Band: the rows per CTA that fit the per-CTA shared-memory target
 // IPT_COL_SMEM (default 54000 B, four CTAs per SM: the best of the round-1 sweeps over
 // 12-100 KiB, profiles/r01_*).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
