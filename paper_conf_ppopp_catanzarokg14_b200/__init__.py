@@ -29,7 +29,8 @@ STATUS = {0: "IPT_OK", 1: "IPT_ERR_INVALID_ARGUMENT", 2: "IPT_ERR_UNSUPPORTED",
 EXPORTS = ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_status_string", "ipt_plan_info",
            "ipt_launch_count", "ipt_profile_enable", "ipt_profile_read", "ipt_debug_tile_copy",
-           "ipt_debug_aos_copy", "ipt_debug_aos_fill", "ipt_debug_warp_load_dump", "ipt_debug_warp_store")
+           "ipt_debug_aos_copy", "ipt_debug_aos_fill", "ipt_debug_warp_load_dump", "ipt_debug_warp_store",
+           "ipt_debug_aos_gather", "ipt_debug_aos_scatter")
 AOS_DIRECT, AOS_VECTOR, AOS_COALESCED = 0, 1, 2
 PROFILE_KINDS = 8
 KERNEL_KINDS = ("row_shuffle", "col_shuffle", "col_rotate", "skinny")
@@ -70,7 +71,10 @@ _lib.ipt_debug_aos_copy.argtypes = [_vp, _vp, _i64, _int, _int, _vp]
 _lib.ipt_debug_aos_fill.argtypes = [_vp, _i64, _int, _int, _vp]
 _lib.ipt_debug_warp_load_dump.argtypes = [_vp, _vp, _i64, _int, _vp]
 _lib.ipt_debug_warp_store.argtypes = [_vp, _vp, _i64, _int, _vp]
-for _f in ("ipt_debug_aos_copy", "ipt_debug_aos_fill", "ipt_debug_warp_load_dump", "ipt_debug_warp_store"):
+_lib.ipt_debug_aos_gather.argtypes = [_vp, _vp, _vp, _i64, _int, _int, _vp]
+_lib.ipt_debug_aos_scatter.argtypes = [_vp, _vp, _vp, _i64, _int, _int, _vp]
+for _f in ("ipt_debug_aos_copy", "ipt_debug_aos_fill", "ipt_debug_warp_load_dump", "ipt_debug_warp_store",
+           "ipt_debug_aos_gather", "ipt_debug_aos_scatter"):
     getattr(_lib, _f).restype = _int
 for _f in ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_plan_info"):
@@ -209,6 +213,18 @@ def aos_copy(src, dst, count: int, words: int, variant: int, stream=None):
 def aos_fill(dst, count: int, words: int, variant: int, stream=None):
     _check(_lib.ipt_debug_aos_fill(dst.data_ptr(), count, words, variant, _dev_stream(dst, stream)),
            "ipt_debug_aos_fill")
+
+
+def aos_gather(src, idx, dst, count: int, words: int, variant: int, stream=None):
+    """Random-access consumer dst[k] = src[idx[k]] (include/ipt_debug.h)."""
+    _check(_lib.ipt_debug_aos_gather(src.data_ptr(), idx.data_ptr(), dst.data_ptr(), count, words, variant,
+                                     _dev_stream(dst, stream)), "ipt_debug_aos_gather")
+
+
+def aos_scatter(src, idx, dst, count: int, words: int, variant: int, stream=None):
+    """Random-access consumer dst[idx[k]] = src[k] (idx a permutation)."""
+    _check(_lib.ipt_debug_aos_scatter(src.data_ptr(), idx.data_ptr(), dst.data_ptr(), count, words, variant,
+                                      _dev_stream(dst, stream)), "ipt_debug_aos_scatter")
 
 
 def warp_load_dump(src, dump, nchunks: int, words: int, stream=None):

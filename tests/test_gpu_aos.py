@@ -58,3 +58,28 @@ def test_consumer_variants_agree(S, count):
         dst.zero_()
         ipt.aos_fill(dst, count, S, variant)
         assert np.array_equal(dst.cpu().numpy(), ref_fill), (S, count, variant)
+
+
+@pytest.mark.parametrize("S", [1, 2, 3, 4, 5, 7, 8, 12, 16, 24, 31, 32])
+@pytest.mark.parametrize("count", [32 * 500, 32 * 500 + 7, 9])
+def test_random_access_gather_scatter(S, count):
+    """warp_gather_aos / warp_scatter_aos (row f1, PAPER.md :1087, :1099): gather with a
+    random index vector (repeats allowed) equals numpy fancy indexing of the structs; scatter
+    through a random permutation equals numpy's inverse assignment; direct, vector and
+    cooperative variants agree; partial tail warps take the per-lane path."""
+    rng = np.random.default_rng(S * 1000 + count)
+    nsrc = count + 37
+    src_h = workloads.random_words(nsrc * S, 4, seed=S + count).reshape(nsrc, S)
+    idx_h = rng.integers(0, nsrc, size=count, dtype=np.uint32)
+    want = src_h[idx_h]
+    perm = rng.permutation(count).astype(np.uint32)
+    want_sc = np.zeros((count, S), dtype=np.uint32)
+    want_sc[perm] = src_h[:count]
+    src, idx, pidx = dev(src_h.reshape(-1)), dev(idx_h), dev(perm)
+    for variant in (ipt.AOS_DIRECT, ipt.AOS_VECTOR, ipt.AOS_COALESCED):
+        dst = torch.zeros(count * S, dtype=torch.uint32, device="cuda")
+        ipt.aos_gather(src, idx, dst, count, S, variant)
+        assert np.array_equal(dst.cpu().numpy().reshape(count, S), want), (S, count, variant)
+        dst.zero_()
+        ipt.aos_scatter(src, pidx, dst, count, S, variant)
+        assert np.array_equal(dst.cpu().numpy().reshape(count, S), want_sc), (S, count, variant)
