@@ -466,6 +466,34 @@ __device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, 
     } else {
         const T *src = reinterpret_cast<const T *>(buf);
         R2CWalk<true> w(P, im, p);
+        if (i < P.M - P.c + 1) {
+            // f2 = 0 in the whole row: the source walk without the f2 term, and the
+            // destination (row i + l, column p) as one running pointer that moves by 32
+            // columns plus (32 div b + carry) rows per step
+            uint32_t sidx = static_cast<uint32_t>(w.s);
+            int32_t h = w.h, r = i + w.l;
+            r -= r >= P.M ? P.M : 0;
+            char *dst = mbase + static_cast<int64_t>(r) * pitch + static_cast<int64_t>(p) * EB;
+            const int64_t wrap = static_cast<int64_t>(P.M) * pitch;
+            const uint32_t n = static_cast<uint32_t>(P.N);
+#pragma unroll 4
+            for (; p < p_end; p += 32) {
+                *reinterpret_cast<T *>(dst) = src[sidx];
+                h += P.w_dh;
+                const int32_t carry = h >= P.b ? 1 : 0;
+                h -= carry ? P.b : 0;
+                sidx += static_cast<uint32_t>(P.w_ds + carry);
+                sidx -= sidx >= n ? n : 0;
+                const int32_t dl = P.w_dl2 + carry;
+                r += dl;
+                dst += 32 * EB + static_cast<int64_t>(dl) * pitch;
+                if (r >= P.M) {
+                    r -= P.M;
+                    dst -= wrap;
+                }
+            }
+            return;
+        }
 #pragma unroll 4
         for (; p < p_end; p += 32) {
             int32_t r = i + w.l;
