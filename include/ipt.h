@@ -18,6 +18,14 @@
  *
  * Element size: elem_bytes in {4, 8, 16}.  Elements are opaque words (bit-exact moves,
  * no floating-point semantics; NaN payloads, -0.0 and subnormals are preserved).
+ *
+ * Multi-word elements (records): elem_bytes = k*w for any multiple of 4 up to 4096 that is
+ * not 4, 8 or 16 (12, 24, 32, 48, 64 B ...).  `ptr` then needs 4-byte alignment only; w is
+ * the largest of 16, 8, 4 dividing both elem_bytes and the address.  Such a call runs two
+ * word-level permutations of the same engine (the paper's passes move opaque words of any
+ * size): P_{x,y} on k-word elements = P_{x,y*k} on w-byte words
+ * followed by P_{k,x} on each of the y k-by-x blocks, so it moves the buffer twice.  A
+ * strided batch (stride_elems > m*n) runs the second step once per matrix.
  */
 #ifndef IPT_H_
 #define IPT_H_
@@ -37,7 +45,8 @@ typedef enum {
 typedef enum {
     IPT_OK = 0,
     IPT_ERR_INVALID_ARGUMENT = 1, /* negative dims, bad elem_bytes/layout, NULL or misaligned
-                                     ptr, stride < m*n, size overflow; buffer untouched      */
+                                     ptr (to elem_bytes for 4/8/16, else to 4), stride < m*n,
+                                     size overflow; buffer untouched                         */
     IPT_ERR_UNSUPPORTED = 2,      /* shape beyond the implemented on-chip staging limits, or
                                      the device is not sm_100; buffer untouched              */
     IPT_ERR_OUT_OF_MEMORY = 3,    /* scratch allocation failed; buffer untouched            */
@@ -101,7 +110,9 @@ ipt_status_t ipt_soa_to_aos(void *ptr, int64_t count, int64_t fields, int field_
  * rotation one flag per row plus (C2R) gcd(m, n) - 1 wrapped rows; the skinny engine one row
  * of the long dimension.  Batched calls scale it by the batch (the side block capped at
  * max(256 MiB, 1/32 of the data)).  *onchip_per_cta: the largest shared-memory staging buffer
- * of any launched CTA.  Either pointer may be NULL.
+ * of any launched CTA.  Multi-word elem_bytes: the larger of the two word-level steps
+ * (P_{m,n*k} and one P_{k,m} block, words as wide as a 16-byte-aligned base allows).  Either
+ * pointer may be NULL.
  */
 ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *global_bytes,
                                size_t *onchip_per_cta);
@@ -117,7 +128,9 @@ const char *ipt_status_string(ipt_status_t s);
  * column-tile width in elements, out[7] largest on-chip staging bytes per CTA, out[8]
  * CTAs per row of the row pass (0: one CTA per row; K > 0: a K-CTA cluster sharing the
  * row through distributed shared memory, for rows longer than one CTA's shared memory),
- * out[9] global scratch bytes.  Returns IPT_ERR_UNSUPPORTED for shapes beyond limits.
+ * out[9] global scratch bytes.  Multi-word elem_bytes: out[0..3], out[5..9] describe the
+ * first word-level step P_{x,y*k}; out[4] counts the launches of both steps (one matrix).
+ * Returns IPT_ERR_UNSUPPORTED for shapes beyond limits.
  */
 #define IPT_PLAN_INFO_FIELDS 10
 ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,

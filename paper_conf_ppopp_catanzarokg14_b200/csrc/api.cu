@@ -721,6 +721,44 @@ ipt_status_t run_perm(void *ptr, int64_t batch, int64_t stride, int64_t x, int64
     return execute(pl, static_cast<char *>(ptr), batch, stride * eb, static_cast<cudaStream_t>(stream));
 }
 
+// Multi-word elements (the paper's passes move opaque words whatever their
+// size, :1037, :1085).  An element of eb = k*w bytes (w = 16, 8 or 4: the largest that
+// divides both eb and the base address) is moved by two word-level permutations of the
+// engine: P_{x,y} on k-word elements = P_{x,y*k} on words (output row j*k + v holds word v
+// of column j), then P_{k,x} on each of the y k-by-x blocks (block j becomes x rows of k
+// words, i.e. row j of the y-by-x result).  Buffer traffic: twice the one-step engine.
+constexpr int kMaxElemBytes = 4096;
+bool valid_multiword_eb(int eb) { return eb > 0 && eb % 4 == 0 && eb <= kMaxElemBytes && !valid_eb(eb); }
+
+int word_bytes_of(int eb, uintptr_t addr) {
+    for (int w : {16, 8}) if (eb % w == 0 && addr % w == 0) return w;
+    return 4;
+}
+
+ipt_status_t run_perm_any(void *ptr, int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, void *stream) {
+    if (!valid_multiword_eb(eb)) return run_perm(ptr, batch, stride, x, y, eb, stream);
+    if (x < 0 || y < 0 || batch < 0) return IPT_ERR_INVALID_ARGUMENT;
+    if (x != 0 && y > INT64_MAX / x) return IPT_ERR_INVALID_ARGUMENT;
+    const int64_t elems = x * y;
+    const bool packed = stride < 0;
+    if (packed) stride = elems;
+    if (stride < elems) return IPT_ERR_INVALID_ARGUMENT;
+    if (stride != 0 && batch > INT64_MAX / stride) return IPT_ERR_INVALID_ARGUMENT;
+    if (elems != 0 && batch * stride > INT64_MAX / eb) return IPT_ERR_INVALID_ARGUMENT;
+    if (elems == 0 || batch == 0) return IPT_OK;
+    if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % 4 != 0) return IPT_ERR_INVALID_ARGUMENT;
+    if (x <= 1 || y <= 1) return IPT_OK;
+    const int w = word_bytes_of(eb, reinterpret_cast<uintptr_t>(ptr));
+    const int64_t k = eb / w;
+    ipt_status_t s = run_perm(ptr, batch, stride * k, x, y * k, w, stream);  // P_{x, y k}
+    if (s != IPT_OK) return s;
+    if (batch == 1 || stride == elems)  // every k-by-x block of every matrix is k*x words apart
+        return run_perm(ptr, batch * y, k * x, k, x, w, stream);
+    for (int64_t b = 0; b < batch && s == IPT_OK; ++b)
+        s = run_perm(static_cast<char *>(ptr) + b * stride * eb, y, k * x, k, x, w, stream);
+    return s;
+}
+
 // Export -> P_{x,y} (reading C18): c2r(m,n,ROW) = P_{m,n}, c2r(m,n,COL) = P_{n,m};
 // r2c is the inverse: r2c(m,n,ROW) = P_{n,m}, r2c(m,n,COL) = P_{m,n}.
 bool perm_of(bool c2r, int64_t m, int64_t n, int layout, int64_t &x, int64_t &y) {
@@ -807,41 +845,55 @@ extern "C" {
 ipt_status_t ipt_c2r(void *ptr, int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout, void *stream) {
     int64_t x, y;
     if (!perm_of(true, m, n, layout, x, y)) return IPT_ERR_INVALID_ARGUMENT;
-    return run_perm(ptr, 1, -1, x, y, elem_bytes, stream);
+    return run_perm_any(ptr, 1, -1, x, y, elem_bytes, stream);
 }
 
 ipt_status_t ipt_r2c(void *ptr, int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout, void *stream) {
     int64_t x, y;
     if (!perm_of(false, m, n, layout, x, y)) return IPT_ERR_INVALID_ARGUMENT;
-    return run_perm(ptr, 1, -1, x, y, elem_bytes, stream);
+    return run_perm_any(ptr, 1, -1, x, y, elem_bytes, stream);
 }
 
 ipt_status_t ipt_c2r_batched(void *base, int64_t batch, int64_t stride_elems, int64_t m, int64_t n, int elem_bytes,
                              ipt_layout_t layout, void *stream) {
     int64_t x, y;
     if (stride_elems < 0 || !perm_of(true, m, n, layout, x, y)) return IPT_ERR_INVALID_ARGUMENT;
-    return run_perm(base, batch, stride_elems, x, y, elem_bytes, stream);
+    return run_perm_any(base, batch, stride_elems, x, y, elem_bytes, stream);
 }
 
 ipt_status_t ipt_r2c_batched(void *base, int64_t batch, int64_t stride_elems, int64_t m, int64_t n, int elem_bytes,
                              ipt_layout_t layout, void *stream) {
     int64_t x, y;
     if (stride_elems < 0 || !perm_of(false, m, n, layout, x, y)) return IPT_ERR_INVALID_ARGUMENT;
-    return run_perm(base, batch, stride_elems, x, y, elem_bytes, stream);
+    return run_perm_any(base, batch, stride_elems, x, y, elem_bytes, stream);
 }
 
 ipt_status_t ipt_aos_to_soa(void *ptr, int64_t count, int64_t fields, int field_bytes, void *stream) {
-    return run_perm(ptr, 1, -1, count, fields, field_bytes, stream);  // P_{count,fields}
+    return run_perm_any(ptr, 1, -1, count, fields, field_bytes, stream);  // P_{count,fields}
 }
 
 ipt_status_t ipt_soa_to_aos(void *ptr, int64_t count, int64_t fields, int field_bytes, void *stream) {
-    return run_perm(ptr, 1, -1, fields, count, field_bytes, stream);  // P_{fields,count}
+    return run_perm_any(ptr, 1, -1, fields, count, field_bytes, stream);  // P_{fields,count}
 }
 
 ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *global_bytes, size_t *onchip_per_cta) {
-    if (!valid_eb(elem_bytes) || m < 0 || n < 0) return IPT_ERR_INVALID_ARGUMENT;
+    if (!(valid_eb(elem_bytes) || valid_multiword_eb(elem_bytes)) || m < 0 || n < 0) return IPT_ERR_INVALID_ARGUMENT;
     Plan pl;
-    ipt_status_t s = make_plan(m, n, elem_bytes, pl);
+    ipt_status_t s;
+    if (valid_eb(elem_bytes)) {
+        s = make_plan(m, n, elem_bytes, pl);
+    } else {  // the larger of the two word-level steps (16-byte-aligned base assumed)
+        const int w = word_bytes_of(elem_bytes, 0);
+        const int64_t k = elem_bytes / w;
+        if (n != 0 && k > INT64_MAX / n) return IPT_ERR_INVALID_ARGUMENT;
+        Plan p2;
+        s = make_plan(m, n * k, w, pl);
+        if (s == IPT_OK) s = make_plan(k, m, w, p2);
+        if (s == IPT_OK) {
+            pl.scratch = std::max(pl.scratch, p2.scratch);
+            pl.onchip = std::max(pl.onchip, p2.onchip);
+        }
+    }
     if (s != IPT_OK) return s;
     if (global_bytes) *global_bytes = pl.scratch;
     if (onchip_per_cta) *onchip_per_cta = pl.onchip;
@@ -851,16 +903,29 @@ ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *glo
 ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
                            int64_t out[IPT_PLAN_INFO_FIELDS]) {
     int64_t x, y;
-    if (!out || !valid_eb(elem_bytes) || m < 0 || n < 0 || !perm_of(true, m, n, layout, x, y))
+    if (!out || !(valid_eb(elem_bytes) || valid_multiword_eb(elem_bytes)) || m < 0 || n < 0 ||
+        !perm_of(true, m, n, layout, x, y))
         return IPT_ERR_INVALID_ARGUMENT;
     Plan pl;
-    ipt_status_t s = make_plan(x, y, elem_bytes, pl);
+    int64_t extra_launches = 0;
+    ipt_status_t s;
+    if (valid_eb(elem_bytes)) {
+        s = make_plan(x, y, elem_bytes, pl);
+    } else {  // multi-word element: plan of the first word-level step, launches of both
+        const int w = word_bytes_of(elem_bytes, 0);
+        const int64_t k = elem_bytes / w;
+        if (y != 0 && k > INT64_MAX / y) return IPT_ERR_INVALID_ARGUMENT;
+        Plan p2;
+        s = make_plan(x, y * k, w, pl);
+        if (s == IPT_OK) s = make_plan(k, x, w, p2);
+        if (s == IPT_OK) extra_launches = p2.nlaunch;
+    }
     if (s != IPT_OK) return s;
     out[0] = pl.engine;
     out[1] = pl.M;
     out[2] = pl.N;
     out[3] = pl.c;
-    out[4] = pl.nlaunch;
+    out[4] = pl.nlaunch + extra_launches;
     out[5] = pl.engine ? pl.shuf.p.G : 0;
     out[6] = pl.engine ? pl.shuf.p.W : 0;
     out[7] = static_cast<int64_t>(pl.onchip);

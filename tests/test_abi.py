@@ -64,6 +64,13 @@ def test_argument_validation_without_device(ipt):
     assert lib.ipt_c2r(fake + 2, 4, 6, 4, 0, None) == 1      # misaligned to elem_bytes
     assert lib.ipt_c2r(fake, 1 << 40, 1 << 40, 8, 0, None) == 1  # size overflow
     assert lib.ipt_c2r_batched(fake, 2, 10, 4, 6, 4, 0, None) == 1  # stride < m*n
+    # multi-word records: any multiple of 4 up to 4096, 4-byte aligned base
+    assert lib.ipt_c2r(fake, 4, 6, 6, 0, None) == 1          # not a multiple of 4
+    assert lib.ipt_c2r(fake, 4, 6, 4100, 0, None) == 1       # beyond 4096
+    assert lib.ipt_c2r(fake + 2, 4, 6, 12, 0, None) == 1     # misaligned to 4
+    assert lib.ipt_c2r(fake + 4, 1, 6, 12, 0, None) == 0     # identity, 4-byte alignment enough
+    assert lib.ipt_c2r(fake, 1 << 40, 1 << 40, 24, 0, None) == 1  # size overflow
+    assert lib.ipt_c2r_batched(fake, 2, 10, 4, 6, 32, 0, None) == 1  # stride < m*n
     # identities: nothing is enqueued, no device needed
     assert lib.ipt_c2r(fake, 1, 1000, 4, 0, None) == 0
     assert lib.ipt_r2c(fake, 1000, 1, 8, 1, None) == 0
@@ -86,3 +93,4 @@ def test_oracle_and_product_share_nothing():
         if f.endswith((".py", ".c", ".h")):
             text = open(os.path.join(ROOT, "oracle", f)).read()
             assert "import paper_conf" not in text and "csrc" not in text, f
+

@@ -364,3 +364,81 @@ def test_fused_rotation_vector_gather(vec):
         with env_var("IPT_ROW_VEC", vec), env_var("IPT_COL_LAG", lag):
             for eb in (4, 8, 16):
                 run_packed(shapes, eb, ipt.c2r, "row", "c2r", seed=eb * 7 + len(vec))
+
+
+# ---------------------------------------------------------------------------------------
+# Multi-word elements (records): elem_bytes = k*w, run as P_{x,y*k} then
+# P_{k,x} on w-byte words (include/ipt.h).  The oracle moves eb-byte records directly.
+# ---------------------------------------------------------------------------------------
+@pytest.mark.parametrize("eb", [12, 20, 24, 32, 48, 64, 96])
+def test_multiword_small_shapes_bit_exact(eb):
+    shapes = [(m, n) for m, n in workloads.small_shapes(24) if (m * 7 + n) % 5 == 0]
+    run_packed(shapes, eb, ipt.c2r, "row", None, seed=eb)
+    run_packed(shapes[::3], eb, ipt.r2c, "col", None, seed=eb + 1)
+
+
+@pytest.mark.parametrize("m,n,eb", [(1200, 1800, 12), (1800, 1200, 24), (333, 4097, 32), (4096, 3000 // 8, 64),
+                                    (5000, 7, 12), (3, 20000, 48)])
+def test_multiword_config_shapes(m, n, eb):
+    host = workloads.random_words(m * n, eb, seed=m + n + eb)
+    x = to_dev(host)
+    ipt.c2r(x, m, n, elem_bytes=eb)
+    assert dev_bytes(x) == oracle.transpose(vwords(host, eb), m, n).tobytes()
+    ipt.r2c(x, m, n, elem_bytes=eb)
+    assert dev_bytes(x) == np.ascontiguousarray(host).tobytes()
+
+
+@pytest.mark.parametrize("offset", [4, 8, 12])
+def test_multiword_base_alignment(offset):
+    """Bases aligned to 4 or 8 bytes only pick narrower words (the result is the same)."""
+    m, n, eb = 37, 91, 32
+    host = workloads.random_words(m * n + 4, eb, seed=offset)
+    buf = to_dev(host)
+    ipt.c2r(buf.data_ptr() + offset, m, n, elem_bytes=eb)
+    raw = np.ascontiguousarray(host).view(np.uint8).reshape(-1)
+    body = raw[offset:offset + m * n * eb].copy()
+    want = oracle.transpose(body.view(np.dtype((np.void, eb))), m, n).tobytes()
+    got = dev_bytes(buf)
+    assert got[offset:offset + m * n * eb] == want
+    assert got[:offset] == raw[:offset].tobytes() and got[offset + m * n * eb:] == raw[offset + m * n * eb:].tobytes()
+
+
+@pytest.mark.parametrize("packed", [True, False])
+def test_multiword_batched(packed):
+    B, m, n, eb = 5, 61, 45, 24
+    stride = m * n + (0 if packed else 7)
+    host = workloads.random_words(B * stride, eb, seed=B + stride)
+    hv = vwords(host, eb)
+    buf = to_dev(host)
+    ipt.c2r_batched(buf, B, stride, m, n, elem_bytes=eb)
+    got = vwords(buf.cpu().numpy(), eb)
+    for k in range(B):
+        o = k * stride
+        assert got[o:o + m * n].tobytes() == oracle.transpose(hv[o:o + m * n], m, n).tobytes()
+        assert got[o + m * n:o + stride].tobytes() == hv[o + m * n:o + stride].tobytes()
+    ipt.r2c_batched(buf, B, stride, m, n, elem_bytes=eb)
+    assert dev_bytes(buf) == np.ascontiguousarray(host).tobytes()
+
+
+def test_multiword_aos_soa_records():
+    """Skinny entry point with 12-byte fields: count structs of `fields` 12-byte records."""
+    count, fields, eb = 100003, 5, 12
+    host = workloads.random_words(count * fields, eb, seed=3)
+    x = to_dev(host)
+    ipt.aos_to_soa(x, count, fields, field_bytes=eb)
+    assert dev_bytes(x) == oracle.aos_to_soa(vwords(host, eb), count, fields).tobytes()
+    ipt.soa_to_aos(x, count, fields, field_bytes=eb)
+    assert dev_bytes(x) == np.ascontiguousarray(host).tobytes()
+
+
+def test_multiword_scratch_and_plan():
+    """The plan of a record call reports the first word-level step and both steps' launches."""
+    g12, o12 = ipt.scratch_bytes(1200, 1800, 12)
+    g4, o4 = ipt.scratch_bytes(1200, 1800 * 3, 4)
+    assert g12 >= g4 and o12 >= o4
+    info = ipt.plan_info(1200, 1800, 32)  # 32 B = two 16-byte words
+    ref = ipt.plan_info(1200, 3600, 16)
+    assert all(info[k] == ref[k] for k in ("engine", "M", "N", "c"))
+    assert info["launches"] > ref["launches"]
+    with pytest.raises(ipt.IptError):
+        ipt.scratch_bytes(10, 10, 6)

@@ -39,10 +39,14 @@ def random_words(count: int, elem_bytes: int, seed: int) -> np.ndarray:
     """`count` random elements of `elem_bytes` bytes as a numpy array.
 
     4/8-byte elements come back as uint32/uint64; 16-byte elements as a (count, 2)
-    uint64 array (viewed flat as 2*count uint64)."""
+    uint64 array (viewed flat as 2*count uint64); other multiples of 4 bytes (records)
+    as a (count, elem_bytes // 4) uint32 array."""
     rng = np.random.default_rng(seed)
     if elem_bytes == 16:
         return rng.integers(0, 2**64, size=(count, 2), dtype=np.uint64, endpoint=False)
+    if elem_bytes not in _DTYPES:  # records of elem_bytes / 4 random 32-bit words
+        assert elem_bytes % 4 == 0
+        return rng.integers(0, 2**32, size=(count, elem_bytes // 4), dtype=np.uint32, endpoint=False)
     dt = _DTYPES[elem_bytes]
     return rng.integers(0, np.iinfo(dt).max, size=count, dtype=dt, endpoint=True)
 
