@@ -22,10 +22,15 @@
  * Multi-word elements (records): elem_bytes = k*w for any multiple of 4 up to 4096 that is
  * not 4, 8 or 16 (12, 24, 32, 48, 64 B ...).  `ptr` then needs 4-byte alignment only; w is
  * the largest of 16, 8, 4 dividing both elem_bytes and the address.  Such a call runs two
- * word-level permutations of the same engine (the paper's passes move opaque words of any
- * size): P_{x,y} on k-word elements = P_{x,y*k} on w-byte words
- * followed by P_{k,x} on each of the y k-by-x blocks, so it moves the buffer twice.  A
- * strided batch (stride_elems > m*n) runs the second step once per matrix.
+ * word-level permutations (the paper's passes move opaque words of any size,
+ * PAPER.md:1037, :1085), so it moves the buffer twice.  With L = min(x, y) records
+ * (P_{x,y} = the export's permutation): x <= y runs P_{x,y*k} on w-byte words, then P_{k,x}
+ * on each of the y k-by-x blocks (one record-block pass); x > y first splits each row of y
+ * records into k-by-y words (P_{y,k}, same pass), then runs P_{x*k,y} on words.  A block
+ * is staged in shared memory when L*elem_bytes <= 220 KiB, else in a per-CTA slot of
+ * stream-ordered global scratch (one slot per SM or more, <= 1 GiB in total); beyond that
+ * both steps run on the engine (a strided batch, stride_elems > m*n, then runs the second
+ * step once per matrix).
  */
 #ifndef IPT_H_
 #define IPT_H_
@@ -111,8 +116,7 @@ ipt_status_t ipt_soa_to_aos(void *ptr, int64_t count, int64_t fields, int field_
  * of the long dimension.  Batched calls scale it by the batch (the side block capped at
  * max(256 MiB, 1/32 of the data)).  *onchip_per_cta: the largest shared-memory staging buffer
  * of any launched CTA.  Multi-word elem_bytes: the larger of the two word-level steps
- * (P_{m,n*k} and one P_{k,m} block, words as wide as a 16-byte-aligned base allows).  Either
- * pointer may be NULL.
+ * (words as wide as a 16-byte-aligned base allows).  Either pointer may be NULL.
  */
 ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *global_bytes,
                                size_t *onchip_per_cta);
@@ -129,7 +133,7 @@ const char *ipt_status_string(ipt_status_t s);
  * CTAs per row of the row pass (0: one CTA per row; K > 0: a K-CTA cluster sharing the
  * row through distributed shared memory, for rows longer than one CTA's shared memory),
  * out[9] global scratch bytes.  Multi-word elem_bytes: out[0..3], out[5..9] describe the
- * first word-level step P_{x,y*k}; out[4] counts the launches of both steps (one matrix).
+ * engine's word-level step; out[4] counts the launches of both steps (one matrix).
  * Returns IPT_ERR_UNSUPPORTED for shapes beyond limits.
  */
 #define IPT_PLAN_INFO_FIELDS 10

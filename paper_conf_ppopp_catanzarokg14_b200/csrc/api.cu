@@ -728,6 +728,27 @@ ipt_status_t run_perm(void *ptr, int64_t batch, int64_t stride, int64_t x, int64
 // of column j), then P_{k,x} on each of the y k-by-x blocks (block j becomes x rows of k
 // words, i.e. row j of the y-by-x result).  Buffer traffic: twice the one-step engine.
 constexpr int kMaxElemBytes = 4096;
+
+// Staging of the record-block pass for blocks of blk_bytes: slots = 0 in shared memory;
+// slots > 0 CTAs each with a global scratch slot (at least one per SM, up to 4, while the
+// slots fit ~96 MB and stay L2-resident, never more than the blocks); slots = -1 when even
+// one slot per SM would exceed kRecordTmpMax (then both steps run on the engine).
+ipt_status_t record_slots(int64_t blk_bytes, int64_t nblocks, int64_t &slots) {
+    slots = 0;
+    if (env_int("IPT_RECORD_ENGINE", 0)) {  // tests: force both steps onto the engine
+        slots = -1;
+        return IPT_OK;
+    }
+    if (blk_bytes <= static_cast<int64_t>(kRecordSmemMax)) return IPT_OK;
+    int dev = 0, sms = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) {
+        cudaGetLastError();
+        return IPT_ERR_CUDA;
+    }
+    slots = std::min<int64_t>(nblocks, std::max<int64_t>(sms, std::min<int64_t>(4 * sms, (96ll << 20) / blk_bytes)));
+    if (slots * blk_bytes > static_cast<int64_t>(kRecordTmpMax)) slots = -1;
+    return IPT_OK;
+}
 bool valid_multiword_eb(int eb) { return eb > 0 && eb % 4 == 0 && eb <= kMaxElemBytes && !valid_eb(eb); }
 
 int word_bytes_of(int eb, uintptr_t addr) {
@@ -750,6 +771,50 @@ ipt_status_t run_perm_any(void *ptr, int64_t batch, int64_t stride, int64_t x, i
     if (x <= 1 || y <= 1) return IPT_OK;
     const int w = word_bytes_of(eb, reinterpret_cast<uintptr_t>(ptr));
     const int64_t k = eb / w;
+    const int64_t L = std::min(x, y);
+    const int64_t per_mat = std::max(x, y), nblocks = batch * per_mat;
+    int64_t slots = 0;
+    if (record_slots(L * eb, nblocks, slots) != IPT_OK) return IPT_ERR_CUDA;
+    if (slots >= 0 && nblocks < (int64_t(1) << 40)) {
+        // The block step on the shorter side, staged in shared memory (records.cu):
+        //   x <= y: P_{x,y*k} on words, then merge each k-by-x block into x records;
+        //   x >  y: split each row of y records into k-by-y words, then P_{x*k,y} on words
+        //           (row i*k + v holds word v of row i, so P_{x*k,y} leaves record (i,j)
+        //           at row j, words i*k .. i*k+k-1).
+        RecordParams rp{};
+        rp.base = static_cast<char *>(ptr);
+        rp.per_mat = std::max(x, y);
+        rp.nblocks = batch * rp.per_mat;
+        rp.mat_stride_bytes = stride * eb;
+        rp.blk_stride_bytes = L * eb;
+        rp.L = static_cast<uint32_t>(L);
+        rp.k = static_cast<uint32_t>(k);
+        rp.split = x > y;
+        rp.fd_k = make_fastdiv(static_cast<uint32_t>(k));
+        rp.grid = static_cast<uint32_t>(slots);
+        cudaStream_t cst = static_cast<cudaStream_t>(stream);
+        auto blocks = [&] {
+            if (slots) {
+                cudaMemPool_t pool = scratch_pool();
+                if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&rp.tmp),
+                                                     static_cast<size_t>(slots * L * eb), pool, cst) != cudaSuccess) {
+                    cudaGetLastError();
+                    return IPT_ERR_OUT_OF_MEMORY;
+                }
+            }
+            ipt_status_t r = check(launch_record_blocks(rp, w, cst));
+            if (rp.tmp) cudaFreeAsync(rp.tmp, cst);
+            if (r == IPT_OK) g_launches++;
+            return r;
+        };
+        if (x <= y) {
+            ipt_status_t s = run_perm(ptr, batch, stride * k, x, y * k, w, stream);
+            return s == IPT_OK ? blocks() : s;
+        }
+        ipt_status_t s = blocks();
+        return s == IPT_OK ? run_perm(ptr, batch, stride * k, x * k, y, w, stream) : s;
+    }
+    // Blocks too long for one CTA: both steps on the engine.
     ipt_status_t s = run_perm(ptr, batch, stride * k, x, y * k, w, stream);  // P_{x, y k}
     if (s != IPT_OK) return s;
     if (batch == 1 || stride == elems)  // every k-by-x block of every matrix is k*x words apart
@@ -757,6 +822,35 @@ ipt_status_t run_perm_any(void *ptr, int64_t batch, int64_t stride, int64_t x, i
     for (int64_t b = 0; b < batch && s == IPT_OK; ++b)
         s = run_perm(static_cast<char *>(ptr) + b * stride * eb, y, k * x, k, x, w, stream);
     return s;
+}
+
+// Plan description of a record call P_{x,y} (16-byte-aligned base assumed): `pl` is the
+// plan of its word-level engine step, widened by the other step's scratch and staging;
+// `extra` counts the other step's launches.
+ipt_status_t record_plan(int64_t x, int64_t y, int eb, Plan &pl, int64_t &extra) {
+    const int w = word_bytes_of(eb, 0);
+    const int64_t k = eb / w;
+    if (x < 0 || y < 0 || (y != 0 && k > INT64_MAX / y) || (x != 0 && k > INT64_MAX / x))
+        return IPT_ERR_INVALID_ARGUMENT;
+    const int64_t L = std::min(x, y);
+    int64_t slots = 0;
+    if (record_slots(L * eb, std::max(x, y), slots) != IPT_OK) return IPT_ERR_CUDA;
+    if (slots >= 0) {
+        ipt_status_t s = x <= y ? make_plan(x, y * k, w, pl) : make_plan(x * k, y, w, pl);
+        if (s != IPT_OK) return s;
+        extra = 1;
+        if (slots == 0) pl.onchip = std::max(pl.onchip, static_cast<size_t>(L * eb));
+        else pl.scratch = std::max(pl.scratch, static_cast<size_t>(slots * L * eb));
+        return IPT_OK;
+    }
+    Plan p2;
+    ipt_status_t s = make_plan(x, y * k, w, pl);
+    if (s == IPT_OK) s = make_plan(k, x, w, p2);
+    if (s != IPT_OK) return s;
+    extra = p2.nlaunch;
+    pl.scratch = std::max(pl.scratch, p2.scratch);
+    pl.onchip = std::max(pl.onchip, p2.onchip);
+    return IPT_OK;
 }
 
 // Export -> P_{x,y} (reading C18): c2r(m,n,ROW) = P_{m,n}, c2r(m,n,COL) = P_{n,m};
@@ -882,17 +976,9 @@ ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *glo
     ipt_status_t s;
     if (valid_eb(elem_bytes)) {
         s = make_plan(m, n, elem_bytes, pl);
-    } else {  // the larger of the two word-level steps (16-byte-aligned base assumed)
-        const int w = word_bytes_of(elem_bytes, 0);
-        const int64_t k = elem_bytes / w;
-        if (n != 0 && k > INT64_MAX / n) return IPT_ERR_INVALID_ARGUMENT;
-        Plan p2;
-        s = make_plan(m, n * k, w, pl);
-        if (s == IPT_OK) s = make_plan(k, m, w, p2);
-        if (s == IPT_OK) {
-            pl.scratch = std::max(pl.scratch, p2.scratch);
-            pl.onchip = std::max(pl.onchip, p2.onchip);
-        }
+    } else {
+        int64_t extra = 0;
+        s = record_plan(m, n, elem_bytes, pl, extra);
     }
     if (s != IPT_OK) return s;
     if (global_bytes) *global_bytes = pl.scratch;
@@ -911,14 +997,8 @@ ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t la
     ipt_status_t s;
     if (valid_eb(elem_bytes)) {
         s = make_plan(x, y, elem_bytes, pl);
-    } else {  // multi-word element: plan of the first word-level step, launches of both
-        const int w = word_bytes_of(elem_bytes, 0);
-        const int64_t k = elem_bytes / w;
-        if (y != 0 && k > INT64_MAX / y) return IPT_ERR_INVALID_ARGUMENT;
-        Plan p2;
-        s = make_plan(x, y * k, w, pl);
-        if (s == IPT_OK) s = make_plan(k, x, w, p2);
-        if (s == IPT_OK) extra_launches = p2.nlaunch;
+    } else {  // multi-word element: plan of the engine step, launches of both
+        s = record_plan(x, y, elem_bytes, pl, extra_launches);
     }
     if (s != IPT_OK) return s;
     out[0] = pl.engine;

@@ -213,4 +213,21 @@ size_t skinny_row_smem(int n, int T, int eb);
 cudaError_t launch_skinny_row(const SkinnyRowParams &p, int dir, int eb, cudaStream_t st);
 cudaError_t launch_skinny_row_reg(const SkinnyRowParams &p, int dir, cudaStream_t st);
 
+// Record blocks (records.cu, row f3): nblocks = batch * per_mat independent blocks of L
+// records of k w-byte words at base + b*mat_stride_bytes + j*blk_stride_bytes; split: L x k
+// -> k x L words, merge: k x L -> L x k.  Each block is staged whole: L*k*w bytes of smem,
+// or (tmp != null) a slot of global scratch per CTA.
+constexpr size_t kRecordSmemMax = 220 * 1024;
+constexpr size_t kRecordTmpMax = size_t(1) << 30;  // global-staged blocks: scratch cap
+struct RecordParams {
+    char *base;
+    int64_t nblocks, per_mat, mat_stride_bytes, blk_stride_bytes;
+    uint32_t L, k;
+    int32_t split;
+    FastDiv fd_k;
+    char *tmp;      // non-null: blocks staged in global scratch, grid slots of L*k*w bytes
+    uint32_t grid;  // with tmp: CTAs (= scratch slots)
+};
+cudaError_t launch_record_blocks(const RecordParams &p, int w, cudaStream_t st);
+
 }  // namespace ipt

@@ -1,0 +1,78 @@
+// Record blocks: the local step of a multi-word-element transpose.
+//
+// An element of k words (a record of eb = k*w bytes) is transposed with one word-level
+// engine call plus this pass over independent blocks of L records (api.cu run_perm_any):
+//   split: one block = L x k words (L records)     -> k x L words (word v of every record);
+//   merge: one block = k x L words                 -> L x k words (L records).
+// These are the P_{L,k} / P_{k,L} of the paper's Theorem 1 buffer form
+// on one block per CTA at a time: the block is staged whole with coalesced loads, then
+// written back coalesced in its new order, so each byte is read and written once (2*L*eb
+// bytes per block, HBM bound).  Blocks up to kRecordSmemMax are staged in shared memory;
+// longer ones in a per-CTA slot of a global scratch buffer sized to stay L2-resident
+// (Theorem 6's O(max(m, n)) auxiliary space per worker).
+#include "common.cuh"
+#include "plan.h"
+
+namespace ipt {
+
+namespace {
+
+constexpr int kRecThreads = 512;
+
+template <int W, bool GLOBAL>
+__global__ void __launch_bounds__(kRecThreads) record_block_kernel(RecordParams p) {
+    using T = typename Word<W>::T;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    // GLOBAL: this CTA's slot of the scratch buffer (plain loads: written by this CTA,
+    // made visible to its threads by __syncthreads).
+    T *s = GLOBAL ? reinterpret_cast<T *>(p.tmp + static_cast<int64_t>(blockIdx.x) * p.L * p.k * W)
+                  : reinterpret_cast<T *>(smem_raw);
+    const uint32_t L = p.L, k = p.k, n = p.L * p.k;
+    const FastDiv fk = p.fd_k;
+    for (int64_t blk = blockIdx.x; blk < p.nblocks; blk += gridDim.x) {
+        const int64_t b = blk / p.per_mat, j = blk - b * p.per_mat;
+        T *g = reinterpret_cast<T *>(p.base + b * p.mat_stride_bytes + j * p.blk_stride_bytes);
+        for (uint32_t t = threadIdx.x; t < n; t += kRecThreads) s[t] = g[t];
+        __syncthreads();
+        if (p.split) {  // L x k -> k x L: out[v*L + i] = in[i*k + v]
+            for (uint32_t v = 0; v < k; ++v)
+                for (uint32_t i = threadIdx.x; i < L; i += kRecThreads) g[v * L + i] = s[i * k + v];
+        } else {        // k x L -> L x k: out[i*k + v] = in[v*L + i]
+            for (uint32_t o = threadIdx.x; o < n; o += kRecThreads) {
+                const uint32_t i = fdiv(o, fk), v = o - i * k;
+                g[o] = s[v * L + i];
+            }
+        }
+        __syncthreads();  // the buffer is refilled by the next block
+    }
+}
+
+template <int W>
+cudaError_t launch_w(const RecordParams &p, cudaStream_t st) {
+    if (p.tmp) {
+        record_block_kernel<W, true><<<p.grid, kRecThreads, 0, st>>>(p);
+        return cudaGetLastError();
+    }
+    const size_t smem = static_cast<size_t>(p.L) * p.k * W;
+    auto kern = record_block_kernel<W, false>;
+    cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
+    if (e != cudaSuccess) return e;
+    const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), kRecThreads, smem);
+    if (resident < 1) return cudaErrorInvalidConfiguration;
+    const int64_t grid = p.nblocks < resident ? p.nblocks : resident;
+    kern<<<static_cast<unsigned>(grid), kRecThreads, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_record_blocks(const RecordParams &p, int w, cudaStream_t st) {
+    switch (w) {
+        case 4: return launch_w<4>(p, st);
+        case 8: return launch_w<8>(p, st);
+        case 16: return launch_w<16>(p, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+}  // namespace ipt

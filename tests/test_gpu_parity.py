@@ -378,7 +378,7 @@ def test_multiword_small_shapes_bit_exact(eb):
 
 
 @pytest.mark.parametrize("m,n,eb", [(1200, 1800, 12), (1800, 1200, 24), (333, 4097, 32), (4096, 3000 // 8, 64),
-                                    (5000, 7, 12), (3, 20000, 48)])
+                                    (5000, 7, 12), (3, 20000, 48), (2000, 2100, 128), (2100, 2000, 128)])
 def test_multiword_config_shapes(m, n, eb):
     host = workloads.random_words(m * n, eb, seed=m + n + eb)
     x = to_dev(host)
@@ -404,8 +404,10 @@ def test_multiword_base_alignment(offset):
 
 
 @pytest.mark.parametrize("packed", [True, False])
-def test_multiword_batched(packed):
-    B, m, n, eb = 5, 61, 45, 24
+@pytest.mark.parametrize("B,m,n,eb", [(5, 61, 45, 24), (5, 45, 61, 24), (2, 900, 950, 256)])
+def test_multiword_batched(packed, B, m, n, eb):
+    """Small blocks go through the shared-memory record pass; 900 x 256 B blocks (> 220 KiB)
+    are staged in global scratch slots."""
     stride = m * n + (0 if packed else 7)
     host = workloads.random_words(B * stride, eb, seed=B + stride)
     hv = vwords(host, eb)
@@ -417,6 +419,26 @@ def test_multiword_batched(packed):
         assert got[o:o + m * n].tobytes() == oracle.transpose(hv[o:o + m * n], m, n).tobytes()
         assert got[o + m * n:o + stride].tobytes() == hv[o + m * n:o + stride].tobytes()
     ipt.r2c_batched(buf, B, stride, m, n, elem_bytes=eb)
+    assert dev_bytes(buf) == np.ascontiguousarray(host).tobytes()
+
+
+@pytest.mark.parametrize("B,m,n,eb,stride", [(1, 300, 257, 24, None), (3, 97, 130, 32, 97 * 130),
+                                             (3, 130, 97, 12, 130 * 97 + 5)])
+def test_multiword_engine_fallback(B, m, n, eb, stride):
+    """IPT_RECORD_ENGINE=1: both word-level steps on the engine (the path for blocks beyond
+    the record pass's scratch cap), packed and gapped batches."""
+    stride = stride or m * n
+    host = workloads.random_words(B * stride, eb, seed=m * n + eb)
+    hv = vwords(host, eb)
+    buf = to_dev(host)
+    with env_var("IPT_RECORD_ENGINE", "1"):
+        ipt.c2r_batched(buf, B, stride, m, n, elem_bytes=eb)
+        got = vwords(buf.cpu().numpy(), eb)
+        for k in range(B):
+            o = k * stride
+            assert got[o:o + m * n].tobytes() == oracle.transpose(hv[o:o + m * n], m, n).tobytes()
+            assert got[o + m * n:o + stride].tobytes() == hv[o + m * n:o + stride].tobytes()
+        ipt.r2c_batched(buf, B, stride, m, n, elem_bytes=eb)
     assert dev_bytes(buf) == np.ascontiguousarray(host).tobytes()
 
 
