@@ -19,6 +19,14 @@
  * Element size: elem_bytes in {4, 8, 16}.  Elements are opaque words (bit-exact moves,
  * no floating-point semantics; NaN payloads, -0.0 and subnormals are preserved).
  *
+ * Sub-word elements: elem_bytes in {1, 2}, `ptr` 4-byte aligned.  g = 4 / elem_bytes
+ * elements share one 4-byte engine word: with P_{x,y} the export's permutation, y % g == 0
+ * runs P_{x,y/g} on words and then splits each row of x g-tuples into g rows; otherwise
+ * x % g == 0 merges each group of g rows into y g-tuples and runs P_{x/g,y} on words (one
+ * record-block pass + one engine call; the buffer moves twice).  IPT_ERR_UNSUPPORTED when
+ * neither x nor y is a multiple of g, when a batch stride is not a multiple of g, or when
+ * a block of 4*min-side bytes exceeds the record pass's scratch budget.
+ *
  * Multi-word elements (records): elem_bytes = k*w for any multiple of 4 up to 4096 that is
  * not 4, 8 or 16 (12, 24, 32, 48, 64 B ...).  `ptr` then needs 4-byte alignment only; w is
  * the largest of 16, 8, 4 dividing both elem_bytes and the address.  Such a call runs two

@@ -756,7 +756,68 @@ int word_bytes_of(int eb, uintptr_t addr) {
     return 4;
 }
 
+// Sub-word elements (1 or 2 bytes): g = 4 / eb elements share one 4-byte
+// engine word.  y % g == 0: P_{x,y/g} on words (row j' holds x g-tuples of row elements
+// g*j' .. g*j'+g-1), then split each row's x-by-g tuples into g rows of x elements.
+// Otherwise x % g == 0: merge each group of g rows (g-by-y elements -> y g-tuples), then
+// P_{x/g,y} on words (word (j, i') holds elements (g*i'+v, j), i.e. row j of the result).
+// Both x and y indivisible by g is unsupported, as are blocks beyond the record pass's
+// scratch budget and batch strides that are not a whole number of words.
+bool valid_subword_eb(int eb) { return eb == 1 || eb == 2; }
+
+ipt_status_t run_perm_subword(void *ptr, int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, void *stream) {
+    if (x < 0 || y < 0 || batch < 0) return IPT_ERR_INVALID_ARGUMENT;
+    if (x != 0 && y > INT64_MAX / x) return IPT_ERR_INVALID_ARGUMENT;
+    const int64_t elems = x * y;
+    if (stride < 0) stride = elems;
+    if (stride < elems) return IPT_ERR_INVALID_ARGUMENT;
+    if (stride != 0 && batch > INT64_MAX / stride) return IPT_ERR_INVALID_ARGUMENT;
+    if (elems == 0 || batch == 0) return IPT_OK;
+    if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % 4 != 0) return IPT_ERR_INVALID_ARGUMENT;
+    if (x <= 1 || y <= 1) return IPT_OK;
+    const int64_t g = 4 / eb;
+    const bool split = y % g == 0;
+    if ((!split && x % g != 0) || (batch > 1 && stride % g != 0)) return IPT_ERR_UNSUPPORTED;
+    const int64_t L = split ? x : y, per_mat = split ? y / g : x / g, nblocks = batch * per_mat;
+    int64_t slots = 0;
+    if (record_slots(L * 4, nblocks, slots) != IPT_OK) return IPT_ERR_CUDA;
+    if (slots < 0 || L * g >= (int64_t(1) << 32)) return IPT_ERR_UNSUPPORTED;
+    RecordParams rp{};
+    rp.base = static_cast<char *>(ptr);
+    rp.per_mat = per_mat;
+    rp.nblocks = nblocks;
+    rp.mat_stride_bytes = stride * eb;
+    rp.blk_stride_bytes = L * 4;
+    rp.L = static_cast<uint32_t>(L);
+    rp.k = static_cast<uint32_t>(g);
+    rp.split = split;
+    rp.fd_k = make_fastdiv(static_cast<uint32_t>(g));
+    rp.grid = static_cast<uint32_t>(slots);
+    cudaStream_t cst = static_cast<cudaStream_t>(stream);
+    auto blocks = [&] {
+        if (slots) {
+            cudaMemPool_t pool = scratch_pool();
+            if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&rp.tmp), static_cast<size_t>(slots * L * 4),
+                                                 pool, cst) != cudaSuccess) {
+                cudaGetLastError();
+                return IPT_ERR_OUT_OF_MEMORY;
+            }
+        }
+        ipt_status_t r = check(launch_record_blocks(rp, eb, cst));
+        if (rp.tmp) cudaFreeAsync(rp.tmp, cst);
+        if (r == IPT_OK) g_launches++;
+        return r;
+    };
+    if (split) {
+        ipt_status_t s = run_perm(ptr, batch, stride / g, x, y / g, 4, stream);
+        return s == IPT_OK ? blocks() : s;
+    }
+    ipt_status_t s = blocks();
+    return s == IPT_OK ? run_perm(ptr, batch, stride / g, x / g, y, 4, stream) : s;
+}
+
 ipt_status_t run_perm_any(void *ptr, int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, void *stream) {
+    if (valid_subword_eb(eb)) return run_perm_subword(ptr, batch, stride, x, y, eb, stream);
     if (!valid_multiword_eb(eb)) return run_perm(ptr, batch, stride, x, y, eb, stream);
     if (x < 0 || y < 0 || batch < 0) return IPT_ERR_INVALID_ARGUMENT;
     if (x != 0 && y > INT64_MAX / x) return IPT_ERR_INVALID_ARGUMENT;
@@ -828,6 +889,16 @@ ipt_status_t run_perm_any(void *ptr, int64_t batch, int64_t stride, int64_t x, i
 // plan of its word-level engine step, widened by the other step's scratch and staging;
 // `extra` counts the other step's launches.
 ipt_status_t record_plan(int64_t x, int64_t y, int eb, Plan &pl, int64_t &extra) {
+    if (valid_subword_eb(eb)) {  // plan of the packed-word engine step (run_perm_subword)
+        const int64_t g = 4 / eb;
+        if (y % g != 0 && x % g != 0) return IPT_ERR_UNSUPPORTED;
+        ipt_status_t s = y % g == 0 ? make_plan(x, y / g, 4, pl) : make_plan(x / g, y, 4, pl);
+        if (s != IPT_OK) return s;
+        extra = 1;
+        const int64_t blk = 4 * (y % g == 0 ? x : y);
+        if (blk <= static_cast<int64_t>(kRecordSmemMax)) pl.onchip = std::max(pl.onchip, static_cast<size_t>(blk));
+        return IPT_OK;
+    }
     const int w = word_bytes_of(eb, 0);
     const int64_t k = eb / w;
     if (x < 0 || y < 0 || (y != 0 && k > INT64_MAX / y) || (x != 0 && k > INT64_MAX / x))
@@ -971,7 +1042,8 @@ ipt_status_t ipt_soa_to_aos(void *ptr, int64_t count, int64_t fields, int field_
 }
 
 ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *global_bytes, size_t *onchip_per_cta) {
-    if (!(valid_eb(elem_bytes) || valid_multiword_eb(elem_bytes)) || m < 0 || n < 0) return IPT_ERR_INVALID_ARGUMENT;
+    if (!(valid_eb(elem_bytes) || valid_multiword_eb(elem_bytes) || valid_subword_eb(elem_bytes)) || m < 0 || n < 0)
+        return IPT_ERR_INVALID_ARGUMENT;
     Plan pl;
     ipt_status_t s;
     if (valid_eb(elem_bytes)) {
@@ -989,7 +1061,8 @@ ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *glo
 ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
                            int64_t out[IPT_PLAN_INFO_FIELDS]) {
     int64_t x, y;
-    if (!out || !(valid_eb(elem_bytes) || valid_multiword_eb(elem_bytes)) || m < 0 || n < 0 ||
+    if (!out || !(valid_eb(elem_bytes) || valid_multiword_eb(elem_bytes) || valid_subword_eb(elem_bytes)) ||
+        m < 0 || n < 0 ||
         !perm_of(true, m, n, layout, x, y))
         return IPT_ERR_INVALID_ARGUMENT;
     Plan pl;

@@ -52,6 +52,8 @@ __device__ __forceinline__ uint32_t mulmod(uint32_t x, uint32_t y, const FastDiv
 
 // Opaque element words.
 template <int EB> struct Word;
+template <> struct Word<1> { using T = uint8_t; };
+template <> struct Word<2> { using T = uint16_t; };
 template <> struct Word<4> { using T = uint32_t; };
 template <> struct Word<8> { using T = unsigned long long; };
 template <> struct Word<16> { using T = uint4; };

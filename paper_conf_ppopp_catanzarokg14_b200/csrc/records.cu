@@ -4,6 +4,8 @@
 // engine call plus this pass over independent blocks of L records (api.cu run_perm_any):
 //   split: one block = L x k words (L records)     -> k x L words (word v of every record);
 //   merge: one block = k x L words                 -> L x k words (L records).
+// Sub-word elements (1 or 2 bytes) use the same pass with k = 4 / eb elements per 4-byte
+// engine word (api.cu run_perm_subword).
 // These are the P_{L,k} / P_{k,L} of the paper's Theorem 1 buffer form
 // on one block per CTA at a time: the block is staged whole with coalesced loads, then
 // written back coalesced in its new order, so each byte is read and written once (2*L*eb
@@ -68,6 +70,8 @@ cudaError_t launch_w(const RecordParams &p, cudaStream_t st) {
 
 cudaError_t launch_record_blocks(const RecordParams &p, int w, cudaStream_t st) {
     switch (w) {
+        case 1: return launch_w<1>(p, st);
+        case 2: return launch_w<2>(p, st);
         case 4: return launch_w<4>(p, st);
         case 8: return launch_w<8>(p, st);
         case 16: return launch_w<16>(p, st);

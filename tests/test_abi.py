@@ -64,6 +64,11 @@ def test_argument_validation_without_device(ipt):
     assert lib.ipt_c2r(fake + 2, 4, 6, 4, 0, None) == 1      # misaligned to elem_bytes
     assert lib.ipt_c2r(fake, 1 << 40, 1 << 40, 8, 0, None) == 1  # size overflow
     assert lib.ipt_c2r_batched(fake, 2, 10, 4, 6, 4, 0, None) == 1  # stride < m*n
+    # sub-word elements: 4-byte aligned base, one side a multiple of 4 / elem_bytes
+    assert lib.ipt_c2r(fake + 2, 4, 6, 2, 0, None) == 1      # misaligned to 4
+    assert lib.ipt_c2r(fake, 3, 5, 2, 0, None) == 2          # both sides odd: unsupported
+    assert lib.ipt_c2r(fake, 6, 10, 1, 0, None) == 2         # neither side a multiple of 4
+    assert lib.ipt_c2r_batched(fake, 2, 25, 4, 6, 2, 0, None) == 2  # stride not whole words
     # multi-word records: any multiple of 4 up to 4096, 4-byte aligned base
     assert lib.ipt_c2r(fake, 4, 6, 6, 0, None) == 1          # not a multiple of 4
     assert lib.ipt_c2r(fake, 4, 6, 4100, 0, None) == 1       # beyond 4096

@@ -464,3 +464,48 @@ def test_multiword_scratch_and_plan():
     assert info["launches"] > ref["launches"]
     with pytest.raises(ipt.IptError):
         ipt.scratch_bytes(10, 10, 6)
+
+
+# ---------------------------------------------------------------------------------------
+# Sub-word elements (1 and 2 bytes): 4 / eb elements per engine word plus
+# the record-block split/merge pass (include/ipt.h).  Every buffer starts 4-byte aligned.
+# ---------------------------------------------------------------------------------------
+def _subword_roundtrip(m, n, eb, layout="row", seed=0):
+    host = workloads.random_words(m * n, eb, seed)
+    x = to_dev(host)
+    lay = {"row": oracle.ROW_MAJOR, "col": oracle.COL_MAJOR}[layout]
+    ipt.c2r(x, m, n, elem_bytes=eb, layout=layout)
+    assert dev_bytes(x) == oracle.ipt_c2r(host, m, n, lay).tobytes(), (m, n, eb, layout)
+    ipt.r2c(x, m, n, elem_bytes=eb, layout=layout)
+    assert dev_bytes(x) == np.ascontiguousarray(host).tobytes()
+
+
+@pytest.mark.parametrize("eb", [1, 2])
+def test_subword_small_shapes_bit_exact(eb):
+    g = 4 // eb
+    for m, n in workloads.small_shapes(24):
+        if (m % g == 0 or n % g == 0) and (m * 5 + n) % 3 == 0:
+            _subword_roundtrip(m, n, eb, "row" if (m + n) % 2 else "col", seed=m * 31 + n)
+
+
+@pytest.mark.parametrize("m,n,eb", [(1200, 1800, 2), (1200, 1800, 1), (14414, 6565, 2), (6565, 14414, 2),
+                                    (17226, 6052, 1), (3, 20000, 2), (20001, 4, 1), (70001, 2, 2)])
+def test_subword_config_shapes(m, n, eb):
+    _subword_roundtrip(m, n, eb, seed=m ^ n)
+
+
+def test_subword_batched_and_unsupported():
+    B, m, n, eb = 3, 50, 37, 2
+    stride = m * n + 6
+    host = workloads.random_words(B * stride, eb, seed=9)
+    buf = to_dev(host)
+    ipt.c2r_batched(buf, B, stride, m, n, elem_bytes=eb)
+    got = buf.cpu().numpy().view(host.dtype)
+    for k in range(B):
+        o = k * stride
+        assert got[o:o + m * n].tobytes() == oracle.transpose(host[o:o + m * n], m, n).tobytes()
+        assert got[o + m * n:o + stride].tobytes() == host[o + m * n:o + stride].tobytes()
+    ipt.r2c_batched(buf, B, stride, m, n, elem_bytes=eb)
+    assert dev_bytes(buf) == host.tobytes()
+    with pytest.raises(ipt.IptError):
+        ipt.c2r(buf, 7, 9, elem_bytes=2)

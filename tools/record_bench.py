@@ -1,4 +1,4 @@
-"""Throughput of multi-word records against single-word calls of the same bytes.
+"""Throughput of multi-word records and 1/2-byte elements against single-word calls of the same bytes.
 
 For each (m, n, record bytes) it times ipt_c2r on the record matrix and, for comparison, the
 single-word call that moves the same buffer as one 16-byte-word (or 4-byte) transpose
@@ -21,7 +21,8 @@ import torch  # noqa: E402
 import paper_conf_ppopp_catanzarokg14_b200 as ipt  # noqa: E402
 
 SHAPES = [(1200, 1800, 12), (1200, 1800, 32), (14414, 6565, 12), (14414, 6565, 24), (14414, 6565, 32),
-          (6565, 14414, 64), (4096, 3000, 48), (17226, 6052, 20)]
+          (6565, 14414, 64), (4096, 3000, 48), (17226, 6052, 20),
+          (14414, 6565, 2), (6565, 14414, 2), (14412, 6565, 1), (1200, 1800, 2), (1200, 1800, 1)]
 
 
 def time_op(fn, reps, flush):
@@ -46,10 +47,12 @@ def main():
         x = torch.randint(0, 255, (m * n * eb,), dtype=torch.uint8, device="cuda")
         w = 16 if eb % 16 == 0 else 8 if eb % 8 == 0 else 4
         k = eb // w
+        # the single-word call over the same bytes: P_{m, n*k}; sub-word: packed 4-byte words
+        wm, wn = (m, n * k) if eb >= 4 else ((m, n * eb // 4) if n * eb % 4 == 0 else (m * eb // 4, n))
         ipt.c2r(x, m, n, elem_bytes=eb)  # warm-up (plans, pools)
-        ipt.c2r(x, m, n * k, elem_bytes=w)
+        ipt.c2r(x, wm, wn, elem_bytes=w)
         t_rec = time_op(lambda: ipt.c2r(x, m, n, elem_bytes=eb), a.reps, flush)
-        t_word = time_op(lambda: ipt.c2r(x, m, n * k, elem_bytes=w), a.reps, flush)
+        t_word = time_op(lambda: ipt.c2r(x, wm, wn, elem_bytes=w), a.reps, flush)
         by = 2 * m * n * eb
         print(json.dumps({"m": m, "n": n, "record_bytes": eb, "word_bytes": w, "k": k,
                           "record_gbs": round(by / t_rec / 1e9, 1), "record_ms": round(t_rec * 1e3, 3),
