@@ -18,3 +18,5 @@ timeout 600 ncu --set full --clock-control none --import-source on -k regex:row_
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:row_rot -c 1 -s 2 -f -o gpurun_out/rowrot_$TAG \
     python tools/one_shape.py --m 17226 --n 6052 --eb 4 --reps 3 > gpurun_out/ncu_rowrot_$TAG.log 2>&1
 ls -la gpurun_out | tail -5
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:record_block -c 1 -s 1 -f -o gpurun_out/rec_$TAG \
+    python tools/one_shape.py --m 14414 --n 6565 --eb 12 --reps 2 > gpurun_out/ncu_rec_$TAG.log 2>&1
