@@ -792,6 +792,7 @@ ipt_status_t run_perm_subword(void *ptr, int64_t batch, int64_t stride, int64_t 
     rp.k = static_cast<uint32_t>(g);
     rp.split = split;
     rp.fd_k = make_fastdiv(static_cast<uint32_t>(g));
+    rp.fd_L = make_fastdiv(static_cast<uint32_t>(L));
     rp.grid = static_cast<uint32_t>(slots);
     cudaStream_t cst = static_cast<cudaStream_t>(stream);
     auto blocks = [&] {

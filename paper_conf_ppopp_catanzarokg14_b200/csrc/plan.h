@@ -224,7 +224,7 @@ struct RecordParams {
     int64_t nblocks, per_mat, mat_stride_bytes, blk_stride_bytes;
     uint32_t L, k;
     int32_t split;
-    FastDiv fd_k;
+    FastDiv fd_k, fd_L;  // fd_L: sub-word split of ragged rows
     char *tmp;      // non-null: blocks staged in global scratch, grid slots of L*k*w bytes
     uint32_t grid;  // with tmp: CTAs (= scratch slots)
 };

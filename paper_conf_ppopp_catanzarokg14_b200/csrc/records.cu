@@ -21,6 +21,23 @@ namespace {
 
 constexpr int kRecThreads = 512;
 
+// G x G transpose of sub-word elements held in G 32-bit words (G = 4 / W): out[e] element v
+// = in[v] element e.  1-byte: a 4x4 byte transpose in six byte permutes; 2-byte: two.
+template <int W>
+__device__ __forceinline__ void tuple_transpose(const uint32_t (&in)[4 / W], uint32_t (&out)[4 / W]) {
+    if constexpr (W == 1) {
+        const uint32_t t0 = __byte_perm(in[0], in[1], 0x5140), t1 = __byte_perm(in[0], in[1], 0x7362);
+        const uint32_t t2 = __byte_perm(in[2], in[3], 0x5140), t3 = __byte_perm(in[2], in[3], 0x7362);
+        out[0] = __byte_perm(t0, t2, 0x5410);
+        out[1] = __byte_perm(t0, t2, 0x7632);
+        out[2] = __byte_perm(t1, t3, 0x5410);
+        out[3] = __byte_perm(t1, t3, 0x7632);
+    } else {
+        out[0] = __byte_perm(in[0], in[1], 0x5410);
+        out[1] = __byte_perm(in[0], in[1], 0x7632);
+    }
+}
+
 template <int W, bool GLOBAL>
 __global__ void __launch_bounds__(kRecThreads) record_block_kernel(RecordParams p) {
     using T = typename Word<W>::T;
@@ -34,8 +51,60 @@ __global__ void __launch_bounds__(kRecThreads) record_block_kernel(RecordParams 
     for (int64_t blk = blockIdx.x; blk < p.nblocks; blk += gridDim.x) {
         const int64_t b = blk / p.per_mat, j = blk - b * p.per_mat;
         T *g = reinterpret_cast<T *>(p.base + b * p.mat_stride_bytes + j * p.blk_stride_bytes);
-        for (uint32_t t = threadIdx.x; t < n; t += kRecThreads) s[t] = g[t];
-        __syncthreads();
+        if constexpr (W < 4) {
+            // Sub-word elements (k = G = 4 / W): the block is L whole 32-bit words.  With
+            // L % G == 0 every output row is word-aligned too, so thread c moves one G x G
+            // tile: G words in, G words out, transposed in registers.
+            constexpr uint32_t G = 4 / W;
+            uint32_t *g32 = reinterpret_cast<uint32_t *>(g), *s32 = reinterpret_cast<uint32_t *>(s);
+            for (uint32_t t = threadIdx.x; t < L; t += kRecThreads) s32[t] = g32[t];
+            __syncthreads();
+            if (L % G == 0) {
+                const uint32_t wpr = L / G;  // words per row of G elements' worth
+                for (uint32_t c = threadIdx.x; c < wpr; c += kRecThreads) {
+                    uint32_t in[G], out[G];
+                    if (p.split) {  // tuples c*G .. c*G+G-1 -> word c of rows 0..G-1
+#pragma unroll
+                        for (uint32_t e = 0; e < G; ++e) in[e] = s32[c * G + e];
+                        tuple_transpose<W>(in, out);
+#pragma unroll
+                        for (uint32_t v = 0; v < G; ++v) g32[v * wpr + c] = out[v];
+                    } else {        // word c of rows 0..G-1 -> tuples c*G .. c*G+G-1
+#pragma unroll
+                        for (uint32_t v = 0; v < G; ++v) in[v] = s32[v * wpr + c];
+                        tuple_transpose<W>(in, out);
+#pragma unroll
+                        for (uint32_t e = 0; e < G; ++e) g32[c * G + e] = out[e];
+                    }
+                }
+            } else {
+                // Ragged rows (L % G != 0): still whole output words; each of the word's G
+                // elements is located on its own (split: row v = o / L; merge: o / G).
+                using E = typename Word<W>::T;
+                const E *se = reinterpret_cast<const E *>(s32);
+                for (uint32_t t = threadIdx.x; t < L; t += kRecThreads) {
+                    uint32_t word = 0;
+#pragma unroll
+                    for (uint32_t e = 0; e < G; ++e) {
+                        const uint32_t o = t * G + e;
+                        uint32_t src;
+                        if (p.split) {
+                            const uint32_t v = fdiv(o, p.fd_L);
+                            src = (o - v * L) * G + v;
+                        } else {
+                            src = (o % G) * L + o / G;
+                        }
+                        word |= static_cast<uint32_t>(se[src]) << (8 * W * e);
+                    }
+                    g32[t] = word;
+                }
+            }
+            __syncthreads();
+            continue;
+        } else {
+            for (uint32_t t = threadIdx.x; t < n; t += kRecThreads) s[t] = g[t];
+            __syncthreads();
+        }
         if (p.split) {  // L x k -> k x L: out[v*L + i] = in[i*k + v]
             for (uint32_t v = 0; v < k; ++v)
                 for (uint32_t i = threadIdx.x; i < L; i += kRecThreads) g[v * L + i] = s[i * k + v];
