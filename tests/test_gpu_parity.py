@@ -464,6 +464,16 @@ def test_multiword_scratch_and_plan():
     assert info["launches"] > ref["launches"]
     with pytest.raises(ipt.IptError):
         ipt.scratch_bytes(10, 10, 6)
+    # sub-word: the packed-word engine step (y % g == 0: P_{x,y/g}; else P_{x/g,y}) + 1 launch
+    sub = ipt.plan_info(1200, 1800, 2)
+    ref = ipt.plan_info(1200, 900, 4)
+    assert all(sub[k] == ref[k] for k in ("engine", "M", "N", "c"))
+    assert sub["launches"] == ref["launches"] + 1
+    sub = ipt.plan_info(1200, 1801, 1)
+    ref = ipt.plan_info(300, 1801, 4)
+    assert all(sub[k] == ref[k] for k in ("engine", "M", "N", "c"))
+    with pytest.raises(ipt.IptError):
+        ipt.plan_info(7, 9, 2)
 
 
 # ---------------------------------------------------------------------------------------
