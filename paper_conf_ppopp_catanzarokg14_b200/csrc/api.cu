@@ -772,6 +772,7 @@ ipt_status_t run_perm_subword(void *ptr, int64_t batch, int64_t stride, int64_t 
     if (stride < 0) stride = elems;
     if (stride < elems) return IPT_ERR_INVALID_ARGUMENT;
     if (stride != 0 && batch > INT64_MAX / stride) return IPT_ERR_INVALID_ARGUMENT;
+    if (elems != 0 && batch * stride > INT64_MAX / eb) return IPT_ERR_INVALID_ARGUMENT;
     if (elems == 0 || batch == 0) return IPT_OK;
     if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % 4 != 0) return IPT_ERR_INVALID_ARGUMENT;
     if (x <= 1 || y <= 1) return IPT_OK;
