@@ -21,8 +21,9 @@
  *
  * Sub-word elements: elem_bytes in {1, 2}, `ptr` 4-byte aligned.  g = 4 / elem_bytes
  * elements share one 4-byte engine word: with P_{x,y} the export's permutation, y % g == 0
- * runs P_{x,y/g} on words and then splits each row of x g-tuples into g rows; otherwise
- * x % g == 0 merges each group of g rows into y g-tuples and runs P_{x/g,y} on words (one
+ * runs P_{x,y/g} on words and then splits each row of x g-tuples into g rows; x % g == 0
+ * merges each group of g rows into y g-tuples and runs P_{x/g,y} on words (when both are
+ * possible, the one with the shorter blocks: split if x <= y) (one
  * record-block pass + one engine call; the buffer moves twice).  IPT_ERR_UNSUPPORTED when
  * neither x nor y is a multiple of g, when a batch stride is not a multiple of g, or when
  * a block of 4*min-side bytes exceeds the record pass's scratch budget.

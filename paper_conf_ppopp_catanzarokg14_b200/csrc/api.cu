@@ -777,7 +777,8 @@ ipt_status_t run_perm_subword(void *ptr, int64_t batch, int64_t stride, int64_t 
     if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % 4 != 0) return IPT_ERR_INVALID_ARGUMENT;
     if (x <= 1 || y <= 1) return IPT_OK;
     const int64_t g = 4 / eb;
-    const bool split = y % g == 0;
+    // Of the feasible orientations, the one with the shorter blocks (L = x for split, y for merge).
+    const bool split = y % g == 0 && (x % g != 0 || x <= y);
     if ((!split && x % g != 0) || (batch > 1 && stride % g != 0)) return IPT_ERR_UNSUPPORTED;
     const int64_t L = split ? x : y, per_mat = split ? y / g : x / g, nblocks = batch * per_mat;
     int64_t slots = 0;
@@ -894,10 +895,11 @@ ipt_status_t record_plan(int64_t x, int64_t y, int eb, Plan &pl, int64_t &extra)
     if (valid_subword_eb(eb)) {  // plan of the packed-word engine step (run_perm_subword)
         const int64_t g = 4 / eb;
         if (y % g != 0 && x % g != 0) return IPT_ERR_UNSUPPORTED;
-        ipt_status_t s = y % g == 0 ? make_plan(x, y / g, 4, pl) : make_plan(x / g, y, 4, pl);
+        const bool split = y % g == 0 && (x % g != 0 || x <= y);  // as run_perm_subword
+        ipt_status_t s = split ? make_plan(x, y / g, 4, pl) : make_plan(x / g, y, 4, pl);
         if (s != IPT_OK) return s;
         extra = 1;
-        const int64_t blk = 4 * (y % g == 0 ? x : y);
+        const int64_t blk = 4 * (split ? x : y);
         if (blk <= static_cast<int64_t>(kRecordSmemMax)) pl.onchip = std::max(pl.onchip, static_cast<size_t>(blk));
         return IPT_OK;
     }

@@ -118,8 +118,60 @@ __global__ void __launch_bounds__(kRecThreads) record_block_kernel(RecordParams 
     }
 }
 
+// Short blocks (<= kChunkBlockMax bytes; e.g. AoS<->SoA with a few fields): one CTA would
+// idle on a tiny block per barrier pair, so each CTA stages a chunk of consecutive blocks of
+// one matrix (blocks are contiguous: blk_stride = L*k*W) and permutes every element of the
+// chunk, locating it by strength-reduced divisions.
+constexpr uint32_t kChunkBlockMax = 4096, kChunkBytes = 32768;
+
+template <int W>
+__global__ void __launch_bounds__(kRecThreads) record_chunk_kernel(RecordParams p, uint32_t chunk, FastDiv fd_n,
+                                                                   FastDiv fd_L) {
+    using T = typename Word<W>::T;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    T *s = reinterpret_cast<T *>(smem_raw);
+    const uint32_t L = p.L, k = p.k, n = p.L * p.k;
+    const int64_t cpm = (p.per_mat + chunk - 1) / chunk, items = p.nblocks / p.per_mat * cpm;
+    for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
+        const int64_t b = it / cpm, j0 = (it - b * cpm) * chunk;
+        const uint32_t nb = static_cast<uint32_t>(p.per_mat - j0 < chunk ? p.per_mat - j0 : chunk);
+        T *g = reinterpret_cast<T *>(p.base + b * p.mat_stride_bytes + j0 * p.blk_stride_bytes);
+        const uint32_t tot = nb * n;
+        for (uint32_t t = threadIdx.x; t < tot; t += kRecThreads) s[t] = g[t];
+        __syncthreads();
+        for (uint32_t t = threadIdx.x; t < tot; t += kRecThreads) {
+            const uint32_t blk = fdiv(t, fd_n), r = t - blk * n;
+            uint32_t src;
+            if (p.split) {  // out[v*L + i] = in[i*k + v]
+                const uint32_t v = fdiv(r, fd_L), i = r - v * L;
+                src = i * k + v;
+            } else {        // out[i*k + v] = in[v*L + i]
+                const uint32_t i = fdiv(r, p.fd_k), v = r - i * k;
+                src = v * L + i;
+            }
+            g[t] = s[blk * n + src];
+        }
+        __syncthreads();  // the buffer is refilled by the next chunk
+    }
+}
+
 template <int W>
 cudaError_t launch_w(const RecordParams &p, cudaStream_t st) {
+    const size_t blk_bytes = static_cast<size_t>(p.L) * p.k * W;
+    if (!p.tmp && blk_bytes <= kChunkBlockMax && p.per_mat > 1) {
+        const uint32_t chunk = static_cast<uint32_t>(kChunkBytes / blk_bytes);
+        const size_t smem = chunk * blk_bytes;
+        auto kern = record_chunk_kernel<W>;
+        cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
+        if (e != cudaSuccess) return e;
+        const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), kRecThreads, smem);
+        if (resident < 1) return cudaErrorInvalidConfiguration;
+        const int64_t items = p.nblocks / p.per_mat * ((p.per_mat + chunk - 1) / chunk);
+        const int64_t grid = items < resident ? items : resident;
+        kern<<<static_cast<unsigned>(grid), kRecThreads, smem, st>>>(
+            p, chunk, make_fastdiv(p.L * p.k), make_fastdiv(p.L));
+        return cudaGetLastError();
+    }
     if (p.tmp) {
         record_block_kernel<W, true><<<p.grid, kRecThreads, 0, st>>>(p);
         return cudaGetLastError();

@@ -465,7 +465,7 @@ def test_multiword_scratch_and_plan():
     with pytest.raises(ipt.IptError):
         ipt.scratch_bytes(10, 10, 6)
     # sub-word: the packed-word engine step (y % g == 0: P_{x,y/g}; else P_{x/g,y}) + 1 launch
-    sub = ipt.plan_info(1200, 1800, 2)
+    sub = ipt.plan_info(1200, 1800, 2)  # both sides even, x <= y: split
     ref = ipt.plan_info(1200, 900, 4)
     assert all(sub[k] == ref[k] for k in ("engine", "M", "N", "c"))
     assert sub["launches"] == ref["launches"] + 1
@@ -499,7 +499,8 @@ def test_subword_small_shapes_bit_exact(eb):
 
 
 @pytest.mark.parametrize("m,n,eb", [(1200, 1800, 2), (1200, 1800, 1), (14414, 6565, 2), (6565, 14414, 2),
-                                    (17226, 6052, 1), (3, 20000, 2), (20001, 4, 1), (70001, 2, 2)])
+                                    (17226, 6052, 1), (3, 20000, 2), (20001, 4, 1), (70001, 2, 2),
+                                    (1 << 20, 4, 1), (4, 1 << 20, 1), (1 << 20, 2, 2), (1800, 1200, 2)])
 def test_subword_config_shapes(m, n, eb):
     _subword_roundtrip(m, n, eb, seed=m ^ n)
 

@@ -23,7 +23,7 @@ import paper_conf_ppopp_catanzarokg14_b200 as ipt  # noqa: E402
 SHAPES = [(1200, 1800, 12), (1200, 1800, 32), (14414, 6565, 12), (14414, 6565, 24), (14414, 6565, 32),
           (6565, 14414, 64), (4096, 3000, 48), (17226, 6052, 20),
           (14414, 6565, 2), (6565, 14414, 2), (14412, 6565, 1), (14414, 6566, 2), (14412, 6564, 1),
-          (1200, 1800, 2), (1200, 1800, 1)]
+          (1200, 1800, 2), (1200, 1800, 1), (1 << 24, 5, 12), (1 << 25, 3, 2), (1 << 24, 4, 1)]
 
 
 def time_op(fn, reps, flush):
