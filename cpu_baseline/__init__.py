@@ -17,7 +17,7 @@ _lib = None
 def build(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O3", "-march=native", "-fopenmp", "-std=gnu11", "-Wall", "-shared", "-fPIC",
+        subprocess.check_call(["gcc", "-O3", "-fopenmp", "-std=gnu11", "-Wall", "-shared", "-fPIC",
                                _SRC, "-o", tmp])
         os.replace(tmp, _LIB)
     return _LIB
