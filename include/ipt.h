@@ -16,7 +16,8 @@
  * until the stream reaches the end of the call.  The operation is not atomic: if a
  * launch fails mid-sequence (IPT_ERR_CUDA) the buffer content is unspecified.
  *
- * Element size: elem_bytes in {4, 8, 16}.  Elements are opaque words (bit-exact moves,
+ * Element size: elem_bytes in {4, 8, 16} natively (the engine's passes); 1, 2 and any
+ * other multiple of 4 up to 4096 by composition (below).  Elements are opaque words (bit-exact moves,
  * no floating-point semantics; NaN payloads, -0.0 and subnormals are preserved).
  *
  * Sub-word elements: elem_bytes in {1, 2}, `ptr` 4-byte aligned.  g = 4 / elem_bytes
