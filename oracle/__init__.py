@@ -66,6 +66,9 @@ def lib() -> ctypes.CDLL:
         for name in ("oracle_c2r_alg1", "oracle_r2c_alg1"):
             getattr(L, name).restype = ctypes.c_int
             getattr(L, name).argtypes = [_vp, _i64, _i64, ctypes.c_int, ctypes.c_int, _vp, _vp, _vp, _vp]
+        for name in ("oracle_aos_gather", "oracle_aos_scatter"):
+            getattr(L, name).restype = None
+            getattr(L, name).argtypes = [_vp, _vp, _vp, _i64, ctypes.c_int]
         for name in ("oracle_c2r_gather_forms", "oracle_r2c_gather_forms"):
             getattr(L, name).restype = ctypes.c_int
             getattr(L, name).argtypes = [_vp, _i64, _i64, ctypes.c_int, _vp, _vp, _vp, _vp]
@@ -263,3 +266,28 @@ def warp_load_aos_registers(words: np.ndarray, S: int, lanes: int = 32) -> np.nd
         for k in range(S):
             R[k, lane] = w[lane * S + k]
     return R
+
+
+def aos_gather(src: np.ndarray, idx: np.ndarray, words: int) -> np.ndarray:
+    """§6.2 random-access gather (Fig. 9; reading C17): dst[k] =
+    src[idx[k]] struct by struct (structs of `words` 4-byte words).  Plain loops in C."""
+    src = np.ascontiguousarray(src, dtype=np.uint32).reshape(-1)
+    idx = np.ascontiguousarray(idx, dtype=np.uint32).reshape(-1)
+    assert src.size % words == 0 and (idx.size == 0 or int(idx.max()) < src.size // words)
+    dst = np.empty(idx.size * words, dtype=np.uint32)
+    lib().oracle_aos_gather(_ptr(src), _ptr(idx), _ptr(dst), idx.size, words)
+    return dst
+
+
+def aos_scatter(src: np.ndarray, idx: np.ndarray, words: int, ndst: int | None = None) -> np.ndarray:
+    """§6.2 random-access scatter: dst[idx[k]] = src[k] (idx a permutation of the
+    destination structs; destinations not named by idx stay zero)."""
+    src = np.ascontiguousarray(src, dtype=np.uint32).reshape(-1)
+    idx = np.ascontiguousarray(idx, dtype=np.uint32).reshape(-1)
+    count = idx.size
+    assert src.size >= count * words
+    ndst = count if ndst is None else ndst
+    assert count == 0 or int(idx.max()) < ndst
+    dst = np.zeros(ndst * words, dtype=np.uint32)
+    lib().oracle_aos_scatter(_ptr(src), _ptr(idx), _ptr(dst), count, words)
+    return dst

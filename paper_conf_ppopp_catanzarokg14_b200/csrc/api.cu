@@ -468,7 +468,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -539,11 +539,84 @@ void profile_end(ProfRec &r, cudaStream_t st) {
     g_prof.push_back(r);
 }
 
-ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_bytes, cudaStream_t st) {
+// ---- per-call global scratch (Theorem 6: O(max(m, n)) per worker) -------------------
+// One stream-ordered allocation per call, laid out as
+//   [ counters: shuffle pass | rotation pass ][ row flags + ticket ]   <- zeroed (one memset)
+//   [ wrap rows ][ side blocks ]  or, for the skinny engine, [ tmp row ]
+// Nothing is shared between calls, so concurrent calls (other host threads, other
+// streams, cudaStreamPerThread) cannot see each other's counters.
+struct CallScratch {
+    size_t ctr_shuf = 0, ctr_rot = 0;  // column-pass counter blocks (kCtrBytes each)
+    size_t flags = 0;                  // fused rotation: M*batch row flags + the ticket
+    size_t zero_bytes = 0;             // [0, zero_bytes) is zeroed before the first pass
+    size_t wrap = 0, wstride = 0;      // fused rotation: per-matrix copy of rows 0..c-2
+    size_t side = 0;                   // lagged layouts: side blocks
+    size_t total = 0;
+};
+
+size_t al256(size_t x) { return (x + 255) & ~size_t(255); }
+
+// Final plan of a call on `batch` matrices (batches cap the lag) and its scratch layout.
+// Pure host arithmetic: nothing is enqueued.
+void prepare_call(Plan &pl, int64_t batch, CallScratch &cs) {
+    cs = CallScratch{};
+    if (pl.engine == ENG_NONE || batch == 0) return;
+    if (pl.engine == ENG_SKINNY) {
+        cs.total = al256(pl.scratch);
+        return;
+    }
+    const double full = 2.0 * static_cast<double>(pl.M) * static_cast<double>(pl.N) * pl.eb * static_cast<double>(batch);
+    if (pl.side_bytes && batch > 1) {
+        // Batches: keep the side blocks within max(256 MiB, 1/32 of the data) -- a smaller D.
+        const double cap = std::max(256.0 * (1 << 20), full / 2.0 / 32.0);
+        const double per_tile = static_cast<double>(pl.M) * pl.shuf.p.W * pl.eb * static_cast<double>(batch);
+        const int64_t dmax = static_cast<int64_t>(cap / per_tile);
+        if (dmax < pl.shuf.p.lagD) set_lag(pl, dmax);
+    }
+    size_t o = 0;
+    cs.ctr_shuf = o;
+    o += kCtrBytes;
+    if (pl.has_rot) {
+        cs.ctr_rot = o;
+        o += kCtrBytes;
+    }
+    if (pl.row.fuse) {
+        cs.flags = o;
+        o += al256((static_cast<size_t>(pl.M) * static_cast<size_t>(batch) + 1) * 4);
+    }
+    cs.zero_bytes = o;
+    if (pl.row.fuse) {
+        cs.wrap = o;
+        cs.wstride = al256(static_cast<size_t>(pl.c - 1) * pl.N * pl.eb + 16);
+        o += cs.wstride * static_cast<size_t>(batch);
+    }
+    if (pl.side_bytes) {
+        cs.side = o;
+        o += pl.side_bytes * static_cast<size_t>(batch);
+    }
+    cs.total = o;
+}
+
+ipt_status_t pool_alloc(char **p, size_t bytes, cudaStream_t st) {
+    *p = nullptr;
+    if (!bytes) return IPT_OK;
+    cudaMemPool_t pool = scratch_pool();
+    if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(p), bytes, pool, st) != cudaSuccess) {
+        cudaGetLastError();
+        *p = nullptr;
+        return IPT_ERR_OUT_OF_MEMORY;
+    }
+    return IPT_OK;
+}
+
+// Enqueue the passes of a prepared call.  `scratch` holds cs.total bytes (stream-ordered,
+// owned by the caller of this function).
+ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int64_t batch, int64_t stride_bytes,
+                         cudaStream_t st, char *scratch) {
     if (pl0.engine == ENG_NONE || batch == 0) return IPT_OK;
     Plan pl = pl0;
-    // Row groups are numbered in 32 bits (row_shuffle.cu row_group).
-    if (pl.engine != ENG_SKINNY && (pl.M + pl.row.R - 1) / pl.row.R * batch >= (int64_t(1) << 32))
+    // Row groups are numbered in 32 bits (row_shuffle.cu row_group, the fused pass's ticket).
+    if (pl.engine != ENG_SKINNY && (pl.M + pl.row.R - 1) / pl.row.R * batch >= (int64_t(1) << 32) - 1)
         return IPT_ERR_UNSUPPORTED;
     pl.row.base = base;
     pl.row.batch = batch;
@@ -567,12 +640,6 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
         if (s == IPT_OK) g_launches++;
         return s;
     };
-    // The rotation moves only the columns with a non-zero amount: (c - 1) / c of them.
-    const double rot_bytes = full * static_cast<double>(pl.c - 1) / static_cast<double>(pl.c);
-    auto rot = [&] { return launch_col(pl.rot.p, COL_ROT, pl.eb, st, pl.rot.smem); };
-    auto row = [&] {
-        return pl.row.cl_K ? launch_row_cluster(pl.row, pl.row_dir, pl.eb, st) : launch_row(pl.row, pl.row_dir, pl.eb, st);
-    };
     ipt_status_t s;
     if (pl.engine == ENG_SKINNY) {
         // Rolling rows (§6.1; DESIGN.md §"Skinny"): engine view n rows x N, one
@@ -584,12 +651,7 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
         // by another rho rows (plan.h, SkinnyRowParams).
         const int n = static_cast<int>(pl.M);
         const double rowb = 2.0 * static_cast<double>(pl.N) * pl.eb;
-        char *tmp = nullptr;
-        cudaMemPool_t pool = scratch_pool();
-        if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&tmp), pl.scratch, pool, st) != cudaSuccess) {
-            cudaGetLastError();
-            return IPT_ERR_OUT_OF_MEMORY;
-        }
+        char *tmp = scratch;
         s = IPT_OK;
         for (int64_t mat = 0; mat < batch; ++mat) {
             char *A = base + mat * stride_bytes;
@@ -616,51 +678,32 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
             }
             if (s != IPT_OK) break;
         }
-        cudaFreeAsync(tmp, st);
         return s;
     }
-    // Per-call scratch: fused rotation -- row flags (zeroed) and, for C2R, a copy of the
-    // rows the last staircases wrap onto; lagged layouts -- the side tiles.
-    char *fscratch = nullptr;
+    // Column-pass counters, fused-rotation flags + ticket: zeroed in stream order.
+    if (cs.zero_bytes && (s = check(cudaMemsetAsync(scratch, 0, cs.zero_bytes, st))) != IPT_OK) return s;
+    pl.shuf.p.ctr = reinterpret_cast<unsigned int *>(scratch + cs.ctr_shuf);
+    pl.rot.p.ctr = reinterpret_cast<unsigned int *>(scratch + cs.ctr_rot);
+    pl.shuf.p.ticket = pl.rot.p.ticket = env_int("IPT_COL_TICKET", 1) != 0 ? 1 : 0;
+    if (pl.row.fuse) {
+        pl.row.flags = reinterpret_cast<unsigned int *>(scratch + cs.flags);
+        pl.row.ticket = pl.row.flags + pl.M * batch;
+        pl.row.wrap = scratch + cs.wrap;
+        pl.row.wstride = static_cast<int64_t>(cs.wstride);
+    }
+    pl.row.side = pl.shuf.p.side = pl.side_bytes ? scratch + cs.side : nullptr;
     const int64_t pitch = pl.N * pl.eb;
-    const size_t flag_bytes = pl.row.fuse ? (static_cast<size_t>(pl.M * batch) * 4 + 255) & ~size_t(255) : 0;
-    const size_t wrap_row_bytes = pl.row.fuse ? static_cast<size_t>(pl.c - 1) * pitch : 0;
-    const size_t wrap_bytes = pl.engine == ENG_C2R ? (wrap_row_bytes * batch + 255) & ~size_t(255) : 0;
-    if (pl.side_bytes && batch > 1) {
-        // Batches: keep the side blocks within max(256 MiB, 1/32 of the data) -- a smaller D.
-        const double cap = std::max(256.0 * (1 << 20), full / 2.0 / 32.0);
-        const double per_tile = static_cast<double>(pl.M) * pl.shuf.p.W * pl.eb * static_cast<double>(batch);
-        const int64_t dmax = static_cast<int64_t>(cap / per_tile);
-        if (dmax < pl.shuf.p.lagD) set_lag(pl, dmax);
-    }
-    const size_t side_bytes = pl.side_bytes * static_cast<size_t>(batch);
-    if (flag_bytes + wrap_bytes + side_bytes) {
-        cudaMemPool_t pool = scratch_pool();
-        if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&fscratch), flag_bytes + wrap_bytes + side_bytes,
-                                             pool, st) != cudaSuccess) {
-            cudaGetLastError();
-            return IPT_ERR_OUT_OF_MEMORY;
-        }
-        pl.row.flags = reinterpret_cast<unsigned int *>(fscratch);
-        pl.row.wrap = fscratch + flag_bytes;
-        pl.row.side = pl.shuf.p.side = side_bytes ? fscratch + flag_bytes + wrap_bytes : nullptr;
-        ipt_status_t s0 = flag_bytes ? check(cudaMemsetAsync(fscratch, 0, flag_bytes, st)) : IPT_OK;
-        if (s0 == IPT_OK && wrap_bytes)
-            s0 = check(cudaMemcpy2DAsync(fscratch + flag_bytes, wrap_row_bytes, base, stride_bytes, wrap_row_bytes,
-                                         batch, cudaMemcpyDeviceToDevice, st));
-        if (s0 != IPT_OK) {
-            cudaFreeAsync(fscratch, st);
-            return s0;
-        }
-    }
-    struct FreeScratch {
-        char *p;
-        cudaStream_t st;
-        ~FreeScratch() {
-            if (p) cudaFreeAsync(p, st);
-        }
-    } free_scratch{fscratch, st};
     const int passes = budget;
+    // The rotation moves only the columns with a non-zero amount: (c - 1) / c of them.
+    const double rot_bytes = full * static_cast<double>(pl.c - 1) / static_cast<double>(pl.c);
+    auto rot = [&] { return launch_col(pl.rot.p, COL_ROT, pl.eb, st, pl.rot.smem); };
+    auto row = [&] {
+        if (pl.row.fuse) {  // rows 0..c-2 of every matrix into the wrap slots first
+            cudaError_t e = launch_copy_wrap(pl.row, pl.eb, st);
+            if (e != cudaSuccess) return e;
+        }
+        return pl.row.cl_K ? launch_row_cluster(pl.row, pl.row_dir, pl.eb, st) : launch_row(pl.row, pl.row_dir, pl.eb, st);
+    };
     if (pl.engine == ENG_C2R) {
         auto shuf = [&] { return launch_col(pl.shuf.p, COL_C2R_SHUF, pl.eb, st, pl.shuf.smem); };
         if (pl.has_rot && (s = run(PK_ROT, rot_bytes, rot)) != IPT_OK) return s;  // Eq. 23
@@ -674,7 +717,7 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
     }
     // IPT_DEBUG_PASSES stopping between the row and column passes of a lagged plan: put the
     // logical layout back (side tile -> columns [0, W), A columns [0, N - W) -> [W, N)) so
-    // the snapshot compares with the oracle's.
+    // the snapshot compares with the oracle's.  Tests only (small matrices).
     if (pl.side_bytes && passes < (1 << 30)) {
         const int before_second = pl.engine == ENG_C2R ? (pl.has_rot ? 2 : 1) : 1;  // passes up to the lagged state
         if (passes == before_second) {
@@ -699,26 +742,70 @@ ipt_status_t execute(const Plan &pl0, char *base, int64_t batch, int64_t stride_
     return IPT_OK;
 }
 
+// A resolved engine call: plan, scratch layout; run = allocate + launch + free.
+struct Call {
+    Plan pl;
+    CallScratch cs;
+    int64_t batch = 0;
+};
+
+ipt_status_t resolve(int64_t x, int64_t y, int eb, int64_t batch, Call &c) {
+    c = Call{};
+    c.batch = batch;
+    if (x <= 1 || y <= 1 || batch == 0) return IPT_OK;  // identity: engine NONE
+    ipt_status_t s = cached_plan(x, y, eb, c.pl);
+    if (s != IPT_OK) return s;
+    prepare_call(c.pl, batch, c.cs);
+    return IPT_OK;
+}
+
+ipt_status_t launch_resolved(const Call &c, char *base, int64_t stride_bytes, cudaStream_t st, char *scratch) {
+    return launch_call(c.pl, c.cs, base, c.batch, stride_bytes, st, scratch);
+}
+
+ipt_status_t run_resolved(const Call &c, char *base, int64_t stride_bytes, cudaStream_t st) {
+    char *scratch = nullptr;
+    ipt_status_t s = pool_alloc(&scratch, c.cs.total, st);
+    if (s != IPT_OK) return s;
+    s = launch_resolved(c, base, stride_bytes, st, scratch);
+    if (scratch) cudaFreeAsync(scratch, st);
+    return s;
+}
+
 bool valid_eb(int eb) { return eb == 4 || eb == 8 || eb == 16; }
 
-// Validate and run P_{x,y} on `batch` matrices of x*y elements, `stride` elements apart.
-// stride < 0 means "packed" (stride = x*y), used by the single-matrix entry points.
-ipt_status_t run_perm(void *ptr, int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, void *stream) {
-    if (!valid_eb(eb) || x < 0 || y < 0 || batch < 0) return IPT_ERR_INVALID_ARGUMENT;
+// Shared argument checks of every entry point: sizes, strides, overflow, pointer.  Returns
+// IPT_OK with `done` set when there is nothing to do (empty / identity).
+ipt_status_t check_args(void *ptr, int64_t batch, int64_t &stride, int64_t x, int64_t y, int64_t eb, int64_t align,
+                        bool &done) {
+    done = false;
+    if (x < 0 || y < 0 || batch < 0) return IPT_ERR_INVALID_ARGUMENT;
     if (x != 0 && y > INT64_MAX / x) return IPT_ERR_INVALID_ARGUMENT;
     const int64_t elems = x * y;
     if (stride < 0) stride = elems;
     if (stride < elems) return IPT_ERR_INVALID_ARGUMENT;
     if (stride != 0 && batch > INT64_MAX / stride) return IPT_ERR_INVALID_ARGUMENT;
     if (elems != 0 && batch * stride > INT64_MAX / eb) return IPT_ERR_INVALID_ARGUMENT;
-    if (elems == 0 || batch == 0) return IPT_OK;
-    if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % static_cast<uintptr_t>(eb) != 0)
+    if (elems == 0 || batch == 0) {
+        done = true;
+        return IPT_OK;
+    }
+    if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % static_cast<uintptr_t>(align) != 0)
         return IPT_ERR_INVALID_ARGUMENT;
-    if (x <= 1 || y <= 1) return IPT_OK;  // P_{1,y} and P_{x,1} are the identity
-    Plan pl;
-    ipt_status_t s = cached_plan(x, y, eb, pl);
-    if (s != IPT_OK) return s;
-    return execute(pl, static_cast<char *>(ptr), batch, stride * eb, static_cast<cudaStream_t>(stream));
+    if (x <= 1 || y <= 1) done = true;  // P_{1,y} and P_{x,1} are the identity
+    return IPT_OK;
+}
+
+// Validate and run P_{x,y} on `batch` matrices of x*y elements, `stride` elements apart.
+// stride < 0 means "packed" (stride = x*y), used by the single-matrix entry points.
+ipt_status_t run_perm(void *ptr, int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, void *stream) {
+    if (!valid_eb(eb)) return IPT_ERR_INVALID_ARGUMENT;
+    bool done = false;
+    ipt_status_t s = check_args(ptr, batch, stride, x, y, eb, eb, done);
+    if (s != IPT_OK || done) return s;
+    Call c;
+    if ((s = resolve(x, y, eb, batch, c)) != IPT_OK) return s;
+    return run_resolved(c, static_cast<char *>(ptr), stride * eb, static_cast<cudaStream_t>(stream));
 }
 
 // Multi-word elements (the paper's passes move opaque words whatever their
@@ -756,6 +843,50 @@ int word_bytes_of(int eb, uintptr_t addr) {
     return 4;
 }
 
+// A composed call (records, sub-word elements): up to two engine steps and one record-block
+// pass, all resolved (plans, scratch sizes, UNSUPPORTED checks) before anything is
+// enqueued, with ONE scratch allocation for all of them -- so IPT_ERR_UNSUPPORTED and
+// IPT_ERR_OUT_OF_MEMORY leave the buffer untouched, as ipt.h promises.
+struct Composed {
+    Call e1, e2;                // engine steps (e2 only for the all-engine fallback)
+    int64_t e1_stride = 0, e2_stride = 0;  // matrix strides of the engine steps, bytes
+    bool blocks = false;        // a record-block pass
+    bool blocks_first = false;  // the block pass runs before e1 (merge / split orientation)
+    RecordParams rp{};
+    int rec_w = 4;              // launch_record_blocks word argument
+    size_t rec_tmp = 0;         // global slots of the block pass
+    int64_t e2_loops = 0;       // e2 per matrix (strided batch): > 0 loops this many times
+    int64_t e2_mat_stride = 0;  // bytes between those matrices
+};
+
+ipt_status_t run_composed(const Composed &C, char *base, cudaStream_t st) {
+    const size_t s1 = C.e1.cs.total, s2 = C.e2.cs.total;
+    const size_t o_rec = al256(std::max(s1, s2));
+    char *scratch = nullptr;
+    ipt_status_t s = pool_alloc(&scratch, o_rec + C.rec_tmp, st);
+    if (s != IPT_OK) return s;
+    auto blocks = [&]() -> ipt_status_t {
+        RecordParams rp = C.rp;
+        rp.tmp = C.rec_tmp ? scratch + o_rec : nullptr;
+        ipt_status_t r = check(launch_record_blocks(rp, C.rec_w, st));
+        if (r == IPT_OK) g_launches++;
+        return r;
+    };
+    if (C.blocks && C.blocks_first) s = blocks();
+    if (s == IPT_OK) s = launch_resolved(C.e1, base, C.e1_stride, st, scratch);
+    if (s == IPT_OK && C.blocks && !C.blocks_first) s = blocks();
+    if (s == IPT_OK && C.e2.batch) {
+        if (C.e2_loops == 0) {
+            s = launch_resolved(C.e2, base, C.e2_stride, st, scratch);
+        } else {
+            for (int64_t b = 0; b < C.e2_loops && s == IPT_OK; ++b)
+                s = launch_resolved(C.e2, base + b * C.e2_mat_stride, C.e2_stride, st, scratch);
+        }
+    }
+    if (scratch) cudaFreeAsync(scratch, st);
+    return s;
+}
+
 // Sub-word elements (1 or 2 bytes): g = 4 / eb elements share one 4-byte
 // engine word.  y % g == 0: P_{x,y/g} on words (row j' holds x g-tuples of row elements
 // g*j' .. g*j'+g-1), then split each row's x-by-g tuples into g rows of x elements.
@@ -765,17 +896,7 @@ int word_bytes_of(int eb, uintptr_t addr) {
 // scratch budget and batch strides that are not a whole number of words.
 bool valid_subword_eb(int eb) { return eb == 1 || eb == 2; }
 
-ipt_status_t run_perm_subword(void *ptr, int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, void *stream) {
-    if (x < 0 || y < 0 || batch < 0) return IPT_ERR_INVALID_ARGUMENT;
-    if (x != 0 && y > INT64_MAX / x) return IPT_ERR_INVALID_ARGUMENT;
-    const int64_t elems = x * y;
-    if (stride < 0) stride = elems;
-    if (stride < elems) return IPT_ERR_INVALID_ARGUMENT;
-    if (stride != 0 && batch > INT64_MAX / stride) return IPT_ERR_INVALID_ARGUMENT;
-    if (elems != 0 && batch * stride > INT64_MAX / eb) return IPT_ERR_INVALID_ARGUMENT;
-    if (elems == 0 || batch == 0) return IPT_OK;
-    if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % 4 != 0) return IPT_ERR_INVALID_ARGUMENT;
-    if (x <= 1 || y <= 1) return IPT_OK;
+ipt_status_t resolve_subword(int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, Composed &C) {
     const int64_t g = 4 / eb;
     // Of the feasible orientations, the one with the shorter blocks (L = x for split, y for merge).
     const bool split = y % g == 0 && (x % g != 0 || x <= y);
@@ -784,8 +905,8 @@ ipt_status_t run_perm_subword(void *ptr, int64_t batch, int64_t stride, int64_t 
     int64_t slots = 0;
     if (record_slots(L * 4, nblocks, slots) != IPT_OK) return IPT_ERR_CUDA;
     if (slots < 0 || L * g >= (int64_t(1) << 32)) return IPT_ERR_UNSUPPORTED;
-    RecordParams rp{};
-    rp.base = static_cast<char *>(ptr);
+    RecordParams &rp = C.rp;
+    rp = RecordParams{};
     rp.per_mat = per_mat;
     rp.nblocks = nblocks;
     rp.mat_stride_bytes = stride * eb;
@@ -796,59 +917,33 @@ ipt_status_t run_perm_subword(void *ptr, int64_t batch, int64_t stride, int64_t 
     rp.fd_k = make_fastdiv(static_cast<uint32_t>(g));
     rp.fd_L = make_fastdiv(static_cast<uint32_t>(L));
     rp.grid = static_cast<uint32_t>(slots);
-    cudaStream_t cst = static_cast<cudaStream_t>(stream);
-    auto blocks = [&] {
-        if (slots) {
-            cudaMemPool_t pool = scratch_pool();
-            if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&rp.tmp), static_cast<size_t>(slots * L * 4),
-                                                 pool, cst) != cudaSuccess) {
-                cudaGetLastError();
-                return IPT_ERR_OUT_OF_MEMORY;
-            }
-        }
-        ipt_status_t r = check(launch_record_blocks(rp, eb, cst));
-        if (rp.tmp) cudaFreeAsync(rp.tmp, cst);
-        if (r == IPT_OK) g_launches++;
-        return r;
-    };
-    if (split) {
-        ipt_status_t s = run_perm(ptr, batch, stride / g, x, y / g, 4, stream);
-        return s == IPT_OK ? blocks() : s;
-    }
-    ipt_status_t s = blocks();
-    return s == IPT_OK ? run_perm(ptr, batch, stride / g, x / g, y, 4, stream) : s;
+    C.blocks = true;
+    C.blocks_first = !split;
+    C.rec_w = eb;
+    C.rec_tmp = static_cast<size_t>(slots * L * 4);
+    C.e1_stride = stride / g * 4;
+    return split ? resolve(x, y / g, 4, batch, C.e1) : resolve(x / g, y, 4, batch, C.e1);
 }
 
-ipt_status_t run_perm_any(void *ptr, int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, void *stream) {
-    if (valid_subword_eb(eb)) return run_perm_subword(ptr, batch, stride, x, y, eb, stream);
-    if (!valid_multiword_eb(eb)) return run_perm(ptr, batch, stride, x, y, eb, stream);
-    if (x < 0 || y < 0 || batch < 0) return IPT_ERR_INVALID_ARGUMENT;
-    if (x != 0 && y > INT64_MAX / x) return IPT_ERR_INVALID_ARGUMENT;
-    const int64_t elems = x * y;
-    const bool packed = stride < 0;
-    if (packed) stride = elems;
-    if (stride < elems) return IPT_ERR_INVALID_ARGUMENT;
-    if (stride != 0 && batch > INT64_MAX / stride) return IPT_ERR_INVALID_ARGUMENT;
-    if (elems != 0 && batch * stride > INT64_MAX / eb) return IPT_ERR_INVALID_ARGUMENT;
-    if (elems == 0 || batch == 0) return IPT_OK;
-    if (ptr == nullptr || reinterpret_cast<uintptr_t>(ptr) % 4 != 0) return IPT_ERR_INVALID_ARGUMENT;
-    if (x <= 1 || y <= 1) return IPT_OK;
-    const int w = word_bytes_of(eb, reinterpret_cast<uintptr_t>(ptr));
+ipt_status_t resolve_multiword(int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, uintptr_t addr,
+                               Composed &C) {
+    const int w = word_bytes_of(eb, addr);
     const int64_t k = eb / w;
     const int64_t L = std::min(x, y);
     const int64_t per_mat = std::max(x, y), nblocks = batch * per_mat;
     int64_t slots = 0;
     if (record_slots(L * eb, nblocks, slots) != IPT_OK) return IPT_ERR_CUDA;
+    C.e1_stride = stride * eb;  // = stride * k words of w bytes
     if (slots >= 0 && nblocks < (int64_t(1) << 40)) {
         // The block step on the shorter side, staged in shared memory (records.cu):
         //   x <= y: P_{x,y*k} on words, then merge each k-by-x block into x records;
         //   x >  y: split each row of y records into k-by-y words, then P_{x*k,y} on words
         //           (row i*k + v holds word v of row i, so P_{x*k,y} leaves record (i,j)
         //           at row j, words i*k .. i*k+k-1).
-        RecordParams rp{};
-        rp.base = static_cast<char *>(ptr);
-        rp.per_mat = std::max(x, y);
-        rp.nblocks = batch * rp.per_mat;
+        RecordParams &rp = C.rp;
+        rp = RecordParams{};
+        rp.per_mat = per_mat;
+        rp.nblocks = nblocks;
         rp.mat_stride_bytes = stride * eb;
         rp.blk_stride_bytes = L * eb;
         rp.L = static_cast<uint32_t>(L);
@@ -856,75 +951,76 @@ ipt_status_t run_perm_any(void *ptr, int64_t batch, int64_t stride, int64_t x, i
         rp.split = x > y;
         rp.fd_k = make_fastdiv(static_cast<uint32_t>(k));
         rp.grid = static_cast<uint32_t>(slots);
-        cudaStream_t cst = static_cast<cudaStream_t>(stream);
-        auto blocks = [&] {
-            if (slots) {
-                cudaMemPool_t pool = scratch_pool();
-                if (!pool || cudaMallocFromPoolAsync(reinterpret_cast<void **>(&rp.tmp),
-                                                     static_cast<size_t>(slots * L * eb), pool, cst) != cudaSuccess) {
-                    cudaGetLastError();
-                    return IPT_ERR_OUT_OF_MEMORY;
-                }
-            }
-            ipt_status_t r = check(launch_record_blocks(rp, w, cst));
-            if (rp.tmp) cudaFreeAsync(rp.tmp, cst);
-            if (r == IPT_OK) g_launches++;
-            return r;
-        };
-        if (x <= y) {
-            ipt_status_t s = run_perm(ptr, batch, stride * k, x, y * k, w, stream);
-            return s == IPT_OK ? blocks() : s;
-        }
-        ipt_status_t s = blocks();
-        return s == IPT_OK ? run_perm(ptr, batch, stride * k, x * k, y, w, stream) : s;
+        C.blocks = true;
+        C.blocks_first = x > y;
+        C.rec_w = w;
+        C.rec_tmp = static_cast<size_t>(slots * L * eb);
+        return x <= y ? resolve(x, y * k, w, batch, C.e1) : resolve(x * k, y, w, batch, C.e1);
     }
-    // Blocks too long for one CTA: both steps on the engine.
-    ipt_status_t s = run_perm(ptr, batch, stride * k, x, y * k, w, stream);  // P_{x, y k}
+    // Blocks too long for one CTA: both steps on the engine, P_{x, y k} then P_{k, x} on
+    // every k-by-x block.
+    ipt_status_t s = resolve(x, y * k, w, batch, C.e1);
     if (s != IPT_OK) return s;
-    if (batch == 1 || stride == elems)  // every k-by-x block of every matrix is k*x words apart
-        return run_perm(ptr, batch * y, k * x, k, x, w, stream);
-    for (int64_t b = 0; b < batch && s == IPT_OK; ++b)
-        s = run_perm(static_cast<char *>(ptr) + b * stride * eb, y, k * x, k, x, w, stream);
-    return s;
+    if (batch == 1 || stride == x * y) {  // every k-by-x block of every matrix is k*x words apart
+        C.e2_stride = k * x * w;
+        return resolve(k, x, w, batch * y, C.e2);
+    }
+    C.e2_stride = k * x * w;
+    C.e2_loops = batch;
+    C.e2_mat_stride = stride * eb;
+    return resolve(k, x, w, y, C.e2);
 }
 
-// Plan description of a record call P_{x,y} (16-byte-aligned base assumed): `pl` is the
-// plan of its word-level engine step, widened by the other step's scratch and staging;
-// `extra` counts the other step's launches.
-ipt_status_t record_plan(int64_t x, int64_t y, int eb, Plan &pl, int64_t &extra) {
-    if (valid_subword_eb(eb)) {  // plan of the packed-word engine step (run_perm_subword)
-        const int64_t g = 4 / eb;
-        if (y % g != 0 && x % g != 0) return IPT_ERR_UNSUPPORTED;
-        const bool split = y % g == 0 && (x % g != 0 || x <= y);  // as run_perm_subword
-        ipt_status_t s = split ? make_plan(x, y / g, 4, pl) : make_plan(x / g, y, 4, pl);
-        if (s != IPT_OK) return s;
-        extra = 1;
-        const int64_t blk = 4 * (split ? x : y);
-        if (blk <= static_cast<int64_t>(kRecordSmemMax)) pl.onchip = std::max(pl.onchip, static_cast<size_t>(blk));
-        return IPT_OK;
-    }
-    const int w = word_bytes_of(eb, 0);
-    const int64_t k = eb / w;
-    if (x < 0 || y < 0 || (y != 0 && k > INT64_MAX / y) || (x != 0 && k > INT64_MAX / x))
-        return IPT_ERR_INVALID_ARGUMENT;
-    const int64_t L = std::min(x, y);
-    int64_t slots = 0;
-    if (record_slots(L * eb, std::max(x, y), slots) != IPT_OK) return IPT_ERR_CUDA;
-    if (slots >= 0) {
-        ipt_status_t s = x <= y ? make_plan(x, y * k, w, pl) : make_plan(x * k, y, w, pl);
-        if (s != IPT_OK) return s;
-        extra = 1;
-        if (slots == 0) pl.onchip = std::max(pl.onchip, static_cast<size_t>(L * eb));
-        else pl.scratch = std::max(pl.scratch, static_cast<size_t>(slots * L * eb));
-        return IPT_OK;
-    }
-    Plan p2;
-    ipt_status_t s = make_plan(x, y * k, w, pl);
-    if (s == IPT_OK) s = make_plan(k, x, w, p2);
+ipt_status_t run_perm_any(void *ptr, int64_t batch, int64_t stride, int64_t x, int64_t y, int eb, void *stream) {
+    if (valid_eb(eb)) return run_perm(ptr, batch, stride, x, y, eb, stream);
+    if (!valid_subword_eb(eb) && !valid_multiword_eb(eb)) return IPT_ERR_INVALID_ARGUMENT;
+    bool done = false;
+    ipt_status_t s = check_args(ptr, batch, stride, x, y, eb, 4, done);
+    if (s != IPT_OK || done) return s;
+    Composed C;
+    s = valid_subword_eb(eb) ? resolve_subword(batch, stride, x, y, eb, C)
+                             : resolve_multiword(batch, stride, x, y, eb, reinterpret_cast<uintptr_t>(ptr), C);
     if (s != IPT_OK) return s;
-    extra = p2.nlaunch;
-    pl.scratch = std::max(pl.scratch, p2.scratch);
-    pl.onchip = std::max(pl.onchip, p2.onchip);
+    C.rp.base = static_cast<char *>(ptr);
+    return run_composed(C, static_cast<char *>(ptr), static_cast<cudaStream_t>(stream));
+}
+
+// Plan description of a single-word call: the plan, with pl.scratch = the bytes the call
+// allocates (CallScratch of one matrix).
+ipt_status_t engine_plan(int64_t x, int64_t y, int eb, Plan &pl) {
+    ipt_status_t s = make_plan(x, y, eb, pl);
+    if (s != IPT_OK) return s;
+    CallScratch cs;
+    prepare_call(pl, 1, cs);
+    pl.scratch = cs.total;
+    return IPT_OK;
+}
+
+// Plan description of a record / sub-word call P_{x,y} (16-byte-aligned base assumed, one
+// matrix): `pl` is the plan of its (first) word-level engine step, widened by the other
+// steps' scratch and staging; `extra` counts the other steps' launches.  Same resolution
+// as the run (resolve_subword / resolve_multiword), so UNSUPPORTED agrees with execution.
+ipt_status_t record_plan(int64_t x, int64_t y, int eb, Plan &pl, int64_t &extra) {
+    if (x < 0 || y < 0) return IPT_ERR_INVALID_ARGUMENT;
+    if (x != 0 && y > INT64_MAX / x) return IPT_ERR_INVALID_ARGUMENT;
+    pl = Plan{};
+    pl.eb = eb;
+    extra = 0;
+    if (x <= 1 || y <= 1) return IPT_OK;
+    Composed C;
+    ipt_status_t s = valid_subword_eb(eb) ? resolve_subword(1, x * y, x, y, eb, C)
+                                          : resolve_multiword(1, x * y, x, y, eb, 0, C);
+    if (s != IPT_OK) return s;
+    pl = C.e1.pl;
+    pl.scratch = std::max(C.e1.cs.total, C.e2.cs.total) + C.rec_tmp;
+    if (C.blocks) {
+        extra = 1;
+        if (!C.rec_tmp) pl.onchip = std::max(pl.onchip, static_cast<size_t>(C.rp.L) * C.rp.k * C.rec_w);
+    }
+    if (C.e2.batch) {
+        extra += C.e2.pl.nlaunch;
+        pl.onchip = std::max(pl.onchip, C.e2.pl.onchip);
+    }
     return IPT_OK;
 }
 
@@ -961,25 +1057,6 @@ cudaError_t ensure_kernel_attrs(const void *kern, size_t smem, bool nonportable_
     }
     smem_set[key] = lim | ((have | want) & (size_t(1) << 62));
     return cudaSuccess;
-}
-
-unsigned int *group_counters(cudaStream_t st, int n) {
-    if (n > kMaxGroups) return nullptr;
-    static std::mutex mu;
-    static std::unordered_map<std::string, unsigned int *> blocks;
-    int dev = 0;
-    cudaGetDevice(&dev);
-    const std::string key = std::to_string(dev) + "/" + std::to_string(reinterpret_cast<uintptr_t>(st));
-    std::lock_guard<std::mutex> lk(mu);
-    auto it = blocks.find(key);
-    if (it != blocks.end()) return it->second;
-    unsigned int *p = nullptr;
-    if (cudaMalloc(&p, sizeof(unsigned int) * kMaxGroups) != cudaSuccess) {
-        cudaGetLastError();
-        return nullptr;
-    }
-    blocks[key] = p;
-    return p;
 }
 
 int cached_resident_blocks(const void *kern, int threads, size_t smem) {
@@ -1051,7 +1128,7 @@ ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *glo
     Plan pl;
     ipt_status_t s;
     if (valid_eb(elem_bytes)) {
-        s = make_plan(m, n, elem_bytes, pl);
+        s = engine_plan(m, n, elem_bytes, pl);
     } else {
         int64_t extra = 0;
         s = record_plan(m, n, elem_bytes, pl, extra);
@@ -1073,7 +1150,7 @@ ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t la
     int64_t extra_launches = 0;
     ipt_status_t s;
     if (valid_eb(elem_bytes)) {
-        s = make_plan(x, y, elem_bytes, pl);
+        s = engine_plan(x, y, elem_bytes, pl);
     } else {  // multi-word element: plan of the engine step, launches of both
         s = record_plan(x, y, elem_bytes, pl, extra_launches);
     }
@@ -1127,7 +1204,16 @@ ipt_status_t ipt_debug_tile_copy(void *ptr, int64_t M, int64_t N, int elem_bytes
     p.resident = col_resident_ctas(COL_COPY, elem_bytes, tile_bytes, smem, pipe, p.threads);
     if (p.resident < p.G) return IPT_ERR_UNSUPPORTED;
     finish_col(p, 1);
-    return check(launch_col(p, COL_COPY, elem_bytes, static_cast<cudaStream_t>(stream), smem));
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    char *ctr = nullptr;
+    ipt_status_t s = pool_alloc(&ctr, kCtrBytes, st);
+    if (s != IPT_OK) return s;
+    s = check(cudaMemsetAsync(ctr, 0, kCtrBytes, st));
+    p.ctr = reinterpret_cast<unsigned int *>(ctr);
+    p.ticket = 1;
+    if (s == IPT_OK) s = check(launch_col(p, COL_COPY, elem_bytes, st, smem));
+    cudaFreeAsync(ctr, st);
+    return s;
 }
 
 void ipt_profile_enable(int on) { g_prof_on.store(on ? 1 : 0); }

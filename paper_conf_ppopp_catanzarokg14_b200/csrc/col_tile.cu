@@ -416,14 +416,16 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
 template <int EB, int MODE, int TWB>
 __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
-    // Unit order.  Barrier mode: a dispatch ticket (an atomic), so a tile's G members are G
-    // consecutive dispatches -- the whole group is co-resident.  Lagged layouts only ever wait
-    // for units of smaller index, and CTAs are dispatched in blockIdx order (the premise of
-    // single-pass scans' decoupled look-back), so the block index serves and the ticket's
-    // atomic round trip (~5 % of a loads-only pass, IPT_COL_DEBUG=3) is saved.
+    // Unit order = dispatch-ticket order (an atomic taken at start).  Barrier mode: a tile's
+    // G members are G consecutive dispatches, so the whole group is co-resident.  Lagged
+    // layouts only ever wait for units of smaller ticket, which were taken by CTAs already
+    // running: no assumption about the order in which the hardware dispatches blocks, or
+    // about co-residency with other kernels (MPS, other streams).  P.ticket = 0
+    // (IPT_COL_TICKET=0, measurement only) uses the block index instead in lagged mode,
+    // which relies on blocks being dispatched in index order.
     __shared__ unsigned int s_ticket;
     unsigned int ticket = blockIdx.x;
-    if (P.lag == LAG_NONE && P.dbg != 3) {
+    if ((P.lag == LAG_NONE || P.ticket) && P.dbg != 3) {
         if (threadIdx.x == 0) s_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
         __syncthreads();
         ticket = s_ticket;
@@ -672,11 +674,8 @@ cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, s
     const int64_t grid = P.pipe ? std::min<int64_t>(P.resident, units)
                                 : P.G == 1 ? (P.total_tiles + P.tpc - 1) / P.tpc : units;
     if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
-    // Ticket + group counters: the stream's own block, zeroed in stream order.
-    P.ctr = group_counters(st, kCtrSlots + 1);
-    if (!P.ctr) return cudaErrorMemoryAllocation;
-    e = cudaMemsetAsync(P.ctr, 0, sizeof(unsigned int) * (kTicketSlot + 1), st);
-    if (e != cudaSuccess) return e;
+    // Ticket + group counters: the call's own zeroed scratch (api.cu CallScratch).
+    if (!P.ctr) return cudaErrorInvalidValue;
     void *args[] = {&P};
     const int threads = P.threads > 0 ? P.threads : kColThreads;
     return cudaLaunchKernel(kern, dim3(static_cast<unsigned>(grid)), dim3(threads), args, smem, st);

@@ -38,6 +38,12 @@ __host__ __device__ inline char *side_matrix(char *side, int64_t sstride, int64_
     char *raw = side + mat * sstride;
     return raw + ((reinterpret_cast<uintptr_t>(A_mat) - reinterpret_cast<uintptr_t>(raw)) & 15);
 }
+// Wrap rows of the fused rotation: matrix k's copy of rows 0..c-2, placed so that copy row i
+// has the same address mod 16 as row i of the matrix (staged with the same 16-byte copies).
+__host__ __device__ inline char *wrap_matrix(char *wrap, int64_t wstride, int64_t mat, const char *A_mat) {
+    char *raw = wrap + mat * wstride;
+    return raw + ((reinterpret_cast<uintptr_t>(A_mat) - reinterpret_cast<uintptr_t>(raw)) & 15);
+}
 // Row-shuffle directions.
 enum RowDir : int {
     ROW_C2R = 0,  // out[i][j] = in[i][d'^{-1}_i(j)]  (Eq. 31)
@@ -89,7 +95,11 @@ struct RowParams {
     int32_t segp;            // C2R staircase: shared bytes per source segment (b elements)
     FastDiv fd_cps;          // segp / 16 (16-byte chunks per segment)
     unsigned int *flags;     // per-row "read" flags (M * batch, zeroed per call)
-    const char *wrap;        // C2R: copy of rows 0..c-2 of every matrix (batch x (c-1) rows)
+    unsigned int *ticket;    // row-group dispatch ticket of the fused pass (zeroed per call)
+    char *wrap;              // copy of rows 0..c-2 of every matrix (wrap_matrix(); taken before
+                             // the fused pass: C2R staircases past row M-1 read it, R2C reads
+                             // rows 0..c-2 from it so that writes into them need no wait)
+    int64_t wstride;         // bytes reserved per matrix in `wrap`
 };
 constexpr int kMaxFuseC = 32;
 
@@ -107,7 +117,9 @@ struct ColParams {
     int32_t ngroups;    // groups in the persistent grid (grid = ngroups * G)
     int32_t resident;   // co-resident CTAs of this configuration (SMs x CTAs per SM)
     int64_t total_tiles;  // ntiles * batch
-    unsigned int *ctr;  // per-group arrival counters (stream-ordered scratch, launch_col)
+    unsigned int *ctr;  // arrival counters + dispatch ticket: kCtrSlots + 1 words of the call's
+                        // stream-ordered scratch, zeroed before the launch (api.cu CallScratch)
+    int32_t ticket;     // 1: units in dispatch-ticket order (an atomic per CTA); 0: block index
     int32_t rot_sign;   // COL_ROT: +1 (C2R pre-rotation) or -1 (R2C post-rotation)
     int32_t wide_a;     // a >= 2^16
     FastDiv fd_G, fd_nt;  // ticket -> (tile, band), tile -> (matrix, column tile)
@@ -154,15 +166,16 @@ struct SkinnyRowParams {
 cudaError_t ensure_kernel_attrs(const void *kern, size_t smem, bool nonportable_cluster);
 int cached_resident_blocks(const void *kern, int threads, size_t smem);  // SMs x blocks per SM
 
-// Group-barrier counters of the column passes: one block per (device, stream), allocated
-// on first use and reused by every later launch on that stream (launches on one stream
-// are serialised; different streams never share a block).  Slots [0, kCtrSlots) are the
+// Group-barrier counters of a column pass: kCtrSlots + 1 words of the CALL's scratch
+// (allocated and zeroed in stream order per call, so concurrent calls -- other threads,
+// other streams, cudaStreamPerThread -- never share them).  Slots [0, kCtrSlots) are the
 // per-tile arrival counters (tile t uses slot t mod kCtrSlots), slot kTicketSlot is the
 // dispatch ticket.
 constexpr int kCtrSlots = 4096;  // a power of two
 constexpr int kTicketSlot = kCtrSlots;
-constexpr int kMaxGroups = kCtrSlots + 1;
-unsigned int *group_counters(cudaStream_t st, int n);
+constexpr size_t kCtrBytes = (sizeof(unsigned int) * (kCtrSlots + 1) + 255) & ~size_t(255);
+// Copy rows 0..c-2 of every matrix into the wrap buffer (row_shuffle.cu).
+cudaError_t launch_copy_wrap(const RowParams &p, int eb, cudaStream_t st);
 
 // Launchers (col_tile.cu / row_shuffle.cu).  They return the CUDA error of the launch.
 size_t row_smem_bytes(int64_t N, int eb);

@@ -19,6 +19,7 @@
 // so a lane spends a handful of integer adds per element (§4.4's strength reduction
 // taken one step further); f2 can only be 1 in the last c - 1 rows, which take a
 // slower walk that tracks l.
+#include <algorithm>
 #include <array>
 #include <map>
 #include <mutex>
@@ -507,14 +508,14 @@ __device__ __forceinline__ void gather_row_rot(const RowParams &P, char *mbase, 
 template <int EB, int DIR, int NBUF>
 __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ uint32_t s_cur, s_next;
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
     const uint32_t rowbuf = static_cast<uint32_t>(row_fused_smem_bytes(P, EB, DIR));
     const uint32_t bufbytes = rowbuf * static_cast<uint32_t>(P.R);
     const uint32_t padoff = static_cast<uint32_t>(P.c) * static_cast<uint32_t>(P.segp);  // C2R pad table
     const uint32_t sbase = smem_u32(smem);
-    const int64_t wrap_stride = static_cast<int64_t>(P.c - 1) * pitch;
     const int32_t gpm = (P.M + P.R - 1) / P.R;
-    const int64_t groups_total = static_cast<int64_t>(gpm) * P.batch;
+    const uint32_t groups_total = static_cast<uint32_t>(gpm) * static_cast<uint32_t>(P.batch);  // < 2^32 (planner)
     const int wn = (blockDim.x >> 5) / P.R;
     const int team = (threadIdx.x >> 5) / wn, wl = (threadIdx.x >> 5) - team * wn;
     const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;
@@ -524,18 +525,44 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P)
     const int32_t vdl = static_cast<int32_t>(vD % P.c);
     const int32_t vdh = static_cast<int32_t>((static_cast<int64_t>(P.ainv) * ((vD / P.c) % P.b)) % P.b);
 
+    // Work order.  Groups are handed out by a dispatch ticket (an atomic), C2R in ascending
+    // row order, R2C in descending row order within each matrix, so that every row a group
+    // waits for (C2R: rows i0-1 .. i0-c+1; R2C: rows i0+nr .. i0+nr+c-2 < M) belongs to a
+    // group with a SMALLER ticket -- one already taken by a running CTA.  The rows whose
+    // readers would otherwise come later (C2R: staircases past row M-1; R2C: writes of the
+    // last rows' blocks into rows 0..c-2) read the wrap copy of rows 0..c-2 instead, taken
+    // before this pass.  Progress (no co-residency assumption, no dispatch-order assumption):
+    // a group is flagged once it is staged and its CTA's previous group has been gathered; a
+    // gather waits only for flags of smaller tickets; by induction on the ticket, the
+    // smallest unflagged group gets flagged.
+    auto group_of = [&](uint32_t t) {
+        const uint32_t mat = fdiv(t, P.fd_gpm);
+        uint32_t gm = t - mat * static_cast<uint32_t>(gpm);
+        if (DIR == ROW_R2C) gm = static_cast<uint32_t>(gpm) - 1 - gm;
+        RowGroup G;
+        G.mat = mat;
+        G.i0 = static_cast<int32_t>(gm) * P.R;
+        G.nr = min(P.R, P.M - G.i0);
+        return G;
+    };
+    auto a_row = [&](const RowGroup &G, char *mb, int32_t i) -> const char * {
+        // R2C: rows 0..c-2 from their wrap copy (same address mod 16 as the row)
+        if (DIR == ROW_R2C && i < P.c - 1) return wrap_matrix(P.wrap, P.wstride, G.mat, mb) + i * pitch;
+        return mb + i * pitch;
+    };
     auto stage = [&](const RowGroup &G, int b) {
         char *mb = P.base + G.mat * P.mat_stride_bytes;
         for (int32_t rr = 0; rr < G.nr; ++rr) {
             const uint32_t o = b * bufbytes + rr * rowbuf;
+            const int32_t i = G.i0 + rr;
             if (DIR == ROW_C2R)
-                stage_stair<EB>(P, mb, P.wrap + G.mat * wrap_stride, G.i0 + rr, sbase + o,
+                stage_stair<EB>(P, mb, wrap_matrix(P.wrap, P.wstride, G.mat, mb), i, sbase + o,
                                 reinterpret_cast<int32_t *>(smem + o + padoff));
             else if (P.shW)
-                stage_row_lagged<EB>(P, mb + (G.i0 + rr) * pitch,
-                                     side_matrix(P.side, P.sstride, G.mat, mb) + (G.i0 + rr) * P.spitch, sbase + o);
+                stage_row_lagged<EB>(P, a_row(G, mb, i), side_matrix(P.side, P.sstride, G.mat, mb) + i * P.spitch,
+                                     sbase + o);
             else
-                stage_row_chunks<EB>(mb + (G.i0 + rr) * pitch, P.N * EB, sbase + o);
+                stage_row_chunks<EB>(a_row(G, mb, i), P.N * EB, sbase + o);
         }
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
@@ -550,10 +577,9 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P)
     };
     auto wait_deps = [&](const RowGroup &G) {  // every row the group overwrites has been read
         if (threadIdx.x >= 1 && threadIdx.x < P.c) {
-            int32_t y = DIR == ROW_C2R ? G.i0 - static_cast<int32_t>(threadIdx.x)
-                                       : G.i0 + G.nr - 1 + static_cast<int32_t>(threadIdx.x);
-            if (y >= P.M) y -= P.M;
-            if (y >= 0) {
+            const int32_t y = DIR == ROW_C2R ? G.i0 - static_cast<int32_t>(threadIdx.x)
+                                             : G.i0 + G.nr - 1 + static_cast<int32_t>(threadIdx.x);
+            if (y >= 0 && y < P.M) {
                 const unsigned int *f = P.flags + G.mat * P.M + y;
                 unsigned int v;
                 while (true) {
@@ -565,26 +591,31 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P)
         }
         __syncthreads();
     };
-    // NBUF = 2: group g + grid is staged while group g is gathered, and flagged as soon as
-    // the gather of group g is done -- a full group ahead of the moment its neighbours wait.
-    int64_t g = blockIdx.x;
-    RowGroup G = row_group(P, g, gpm);
-    if (g < groups_total) {
-        stage(G, 0);
-        asm volatile("cp.async.wait_group 0;" ::: "memory");
-        __syncthreads();
-        set_flags(G);
+    if (threadIdx.x == 0) {
+        s_cur = atomicAdd(P.ticket, 1u);
+        s_next = s_cur < groups_total ? atomicAdd(P.ticket, 1u) : groups_total;
     }
+    __syncthreads();
+    uint32_t tc = s_cur, tn = s_next;
+    if (tc >= groups_total) return;
+    // NBUF = 2: the next group is staged while the current one is gathered, and flagged as
+    // soon as the gather of the current group is done -- a full group ahead of the moment
+    // its neighbours wait.  The ticket after it is taken during the gather.
+    RowGroup G = group_of(tc);
+    stage(G, 0);
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncthreads();
+    set_flags(G);
     int buf = 0;
-    for (; g < groups_total; g += gridDim.x) {
+    while (tc < groups_total) {
         char *mbase = P.base + G.mat * P.mat_stride_bytes;
-        const int64_t ng = g + gridDim.x;
-        const RowGroup NG = row_group(P, ng, gpm);
-        const bool more = ng < groups_total;
+        const bool more = tn < groups_total;
+        const RowGroup NG = more ? group_of(tn) : G;
         if (NBUF == 2 && more) stage(NG, buf ^ 1);
         if (NBUF == 1 && more)  // single buffer: the next group's rows stream into L2 meanwhile
             prefetch_l2(P.base + NG.mat * P.mat_stride_bytes + NG.i0 * pitch, static_cast<int64_t>(NG.nr) * pitch);
         wait_deps(G);
+        if (threadIdx.x == 0 && more) s_next = atomicAdd(P.ticket, 1u);  // published by the barrier below
 
         if (team < G.nr) {
             const int32_t i = G.i0 + team;
@@ -617,7 +648,31 @@ __global__ void __launch_bounds__(kRowThreadsMax, 4) row_rot_kernel(RowParams P)
             }
         }
         if (NBUF == 2) buf ^= 1;
+        tc = tn;
         G = NG;
+        tn = more ? s_next : groups_total;
+    }
+}
+
+// Copy rows 0..c-2 of every matrix of the batch into its wrap slot (wrap_matrix: same address
+// mod 16 as the rows, so the body moves with 16-byte accesses; every offset is a multiple of 4).
+__global__ void __launch_bounds__(256) copy_wrap_kernel(char *base, int64_t mat_stride, int64_t batch, char *wrap,
+                                                        int64_t wstride, int64_t bytes) {
+    for (int64_t mat = blockIdx.y; mat < batch; mat += gridDim.y) {
+        const char *src = base + mat * mat_stride;
+        char *dst = wrap_matrix(wrap, wstride, mat, src);
+        const int64_t mis = static_cast<int64_t>((16 - (reinterpret_cast<uintptr_t>(src) & 15)) & 15);
+        const int64_t head = bytes < mis ? bytes : mis;
+        const int64_t body = (bytes - head) & ~int64_t(15);
+        const int64_t tid = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+        const int64_t nth = static_cast<int64_t>(gridDim.x) * blockDim.x;
+        for (int64_t k = tid; k < body / 16; k += nth)
+            stg16(dst + head + 16 * k, ldg16(src + head + 16 * k));
+        if (tid < head / 4)
+            reinterpret_cast<uint32_t *>(dst)[tid] = reinterpret_cast<const uint32_t *>(src)[tid];
+        const int64_t t0 = head + body;
+        if (tid < (bytes - t0) / 4)
+            reinterpret_cast<uint32_t *>(dst + t0)[tid] = reinterpret_cast<const uint32_t *>(src + t0)[tid];
     }
 }
 
@@ -885,7 +940,8 @@ cudaError_t launch_row_rot_t(const RowParams &P, cudaStream_t st) {
     cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
     if (e != cudaSuccess) return e;
     const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), threads, smem);
-    if (resident <= P.c) return cudaErrorInvalidConfiguration;  // the flag waits need > c co-resident CTAs
+    if (resident < 1) return cudaErrorInvalidConfiguration;
+    if (!P.ticket || !P.flags || !P.wrap) return cudaErrorInvalidValue;
     const int64_t rows = static_cast<int64_t>((P.M + P.R - 1) / P.R) * P.batch;
     int64_t grid = resident;
     if (grid > rows) grid = rows;
@@ -904,6 +960,17 @@ cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
 }
 
 }  // namespace
+
+cudaError_t launch_copy_wrap(const RowParams &P, int eb, cudaStream_t st) {
+    (void)eb;
+    const int64_t bytes = static_cast<int64_t>(P.c - 1) * P.N * eb;
+    if (bytes <= 0) return cudaSuccess;
+    const int64_t chunks = (bytes + 16 * 256 - 1) / (16 * 256);
+    const unsigned gx = static_cast<unsigned>(std::min<int64_t>(chunks, 64));
+    const unsigned gy = static_cast<unsigned>(std::min<int64_t>(P.batch, 65535));
+    copy_wrap_kernel<<<dim3(gx, gy), 256, 0, st>>>(P.base, P.mat_stride_bytes, P.batch, P.wrap, P.wstride, bytes);
+    return cudaGetLastError();
+}
 
 size_t row_smem_bytes(int64_t N, int eb) { return (static_cast<size_t>(N) * eb + 31) & ~size_t(15); }
 int row_block_threads() { return kRowThreadsMax; }

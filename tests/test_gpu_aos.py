@@ -64,17 +64,17 @@ def test_consumer_variants_agree(S, count):
 @pytest.mark.parametrize("count", [32 * 500, 32 * 500 + 7, 9])
 def test_random_access_gather_scatter(S, count):
     """warp_gather_aos / warp_scatter_aos (row f1, PAPER.md :1087, :1099): gather with a
-    random index vector (repeats allowed) equals numpy fancy indexing of the structs; scatter
-    through a random permutation equals numpy's inverse assignment; direct, vector and
-    cooperative variants agree; partial tail warps take the per-lane path."""
+    random index vector (repeats allowed) and scatter through a random permutation equal
+    the oracle's struct-by-struct definitions (oracle.aos_gather / aos_scatter, pinned to
+    numpy in test_oracle.py), bit for bit; direct, vector and cooperative variants all
+    match; partial tail warps take the per-lane path."""
     rng = np.random.default_rng(S * 1000 + count)
     nsrc = count + 37
     src_h = workloads.random_words(nsrc * S, 4, seed=S + count).reshape(nsrc, S)
     idx_h = rng.integers(0, nsrc, size=count, dtype=np.uint32)
-    want = src_h[idx_h]
+    want = oracle.aos_gather(src_h, idx_h, S).reshape(count, S)       # plain loops (oracle)
     perm = rng.permutation(count).astype(np.uint32)
-    want_sc = np.zeros((count, S), dtype=np.uint32)
-    want_sc[perm] = src_h[:count]
+    want_sc = oracle.aos_scatter(src_h[:count], perm, S).reshape(count, S)
     src, idx, pidx = dev(src_h.reshape(-1)), dev(idx_h), dev(perm)
     for variant in (ipt.AOS_DIRECT, ipt.AOS_VECTOR, ipt.AOS_COALESCED):
         dst = torch.zeros(count * S, dtype=torch.uint32, device="cuda")

@@ -196,3 +196,21 @@ def test_config5a_full_size():
     check_identity_chunked(x, m * n, eb)
     del x
     torch.cuda.empty_cache()
+
+
+def test_config5a_prime_gcd_5000():
+    """BASELINE config 5a, second shape: m = 125000, n = 140000 fp64 (140 GB), gcd 5000 > 32:
+    cluster row pass + the separate rotation pass (Eq. 36) over 140000-row column tiles +
+    the column shuffle.  10^6 sampled outputs checked one by one with the oracle's Eqs. 7-8,
+    then the full round trip r2c(c2r(x)) == x compared on the device."""
+    m, n, eb = 125000, 140000, 8
+    need_bytes(m * n * eb)
+    info = ipt.plan_info(m, n, eb)
+    assert info["c"] == 5000 and info["row_cluster"] >= 2 and info["launches"] == 3, info
+    x = index_tensor(m * n, eb)
+    ipt.c2r(x, m, n, elem_bytes=eb)
+    check_index_transpose(x, m, n, eb, 1_000_000, seed=7)
+    ipt.r2c(x, m, n, elem_bytes=eb)
+    check_identity_chunked(x, m * n, eb)
+    del x
+    torch.cuda.empty_cache()

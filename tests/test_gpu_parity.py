@@ -520,3 +520,163 @@ def test_subword_batched_and_unsupported():
     assert dev_bytes(buf) == host.tobytes()
     with pytest.raises(ipt.IptError):
         ipt.c2r(buf, 7, 9, elem_bytes=2)
+
+
+# ---------------------------------------------------------------------------------------
+# Round 2: every call the bench times, compared in full; scale cases of the separate
+# rotation and of the fused pass; robustness of the fused pass's cross-CTA waits.
+# ---------------------------------------------------------------------------------------
+def _oracle_pool():
+    import concurrent.futures as cf
+    return cf.ThreadPoolExecutor(max_workers=4)  # ctypes releases the GIL in the oracle
+
+
+def _fast_words(count, eb, seed):
+    return workloads.fast_random_words(count, eb, seed)
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+@pytest.mark.timeout(1800)
+def test_bench_sweep_calls_full(eb):
+    """The exact calls bench.py times (workloads.sweep_shapes(48), BASELINE configs[1]):
+    ipt_c2r(m, n) and ipt_r2c(m, n) of every shape, each compared IN FULL with the oracle's
+    plain transpose (Theorem 1 buffer form; c2r = P_{m,n}, r2c = P_{n,m}, reading C18).
+    Covers gcd 1, the fused rotation (gcd 2..32), the separate rotation (gcd > 32) and
+    both engines as the planner picks them."""
+    shapes = workloads.sweep_shapes(48)
+    pool = _oracle_pool()
+    maxel = max(m * n for m, n in shapes)
+    dbuf = torch.empty(maxel * eb, dtype=torch.uint8, device=DEV)
+    pending = []
+    for k, (m, n) in enumerate(shapes):
+        for op in ("c2r", "r2c"):
+            host = _fast_words(m * n, eb, seed=1000 * k + (op == "r2c") + 10 * eb)
+            want = pool.submit(getattr(oracle, "ipt_" + op), host, m, n)
+            x = dbuf[:m * n * eb]
+            x.copy_(torch.from_numpy(host.view(np.uint8)))
+            getattr(ipt, op)(x, m, n, elem_bytes=eb)
+            got = x.cpu().numpy()
+            pending.append(((m, n, op), got, want))
+            while len(pending) > 3:
+                key, g, w = pending.pop(0)
+                assert g.tobytes() == w.result().tobytes(), key
+    for key, g, w in pending:
+        assert g.tobytes() == w.result().tobytes(), key
+    pool.shutdown()
+
+
+@pytest.mark.parametrize("m,n,eb", [(19800, 13200, 4), (13200, 19800, 4), (14000, 10500, 8), (6000, 9000, 16)])
+def test_separate_rotation_at_hbm_scale(m, n, eb):
+    """gcd > 32: the column rotation (Eq. 23 before / Eq. 36 after) runs as its own
+    column-tile pass (COL_ROT) on matrices far larger than L2 (0.8-1.1 GB), compared in
+    full with the oracle in both directions."""
+    import math
+    assert math.gcd(m, n) > 32
+    assert ipt.plan_info(m, n, eb)["launches"] == 3
+    host = _fast_words(m * n, eb, seed=m + n + eb)
+    x = to_dev(host)
+    ipt.c2r(x, m, n, elem_bytes=eb)
+    assert dev_bytes(x) == oracle.ipt_c2r(vwords(host, eb), m, n).tobytes()
+    ipt.r2c(x, m, n, elem_bytes=eb)
+    assert dev_bytes(x) == np.ascontiguousarray(host).tobytes()
+    y = to_dev(host)
+    ipt.r2c(y, m, n, elem_bytes=eb)
+    assert dev_bytes(y) == oracle.ipt_r2c(vwords(host, eb), m, n).tobytes()
+
+
+def test_fused_c2r_beyond_2gib():
+    """Fused rotation + row pass (gcd 2) with the C2R engine on a matrix of > 2 GiB, alone and
+    as a batch of two (matrix stride > 2^31 bytes: the wrap rows are copied by a kernel, not
+    a pitched memcpy), compared in full."""
+    m, n, eb = 30002, 18002, 4
+    info = ipt.plan_info(m, n, eb)
+    assert info["engine"] == "c2r" and info["c"] == 2 and info["launches"] == 2, info
+    assert m * n * eb > (1 << 31)
+    host = _fast_words(m * n, eb, seed=2)
+    x = to_dev(host)
+    ipt.c2r(x, m, n, elem_bytes=eb)
+    assert dev_bytes(x) == oracle.transpose(host, m, n).tobytes()
+    ipt.r2c(x, m, n, elem_bytes=eb)
+    assert dev_bytes(x) == host.tobytes()
+    del x
+    m2, n2 = 24002, 12002  # gcd 2; 1.15 GB each, stride 1.15 GB * 1 + gap
+    assert math.gcd(m2, n2) == 2
+    stride = m2 * n2 + 16
+    hb = _fast_words(2 * stride, eb, seed=3)
+    x = to_dev(hb)
+    ipt.c2r_batched(x, 2, stride, m2, n2, elem_bytes=eb)
+    got = x.cpu().numpy().view(np.uint32)
+    for k in range(2):
+        o = k * stride
+        assert got[o:o + m2 * n2].tobytes() == oracle.transpose(hb[o:o + m2 * n2], m2, n2).tobytes(), k
+        assert got[o + m2 * n2:o + stride].tobytes() == hb[o + m2 * n2:o + stride].tobytes()
+    ipt.r2c_batched(x, 2, stride, m2, n2, elem_bytes=eb)
+    assert dev_bytes(x) == hb.tobytes()
+
+
+@pytest.mark.timeout(600)
+def test_fused_rotation_concurrent_with_busy_kernels():
+    """The fused pass's cross-CTA waits must not assume co-residency: both fused directions
+    (C2R staircases and R2C post-rotation, gcd 2..32) run on two streams while a third
+    stream keeps the SMs busy with long GEMMs, so the fused kernels start with only part of
+    their grid resident.  Work order by ticket guarantees progress (row_shuffle.cu
+    row_rot_kernel); results compared in full."""
+    shapes = [(6 * 1201, 6 * 1007, 4), (4 * 999, 4 * 1250, 8), (2 * 3001, 2 * 2203, 4), (30 * 137, 30 * 151, 4)]
+    hosts = [_fast_words(m * n, eb, seed=i) for i, (m, n, eb) in enumerate(shapes)]
+    xs = [to_dev(h) for h in hosts]
+    a = torch.randn(8192, 8192, device=DEV, dtype=torch.bfloat16)
+    torch.cuda.synchronize()
+    busy, s1, s2 = torch.cuda.Stream(), torch.cuda.Stream(), torch.cuda.Stream()
+    for rep in range(3):
+        with torch.cuda.stream(busy):
+            for _ in range(20):
+                a = (a @ a).clamp_(-1, 1)
+        for k, ((m, n, eb), x) in enumerate(zip(shapes, xs)):
+            s = s1 if k % 2 == 0 else s2
+            for engine in ("c2r", "r2c"):
+                with forced_engine(engine), torch.cuda.stream(s):
+                    ipt.c2r(x, m, n, elem_bytes=eb, stream=s)
+                    ipt.r2c(x, m, n, elem_bytes=eb, stream=s)
+        with torch.cuda.stream(s1):
+            ipt.c2r(xs[0], *shapes[0][:2], elem_bytes=shapes[0][2], stream=s1)
+            ipt.r2c(xs[0], *shapes[0][:2], elem_bytes=shapes[0][2], stream=s1)
+    torch.cuda.synchronize()
+    for (m, n, eb), x, h in zip(shapes, xs, hosts):
+        assert dev_bytes(x) == h.tobytes(), (m, n, eb)
+        with forced_engine("r2c"):
+            ipt.c2r(x, m, n, elem_bytes=eb)
+        assert dev_bytes(x) == oracle.transpose(vwords(h, eb), m, n).tobytes(), (m, n, eb)
+
+
+def test_concurrent_calls_from_threads_share_no_counters():
+    """ipt.h: thread-safe and reentrant.  Several host threads issue calls on their own
+    streams and on cudaStreamPerThread-style shared handles at once; every call owns its
+    counters (per-call scratch), so all results are exact."""
+    import threading
+    shapes = [(1811, 2903, 4), (4099, 1024, 8), (1200, 1800, 4), (3000, 4096, 4)]
+    hosts = [_fast_words(m * n, eb, seed=50 + i) for i, (m, n, eb) in enumerate(shapes)]
+    xs = [to_dev(h) for h in hosts]
+    torch.cuda.synchronize()
+    errors = []
+
+    def work(k):
+        try:
+            m, n, eb = shapes[k]
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                for _ in range(5):
+                    ipt.c2r(xs[k], m, n, elem_bytes=eb, stream=s)
+                    ipt.r2c(xs[k], m, n, elem_bytes=eb, stream=s)
+                ipt.c2r(xs[k], m, n, elem_bytes=eb, stream=s)
+            s.synchronize()
+        except Exception as e:  # pragma: no cover
+            errors.append(e)
+
+    ts = [threading.Thread(target=work, args=(k,)) for k in range(len(shapes))]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    assert not errors, errors
+    for (m, n, eb), x, h in zip(shapes, xs, hosts):
+        assert dev_bytes(x) == oracle.transpose(vwords(h, eb), m, n).tobytes(), (m, n, eb)

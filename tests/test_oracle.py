@@ -108,7 +108,8 @@ def test_theorem2_swapped_dimensions_transpose_column_major():
 # Brute force: Algorithm 1, its inverse, and the §4 gather forms on every small shape
 # ---------------------------------------------------------------------------------------
 def test_bruteforce_alg1_and_gather_forms_eb4():
-    for m, n in workloads.small_shapes(40):
+    """Every m, n <= 64 (north_star: brute force over all m, n <= 64, coprime and not)."""
+    for m, n in workloads.small_shapes(64):
         X = words(m * n, 4, seed=m * 1000 + n)
         ref = np_P(X, m, n)
         y = oracle.c2r_alg1(X, m, n)
@@ -118,9 +119,9 @@ def test_bruteforce_alg1_and_gather_forms_eb4():
         assert same(oracle.r2c_gather_forms(y, m, n), X), (m, n)
 
 
-@pytest.mark.parametrize("eb", [1, 8, 16])
+@pytest.mark.parametrize("eb", [1, 2, 8, 16, 12])
 def test_bruteforce_other_element_sizes(eb):
-    for m, n in workloads.small_shapes(14):
+    for m, n in workloads.small_shapes(40):
         X = words(m * n, eb, seed=m * 1000 + n)
         ref = np_P(X, m, n)
         assert same(oracle.c2r_alg1(X, m, n), ref), (m, n)
@@ -247,3 +248,25 @@ def test_warp_register_mapping():
         # the register array is the R2C(S, 32) of the loaded chunk: chunk word k*32+l (the
         # coalesced load order, Eq. 4 column-major view) ... equals numpy's P_{32,S}.
         assert same(R.ravel(), np_P(w, 32, S))
+
+
+@pytest.mark.parametrize("S", [1, 2, 3, 5, 16, 32])
+def test_aos_gather_scatter_against_numpy(S):
+    """Pins oracle.aos_gather / aos_scatter (Fig. 9 random-access AoS)
+    to numpy fancy indexing of the struct array, an independent implementation; plus the
+    invariants: gathering through a permutation and scattering back through the same
+    permutation is the identity, and a gather with the identity index is a copy."""
+    rng = np.random.default_rng(S)
+    nsrc, count = 301, 257
+    src = rng.integers(0, 2**32, size=(nsrc, S), dtype=np.uint32)
+    idx = rng.integers(0, nsrc, size=count, dtype=np.uint32)          # repeats allowed
+    assert same(oracle.aos_gather(src, idx, S), src[idx].reshape(-1))
+    perm = rng.permutation(count).astype(np.uint32)
+    want = np.zeros((count, S), dtype=np.uint32)
+    want[perm] = src[:count]
+    got = oracle.aos_scatter(src[:count], perm, S)
+    assert same(got, want.reshape(-1))
+    assert same(oracle.aos_scatter(oracle.aos_gather(src[:count], perm, S), perm, S), src[:count].reshape(-1))
+    ident = np.arange(nsrc, dtype=np.uint32)
+    assert same(oracle.aos_gather(src, ident, S), src.reshape(-1))
+    assert oracle.aos_gather(src, idx[:0], S).size == 0
