@@ -12,9 +12,12 @@ data stay meaningful).  Every call is timed alone with CUDA events on the launch
 stream; L2 is flushed (a 256 MiB write, > the 126 MB L2) before every timed call, outside
 the events.  Throughput per call follows Eq. 37: 2 m n s / t, GB = 1e9 B.
 
-value   = median over all timed calls of the per-call GB/s (the paper's statistic);
-          with N ranks each rank transposes its own S independent shapes (weak scaling,
-          no collective on the data path) and value = the sum of the rank medians.
+value   = median over all timed calls of the per-call GB/s (the paper's statistic).  With N
+          ranks every rank runs the SAME S shapes (weak scaling, no collective on the data
+          path); call k's time is the max over ranks and its GB/s is N x 2 m n s / that time.
+moved   = the same median over the call's algorithmic bytes (4 m n s for two passes).
+extras  = cfg5b (batch of 4096 4096x3000 fp32, sharded over the ranks; strong scaling),
+          cfg3 (skinny AoS<->SoA, median over n) and cfg5a (~140 GB fp64) at N = 1.
 e2e     = the same median, each call timed from a pinned-host H2D copy through ipt_c2r
           to the D2H copy of the result (public API, host buffers).
 roofline= the dominant kernel's algorithmic bytes / its event-timed device time against
@@ -53,7 +56,8 @@ def parse_args():
     p.add_argument("--steps", type=int, default=6)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    p.add_argument("--shapes", type=int, default=48, help="sweep shapes per rank per step")
+    p.add_argument("--shapes", type=int, default=200, help="sweep shapes per step (the same on every rank)")
+    p.add_argument("--no-extras", action="store_true", help="skip the cfg3 / cfg5a / cfg5b keys")
     p.add_argument("--e2e-shapes", type=int, default=8)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--profile-only", action="store_true", help="one short untimed pass (for ncu)")
@@ -239,8 +243,9 @@ def run_reference(args, rank, world):
 
 
 def rank_shapes(rank, S):
-    """Rank r transposes sweep shapes [r*S, (r+1)*S): independent matrices, weak scaling."""
-    return workloads.sweep_shapes(S * (rank + 1))[S * rank:]
+    """Every rank transposes the SAME S sweep shapes (so that N=1 and N>1 time the same
+    workload per GPU; weak scaling: the job's work grows with N, no data-path collective)."""
+    return workloads.sweep_shapes(S)
 
 
 def shard_batch(batch, rank, world):
@@ -257,25 +262,52 @@ def reduce_over_ranks(sum_vals, max_vals, world, device):
         return list(sum_vals), list(max_vals)
     import torch
     import torch.distributed as dist
-    s = torch.tensor(list(sum_vals), dtype=torch.float64, device=device)
-    m = torch.tensor(list(max_vals), dtype=torch.float64, device=device)
-    dist.all_reduce(s, op=dist.ReduceOp.SUM)
-    dist.all_reduce(m, op=dist.ReduceOp.MAX)
-    return [float(v) for v in s], [float(v) for v in m]
+    out = []
+    for vals, op in ((sum_vals, dist.ReduceOp.SUM), (max_vals, dist.ReduceOp.MAX)):
+        vals = list(vals)
+        if vals:
+            t = torch.tensor(vals, dtype=torch.float64, device=device)
+            dist.all_reduce(t, op=op)
+            vals = [float(v) for v in t]
+        out.append(vals)
+    return out[0], out[1]
 
 
-def run_batched(args, rank, world, local_rank):
-    """Config 5b: `--batch` independent 4096 x 3000 float32 matrices (default 4096, 201 GB)
-    sharded contiguously over the ranks (strong scaling); each rank transposes its shard
-    with ipt_c2r_batched in resident chunks of at most --chunk matrices.  value =
-    total Eq. 37 bytes / max-over-ranks device time."""
+def aggregate_calls(call_bytes, call_ms, world, device):
+    """Multi-GPU semantics of the sweep metric.  Every rank runs the same calls in the same
+    order; call k's job time is the MAX over ranks of its device time, and its job
+    throughput is (world x its Eq. 37 bytes) / that time.  value = the median over calls
+    (at world = 1: the plain per-call median, the paper's statistic).  Also returns the
+    aggregate throughput = all ranks' bytes / the max over ranks of the summed device time."""
+    _, t_max = reduce_over_ranks([], list(call_ms), world, device)
+    per_call = [world * b / (t * 1e-3) / 1e9 for b, t in zip(call_bytes, t_max)]
+    _, (tot_max,) = reduce_over_ranks([], [sum(call_ms)], world, device)
+    aggregate = world * sum(call_bytes) / (tot_max * 1e-3) / 1e9
+    return per_call, t_max, aggregate
+
+
+def algorithmic_bytes(ipt, m, n, eb, op):
+    """What the engine must move for one call: one read + one write of every
+    element per pass -- 4 m n s for two passes (gcd 1, or the rotation fused), plus
+    2 m n s (c - 1) / c for a separate rotation pass."""
+    info = ipt.plan_info(m, n, eb) if op == "c2r" else ipt.plan_info(n, m, eb)
+    c = info["c"]
+    extra = 2.0 * (c - 1) / c if info["launches"] >= 3 and info["engine"] in ("c2r", "r2c") else 0.0
+    return (4.0 + extra) * m * n * eb
+
+
+def measure_batched(args, rank, world, local_rank, steps=2, warmup=1):
+    """Config 5b: `args.batch` independent 4096 x 3000 float32 matrices (default 4096, 201 GB)
+    sharded contiguously over the ranks (strong scaling); each rank transposes its shard with
+    ipt_c2r_batched / ipt_r2c_batched in resident chunks of at most --chunk matrices (one GPU
+    cannot hold 201 GB: the chunks reuse one 25 GB buffer).  value = total Eq. 37 bytes /
+    max-over-ranks device time."""
     import torch
     import torch.distributed as dist
 
     import paper_conf_ppopp_catanzarokg14_b200 as ipt
 
     dev = torch.device("cuda", local_rank)
-    torch.cuda.set_device(dev)
     m, n, eb = workloads.CONFIG5B["m"], workloads.CONFIG5B["n"], workloads.CONFIG5B["elem_bytes"]
     lo, hi = shard_batch(args.batch, rank, world)
     mine = hi - lo
@@ -299,46 +331,41 @@ def run_batched(args, rank, world, local_rank):
             if record is not None:
                 record.append((e0, e1))
 
-    for _ in range(args.warmup):
+    for _ in range(warmup):
         step(None)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     launches0 = ipt.launch_count()
     rec = []
-    for _ in range(args.steps):
+    for _ in range(steps):
         step(rec)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    dev_ms = sum(e0.elapsed_time(e1) for e0, e1 in rec) / args.steps
+    dev_ms = sum(e0.elapsed_time(e1) for e0, e1 in rec) / steps
     (total_bytes,), (t_max,) = reduce_over_ranks([2.0 * mine * m * n * eb], [dev_ms], world, dev)
-    if rank != 0:
-        return
-    peak, peak_src = hbm_peak()
+    del buf
+    torch.cuda.empty_cache()
+    peak, _ = hbm_peak()
     value = total_bytes / (t_max * 1e-3) / 1e9
-    print(json.dumps({
-        "metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": round(t_max, 3), "higher_is_better": True, "scaling": "strong",
-        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": f"cfg5b: batch of {args.batch} independent {m}x{n} float32 matrices, "
-                               f"contiguous shards per rank, chunks of <= {args.chunk} resident matrices",
-                   "parallelism": f"batch sharding x{world}, no data-path collective",
-                   "l2": "inputs (>= 25 GB per chunk) far larger than L2"},
-        "impl": "ours", "frac_of_hbm_peak_per_gpu": round(value / world / peak, 4),
-        "gpu_launches": ipt.launch_count() - launches0}), flush=True)
+    return {"value": round(value, 2), "unit": UNIT, "metric": "Eq. 37 GB/s of the whole batch (2 m n s per matrix)",
+            "n_gpus": world, "scaling": "strong", "ms_per_step": round(t_max, 3), "steps": steps,
+            "workload": f"cfg5b: {args.batch} independent {m}x{n} float32 matrices, contiguous shards per rank, "
+                        f"chunks of <= {args.chunk} resident matrices (c2r / r2c alternating)",
+            "frac_of_hbm_peak_per_gpu": round(value / world / peak, 4),
+            "moved_GBps": round(2 * value, 2), "gpu_launches": ipt.launch_count() - launches0}
 
 
-def run_skinny(args, rank, world, local_rank):
-    """Config 3: AoS -> SoA and SoA -> AoS of 2**26 structs x n 4-byte fields, n = 2..32
+def measure_skinny(args, local_rank, steps=1, warmup=1):
+    """Config 3: AoS -> SoA and SoA -> AoS of args.count structs x n 4-byte fields, n = 2..32
     (ipt_aos_to_soa / ipt_soa_to_aos, the skinny engine).  value = median over all calls of
-    Eq. 37 GB/s (2 * count * n * 4 / t); per-n numbers in `per_n`."""
+    Eq. 37 GB/s (2 * count * n * 4 / t); per-n medians; per-kernel event times."""
     import torch
 
     import paper_conf_ppopp_catanzarokg14_b200 as ipt
 
     dev = torch.device("cuda", local_rank)
-    torch.cuda.set_device(dev)
     count = args.count
     ns = workloads.skinny_field_counts()
     buf = torch.randint(0, 255, (count * max(ns) * 4,), dtype=torch.uint8, device=dev)
@@ -354,7 +381,7 @@ def run_skinny(args, rank, world, local_rank):
         if rec is not None:
             rec.append((n, op.__name__, e0, e1))
 
-    for _ in range(args.warmup):
+    for _ in range(warmup):
         for n in ns:
             one(n, ipt.aos_to_soa, None)
             one(n, ipt.soa_to_aos, None)
@@ -363,7 +390,7 @@ def run_skinny(args, rank, world, local_rank):
     ipt.profile_enable(True)
     ipt.profile_read()
     rec = []
-    for _ in range(args.steps):
+    for _ in range(steps):
         for n in ns:
             one(n, ipt.aos_to_soa, rec)
             one(n, ipt.soa_to_aos, rec)
@@ -377,32 +404,93 @@ def run_skinny(args, rank, world, local_rank):
         g = 2.0 * count * n * 4 / (ms * 1e-3) / 1e9
         rates.append(g)
         per_n.setdefault(f"{name}_n{n}", []).append(g)
-    peak, peak_src = hbm_peak()
+    del buf, flush
+    torch.cuda.empty_cache()
+    peak, _ = hbm_peak()
     value = statistics.median(rates)
-    dom = max(kern.items(), key=lambda kv: kv[1][1]) if kern else None
-    roof = None
-    if dom:
-        name, (nl, ms, by) = dom
-        achieved = by / (ms * 1e-3) / 1e9
-        roof = {"bound": "hbm", "kernel": name, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4), "peak_source": peak_src, "traffic": None,
-                "share_of_device_time": round(ms / sum(v[1] for v in kern.values()), 3)}
-    if rank == 0:
-        print(json.dumps({
-            "metric": "median in-place AoS<->SoA GB/s (Eq. 37) over n = 2..32 fields", "value": round(value, 2),
-            "unit": UNIT, "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(dev_ms / args.steps, 3), "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": f"cfg3 skinny: {count} structs x n 4-byte fields, n = 2..32, "
-                                   "ipt_aos_to_soa then ipt_soa_to_aos", "l2": "flushed before every timed call"},
-            "impl": "ours", "frac_of_hbm_peak": round(value / peak, 4), "max_GBps": round(max(rates), 2),
+    return {"value": round(value, 2), "unit": UNIT, "metric": "median in-place AoS<->SoA GB/s (Eq. 37) over n = 2..32",
+            "workload": f"cfg3 skinny: {count} structs x n 4-byte fields, n = 2..32, ipt_aos_to_soa then "
+                        "ipt_soa_to_aos, L2 flushed before every call",
+            "frac_of_hbm_peak": round(value / peak, 4), "max_GBps": round(max(rates), 2),
+            "ceiling_note": "(2 + 1/n) passes for odd n, 3 for even n: eff <= copy / (2 + 1/n) or copy / 3",
             "per_n": {k: round(statistics.median(v), 1) for k, v in per_n.items()},
-            "paper_context": {"K20c_skinny_median_GBps": 34.3, "K20c_skinny_max_GBps": 51,
-                              "source": "PAPER.md:1069 (64-bit fields, other hardware)"},
-            "roofline": roof,
             "kernels": {k: {"launches": v[0], "ms": round(v[1], 3), "GBps": round(v[2] / (v[1] * 1e-3) / 1e9, 1)}
                         for k, v in kern.items()},
-            "gpu_launches": ipt.launch_count() - launches0}), flush=True)
+            "ms_per_step": round(dev_ms / steps, 3), "gpu_launches": ipt.launch_count() - launches0}
+
+
+def measure_huge(local_rank, shapes=((120011, 145820), (125000, 140000)), eb=8):
+    """Config 5a: in-place transpose of ~140 GB float64 matrices on one GPU (c2r then r2c,
+    one warm-up pair, one timed pair per shape).  Skipped when the device lacks the memory."""
+    import torch
+
+    import paper_conf_ppopp_catanzarokg14_b200 as ipt
+
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.empty_cache()
+    out = {}
+    stream = torch.cuda.current_stream(dev)
+    for (m, n) in shapes:
+        free, _ = torch.cuda.mem_get_info(dev)
+        need = m * n * eb
+        key = f"{m}x{n}"
+        if free < need + (3 << 30):
+            out[key] = {"skipped": f"needs {need / 1e9:.1f} GB, {free / 1e9:.1f} GB free"}
+            continue
+        x = torch.empty(need, dtype=torch.uint8, device=dev)
+        ipt.c2r(x, m, n, elem_bytes=eb)
+        ipt.r2c(x, m, n, elem_bytes=eb)
+        torch.cuda.synchronize()
+        ipt.profile_enable(True)
+        ipt.profile_read()
+        res = {}
+        for op in ("c2r", "r2c"):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            getattr(ipt, op)(x, m, n, elem_bytes=eb, stream=stream.cuda_stream)
+            e1.record(stream)
+            e1.synchronize()
+            ms = e0.elapsed_time(e1)
+            res[op + "_GBps"] = round(2.0 * m * n * eb / (ms * 1e-3) / 1e9, 1)
+            res[op + "_ms"] = round(ms, 2)
+        ipt.profile_enable(False)
+        kern = ipt.profile_read()
+        info = ipt.plan_info(m, n, eb)
+        res.update({"bytes": need, "gcd": info["c"], "engine": info["engine"], "row_cluster_K": info["row_cluster"],
+                    "launches": info["launches"], "scratch_bytes": info["scratch_bytes"],
+                    "kernels": {k: {"launches": v[0], "ms": round(v[1], 3),
+                                    "GBps": round(v[2] / (v[1] * 1e-3) / 1e9, 1)} for k, v in kern.items()}})
+        out[key] = res
+        del x
+        torch.cuda.empty_cache()
+    return {"workload": "cfg5a: 120011x145820 (gcd 1) and 125000x140000 (gcd 5000) float64, ~140 GB each, "
+                        "one GPU; Eq. 37 GB/s per call (device events)", "shapes": out}
+
+
+def run_batched(args, rank, world, local_rank):
+    import torch
+    torch.cuda.set_device(local_rank)
+    res = measure_batched(args, rank, world, local_rank, steps=args.steps, warmup=args.warmup)
+    if rank == 0:
+        print(json.dumps({"metric": METRIC, "value": res["value"], "unit": UNIT, "n_gpus": world,
+                          "steps": args.steps, "warmup": args.warmup, "ms_per_step": res["ms_per_step"],
+                          "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+                          "data": "synthetic", "config": {"workload": res["workload"]}, "impl": "ours",
+                          "frac_of_hbm_peak_per_gpu": res["frac_of_hbm_peak_per_gpu"],
+                          "gpu_launches": res["gpu_launches"]}), flush=True)
+
+
+def run_skinny(args, rank, world, local_rank):
+    import torch
+    torch.cuda.set_device(local_rank)
+    res = measure_skinny(args, local_rank, steps=args.steps, warmup=args.warmup)
+    if rank == 0:
+        print(json.dumps({"metric": res["metric"], "value": res["value"], "unit": UNIT, "n_gpus": world,
+                          "steps": args.steps, "warmup": args.warmup, "ms_per_step": res["ms_per_step"],
+                          "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+                          "data": "synthetic", "config": {"workload": res["workload"]}, "impl": "ours",
+                          **{k: v for k, v in res.items() if k not in ("value", "metric", "workload", "ms_per_step")}}),
+              flush=True)
 
 
 def run_ours(args, rank, world, local_rank):
@@ -420,9 +508,15 @@ def run_ours(args, rank, world, local_rank):
     bufs = {eb: torch.randint(0, 255, (maxel * eb,), dtype=torch.uint8, device=dev) for eb in ebs}
     flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream(dev)
+    alg = {}
+    for (m, n) in shapes:
+        for eb in ebs:
+            for op in ("c2r", "r2c"):
+                alg[(m, n, eb, op)] = algorithmic_bytes(ipt, m, n, eb, op)
 
     def one_step(step, record):
-        op = ipt.c2r if step % 2 == 0 else ipt.r2c
+        opn = "c2r" if step % 2 == 0 else "r2c"
+        op = getattr(ipt, opn)
         for (m, n) in shapes:
             for eb in ebs:
                 flush.zero_()
@@ -433,7 +527,7 @@ def run_ours(args, rank, world, local_rank):
                 op(bufs[eb], m, n, elem_bytes=eb, stream=stream.cuda_stream)
                 if record is not None:
                     e1.record(stream)
-                    record.append((m, n, eb, e0, e1))
+                    record.append((m, n, eb, opn, e0, e1))
 
     if args.profile_only:
         one_step(0, None)
@@ -468,17 +562,13 @@ def run_ours(args, rank, world, local_rank):
     launches = ipt.launch_count() - launches0
     clk = clocks.stop()
 
-    per_call = []
-    by_eb = {eb: [] for eb in ebs}
-    dev_ms = 0.0
-    for (m, n, eb, e0, e1) in rec:
-        ms = e0.elapsed_time(e1)
-        dev_ms += ms
-        g = 2.0 * m * n * eb / (ms * 1e-3) / 1e9
-        per_call.append(g)
-        by_eb[eb].append(g)
-    median = statistics.median(per_call)
-    ms_step = dev_ms / args.steps
+    call_ms = [e0.elapsed_time(e1) for (_, _, _, _, e0, e1) in rec]
+    call_bytes = [2.0 * m * n * eb for (m, n, eb, _, _, _) in rec]
+    per_call, t_max, aggregate = aggregate_calls(call_bytes, call_ms, world, dev)
+    moved = [world * alg[(m, n, eb, op)] / (t * 1e-3) / 1e9 for (m, n, eb, op, _, _), t in zip(rec, t_max)]
+    by_eb = {eb: [g for g, r in zip(per_call, rec) if r[2] == eb] for eb in ebs}
+    value = statistics.median(per_call)
+    ms_step = sum(t_max) / args.steps
 
     # ---- e2e through the public API with host buffers --------------------------------
     e2e_shapes = shapes[:args.e2e_shapes]
@@ -504,14 +594,21 @@ def run_ours(args, rank, world, local_rank):
                 if rep == 1:
                     e2e_rates.append(2.0 * nb / (e0.elapsed_time(e1) * 1e-3) / 1e9)
             h2d += nb
-    e2e = {"value": round(statistics.median(e2e_rates), 2), "unit": UNIT,
-           "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": h2d,
-           "note": f"median over {len(e2e_rates)} calls: pinned host -> H2D -> ipt_c2r -> D2H, first "
-                   f"{len(e2e_shapes)} sweep shapes x fp32/fp64"}
+    e2e_med = statistics.median(e2e_rates)
+    (e2e_sum,), _ = reduce_over_ranks([e2e_med], [], world, dev)
+    e2e = {"value": round(e2e_sum, 2), "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": h2d,
+           "note": f"median over {len(e2e_rates)} calls per rank (summed over ranks): pinned host -> H2D -> ipt_c2r "
+                   f"-> D2H, first {len(e2e_shapes)} sweep shapes x fp32/fp64; bound by the host link"}
+    del bufs, flush
+    torch.cuda.empty_cache()
 
-    # ---- aggregate over ranks (max time, summed medians) ------------------------------
-    (value, e2e_value), (ms_step,) = reduce_over_ranks([median, e2e["value"]], [ms_step], world, dev)
-    e2e["value"] = round(e2e_value, 2)
+    # ---- the other BASELINE configs, folded into the same line ------------------------
+    extras = {}
+    if not args.no_extras:
+        extras["cfg5b_batched"] = measure_batched(args, rank, world, local_rank)
+        if world == 1:
+            extras["cfg3_skinny"] = measure_skinny(args, local_rank)
+            extras["cfg5a_huge"] = measure_huge(local_rank)
     if rank != 0:
         return
 
@@ -528,8 +625,10 @@ def run_ours(args, rank, world, local_rank):
                 "traffic_algorithmic": tr.get("algorithmic_bytes_per_launch") if tr else None,
                 "traffic_source": tr.get("source") if tr else None,
                 "launches": nl, "share_of_device_time": round(ms / sum(v[1] for v in kern.values()), 3)}
-    kernels = {k: {"launches": v[0], "ms": round(v[1], 3), "GBps": round(v[2] / (v[1] * 1e-3) / 1e9, 1)}
+    kernels = {k: {"launches": v[0], "ms": round(v[1], 3), "GBps": round(v[2] / (v[1] * 1e-3) / 1e9, 1),
+                   "frac_of_hbm_peak": round(v[2] / (v[1] * 1e-3) / 1e9 / peak, 4)}
                for k, v in kern.items()}
+    moved_med = statistics.median(moved)
     out = {"metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": round(ms_step, 3), "higher_is_better": True, "scaling": "weak",
            "vs_baseline": None, "dtype": "f32+f64", "data": "synthetic",
@@ -537,18 +636,29 @@ def run_ours(args, rank, world, local_rank):
                                   "float32+float64, ipt_c2r/ipt_r2c alternating steps",
                       "shapes_per_rank": S, "elem_bytes": list(ebs), "calls_per_step": S * len(ebs),
                       "l2": "flushed before every timed call (256 MiB write > 126 MB L2)",
-                      "parallelism": f"replicas x{world} (independent matrices per rank, no data-path collective)",
+                      "parallelism": f"replicas x{world}: every rank runs the same shapes; per call the max over "
+                                     "ranks of its device time (no data-path collective)",
                       "engine": "paper heuristic PAPER.md:959 (C2R if m > n else R2C)"},
            "impl": "ours",
+           "statistic": "median over calls of Eq. 37 GB/s = world x 2 m n s / max-over-ranks call time "
+                        "(PAPER.md:789-795, GB = 1e9 B)",
            "median_GBps_fp32": round(statistics.median(by_eb[4]), 2),
            "median_GBps_fp64": round(statistics.median(by_eb[8]), 2),
            "p10_GBps": round(sorted(per_call)[len(per_call) // 10], 2),
            "p90_GBps": round(sorted(per_call)[(9 * len(per_call)) // 10], 2),
+           "aggregate_GBps": round(aggregate, 2),
            "frac_of_hbm_peak": round(value / world / peak, 4),
+           "frac_of_spec_8TBps": round(value / world / 8000.0, 4),
+           "moved_GBps": round(moved_med, 2),
+           "moved_frac_of_hbm_peak": round(moved_med / world / peak, 4),
+           "moved_frac_of_spec_8TBps": round(moved_med / world / 8000.0, 4),
+           "moved_note": "algorithmic bytes of the call's passes (4 m n s, + 2 m n s (c-1)/c for a separate "
+                         "rotation) / call time, median over calls; 2-pass ceiling of Eq. 37 = 50% of copy",
            "paper_context": {"K20c_median_GBps_fp64": 19.53, "K20c_median_GBps_fp32": 14.23,
                              "source": "PAPER.md:1027-1033 Table 2 (other hardware; context only)"},
            "roofline": roof, "kernels": kernels, "gpu_launches": launches, "e2e": e2e, "clocks": clk,
            "wall_s_timed_region": round(t_wall, 3)}
+    out.update(extras)
     if world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = cpu_baseline()
         out["cpu_tuned"] = cpu_tuned()

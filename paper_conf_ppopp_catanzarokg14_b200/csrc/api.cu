@@ -701,6 +701,7 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
         if (pl.row.fuse) {  // rows 0..c-2 of every matrix into the wrap slots first
             cudaError_t e = launch_copy_wrap(pl.row, pl.eb, st);
             if (e != cudaSuccess) return e;
+            g_launches++;
         }
         return pl.row.cl_K ? launch_row_cluster(pl.row, pl.row_dir, pl.eb, st) : launch_row(pl.row, pl.row_dir, pl.eb, st);
     };

@@ -189,16 +189,9 @@ __device__ __forceinline__ void unit_prepass(const ColParams &P, const Unit &U, 
 // (one more chunk when the segment is misaligned; 16-byte elements never are).
 template <int EB, int TWB> constexpr int chunks_per_row() { return TWB / 16 + (EB < 16 ? 1 : 0); }
 
-// Load: every input row ("slot" t) is staged as the 16-byte-aligned hull of its tile row
-// with 16-byte cp.async (element-granular cp.async runs at ~70% of the 16-byte rate on
-// B200 for 4-byte elements: tools/tile_probe.cu), the last chunk with a src-size so no
-// byte past the tile's row end is read; sbase[t] records where its first element landed.
-// The skew / rotation / permutation is applied when the store phase reads shared memory.
-// Not committed here.
-template <int EB, int MODE, int TWB>
-__device__ __forceinline__ void unit_load(const ColParams &P, const Unit &U, const int32_t *srow, uint32_t *sbase,
-                                          uint32_t rows_s, int nthr) {
-    if (U.skip) return;
+template <int EB, int MODE, int TWB, bool EXACT>
+__device__ __forceinline__ void unit_load_t(const ColParams &P, const Unit &U, const int32_t *srow, uint32_t *sbase,
+                                            uint32_t rows_s, int nthr) {
     constexpr int CPR = chunks_per_row<EB, TWB>();
     constexpr int LPS = CPR < 32 ? CPR : 32;  // lanes per slot
     constexpr int RPI = 32 / LPS;             // slots per warp iteration
@@ -212,46 +205,68 @@ __device__ __forceinline__ void unit_load(const ColParams &P, const Unit &U, con
     if (t >= U.nslots) return;
     const int64_t pitch = U.in_pitch;
     const int32_t c16 = c * 16;
-    const int32_t rem0 = U.wt * EB - c16;  // + off: bytes of the hull from this chunk on
     uint32_t dst = rows_s + t * HS + c16;
     const uint32_t dst_inc = step * HS;
-    // Chunks c (+ 32, ...) of slot t's hull; rp = the slot's first tile element in global.
-    auto issue = [&](const char *rp) {
-        const int32_t off = static_cast<int32_t>(reinterpret_cast<uintptr_t>(rp) & 15u);
-        if (c == 0) sbase[t] = dst + off;
+    uint32_t *sb = sbase + t;
+    // Chunks c (+ 32, ...) of slot t's hull; q = the slot's first tile element + 16 c.
+    auto issue = [&](const char *q) {
+        const uint32_t off = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(q)) & 15u;
+        if (c == 0) *sb = dst + off;
 #pragma unroll
         for (int k = 0; k < CPL; ++k) {
             if (CPL > 1 && c + 32 * k >= CPR) break;
-            const char *src = rp - off + c16 + 512 * k;
+            const char *src = reinterpret_cast<const char *>(reinterpret_cast<uintptr_t>(q + 512 * k) & ~uintptr_t(15));
             const uint32_t d = dst + 512 * k;
-            const int32_t rem = rem0 + off - 512 * k;
-            if (rem >= 16) {
+            if (!EXACT) {
                 asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(d), "l"(src) : "memory");
-            } else if (rem > 0) {  // row end: read only the tile's bytes (never past the buffer)
-                asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(d), "l"(src), "r"(rem) : "memory");
+            } else {
+                const int32_t rem = U.wt * EB + static_cast<int32_t>(off) - c16 - 512 * k;  // hull bytes from here
+                if (rem >= 16) {
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(d), "l"(src) : "memory");
+                } else if (rem > 0) {  // row end: read only the tile's bytes (never past the buffer)
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(d), "l"(src), "r"(rem) : "memory");
+                }
             }
         }
     };
     if (MODE == COL_R2C_SHUF) {
-        for (; t < U.nslots; t += step, dst += dst_inc) issue(U.inp + static_cast<int64_t>(srow[t]) * pitch);
+        for (; t < U.nslots; t += step, dst += dst_inc, sb += step) issue(U.inp + static_cast<int64_t>(srow[t]) * pitch + c16);
     } else if (step <= P.M) {
         // contiguous (cyclic) input rows rowbase + t: incremental row index and pointer
-        int32_t g = mod_M(U.rowbase + t, P.kshM, P.fd_M);
-        const char *rp = U.inp + static_cast<int64_t>(g) * pitch;
-        const int64_t rp_inc = step * pitch, rp_wrap = static_cast<int64_t>(P.M) * pitch;
-        for (; t < U.nslots; t += step, dst += dst_inc) {
-            issue(rp);
-            g += step;
-            rp += rp_inc;
-            if (g >= P.M) {
-                g -= P.M;
-                rp -= rp_wrap;
-            }
-        }
+        // Each lane's rows wrap past M - 1 at most once (nslots <= M + W - 1 rows from
+        // rowbase): two plain pointer walks, split where the wrap happens.
+        const int32_t g = mod_M(U.rowbase + t, P.kshM, P.fd_M);
+        const char *rp = U.inp + static_cast<int64_t>(g) * pitch + c16;
+        const int64_t rp_inc = step * pitch;
+        const uint32_t *sb_end = sbase + U.nslots;
+        const int32_t n1 = (P.M - 1 - g) / step + 1;  // iterations before the wrap
+        const uint32_t *sb_wrap = sb + static_cast<int64_t>(n1) * step;
+        const uint32_t *stop1 = sb_wrap < sb_end ? sb_wrap : sb_end;
+#pragma unroll 4
+        for (; sb < stop1; sb += step, dst += dst_inc, rp += rp_inc) issue(rp);
+        rp -= static_cast<int64_t>(P.M) * pitch;
+#pragma unroll 4
+        for (; sb < sb_end; sb += step, dst += dst_inc, rp += rp_inc) issue(rp);
     } else {  // tiny M: fewer rows than one step
-        for (; t < U.nslots; t += step, dst += dst_inc)
-            issue(U.inp + static_cast<int64_t>(mod_M(U.rowbase + t, P.kshM, P.fd_M)) * pitch);
+        for (; t < U.nslots; t += step, dst += dst_inc, sb += step)
+            issue(U.inp + static_cast<int64_t>(mod_M(U.rowbase + t, P.kshM, P.fd_M)) * pitch + c16);
     }
+}
+
+// Load: every input row ("slot" t) is staged as the 16-byte-aligned hull of its tile row
+// with 16-byte cp.async (element-granular cp.async runs at ~70% of the 16-byte rate on
+// B200 for 4-byte elements: tools/tile_probe.cu); sbase[t] records where its first element
+// landed.  The skew / rotation / permutation is applied when the store phase reads shared
+// memory.  The rightmost tile of a row (its hull may end past the last byte of the buffer)
+// reads exactly the tile's bytes (src-size); every other tile reads whole 16-byte chunks:
+// bytes past the tile belong to the next tile of the same row and are never used.  Per slot
+// and lane: one 64-bit pointer step, one AND, one cp.async.  Not committed here.
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ void unit_load(const ColParams &P, const Unit &U, const int32_t *srow, uint32_t *sbase,
+                                          uint32_t rows_s, int nthr) {
+    if (U.skip) return;
+    if (U.j0 + U.wt >= P.N) unit_load_t<EB, MODE, TWB, true>(P, U, srow, sbase, rows_s, nthr);
+    else unit_load_t<EB, MODE, TWB, false>(P, U, srow, sbase, rows_s, nthr);
 }
 
 template <int EB>

@@ -1,7 +1,8 @@
 """Multi-process (world_size 2, gloo, CPU) coverage of the N>1 bench path.
 
-The data path has no collective: ranks own disjoint, contiguous shards of independent
-matrices; the only collectives are the timing/throughput reductions (SUM, MAX).  These
+The data path has no collective: in the sweep every rank transposes the same shapes in its
+own memory, in config 5b ranks own disjoint contiguous shards of independent matrices; the
+only collectives are the timing/throughput reductions (SUM, MAX).  These
 tests run the bench's own sharding and reduction helpers in two real processes.
 """
 import os
@@ -32,7 +33,11 @@ def _worker(rank, world, port, out):
         sums, maxs = bench.reduce_over_ranks([rank + 1.0, 10.0 * rank], [rank * 3.0 + 1], world, "cpu")
         shapes = bench.rank_shapes(rank, 4)
         lo, hi = bench.shard_batch(4096, rank, world)
-        out[rank] = (sums, maxs, shapes, (lo, hi))
+        # the sweep metric: same calls on every rank, per call the max time over ranks
+        call_bytes = [2e9, 4e9, 1e9]
+        call_ms = [1.0, 2.0, 4.0] if rank == 0 else [2.0, 1.0, 4.0]
+        per_call, t_max, agg = bench.aggregate_calls(call_bytes, call_ms, world, "cpu")
+        out[rank] = (sums, maxs, shapes, (lo, hi), per_call, t_max, agg)
     finally:
         dist.destroy_process_group()
 
@@ -47,8 +52,13 @@ def test_two_rank_sharding_and_reductions(world):
     # reductions: SUM and MAX of the per-rank values, identical on every rank
     assert r0[0] == r1[0] == [3.0, 10.0]
     assert r0[1] == r1[1] == [4.0]
-    # independent shapes per rank (no rank repeats another's matrices)
-    assert len(r0[2]) == len(r1[2]) == 4 and not set(r0[2]) & set(r1[2])
+    # the same shapes on every rank (N = 1 and N > 1 time the same per-GPU workload)
+    assert len(r0[2]) == len(r1[2]) == 4 and r0[2] == r1[2]
+    # per call: max over ranks of the time, job throughput = world x bytes / that time
+    assert r0[5] == r1[5] == [2.0, 2.0, 4.0]
+    assert r0[4] == r1[4] == [2 * 2e9 / 2e-3 / 1e9, 2 * 4e9 / 2e-3 / 1e9, 2 * 1e9 / 4e-3 / 1e9]
+    # aggregate: both ranks' bytes over the max of the summed times (7 ms on both)
+    assert abs(r0[6] - 2 * 7e9 / 7e-3 / 1e9) < 1e-6 and r0[6] == r1[6]
     # config 5b: contiguous shards covering [0, 4096) exactly once
     assert r0[3] == (0, 2048) and r1[3] == (2048, 4096)
 
