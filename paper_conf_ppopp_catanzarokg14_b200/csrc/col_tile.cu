@@ -233,20 +233,20 @@ __device__ __forceinline__ void unit_load_t(const ColParams &P, const Unit &U, c
         for (; t < U.nslots; t += step, dst += dst_inc, sb += step) issue(U.inp + static_cast<int64_t>(srow[t]) * pitch + c16);
     } else if (step <= P.M) {
         // contiguous (cyclic) input rows rowbase + t: incremental row index and pointer
-        // Each lane's rows wrap past M - 1 at most once (nslots <= M + W - 1 rows from
-        // rowbase): two plain pointer walks, split where the wrap happens.
-        const int32_t g = mod_M(U.rowbase + t, P.kshM, P.fd_M);
+        // Plain pointer walks between the points where a lane's rows wrap past M - 1 (once
+        // for big M; small M with a halo longer than M wraps more often).
+        int32_t g = mod_M(U.rowbase + t, P.kshM, P.fd_M);
         const char *rp = U.inp + static_cast<int64_t>(g) * pitch + c16;
-        const int64_t rp_inc = step * pitch;
+        const int64_t rp_inc = step * pitch, rp_wrap = static_cast<int64_t>(P.M) * pitch;
         const uint32_t *sb_end = sbase + U.nslots;
-        const int32_t n1 = (P.M - 1 - g) / step + 1;  // iterations before the wrap
-        const uint32_t *sb_wrap = sb + static_cast<int64_t>(n1) * step;
-        const uint32_t *stop1 = sb_wrap < sb_end ? sb_wrap : sb_end;
+        while (sb < sb_end) {
+            const int32_t n = (P.M - 1 - g) / step + 1;  // iterations before the wrap
+            const uint32_t *stop = sb_end - sb > static_cast<int64_t>(n) * step ? sb + static_cast<int64_t>(n) * step : sb_end;
 #pragma unroll 4
-        for (; sb < stop1; sb += step, dst += dst_inc, rp += rp_inc) issue(rp);
-        rp -= static_cast<int64_t>(P.M) * pitch;
-#pragma unroll 4
-        for (; sb < sb_end; sb += step, dst += dst_inc, rp += rp_inc) issue(rp);
+            for (; sb < stop; sb += step, dst += dst_inc, rp += rp_inc) issue(rp);
+            g += n * step - P.M;
+            rp -= rp_wrap;
+        }
     } else {  // tiny M: fewer rows than one step
         for (; t < U.nslots; t += step, dst += dst_inc, sb += step)
             issue(U.inp + static_cast<int64_t>(mod_M(U.rowbase + t, P.kshM, P.fd_M)) * pitch + c16);

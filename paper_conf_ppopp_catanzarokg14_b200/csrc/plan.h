@@ -85,6 +85,7 @@ struct RowParams {
     int32_t vec;             // fused C2R: vectorised gather for rows with f2 = 0 (IPT_ROW_VEC)
     int32_t R;               // rows per CTA stage (row groups; a power of two dividing the warps)
     int32_t db_max;          // double-buffer the row stage while two buffers fit in this many bytes
+    int32_t pipe;            // 1: warp-specialised pass (bulk-copy producer warp, row_pipe_kernel)
     FastDiv fd_gpm;          // ceil(M / R): row groups per matrix
     // Lagged layout shared with the column shuffle (col_tile.cu): logical columns [0, shW)
     // of row i live in the side tile, side + (mat M + i) spitch; columns [shW, N) at A

@@ -916,6 +916,262 @@ cudaError_t row_cluster_dispatch(const RowParams &P, int dir, int eb, cudaStream
 
 
 
+// ---- Warp-specialised row pass (default; IPT_ROW_PIPE=0 keeps the kernels above) ------
+// One PRODUCER warp stages row groups with TMA bulk copies (cp.async.bulk, one per row part:
+// the 16-byte-aligned interior; the at most 3 + 3 words of ragged head / tail with 4-byte
+// cp.async) into NBUF mbarrier-tracked buffers; NW CONSUMER warps gather and write the
+// rows.  full[b]: 1 arrival (lane 0, after publishing the group id) + 32 cp.async arrivals
+// (one per producer lane, each deferred until that lane's small copies landed) + the bulk
+// bytes; empty[b]: one arrival per consumer warp once it no longer reads the buffer.  No
+// CTA-wide barrier on the data path: warps run ahead / behind independently.  Same shared-
+// memory layouts as the kernels above, so the gathers (gather_row, gather_row_rot*) are
+// shared.  Fused rotation (FUSE): the producer takes row groups by ticket (row_rot_kernel's
+// order and progress argument) and sets a group's "read" flags as soon as its data have
+// landed -- not after the CTA's previous gather -- so the neighbours' waits are short.
+__device__ __forceinline__ void pmbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void pmbar_expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" :: "r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void pmbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" :: "r"(bar) : "memory");
+}
+__device__ __forceinline__ void pmbar_arrive_cpasync(uint32_t bar) {
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" :: "r"(bar) : "memory");
+}
+__device__ __forceinline__ void pmbar_wait(uint32_t bar, uint32_t parity) {
+    asm volatile("{\n .reg .pred p;\n WAIT_%=:\n"
+                 " mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%0], %1;\n"
+                 " @!p bra WAIT_%=;\n}" :: "r"(bar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 :: "r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+
+// Stage one contiguous part of a row: global bytes [gs, gs + nb) land at shared byte
+// sd16 + (x - floor16(gs)) (sd16 16-byte aligned).  Interior by one bulk copy (expect_tx
+// first), ragged ends word by word with 4-byte cp.async (every offset is a multiple of 4).
+__device__ __forceinline__ void stage_part(const char *gs, int32_t nb, uint32_t sd16, uint32_t bar) {
+    if (nb <= 0) return;
+    const uintptr_t g = reinterpret_cast<uintptr_t>(gs);
+    const uintptr_t g16 = g & ~uintptr_t(15);
+    const uintptr_t a0 = (g + 15) & ~uintptr_t(15), a1 = (g + nb) & ~uintptr_t(15);
+    auto word = [&](uintptr_t x) {
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(sd16 + static_cast<uint32_t>(x - g16)),
+                     "l"(reinterpret_cast<const void *>(x)) : "memory");
+    };
+    if (a1 > a0) {
+        const uint32_t bytes = static_cast<uint32_t>(a1 - a0);
+        pmbar_expect_tx(bar, bytes);
+        bulk_g2s(sd16 + static_cast<uint32_t>(a0 - g16), reinterpret_cast<const void *>(a0), bytes, bar);
+        for (uintptr_t x = g; x < a0; x += 4) word(x);
+        for (uintptr_t x = a1; x < g + nb; x += 4) word(x);
+    } else {
+        for (uintptr_t x = g; x < g + nb; x += 4) word(x);
+    }
+}
+
+template <int EB, int DIR, bool FUSE, int NBUF, int NW>
+__global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kernel(RowParams P) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ __align__(8) uint64_t bar_full[NBUF], bar_empty[NBUF];
+    __shared__ uint32_t s_group[NBUF];
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    const uint32_t rowbuf = FUSE ? static_cast<uint32_t>(row_fused_smem_bytes(P, EB, DIR))
+                                 : static_cast<uint32_t>((static_cast<uint32_t>(P.N) * EB + 31) & ~15u);
+    const uint32_t bufbytes = rowbuf * static_cast<uint32_t>(P.R);
+    const uint32_t padoff = static_cast<uint32_t>(P.c) * static_cast<uint32_t>(P.segp);  // C2R pad table
+    const uint32_t sbase = smem_u32(smem);
+    const int32_t gpm = (P.M + P.R - 1) / P.R;
+    const uint32_t groups_total = static_cast<uint32_t>(gpm) * static_cast<uint32_t>(P.batch);  // < 2^32 (planner)
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t kDone = 0xffffffffu;
+    if (threadIdx.x == 0) {
+        for (int b = 0; b < NBUF; ++b) {
+            pmbar_init(smem_u32(&bar_full[b]), 33);
+            pmbar_init(smem_u32(&bar_empty[b]), NW);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    auto group_of = [&](uint32_t t) {
+        const uint32_t mat = fdiv(t, P.fd_gpm);
+        uint32_t gm = t - mat * static_cast<uint32_t>(gpm);
+        if (FUSE && DIR == ROW_R2C) gm = static_cast<uint32_t>(gpm) - 1 - gm;
+        RowGroup G;
+        G.mat = mat;
+        G.i0 = static_cast<int32_t>(gm) * P.R;
+        G.nr = min(P.R, P.M - G.i0);
+        return G;
+    };
+    auto mat_base = [&](const RowGroup &G) { return P.base + G.mat * P.mat_stride_bytes; };
+
+    if (warp == NW) {
+        // ================================ producer ================================
+        uint32_t tk = blockIdx.x;  // non-fused: grid-stride order
+        for (uint32_t k = 0;; ++k) {
+            const int b = static_cast<int>(k % NBUF);
+            const uint32_t fb = smem_u32(&bar_full[b]);
+            if (k >= NBUF) pmbar_wait(smem_u32(&bar_empty[b]), ((k / NBUF) - 1) & 1);
+            uint32_t t = 0;
+            if (lane == 0) t = FUSE ? atomicAdd(P.ticket, 1u) : tk;
+            t = __shfl_sync(0xffffffffu, t, 0);
+            tk += gridDim.x;
+            const bool done = t >= groups_total;
+            if (lane == 0) s_group[b] = done ? kDone : t;
+            if (!done) {
+                const RowGroup G = group_of(t);
+                char *mb = mat_base(G);
+                const uint32_t sb0 = sbase + b * bufbytes;
+                if (FUSE && DIR == ROW_C2R) {
+                    // staircase: segment rho of row i = source columns [rho b, rho b + b) of
+                    // row i + rho (rows past M - 1 from the wrap copy), each in its own
+                    // 16-byte-aligned region; padl[rho] maps a source index to its byte
+                    const int32_t Lb = P.b * EB;
+                    char *wb = wrap_matrix(P.wrap, P.wstride, G.mat, mb);
+                    for (int32_t pi = lane; pi < G.nr * P.c; pi += 32) {
+                        const int32_t rr = pi / P.c, rho = pi - rr * P.c;
+                        const int32_t y = G.i0 + rr + rho;
+                        const char *S = (y < P.M ? mb + y * pitch : wb + (y - P.M) * pitch) + static_cast<int64_t>(rho) * Lb;
+                        const uint32_t reg = sb0 + rr * rowbuf + rho * P.segp;
+                        int32_t *padl = reinterpret_cast<int32_t *>(smem + b * bufbytes + rr * rowbuf + padoff);
+                        padl[rho] = rho * P.segp + static_cast<int32_t>(reinterpret_cast<uintptr_t>(S) & 15) - rho * Lb;
+                        stage_part(S, Lb, reg, fb);
+                    }
+                } else {
+                    // whole rows (R2C fused: rows 0..c-2 from the wrap copy); lagged R2C rows
+                    // in two parts (side row, row), both at the row's alignment
+                    const int parts = (DIR == ROW_R2C && P.shW) ? 2 : 1;
+                    for (int32_t pi = lane; pi < G.nr * parts; pi += 32) {
+                        const int32_t rr = pi / parts, part = pi - rr * parts;
+                        const int32_t i = G.i0 + rr;
+                        const char *row = (FUSE && DIR == ROW_R2C && i < P.c - 1)
+                                              ? wrap_matrix(P.wrap, P.wstride, G.mat, mb) + i * pitch
+                                              : mb + i * pitch;
+                        const uint32_t reg = sb0 + rr * rowbuf;
+                        if (parts == 1) {
+                            stage_part(row, P.N * EB, reg, fb);
+                        } else if (part == 0) {
+                            stage_part(side_matrix(P.side, P.sstride, G.mat, mb) + i * P.spitch, P.shW * EB, reg, fb);
+                        } else {
+                            stage_part(row, (P.N - P.shW) * EB, reg + P.shW * EB, fb);
+                        }
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) pmbar_arrive(fb);  // publishes s_group[b] and the pad tables
+            pmbar_arrive_cpasync(fb);
+            if (done) break;
+            if (FUSE) {
+                // the group's reads are complete once its data have landed: flag its rows
+                // (relaxed: the reads are done, the flag orders nothing else; row_rot_kernel)
+                pmbar_wait(fb, (k / NBUF) & 1);
+                const RowGroup G = group_of(t);
+                if (lane < G.nr)
+                    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;"
+                                 :: "l"(P.flags + G.mat * P.M + G.i0 + lane), "r"(1u) : "memory");
+            } else if (NBUF == 1 && tk < groups_total && lane == 0) {
+                // single buffer: the next group's rows stream into L2 while this one is gathered
+                const RowGroup NG = group_of(tk);
+                const char *a = mat_base(NG) + NG.i0 * pitch;
+                const uintptr_t a0 = (reinterpret_cast<uintptr_t>(a) + 15) & ~uintptr_t(15);
+                const uintptr_t a1 = (reinterpret_cast<uintptr_t>(a) + NG.nr * pitch) & ~uintptr_t(15);
+                for (uintptr_t x = a0; x < a1; x += 32768) {
+                    const uint32_t sz = a1 - x < 32768 ? static_cast<uint32_t>(a1 - x) : 32768u;
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(x), "r"(sz) : "memory");
+                }
+            }
+        }
+        return;
+    }
+
+    // ================================ consumers ================================
+    const int wn = NW / P.R;  // warps per row team
+    const int team = warp / wn, wl = warp - team * wn;
+    const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;
+    const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
+    const int64_t vD = static_cast<int64_t>(wn) * 32 * (16 / EB);
+    const int32_t vdl = FUSE ? static_cast<int32_t>(vD % P.c) : 0;
+    const int32_t vdh = FUSE ? static_cast<int32_t>((static_cast<int64_t>(P.ainv) * ((vD / P.c) % P.b)) % P.b) : 0;
+    for (uint32_t k = 0;; ++k) {
+        const int b = static_cast<int>(k % NBUF);
+        pmbar_wait(smem_u32(&bar_full[b]), (k / NBUF) & 1);
+        const uint32_t t = s_group[b];
+        if (t == kDone) break;
+        const RowGroup G = group_of(t);
+        char *mbase = mat_base(G);
+        if (FUSE) {
+            // every row this group overwrites has been read (flags of smaller tickets)
+            if (lane >= 1 && lane < P.c) {
+                const int32_t y = DIR == ROW_C2R ? G.i0 - lane : G.i0 + G.nr - 1 + lane;
+                if (y >= 0 && y < P.M) {
+                    const unsigned int *f = P.flags + G.mat * P.M + y;
+                    unsigned int v;
+                    while (true) {
+                        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
+                        if (v) break;
+                        __nanosleep(32);
+                    }
+                }
+            }
+            __syncwarp();
+        }
+        if (team < G.nr) {
+            const int32_t i = G.i0 + team;
+            const unsigned char *buf = smem + b * bufbytes + team * rowbuf;
+            if (!FUSE) {
+                char *row = mbase + i * pitch;
+                const unsigned char *st = buf + (reinterpret_cast<uintptr_t>(row) & 15);
+                char *srow = P.shW ? side_matrix(P.side, P.sstride, G.mat, mbase) + i * P.spitch : nullptr;
+                if (i >= P.M - P.c + 1) gather_row<EB, DIR, true>(P, row, srow, st, i, p_begin, p_end);
+                else gather_row<EB, DIR, false>(P, row, srow, st, i, p_begin, p_end);
+            } else {
+                char *srow = P.shW ? side_matrix(P.side, P.sstride, G.mat, mbase) + i * P.spitch : nullptr;
+                if (DIR == ROW_C2R) {
+                    if (P.vec && i < P.M - P.c + 1)
+                        gather_row_rot_c2r_vec<EB>(P, mbase, srow, buf, reinterpret_cast<const int32_t *>(buf + padoff), i,
+                                                   wl * 32 + lane, wn * 32, vdl, vdh);
+                    else
+                        gather_row_rot<EB, DIR>(P, mbase, srow, buf, reinterpret_cast<const int32_t *>(buf + padoff), i,
+                                                p_begin, p_end);
+                } else {
+                    gather_row_rot<EB, DIR>(P, mbase, srow, buf + (reinterpret_cast<uintptr_t>(mbase + i * pitch) & 15),
+                                            nullptr, i, p_begin, p_end);
+                }
+            }
+        }
+        __syncwarp();
+        if (lane == 0) pmbar_arrive(smem_u32(&bar_empty[b]));
+    }
+}
+
+template <int EB, int DIR, bool FUSE, int NBUF, int NW>
+cudaError_t launch_row_pipe_t(const RowParams &P, cudaStream_t st) {
+    const size_t rowbuf = FUSE ? row_fused_smem_bytes(P, EB, DIR) : row_smem_bytes(P.N, EB);
+    const size_t smem = NBUF * P.R * rowbuf;
+    auto kern = row_pipe_kernel<EB, DIR, FUSE, NBUF, NW>;
+    cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
+    if (e != cudaSuccess) return e;
+    const int threads = NW * 32 + 32;
+    const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), threads, smem);
+    if (resident < 1) return cudaErrorInvalidConfiguration;
+    if (FUSE && (!P.ticket || !P.flags || !P.wrap)) return cudaErrorInvalidValue;
+    const int64_t groups = static_cast<int64_t>((P.M + P.R - 1) / P.R) * P.batch;
+    int64_t grid = resident;
+    if (grid > groups) grid = groups;
+    kern<<<static_cast<unsigned>(grid), threads, smem, st>>>(P);
+    return cudaGetLastError();
+}
+
+template <int EB, int DIR, bool FUSE, int NBUF>
+cudaError_t launch_row_pipe_n(const RowParams &P, cudaStream_t st) {
+    return row_threads(P.N, EB) == 512 ? launch_row_pipe_t<EB, DIR, FUSE, NBUF, 16>(P, st)
+                                       : launch_row_pipe_t<EB, DIR, FUSE, NBUF, 8>(P, st);
+}
+
 template <int EB, int DIR, int NBUF>
 cudaError_t launch_row_t(const RowParams &P, cudaStream_t st) {
     const size_t smem = NBUF * P.R * row_smem_bytes(P.N, EB);
@@ -951,6 +1207,15 @@ cudaError_t launch_row_rot_t(const RowParams &P, cudaStream_t st) {
 
 template <int EB, int DIR>
 cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
+    if (P.pipe) {
+        if (P.fuse)
+            return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max)
+                       ? launch_row_pipe_n<EB, DIR, true, 2>(P, st)
+                       : launch_row_pipe_n<EB, DIR, true, 1>(P, st);
+        return 2 * P.R * row_smem_bytes(P.N, EB) <= static_cast<size_t>(P.db_max)
+                   ? launch_row_pipe_n<EB, DIR, false, 2>(P, st)
+                   : launch_row_pipe_n<EB, DIR, false, 1>(P, st);
+    }
     if (P.fuse)
         return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max)
                    ? launch_row_rot_t<EB, DIR, 2>(P, st)
