@@ -417,7 +417,7 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         rsm = rowbuf * rp.R;
     }
     rp.db_max = env_int("IPT_ROW_DB_MAX", 112 * 1024);
-    rp.pipe = env_int("IPT_ROW_PIPE", 1) != 0 ? 1 : 0;
+    rp.pipe = env_int("IPT_ROW_PIPE", 1);
     rp.fd_gpm = make_fastdiv(static_cast<uint32_t>((pl.M + rp.R - 1) / rp.R));
 
     ipt_status_t s = plan_col(dev, pl, engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.shuf);

@@ -945,6 +945,12 @@ __device__ __forceinline__ void pmbar_wait(uint32_t bar, uint32_t parity) {
                  " mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%0], %1;\n"
                  " @!p bra WAIT_%=;\n}" :: "r"(bar), "r"(parity) : "memory");
 }
+__device__ __forceinline__ bool pmbar_test(uint32_t bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile("{\n .reg .pred p;\n mbarrier.test_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n"
+                 " selp.u32 %0, 1, 0, p;\n}" : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
+    return ok != 0;
+}
 __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                  :: "r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
@@ -1010,15 +1016,63 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
 
     if (warp == NW) {
         // ================================ producer ================================
+        // FUSE: a group's flags are set as soon as its data have landed: while the
+        // producer waits for a free buffer it polls the landings of the groups it issued
+        // (at most NBUF pending).  Progress: every wait of this CTA (free buffers, landings)
+        // depends only on groups with smaller tickets (row_rot_kernel's induction).
+        auto set_flags = [&](uint32_t t) {
+            const RowGroup G = group_of(t);
+            if (lane < G.nr)
+                asm volatile("st.relaxed.gpu.global.u32 [%0], %1;"
+                             :: "l"(P.flags + G.mat * P.M + G.i0 + lane), "r"(1u) : "memory");
+        };
+        uint32_t pend_t[NBUF + 1], pend_k[NBUF + 1];  // issued, not yet flagged (oldest first)
+        int npend = 0;
+        auto poll = [&](bool block) {  // flag the landed pending groups (block: all of them)
+            while (npend > 0) {
+                const uint32_t fb0 = smem_u32(&bar_full[pend_k[0] % NBUF]);
+                bool ok = lane == 0 ? (block ? (pmbar_wait(fb0, (pend_k[0] / NBUF) & 1), true)
+                                             : pmbar_test(fb0, (pend_k[0] / NBUF) & 1))
+                                    : false;
+                ok = __shfl_sync(0xffffffffu, ok ? 1 : 0, 0) != 0;
+                if (!ok) return;
+                set_flags(pend_t[0]);
+                for (int q = 1; q < npend; ++q) {
+                    pend_t[q - 1] = pend_t[q];
+                    pend_k[q - 1] = pend_k[q];
+                }
+                --npend;
+            }
+        };
         uint32_t tk = blockIdx.x;  // non-fused: grid-stride order
         for (uint32_t k = 0;; ++k) {
             const int b = static_cast<int>(k % NBUF);
             const uint32_t fb = smem_u32(&bar_full[b]);
-            if (k >= NBUF) pmbar_wait(smem_u32(&bar_empty[b]), ((k / NBUF) - 1) & 1);
-            uint32_t t = 0;
-            if (lane == 0) t = FUSE ? atomicAdd(P.ticket, 1u) : tk;
-            t = __shfl_sync(0xffffffffu, t, 0);
-            tk += gridDim.x;
+            if (k >= NBUF) {
+                const uint32_t eb_ = smem_u32(&bar_empty[b]), ep = ((k / NBUF) - 1) & 1;
+                if (FUSE) {
+                    while (true) {
+                        poll(false);
+                        bool ok = lane == 0 ? pmbar_test(eb_, ep) : false;
+                        if (__shfl_sync(0xffffffffu, ok ? 1 : 0, 0)) break;
+                        __nanosleep(20);
+                    }
+                    __syncwarp();
+                    pmbar_wait(eb_, ep);  // every lane observes the release (acquire)
+                    poll(false);          // group k - NBUF has landed (its consumers are done)
+                } else {
+                    pmbar_wait(eb_, ep);
+                }
+            }
+            // fused: the ticket is taken only now, when its group is staged at once (a ticket
+            // held while the CTA waits for a buffer would stall the groups after it)
+            uint32_t t = tk;
+            if (FUSE) {
+                if (lane == 0) t = atomicAdd(P.ticket, 1u);
+                t = __shfl_sync(0xffffffffu, t, 0);
+            } else {
+                tk += gridDim.x;
+            }
             const bool done = t >= groups_total;
             if (lane == 0) s_group[b] = done ? kDone : t;
             if (!done) {
@@ -1064,15 +1118,15 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
             __syncwarp();
             if (lane == 0) pmbar_arrive(fb);  // publishes s_group[b] and the pad tables
             pmbar_arrive_cpasync(fb);
-            if (done) break;
             if (FUSE) {
                 // the group's reads are complete once its data have landed: flag its rows
                 // (relaxed: the reads are done, the flag orders nothing else; row_rot_kernel)
-                pmbar_wait(fb, (k / NBUF) & 1);
-                const RowGroup G = group_of(t);
-                if (lane < G.nr)
-                    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;"
-                                 :: "l"(P.flags + G.mat * P.M + G.i0 + lane), "r"(1u) : "memory");
+                if (!done) {
+                    pend_t[npend] = t;
+                    pend_k[npend] = k;
+                    ++npend;
+                }
+                poll(done || NBUF == 1);
             } else if (NBUF == 1 && tk < groups_total && lane == 0) {
                 // single buffer: the next group's rows stream into L2 while this one is gathered
                 const RowGroup NG = group_of(tk);
@@ -1084,6 +1138,7 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
                     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(x), "r"(sz) : "memory");
                 }
             }
+            if (done) break;
         }
         return;
     }
@@ -1208,13 +1263,15 @@ cudaError_t launch_row_rot_t(const RowParams &P, cudaStream_t st) {
 template <int EB, int DIR>
 cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
     if (P.pipe) {
-        if (P.fuse)
-            return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max)
-                       ? launch_row_pipe_n<EB, DIR, true, 2>(P, st)
-                       : launch_row_pipe_n<EB, DIR, true, 1>(P, st);
-        return 2 * P.R * row_smem_bytes(P.N, EB) <= static_cast<size_t>(P.db_max)
-                   ? launch_row_pipe_n<EB, DIR, false, 2>(P, st)
-                   : launch_row_pipe_n<EB, DIR, false, 1>(P, st);
+        // Fused rotation: row_rot_kernel stays the default (the pipelined variant measured
+        // 0.89x of it on the fused sweep shapes, tools/ab_calls.py r02f); IPT_ROW_PIPE=2
+        // selects the pipelined one where two buffers fit.
+        if (P.fuse && P.pipe == 2 && 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max))
+            return launch_row_pipe_n<EB, DIR, true, 2>(P, st);
+        if (!P.fuse)
+            return 2 * P.R * row_smem_bytes(P.N, EB) <= static_cast<size_t>(P.db_max)
+                       ? launch_row_pipe_n<EB, DIR, false, 2>(P, st)
+                       : launch_row_pipe_n<EB, DIR, false, 1>(P, st);
     }
     if (P.fuse)
         return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max)
