@@ -303,6 +303,7 @@ __device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, co
     constexpr int LPR = W < 32 ? W : 32;  // lanes per tile row
     constexpr int RPW = 32 / LPR;         // tile rows per warp instruction
     constexpr int CPL = W / LPR;          // columns per lane
+    constexpr int U8 = EB == 16 ? 4 : 8;  // rows in flight per lane (independent shared loads)
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = nthr >> 5;
     const int w0 = lane % LPR, sub = lane / LPR;
     if (U.skip) return;
@@ -316,21 +317,26 @@ __device__ __forceinline__ void unit_store(const ColParams &P, const Unit &U, co
         char *colp = U.outp + w * EB;
         const uint32_t *sb = sbase + dw_of<EB, MODE, TWB>(P, U, w);
         const uint32_t wo = w * EB;
-        uint32_t v[4];
-        if (MODE == COL_C2R_SHUF) {
-#pragma unroll 4
-            for (; k < U.nrows; k += step) {
-                lds_elem<EB>(v, sb[k] + wo);
-                stg_elem<EB>(colp + orow[k], v);
+        // Batches of U8 rows: all the batch's slot addresses and row offsets first, then its
+        // element loads, then its stores -- U8 independent load chains per lane instead of a
+        // dependent lds -> lds -> stg chain per row.
+        for (; k + (U8 - 1) * step < U.nrows; k += U8 * step) {
+            uint32_t a[U8], v[U8][EB / 4];
+            int64_t o[U8];
+#pragma unroll
+            for (int u = 0; u < U8; ++u) {
+                a[u] = sb[k + u * step] + wo;
+                o[u] = MODE == COL_C2R_SHUF ? orow[k + u * step] : static_cast<int64_t>(U.r0 + k + u * step) * pitch;
             }
-        } else {
-            char *g = colp + static_cast<int64_t>(U.r0 + k) * pitch;
-            const int64_t g_inc = step * pitch;
-#pragma unroll 4
-            for (; k < U.nrows; k += step, g += g_inc) {
-                lds_elem<EB>(v, sb[k] + wo);
-                stg_elem<EB>(g, v);
-            }
+#pragma unroll
+            for (int u = 0; u < U8; ++u) lds_elem<EB>(v[u], a[u]);
+#pragma unroll
+            for (int u = 0; u < U8; ++u) stg_elem<EB>(colp + o[u], v[u]);
+        }
+        for (; k < U.nrows; k += step) {
+            uint32_t v[EB / 4];
+            lds_elem<EB>(v, sb[k] + wo);
+            stg_elem<EB>(colp + (MODE == COL_C2R_SHUF ? orow[k] : static_cast<int64_t>(U.r0 + k) * pitch), v);
         }
     }
 }
@@ -402,12 +408,18 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
         if (D.arrive && threadIdx.x == 0) atomicAdd(P.ctr + (tt % kCtrSlots), 1u);
         return;
     }
-    if (P.dbg != 4) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
-    if (MODE == COL_R2C_SHUF) __syncthreads();
+    // R2C: the loads need the scattered source rows (prepass first); otherwise the loads go
+    // out first and the C2R destination rows are computed while they are in flight.
+    if (MODE == COL_R2C_SHUF) {
+        if (P.dbg != 4) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
+        __syncthreads();
+    }
     if (P.dbg != 2)  // measurement knob: 2 = skip the loads
         unit_load<EB, MODE, TWB>(P, U, srow, sbase, static_cast<uint32_t>(__cvta_generic_to_shared(smem + L.rows)),
                                  blockDim.x);
-    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    if (MODE != COL_R2C_SHUF && P.dbg != 4) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
     __syncthreads();  // every thread's staged data is in shared memory
     if (threadIdx.x == 0) {
         // The arrival only says "this unit's reads of its input are complete" (write-after-

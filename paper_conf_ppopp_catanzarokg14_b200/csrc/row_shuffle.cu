@@ -1031,11 +1031,13 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
         auto poll = [&](bool block) {  // flag the landed pending groups (block: all of them)
             while (npend > 0) {
                 const uint32_t fb0 = smem_u32(&bar_full[pend_k[0] % NBUF]);
-                bool ok = lane == 0 ? (block ? (pmbar_wait(fb0, (pend_k[0] / NBUF) & 1), true)
-                                             : pmbar_test(fb0, (pend_k[0] / NBUF) & 1))
-                                    : false;
-                ok = __shfl_sync(0xffffffffu, ok ? 1 : 0, 0) != 0;
-                if (!ok) return;
+                // every lane observes the phase itself (acquire), the warp agrees on the result
+                bool ok = block ? (pmbar_wait(fb0, (pend_k[0] / NBUF) & 1), true)
+                                : pmbar_test(fb0, (pend_k[0] / NBUF) & 1);
+                if (!__all_sync(0xffffffffu, ok)) {
+                    if (block) continue;
+                    return;
+                }
                 set_flags(pend_t[0]);
                 for (int q = 1; q < npend; ++q) {
                     pend_t[q - 1] = pend_t[q];
@@ -1053,13 +1055,12 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
                 if (FUSE) {
                     while (true) {
                         poll(false);
-                        bool ok = lane == 0 ? pmbar_test(eb_, ep) : false;
-                        if (__shfl_sync(0xffffffffu, ok ? 1 : 0, 0)) break;
+                        const bool ok = pmbar_test(eb_, ep);  // per lane: acquire
+                        if (__all_sync(0xffffffffu, ok)) break;
+                        if (ok) pmbar_wait(eb_, ep);  // (a phase once complete stays complete)
                         __nanosleep(20);
                     }
-                    __syncwarp();
-                    pmbar_wait(eb_, ep);  // every lane observes the release (acquire)
-                    poll(false);          // group k - NBUF has landed (its consumers are done)
+                    poll(false);  // group k - NBUF has landed (its consumers are done)
                 } else {
                     pmbar_wait(eb_, ep);
                 }
