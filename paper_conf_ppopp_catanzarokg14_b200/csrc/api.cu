@@ -416,6 +416,20 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         while (rp.R * 2 <= nw && rp.R * 2 * rowbuf <= target) rp.R *= 2;
         rsm = rowbuf * rp.R;
     }
+    // Chunked fused pass (row_chunk_kernel; IPT_ROW_CHUNK=0 keeps the flag-based
+    // row_rot_kernel): chunks of cK = max(R, IPT_ROW_CHUNK_K (c-1)) rows, so the boundary copy
+    // costs 2 (c-1) / cK of a pass.
+    if (rp.fuse && env_int("IPT_ROW_CHUNK", 1) != 0) {
+        int64_t K = std::max<int64_t>(rp.R, static_cast<int64_t>(env_int("IPT_ROW_CHUNK_K", 16)) * (pl.c - 1));
+        K = (K + rp.R - 1) / rp.R * rp.R;
+        const int64_t Mr = (pl.M + rp.R - 1) / rp.R * rp.R;
+        if (K > Mr) K = Mr;
+        rp.chunk = 1;
+        rp.cK = static_cast<int32_t>(K);
+        rp.nch = static_cast<int32_t>((pl.M + K - 1) / K);
+        rp.fd_nch = make_fastdiv(static_cast<uint32_t>(rp.nch));
+        rp.rpitch = ((pl.N * eb + 15) & ~int64_t(15)) + 16;
+    }
     rp.db_max = env_int("IPT_ROW_DB_MAX", 112 * 1024);
     rp.pipe = env_int("IPT_ROW_PIPE", 1);
     rp.fd_gpm = make_fastdiv(static_cast<uint32_t>((pl.M + rp.R - 1) / rp.R));
@@ -469,7 +483,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -551,6 +565,7 @@ struct CallScratch {
     size_t flags = 0;                  // fused rotation: M*batch row flags + the ticket
     size_t zero_bytes = 0;             // [0, zero_bytes) is zeroed before the first pass
     size_t wrap = 0, wstride = 0;      // fused rotation: per-matrix copy of rows 0..c-2
+    size_t bnd = 0;                    // chunked fused pass: boundary rows
     size_t side = 0;                   // lagged layouts: side blocks
     size_t total = 0;
 };
@@ -581,15 +596,21 @@ void prepare_call(Plan &pl, int64_t batch, CallScratch &cs) {
         cs.ctr_rot = o;
         o += kCtrBytes;
     }
-    if (pl.row.fuse) {
+    const bool flagged = pl.row.fuse && !pl.row.chunk;  // row_rot_kernel / pipelined fused pass
+    if (flagged) {
         cs.flags = o;
         o += al256((static_cast<size_t>(pl.M) * static_cast<size_t>(batch) + 1) * 4);
     }
     cs.zero_bytes = o;
-    if (pl.row.fuse) {
+    if (flagged) {
         cs.wrap = o;
         cs.wstride = al256(static_cast<size_t>(pl.c - 1) * pl.N * pl.eb + 16);
         o += cs.wstride * static_cast<size_t>(batch);
+    }
+    if (pl.row.fuse && pl.row.chunk) {
+        cs.bnd = o;
+        o += al256(static_cast<size_t>(pl.row.nch) * static_cast<size_t>(batch) * static_cast<size_t>(pl.c - 1) *
+                   static_cast<size_t>(pl.row.rpitch));
     }
     if (pl.side_bytes) {
         cs.side = o;
@@ -686,11 +707,15 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
     pl.shuf.p.ctr = reinterpret_cast<unsigned int *>(scratch + cs.ctr_shuf);
     pl.rot.p.ctr = reinterpret_cast<unsigned int *>(scratch + cs.ctr_rot);
     pl.shuf.p.ticket = pl.rot.p.ticket = env_int("IPT_COL_TICKET", 1) != 0 ? 1 : 0;
-    if (pl.row.fuse) {
+    if (pl.row.fuse && !pl.row.chunk) {
         pl.row.flags = reinterpret_cast<unsigned int *>(scratch + cs.flags);
         pl.row.ticket = pl.row.flags + pl.M * batch;
         pl.row.wrap = scratch + cs.wrap;
         pl.row.wstride = static_cast<int64_t>(cs.wstride);
+    }
+    if (pl.row.fuse && pl.row.chunk) {
+        if (static_cast<int64_t>(pl.row.nch) * batch >= (int64_t(1) << 32)) return IPT_ERR_UNSUPPORTED;
+        pl.row.bnd = scratch + cs.bnd;
     }
     pl.row.side = pl.shuf.p.side = pl.side_bytes ? scratch + cs.side : nullptr;
     const int64_t pitch = pl.N * pl.eb;
@@ -699,8 +724,8 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
     const double rot_bytes = full * static_cast<double>(pl.c - 1) / static_cast<double>(pl.c);
     auto rot = [&] { return launch_col(pl.rot.p, COL_ROT, pl.eb, st, pl.rot.smem); };
     auto row = [&] {
-        if (pl.row.fuse) {  // rows 0..c-2 of every matrix into the wrap slots first
-            cudaError_t e = launch_copy_wrap(pl.row, pl.eb, st);
+        if (pl.row.fuse) {  // chunk boundary rows / rows 0..c-2 of every matrix copied first
+            cudaError_t e = pl.row.chunk ? launch_copy_bounds(pl.row, pl.eb, st) : launch_copy_wrap(pl.row, pl.eb, st);
             if (e != cudaSuccess) return e;
             g_launches++;
         }

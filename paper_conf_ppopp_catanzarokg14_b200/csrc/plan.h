@@ -44,6 +44,13 @@ __host__ __device__ inline char *wrap_matrix(char *wrap, int64_t wstride, int64_
     char *raw = wrap + mat * wstride;
     return raw + ((reinterpret_cast<uintptr_t>(A_mat) - reinterpret_cast<uintptr_t>(raw)) & 15);
 }
+// Boundary row r (< c-1) of chunk x of matrix `mat` (chunked fused pass), placed at the same
+// address mod 16 as the matrix row it copies (A_row), so it stages like that row.
+__host__ __device__ inline char *bnd_row(char *bnd, int64_t rpitch, int64_t nch, int32_t c, int64_t mat, int64_t x,
+                                         int32_t r, const char *A_row) {
+    char *raw = bnd + ((mat * nch + x) * (c - 1) + r) * rpitch;
+    return raw + ((reinterpret_cast<uintptr_t>(A_row) - reinterpret_cast<uintptr_t>(raw)) & 15);
+}
 // Row-shuffle directions.
 enum RowDir : int {
     ROW_C2R = 0,  // out[i][j] = in[i][d'^{-1}_i(j)]  (Eq. 31)
@@ -101,6 +108,17 @@ struct RowParams {
                              // the fused pass: C2R staircases past row M-1 read it, R2C reads
                              // rows 0..c-2 from it so that writes into them need no wait)
     int64_t wstride;         // bytes reserved per matrix in `wrap`
+    // Chunked fused pass (row_chunk_kernel, default for the fused rotation): every matrix
+    // is cut into nch chunks of cK consecutive rows; a CTA processes a chunk's row groups in
+    // order (C2R ascending, R2C descending).  The first c-1 rows of every chunk are copied to
+    // `bnd` before the pass (launch_copy_bounds): C2R staircases that cross into the next
+    // chunk (or past row M-1: chunk 0) and R2C reads of a chunk's own first rows use the copy,
+    // so no CTA ever waits for another.
+    int32_t chunk;           // 1: chunked fused pass
+    int32_t cK, nch;         // rows per chunk (a multiple of R), chunks per matrix
+    FastDiv fd_nch;
+    char *bnd;               // boundary rows: bnd_row()
+    int64_t rpitch;          // bytes per boundary row slot (N eb rounded up to 16, + 16)
 };
 constexpr int kMaxFuseC = 32;
 
@@ -177,6 +195,8 @@ constexpr int kTicketSlot = kCtrSlots;
 constexpr size_t kCtrBytes = (sizeof(unsigned int) * (kCtrSlots + 1) + 255) & ~size_t(255);
 // Copy rows 0..c-2 of every matrix into the wrap buffer (row_shuffle.cu).
 cudaError_t launch_copy_wrap(const RowParams &p, int eb, cudaStream_t st);
+// Copy the first c-1 rows of every chunk into the boundary rows (chunked fused pass).
+cudaError_t launch_copy_bounds(const RowParams &p, int eb, cudaStream_t st);
 
 // Launchers (col_tile.cu / row_shuffle.cu).  They return the CUDA error of the launch.
 size_t row_smem_bytes(int64_t N, int eb);

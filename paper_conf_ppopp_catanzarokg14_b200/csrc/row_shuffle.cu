@@ -1204,6 +1204,225 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
     }
 }
 
+// ---- Chunked fused rotation + row pass (default for 1 < c <= kMaxFuseC) ---------------
+// Same producer / consumer structure and staging as row_pipe_kernel<FUSE>, but the work unit
+// is a CHUNK of cK consecutive rows of one matrix, whose row groups a CTA processes in order:
+//  * C2R (Eq. 23 then Eq. 31): writing row i overwrites segments that only the staircases of
+//    rows i-c+1 .. i read; those of the same chunk were staged (landed) before row i's group
+//    is gathered (the consumer takes groups in order), those of the previous chunk read the
+//    boundary copy of this chunk's first c-1 rows instead.
+//  * R2C (Eq. 24 then Eq. 36), descending: row i's blocks go to rows i .. i+c-1, staged
+//    earlier in the chunk; rows of the next chunk (or rows 0..c-2 past row M-1) are read by
+//    their own chunk from its boundary copy.
+// So no CTA waits for another: no flags, no tickets, no co-residency assumption.  Extra
+// traffic: the boundary copy, 2 (c-1) / cK of a pass.
+template <int EB, int DIR, int NBUF, int NW>
+__global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_chunk_kernel(RowParams P) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ __align__(8) uint64_t bar_full[NBUF], bar_empty[NBUF];
+    const int64_t pitch = static_cast<int64_t>(P.N) * EB;
+    const uint32_t rowbuf = static_cast<uint32_t>(row_fused_smem_bytes(P, EB, DIR));
+    const uint32_t bufbytes = rowbuf * static_cast<uint32_t>(P.R);
+    const uint32_t padoff = static_cast<uint32_t>(P.c) * static_cast<uint32_t>(P.segp);  // C2R pad table
+    const uint32_t sbase = smem_u32(smem);
+    const int64_t total_chunks = static_cast<int64_t>(P.nch) * P.batch;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int b = 0; b < NBUF; ++b) {
+            pmbar_init(smem_u32(&bar_full[b]), 33);
+            pmbar_init(smem_u32(&bar_empty[b]), NW);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    // The (chunk, group) sequence of this CTA -- walked identically by producer and consumers.
+    struct Seq {
+        int64_t ch, mat;
+        int32_t x, r0, r1, ng, gi;
+    };
+    auto chunk_at = [&](Seq &q, int64_t ch) {
+        q.ch = ch;
+        if (ch >= total_chunks) return false;
+        q.mat = static_cast<int64_t>(fdiv(static_cast<uint32_t>(ch), P.fd_nch));  // total_chunks < 2^32
+        q.x = static_cast<int32_t>(ch - q.mat * P.nch);
+        q.r0 = q.x * P.cK;
+        q.r1 = min(P.M, q.r0 + P.cK);
+        q.ng = (q.r1 - q.r0 + P.R - 1) / P.R;
+        q.gi = 0;
+        return true;
+    };
+    auto advance = [&](Seq &q) {  // next group; false at the end of this CTA's work
+        if (++q.gi < q.ng) return true;
+        return chunk_at(q, q.ch + gridDim.x);
+    };
+    auto group_of = [&](const Seq &q) {
+        RowGroup G;
+        G.mat = q.mat;
+        const int32_t g = DIR == ROW_C2R ? q.gi : q.ng - 1 - q.gi;
+        G.i0 = q.r0 + g * P.R;
+        G.nr = min(P.R, q.r1 - G.i0);
+        return G;
+    };
+    auto mat_base = [&](int64_t mat) { return P.base + mat * P.mat_stride_bytes; };
+
+    if (warp == NW) {
+        // ================================ producer ================================
+        Seq q;
+        bool more = chunk_at(q, blockIdx.x);
+        for (uint32_t k = 0; more; ++k) {
+            const int b = static_cast<int>(k % NBUF);
+            const uint32_t fb = smem_u32(&bar_full[b]);
+            if (k >= NBUF) pmbar_wait(smem_u32(&bar_empty[b]), ((k / NBUF) - 1) & 1);
+            const RowGroup G = group_of(q);
+            char *mb = mat_base(G.mat);
+            const uint32_t sb0 = sbase + b * bufbytes;
+            if (DIR == ROW_C2R) {
+                // staircase: segment rho of row i = source columns [rho b, rho b + b) of row
+                // i + rho -- from the boundary copy of the next chunk (chunk 0 past row M-1)
+                const int32_t Lb = P.b * EB;
+                for (int32_t pi = lane; pi < G.nr * P.c; pi += 32) {
+                    const int32_t rr = pi / P.c, rho = pi - rr * P.c;
+                    const int32_t y = G.i0 + rr + rho;
+                    const char *rowp;
+                    if (y < q.r1) {
+                        rowp = mb + y * pitch;
+                    } else if (y < P.M) {
+                        rowp = bnd_row(P.bnd, P.rpitch, P.nch, P.c, G.mat, q.x + 1, y - q.r1, mb + y * pitch);
+                    } else {
+                        rowp = bnd_row(P.bnd, P.rpitch, P.nch, P.c, G.mat, 0, y - P.M, mb + (y - P.M) * pitch);
+                    }
+                    const char *S = rowp + static_cast<int64_t>(rho) * Lb;
+                    const uint32_t reg = sb0 + rr * rowbuf + rho * P.segp;
+                    int32_t *padl = reinterpret_cast<int32_t *>(smem + b * bufbytes + rr * rowbuf + padoff);
+                    padl[rho] = rho * P.segp + static_cast<int32_t>(reinterpret_cast<uintptr_t>(S) & 15) - rho * Lb;
+                    stage_part(S, Lb, reg, fb);
+                }
+            } else {
+                // whole rows, the chunk's first c-1 from its boundary copy; lagged rows in two
+                // parts (side row, row), both at the row's alignment
+                const int parts = P.shW ? 2 : 1;
+                for (int32_t pi = lane; pi < G.nr * parts; pi += 32) {
+                    const int32_t rr = pi / parts, part = pi - rr * parts;
+                    const int32_t i = G.i0 + rr;
+                    const char *row = i - q.r0 < P.c - 1
+                                          ? bnd_row(P.bnd, P.rpitch, P.nch, P.c, G.mat, q.x, i - q.r0, mb + i * pitch)
+                                          : mb + i * pitch;
+                    const uint32_t reg = sb0 + rr * rowbuf;
+                    if (parts == 1) {
+                        stage_part(row, P.N * EB, reg, fb);
+                    } else if (part == 0) {
+                        stage_part(side_matrix(P.side, P.sstride, G.mat, mb) + i * P.spitch, P.shW * EB, reg, fb);
+                    } else {
+                        stage_part(row, (P.N - P.shW) * EB, reg + P.shW * EB, fb);
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) pmbar_arrive(fb);  // publishes the pad tables
+            pmbar_arrive_cpasync(fb);
+            more = advance(q);
+            if (NBUF == 1 && more && lane == 0) {
+                // single buffer: the next group's rows stream into L2 while this one is gathered
+                const RowGroup NG = group_of(q);
+                const char *a = mat_base(NG.mat) + NG.i0 * pitch;
+                const uintptr_t a0 = (reinterpret_cast<uintptr_t>(a) + 15) & ~uintptr_t(15);
+                const uintptr_t a1 = (reinterpret_cast<uintptr_t>(a) + NG.nr * pitch) & ~uintptr_t(15);
+                for (uintptr_t xx = a0; xx < a1; xx += 32768) {
+                    const uint32_t sz = a1 - xx < 32768 ? static_cast<uint32_t>(a1 - xx) : 32768u;
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(xx), "r"(sz) : "memory");
+                }
+            }
+        }
+        return;
+    }
+
+    // ================================ consumers ================================
+    const int wn = NW / P.R;  // warps per row team
+    const int team = warp / wn, wl = warp - team * wn;
+    const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;
+    const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
+    const int64_t vD = static_cast<int64_t>(wn) * 32 * (16 / EB);
+    const int32_t vdl = static_cast<int32_t>(vD % P.c);
+    const int32_t vdh = static_cast<int32_t>((static_cast<int64_t>(P.ainv) * ((vD / P.c) % P.b)) % P.b);
+    Seq q;
+    bool more = chunk_at(q, blockIdx.x);
+    for (uint32_t k = 0; more; ++k) {
+        const int b = static_cast<int>(k % NBUF);
+        pmbar_wait(smem_u32(&bar_full[b]), (k / NBUF) & 1);
+        const RowGroup G = group_of(q);
+        char *mbase = mat_base(G.mat);
+        if (team < G.nr) {
+            const int32_t i = G.i0 + team;
+            const unsigned char *buf = smem + b * bufbytes + team * rowbuf;
+            char *srow = P.shW ? side_matrix(P.side, P.sstride, G.mat, mbase) + i * P.spitch : nullptr;
+            if (DIR == ROW_C2R) {
+                if (P.vec && i < P.M - P.c + 1)
+                    gather_row_rot_c2r_vec<EB>(P, mbase, srow, buf, reinterpret_cast<const int32_t *>(buf + padoff), i,
+                                               wl * 32 + lane, wn * 32, vdl, vdh);
+                else
+                    gather_row_rot<EB, DIR>(P, mbase, srow, buf, reinterpret_cast<const int32_t *>(buf + padoff), i,
+                                            p_begin, p_end);
+            } else {
+                gather_row_rot<EB, DIR>(P, mbase, srow, buf + (reinterpret_cast<uintptr_t>(mbase + i * pitch) & 15),
+                                        nullptr, i, p_begin, p_end);
+            }
+        }
+        __syncwarp();
+        if (lane == 0) pmbar_arrive(smem_u32(&bar_empty[b]));
+        more = advance(q);
+    }
+}
+
+// Boundary copy of the chunked fused pass: rows [x cK, x cK + c - 1) (clamped to M) of every
+// chunk x of every matrix into bnd_row() slots; one CTA per (matrix, chunk), threads over the
+// row's 16-byte chunks (same address mod 16 on both sides; every offset is a multiple of 4).
+__global__ void __launch_bounds__(256) copy_bounds_kernel(RowParams P, int64_t pitch) {
+    const int64_t slots = static_cast<int64_t>(P.nch) * P.batch;
+    for (int64_t sl = blockIdx.x; sl < slots; sl += gridDim.x) {
+        const int64_t mat = sl / P.nch;
+        const int32_t x = static_cast<int32_t>(sl - mat * P.nch);
+        const int32_t r0 = x * P.cK, nr = min(P.c - 1, P.M - r0);
+        char *mb = P.base + mat * P.mat_stride_bytes;
+        for (int32_t r = 0; r < nr; ++r) {
+            const char *src = mb + (r0 + r) * pitch;
+            char *dst = bnd_row(P.bnd, P.rpitch, P.nch, P.c, mat, x, r, src);
+            const int64_t mis = static_cast<int64_t>((16 - (reinterpret_cast<uintptr_t>(src) & 15)) & 15);
+            const int64_t head = pitch < mis ? pitch : mis;
+            const int64_t body = (pitch - head) & ~int64_t(15);
+            for (int64_t kk = threadIdx.x; kk < body / 16; kk += blockDim.x)
+                stg16(dst + head + 16 * kk, ldg16(src + head + 16 * kk));
+            if (threadIdx.x < head / 4)
+                reinterpret_cast<uint32_t *>(dst)[threadIdx.x] = reinterpret_cast<const uint32_t *>(src)[threadIdx.x];
+            const int64_t t0 = head + body;
+            if (threadIdx.x < (pitch - t0) / 4)
+                reinterpret_cast<uint32_t *>(dst + t0)[threadIdx.x] = reinterpret_cast<const uint32_t *>(src + t0)[threadIdx.x];
+        }
+    }
+}
+
+template <int EB, int DIR, int NBUF, int NW>
+cudaError_t launch_row_chunk_t(const RowParams &P, cudaStream_t st) {
+    const size_t smem = NBUF * P.R * row_fused_smem_bytes(P, EB, DIR);
+    auto kern = row_chunk_kernel<EB, DIR, NBUF, NW>;
+    cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
+    if (e != cudaSuccess) return e;
+    const int threads = NW * 32 + 32;
+    const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), threads, smem);
+    if (resident < 1) return cudaErrorInvalidConfiguration;
+    if (!P.bnd) return cudaErrorInvalidValue;
+    const int64_t chunks = static_cast<int64_t>(P.nch) * P.batch;
+    int64_t grid = resident;
+    if (grid > chunks) grid = chunks;
+    kern<<<static_cast<unsigned>(grid), threads, smem, st>>>(P);
+    return cudaGetLastError();
+}
+
+template <int EB, int DIR, int NBUF>
+cudaError_t launch_row_chunk_n(const RowParams &P, cudaStream_t st) {
+    return row_threads(P.N, EB) == 512 ? launch_row_chunk_t<EB, DIR, NBUF, 16>(P, st)
+                                       : launch_row_chunk_t<EB, DIR, NBUF, 8>(P, st);
+}
+
 template <int EB, int DIR, bool FUSE, int NBUF, int NW>
 cudaError_t launch_row_pipe_t(const RowParams &P, cudaStream_t st) {
     const size_t rowbuf = FUSE ? row_fused_smem_bytes(P, EB, DIR) : row_smem_bytes(P.N, EB);
@@ -1263,6 +1482,10 @@ cudaError_t launch_row_rot_t(const RowParams &P, cudaStream_t st) {
 
 template <int EB, int DIR>
 cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
+    if (P.fuse && P.chunk)
+        return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max)
+                   ? launch_row_chunk_n<EB, DIR, 2>(P, st)
+                   : launch_row_chunk_n<EB, DIR, 1>(P, st);
     if (P.pipe) {
         // Fused rotation: row_rot_kernel stays the default (the pipelined variant measured
         // 0.89x of it on the fused sweep shapes, tools/ab_calls.py r02f); IPT_ROW_PIPE=2
@@ -1292,6 +1515,14 @@ cudaError_t launch_copy_wrap(const RowParams &P, int eb, cudaStream_t st) {
     const unsigned gx = static_cast<unsigned>(std::min<int64_t>(chunks, 64));
     const unsigned gy = static_cast<unsigned>(std::min<int64_t>(P.batch, 65535));
     copy_wrap_kernel<<<dim3(gx, gy), 256, 0, st>>>(P.base, P.mat_stride_bytes, P.batch, P.wrap, P.wstride, bytes);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_copy_bounds(const RowParams &P, int eb, cudaStream_t st) {
+    const int64_t slots = static_cast<int64_t>(P.nch) * P.batch;
+    if (P.c <= 1 || slots <= 0) return cudaSuccess;
+    const unsigned grid = static_cast<unsigned>(std::min<int64_t>(slots, 4096));
+    copy_bounds_kernel<<<grid, 256, 0, st>>>(P, static_cast<int64_t>(P.N) * eb);
     return cudaGetLastError();
 }
 
