@@ -419,9 +419,20 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     // Chunked fused pass (row_chunk_kernel; IPT_ROW_CHUNK=0 keeps the flag-based
     // row_rot_kernel): chunks of cK = max(R, IPT_ROW_CHUNK_K (c-1)) rows, so the boundary copy
     // costs 2 (c-1) / cK of a pass.
-    if (rp.fuse && env_int("IPT_ROW_CHUNK", 1) != 0) {
-        int64_t K = std::max<int64_t>(rp.R, static_cast<int64_t>(env_int("IPT_ROW_CHUNK_K", 16)) * (pl.c - 1));
-        K = (K + rp.R - 1) / rp.R * rp.R;
+    // Used where it measured faster than row_rot_kernel (tools/ab_calls.py, r02j): both row
+    // buffers fit (double buffering), the boundary traffic is <= 25 % of a pass (cK >= 8 (c-1)),
+    // and there are >= 2 chunks per SM in a single-matrix call (small c).
+    const int64_t ckmul = env_int("IPT_ROW_CHUNK_K", 16);
+    const size_t fbuf = rp.fuse ? row_fused_smem_bytes(rp, eb, pl.row_dir) : 0;
+    const int64_t par_rows = (pl.M + 8 * dev.sms - 1) / (8 * dev.sms);  // ~8 chunks per SM
+    int64_t K = std::max<int64_t>({static_cast<int64_t>(rp.R), 8 * (pl.c - 1),
+                                   std::min<int64_t>(ckmul * (pl.c - 1), par_rows)});
+    K = (K + rp.R - 1) / rp.R * rp.R;
+    const int chunk_env = env_int("IPT_ROW_CHUNK", -1);  // -1 auto, 0 off, 1 force
+    const bool chunk_ok = 2 * rp.R * fbuf <= static_cast<size_t>(env_int("IPT_ROW_DB_MAX", 112 * 1024)) &&
+                          (pl.M + K - 1) / K >= 2 * dev.sms;
+    if (rp.fuse && (chunk_env == 1 || (chunk_env == -1 && chunk_ok))) {
+        if (chunk_env == 1) K = std::max<int64_t>(rp.R, ckmul * (pl.c - 1)) + rp.R - 1, K = K / rp.R * rp.R;
         const int64_t Mr = (pl.M + rp.R - 1) / rp.R * rp.R;
         if (K > Mr) K = Mr;
         rp.chunk = 1;
