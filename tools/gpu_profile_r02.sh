@@ -16,7 +16,10 @@ ncu)
   timeout 600 $NCU -k regex:row_pipe -c 1 -s 2 -o $REP/rowpipe_$TAG \
       python tools/one_shape.py --m 14414 --n 6565 --eb 4 --reps 3 > gpurun_out/ncu_rowpipe_$TAG.log 2>&1
   timeout 600 $NCU -k regex:row_rot -c 1 -s 2 -o $REP/rowrot_$TAG \
-      python tools/one_shape.py --m 17226 --n 6052 --eb 4 --reps 3 > gpurun_out/ncu_rowrot_$TAG.log 2>&1
+      python tools/one_shape.py --m 13497 --n 16245 --eb 8 --reps 3 > gpurun_out/ncu_rowrot_$TAG.log 2>&1
+  # chunked fused pass (gcd 2, rows of 24 KB)
+  timeout 600 $NCU -k regex:row_chunk -c 1 -s 2 -o $REP/rowchunk_$TAG \
+      python tools/one_shape.py --m 17226 --n 6052 --eb 4 --reps 3 > gpurun_out/ncu_rowchunk_$TAG.log 2>&1
   # separate rotation pass at HBM scale (gcd 6600): col_tile_kernel<4,0,128> is COL_ROT
   timeout 600 $NCU -k regex:col_tile_kernel -c 1 -s 2 -o $REP/colrot_$TAG \
       python tools/one_shape.py --m 19800 --n 13200 --eb 4 --reps 2 > gpurun_out/ncu_colrot_$TAG.log 2>&1
