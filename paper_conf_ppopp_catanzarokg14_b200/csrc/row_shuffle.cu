@@ -924,10 +924,8 @@ cudaError_t row_cluster_dispatch(const RowParams &P, int dir, int eb, cudaStream
 // (one per producer lane, each deferred until that lane's small copies landed) + the bulk
 // bytes; empty[b]: one arrival per consumer warp once it no longer reads the buffer.  No
 // CTA-wide barrier on the data path: warps run ahead / behind independently.  Same shared-
-// memory layouts as the kernels above, so the gathers (gather_row, gather_row_rot*) are
-// shared.  Fused rotation (FUSE): the producer takes row groups by ticket (row_rot_kernel's
-// order and progress argument) and sets a group's "read" flags as soon as its data have
-// landed -- not after the CTA's previous gather -- so the neighbours' waits are short.
+// memory layout as row_shuffle_kernel, so the gather (gather_row) is shared; the chunked
+// fused pass below uses the same structure.
 __device__ __forceinline__ void pmbar_init(uint32_t bar, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(bar), "r"(count) : "memory");
 }
@@ -944,12 +942,6 @@ __device__ __forceinline__ void pmbar_wait(uint32_t bar, uint32_t parity) {
     asm volatile("{\n .reg .pred p;\n WAIT_%=:\n"
                  " mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%0], %1;\n"
                  " @!p bra WAIT_%=;\n}" :: "r"(bar), "r"(parity) : "memory");
-}
-__device__ __forceinline__ bool pmbar_test(uint32_t bar, uint32_t parity) {
-    uint32_t ok;
-    asm volatile("{\n .reg .pred p;\n mbarrier.test_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n"
-                 " selp.u32 %0, 1, 0, p;\n}" : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
-    return ok != 0;
 }
 __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
@@ -979,21 +971,17 @@ __device__ __forceinline__ void stage_part(const char *gs, int32_t nb, uint32_t 
     }
 }
 
-template <int EB, int DIR, bool FUSE, int NBUF, int NW>
+template <int EB, int DIR, int NBUF, int NW>
 __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kernel(RowParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ __align__(8) uint64_t bar_full[NBUF], bar_empty[NBUF];
-    __shared__ uint32_t s_group[NBUF];
     const int64_t pitch = static_cast<int64_t>(P.N) * EB;
-    const uint32_t rowbuf = FUSE ? static_cast<uint32_t>(row_fused_smem_bytes(P, EB, DIR))
-                                 : static_cast<uint32_t>((static_cast<uint32_t>(P.N) * EB + 31) & ~15u);
+    const uint32_t rowbuf = static_cast<uint32_t>((static_cast<uint32_t>(P.N) * EB + 31) & ~15u);
     const uint32_t bufbytes = rowbuf * static_cast<uint32_t>(P.R);
-    const uint32_t padoff = static_cast<uint32_t>(P.c) * static_cast<uint32_t>(P.segp);  // C2R pad table
     const uint32_t sbase = smem_u32(smem);
     const int32_t gpm = (P.M + P.R - 1) / P.R;
     const uint32_t groups_total = static_cast<uint32_t>(gpm) * static_cast<uint32_t>(P.batch);  // < 2^32 (planner)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t kDone = 0xffffffffu;
     if (threadIdx.x == 0) {
         for (int b = 0; b < NBUF; ++b) {
             pmbar_init(smem_u32(&bar_full[b]), 33);
@@ -1002,135 +990,42 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
-    auto group_of = [&](uint32_t t) {
-        const uint32_t mat = fdiv(t, P.fd_gpm);
-        uint32_t gm = t - mat * static_cast<uint32_t>(gpm);
-        if (FUSE && DIR == ROW_R2C) gm = static_cast<uint32_t>(gpm) - 1 - gm;
-        RowGroup G;
-        G.mat = mat;
-        G.i0 = static_cast<int32_t>(gm) * P.R;
-        G.nr = min(P.R, P.M - G.i0);
-        return G;
-    };
+    // Row groups in grid-stride order: CTA blockIdx.x takes groups blockIdx.x + k gridDim.x
+    // (producer and consumers walk the same sequence).
     auto mat_base = [&](const RowGroup &G) { return P.base + G.mat * P.mat_stride_bytes; };
 
     if (warp == NW) {
         // ================================ producer ================================
-        // FUSE: a group's flags are set as soon as its data have landed: while the
-        // producer waits for a free buffer it polls the landings of the groups it issued
-        // (at most NBUF pending).  Progress: every wait of this CTA (free buffers, landings)
-        // depends only on groups with smaller tickets (row_rot_kernel's induction).
-        auto set_flags = [&](uint32_t t) {
-            const RowGroup G = group_of(t);
-            if (lane < G.nr)
-                asm volatile("st.relaxed.gpu.global.u32 [%0], %1;"
-                             :: "l"(P.flags + G.mat * P.M + G.i0 + lane), "r"(1u) : "memory");
-        };
-        uint32_t pend_t[NBUF + 1], pend_k[NBUF + 1];  // issued, not yet flagged (oldest first)
-        int npend = 0;
-        auto poll = [&](bool block) {  // flag the landed pending groups (block: all of them)
-            while (npend > 0) {
-                const uint32_t fb0 = smem_u32(&bar_full[pend_k[0] % NBUF]);
-                // every lane observes the phase itself (acquire), the warp agrees on the result
-                bool ok = block ? (pmbar_wait(fb0, (pend_k[0] / NBUF) & 1), true)
-                                : pmbar_test(fb0, (pend_k[0] / NBUF) & 1);
-                if (!__all_sync(0xffffffffu, ok)) {
-                    if (block) continue;
-                    return;
-                }
-                set_flags(pend_t[0]);
-                for (int q = 1; q < npend; ++q) {
-                    pend_t[q - 1] = pend_t[q];
-                    pend_k[q - 1] = pend_k[q];
-                }
-                --npend;
-            }
-        };
-        uint32_t tk = blockIdx.x;  // non-fused: grid-stride order
-        for (uint32_t k = 0;; ++k) {
+        uint32_t t = blockIdx.x;
+        for (uint32_t k = 0; t < groups_total; ++k, t += gridDim.x) {
             const int b = static_cast<int>(k % NBUF);
             const uint32_t fb = smem_u32(&bar_full[b]);
-            if (k >= NBUF) {
-                const uint32_t eb_ = smem_u32(&bar_empty[b]), ep = ((k / NBUF) - 1) & 1;
-                if (FUSE) {
-                    while (true) {
-                        poll(false);
-                        const bool ok = pmbar_test(eb_, ep);  // per lane: acquire
-                        if (__all_sync(0xffffffffu, ok)) break;
-                        if (ok) pmbar_wait(eb_, ep);  // (a phase once complete stays complete)
-                        __nanosleep(20);
-                    }
-                    poll(false);  // group k - NBUF has landed (its consumers are done)
+            if (k >= NBUF) pmbar_wait(smem_u32(&bar_empty[b]), ((k / NBUF) - 1) & 1);
+            const RowGroup G = row_group(P, t, gpm);
+            char *mb = mat_base(G);
+            const uint32_t sb0 = sbase + b * bufbytes;
+            // whole rows; lagged R2C rows in two parts (side row, row), both at the row's alignment
+            const int parts = (DIR == ROW_R2C && P.shW) ? 2 : 1;
+            for (int32_t pi = lane; pi < G.nr * parts; pi += 32) {
+                const int32_t rr = pi / parts, part = pi - rr * parts;
+                const int32_t i = G.i0 + rr;
+                const char *row = mb + i * pitch;
+                const uint32_t reg = sb0 + rr * rowbuf;
+                if (parts == 1) {
+                    stage_part(row, P.N * EB, reg, fb);
+                } else if (part == 0) {
+                    stage_part(side_matrix(P.side, P.sstride, G.mat, mb) + i * P.spitch, P.shW * EB, reg, fb);
                 } else {
-                    pmbar_wait(eb_, ep);
-                }
-            }
-            // fused: the ticket is taken only now, when its group is staged at once (a ticket
-            // held while the CTA waits for a buffer would stall the groups after it)
-            uint32_t t = tk;
-            if (FUSE) {
-                if (lane == 0) t = atomicAdd(P.ticket, 1u);
-                t = __shfl_sync(0xffffffffu, t, 0);
-            } else {
-                tk += gridDim.x;
-            }
-            const bool done = t >= groups_total;
-            if (lane == 0) s_group[b] = done ? kDone : t;
-            if (!done) {
-                const RowGroup G = group_of(t);
-                char *mb = mat_base(G);
-                const uint32_t sb0 = sbase + b * bufbytes;
-                if (FUSE && DIR == ROW_C2R) {
-                    // staircase: segment rho of row i = source columns [rho b, rho b + b) of
-                    // row i + rho (rows past M - 1 from the wrap copy), each in its own
-                    // 16-byte-aligned region; padl[rho] maps a source index to its byte
-                    const int32_t Lb = P.b * EB;
-                    char *wb = wrap_matrix(P.wrap, P.wstride, G.mat, mb);
-                    for (int32_t pi = lane; pi < G.nr * P.c; pi += 32) {
-                        const int32_t rr = pi / P.c, rho = pi - rr * P.c;
-                        const int32_t y = G.i0 + rr + rho;
-                        const char *S = (y < P.M ? mb + y * pitch : wb + (y - P.M) * pitch) + static_cast<int64_t>(rho) * Lb;
-                        const uint32_t reg = sb0 + rr * rowbuf + rho * P.segp;
-                        int32_t *padl = reinterpret_cast<int32_t *>(smem + b * bufbytes + rr * rowbuf + padoff);
-                        padl[rho] = rho * P.segp + static_cast<int32_t>(reinterpret_cast<uintptr_t>(S) & 15) - rho * Lb;
-                        stage_part(S, Lb, reg, fb);
-                    }
-                } else {
-                    // whole rows (R2C fused: rows 0..c-2 from the wrap copy); lagged R2C rows
-                    // in two parts (side row, row), both at the row's alignment
-                    const int parts = (DIR == ROW_R2C && P.shW) ? 2 : 1;
-                    for (int32_t pi = lane; pi < G.nr * parts; pi += 32) {
-                        const int32_t rr = pi / parts, part = pi - rr * parts;
-                        const int32_t i = G.i0 + rr;
-                        const char *row = (FUSE && DIR == ROW_R2C && i < P.c - 1)
-                                              ? wrap_matrix(P.wrap, P.wstride, G.mat, mb) + i * pitch
-                                              : mb + i * pitch;
-                        const uint32_t reg = sb0 + rr * rowbuf;
-                        if (parts == 1) {
-                            stage_part(row, P.N * EB, reg, fb);
-                        } else if (part == 0) {
-                            stage_part(side_matrix(P.side, P.sstride, G.mat, mb) + i * P.spitch, P.shW * EB, reg, fb);
-                        } else {
-                            stage_part(row, (P.N - P.shW) * EB, reg + P.shW * EB, fb);
-                        }
-                    }
+                    stage_part(row, (P.N - P.shW) * EB, reg + P.shW * EB, fb);
                 }
             }
             __syncwarp();
-            if (lane == 0) pmbar_arrive(fb);  // publishes s_group[b] and the pad tables
+            if (lane == 0) pmbar_arrive(fb);
             pmbar_arrive_cpasync(fb);
-            if (FUSE) {
-                // the group's reads are complete once its data have landed: flag its rows
-                // (relaxed: the reads are done, the flag orders nothing else; row_rot_kernel)
-                if (!done) {
-                    pend_t[npend] = t;
-                    pend_k[npend] = k;
-                    ++npend;
-                }
-                poll(done || NBUF == 1);
-            } else if (NBUF == 1 && tk < groups_total && lane == 0) {
+            const uint32_t tn = t + gridDim.x;
+            if (NBUF == 1 && tn < groups_total && lane == 0) {
                 // single buffer: the next group's rows stream into L2 while this one is gathered
-                const RowGroup NG = group_of(tk);
+                const RowGroup NG = row_group(P, tn, gpm);
                 const char *a = mat_base(NG) + NG.i0 * pitch;
                 const uintptr_t a0 = (reinterpret_cast<uintptr_t>(a) + 15) & ~uintptr_t(15);
                 const uintptr_t a1 = (reinterpret_cast<uintptr_t>(a) + NG.nr * pitch) & ~uintptr_t(15);
@@ -1139,7 +1034,6 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
                     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(x), "r"(sz) : "memory");
                 }
             }
-            if (done) break;
         }
         return;
     }
@@ -1149,55 +1043,20 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
     const int team = warp / wn, wl = warp - team * wn;
     const int32_t seg = ((P.N + wn - 1) / wn + 31) & ~31;
     const int32_t p_begin = wl * seg, p_end = min(P.N, p_begin + seg);
-    const int64_t vD = static_cast<int64_t>(wn) * 32 * (16 / EB);
-    const int32_t vdl = FUSE ? static_cast<int32_t>(vD % P.c) : 0;
-    const int32_t vdh = FUSE ? static_cast<int32_t>((static_cast<int64_t>(P.ainv) * ((vD / P.c) % P.b)) % P.b) : 0;
-    for (uint32_t k = 0;; ++k) {
+    uint32_t t = blockIdx.x;
+    for (uint32_t k = 0; t < groups_total; ++k, t += gridDim.x) {
         const int b = static_cast<int>(k % NBUF);
         pmbar_wait(smem_u32(&bar_full[b]), (k / NBUF) & 1);
-        const uint32_t t = s_group[b];
-        if (t == kDone) break;
-        const RowGroup G = group_of(t);
+        const RowGroup G = row_group(P, t, gpm);
         char *mbase = mat_base(G);
-        if (FUSE) {
-            // every row this group overwrites has been read (flags of smaller tickets)
-            if (lane >= 1 && lane < P.c) {
-                const int32_t y = DIR == ROW_C2R ? G.i0 - lane : G.i0 + G.nr - 1 + lane;
-                if (y >= 0 && y < P.M) {
-                    const unsigned int *f = P.flags + G.mat * P.M + y;
-                    unsigned int v;
-                    while (true) {
-                        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
-                        if (v) break;
-                        __nanosleep(32);
-                    }
-                }
-            }
-            __syncwarp();
-        }
         if (team < G.nr) {
             const int32_t i = G.i0 + team;
             const unsigned char *buf = smem + b * bufbytes + team * rowbuf;
-            if (!FUSE) {
-                char *row = mbase + i * pitch;
-                const unsigned char *st = buf + (reinterpret_cast<uintptr_t>(row) & 15);
-                char *srow = P.shW ? side_matrix(P.side, P.sstride, G.mat, mbase) + i * P.spitch : nullptr;
-                if (i >= P.M - P.c + 1) gather_row<EB, DIR, true>(P, row, srow, st, i, p_begin, p_end);
-                else gather_row<EB, DIR, false>(P, row, srow, st, i, p_begin, p_end);
-            } else {
-                char *srow = P.shW ? side_matrix(P.side, P.sstride, G.mat, mbase) + i * P.spitch : nullptr;
-                if (DIR == ROW_C2R) {
-                    if (P.vec && i < P.M - P.c + 1)
-                        gather_row_rot_c2r_vec<EB>(P, mbase, srow, buf, reinterpret_cast<const int32_t *>(buf + padoff), i,
-                                                   wl * 32 + lane, wn * 32, vdl, vdh);
-                    else
-                        gather_row_rot<EB, DIR>(P, mbase, srow, buf, reinterpret_cast<const int32_t *>(buf + padoff), i,
-                                                p_begin, p_end);
-                } else {
-                    gather_row_rot<EB, DIR>(P, mbase, srow, buf + (reinterpret_cast<uintptr_t>(mbase + i * pitch) & 15),
-                                            nullptr, i, p_begin, p_end);
-                }
-            }
+            char *row = mbase + i * pitch;
+            const unsigned char *st = buf + (reinterpret_cast<uintptr_t>(row) & 15);
+            char *srow = P.shW ? side_matrix(P.side, P.sstride, G.mat, mbase) + i * P.spitch : nullptr;
+            if (i >= P.M - P.c + 1) gather_row<EB, DIR, true>(P, row, srow, st, i, p_begin, p_end);
+            else gather_row<EB, DIR, false>(P, row, srow, st, i, p_begin, p_end);
         }
         __syncwarp();
         if (lane == 0) pmbar_arrive(smem_u32(&bar_empty[b]));
@@ -1205,7 +1064,7 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
 }
 
 // ---- Chunked fused rotation + row pass (default for 1 < c <= kMaxFuseC) ---------------
-// Same producer / consumer structure and staging as row_pipe_kernel<FUSE>, but the work unit
+// Same producer / consumer structure and staging as row_pipe_kernel, but the work unit
 // is a CHUNK of cK consecutive rows of one matrix, whose row groups a CTA processes in order:
 //  * C2R (Eq. 23 then Eq. 31): writing row i overwrites segments that only the staircases of
 //    rows i-c+1 .. i read; those of the same chunk were staged (landed) before row i's group
@@ -1423,17 +1282,15 @@ cudaError_t launch_row_chunk_n(const RowParams &P, cudaStream_t st) {
                                        : launch_row_chunk_t<EB, DIR, NBUF, 8>(P, st);
 }
 
-template <int EB, int DIR, bool FUSE, int NBUF, int NW>
+template <int EB, int DIR, int NBUF, int NW>
 cudaError_t launch_row_pipe_t(const RowParams &P, cudaStream_t st) {
-    const size_t rowbuf = FUSE ? row_fused_smem_bytes(P, EB, DIR) : row_smem_bytes(P.N, EB);
-    const size_t smem = NBUF * P.R * rowbuf;
-    auto kern = row_pipe_kernel<EB, DIR, FUSE, NBUF, NW>;
+    const size_t smem = NBUF * P.R * row_smem_bytes(P.N, EB);
+    auto kern = row_pipe_kernel<EB, DIR, NBUF, NW>;
     cudaError_t e = ensure_kernel_attrs(reinterpret_cast<const void *>(kern), smem, false);
     if (e != cudaSuccess) return e;
     const int threads = NW * 32 + 32;
     const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), threads, smem);
     if (resident < 1) return cudaErrorInvalidConfiguration;
-    if (FUSE && (!P.ticket || !P.flags || !P.wrap)) return cudaErrorInvalidValue;
     const int64_t groups = static_cast<int64_t>((P.M + P.R - 1) / P.R) * P.batch;
     int64_t grid = resident;
     if (grid > groups) grid = groups;
@@ -1441,10 +1298,10 @@ cudaError_t launch_row_pipe_t(const RowParams &P, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-template <int EB, int DIR, bool FUSE, int NBUF>
+template <int EB, int DIR, int NBUF>
 cudaError_t launch_row_pipe_n(const RowParams &P, cudaStream_t st) {
-    return row_threads(P.N, EB) == 512 ? launch_row_pipe_t<EB, DIR, FUSE, NBUF, 16>(P, st)
-                                       : launch_row_pipe_t<EB, DIR, FUSE, NBUF, 8>(P, st);
+    return row_threads(P.N, EB) == 512 ? launch_row_pipe_t<EB, DIR, NBUF, 16>(P, st)
+                                       : launch_row_pipe_t<EB, DIR, NBUF, 8>(P, st);
 }
 
 template <int EB, int DIR, int NBUF>
@@ -1486,17 +1343,10 @@ cudaError_t launch_row_d(const RowParams &P, cudaStream_t st) {
         return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max)
                    ? launch_row_chunk_n<EB, DIR, 2>(P, st)
                    : launch_row_chunk_n<EB, DIR, 1>(P, st);
-    if (P.pipe) {
-        // Fused rotation: row_rot_kernel stays the default (the pipelined variant measured
-        // 0.89x of it on the fused sweep shapes, tools/ab_calls.py r02f); IPT_ROW_PIPE=2
-        // selects the pipelined one where two buffers fit.
-        if (P.fuse && P.pipe == 2 && 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max))
-            return launch_row_pipe_n<EB, DIR, true, 2>(P, st);
-        if (!P.fuse)
-            return 2 * P.R * row_smem_bytes(P.N, EB) <= static_cast<size_t>(P.db_max)
-                       ? launch_row_pipe_n<EB, DIR, false, 2>(P, st)
-                       : launch_row_pipe_n<EB, DIR, false, 1>(P, st);
-    }
+    if (P.pipe && !P.fuse)
+        return 2 * P.R * row_smem_bytes(P.N, EB) <= static_cast<size_t>(P.db_max)
+                   ? launch_row_pipe_n<EB, DIR, 2>(P, st)
+                   : launch_row_pipe_n<EB, DIR, 1>(P, st);
     if (P.fuse)
         return 2 * P.R * row_fused_smem_bytes(P, EB, DIR) <= static_cast<size_t>(P.db_max)
                    ? launch_row_rot_t<EB, DIR, 2>(P, st)

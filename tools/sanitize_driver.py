@@ -41,11 +41,14 @@ def main():
         roundtrip(301, 517, 4, f"gcd1 {eng}")
         roundtrip(517, 301, 8, f"gcd1 {eng}")
         roundtrip(97, 64, 16, f"gcd1 {eng}")
-        # fused rotation (row_rot_kernel) and its pipelined variant
-        roundtrip(2 * 301, 2 * 517, 4, f"fused {eng}")
-        env(IPT_ROW_PIPE=2)
-        roundtrip(6 * 101, 6 * 77, 8, f"fused pipe {eng}")
-        env(IPT_ROW_PIPE=None)
+        # fused rotation: chunked pass (auto for small c) and the flag-based row_rot_kernel
+        env(IPT_ROW_CHUNK=1)
+        roundtrip(2 * 301, 2 * 517, 4, f"fused chunked {eng}")
+        roundtrip(6 * 101, 6 * 77, 8, f"fused chunked {eng}")
+        env(IPT_ROW_CHUNK=0)
+        roundtrip(2 * 301, 2 * 517, 4, f"fused flags {eng}")
+        roundtrip(6 * 101, 6 * 77, 8, f"fused flags {eng}")
+        env(IPT_ROW_CHUNK=None)
         # legacy row kernel
         env(IPT_ROW_PIPE=0)
         roundtrip(301, 517, 4, f"row legacy {eng}")
