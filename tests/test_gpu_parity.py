@@ -680,3 +680,68 @@ def test_concurrent_calls_from_threads_share_no_counters():
     assert not errors, errors
     for (m, n, eb), x, h in zip(shapes, xs, hosts):
         assert dev_bytes(x) == oracle.transpose(vwords(h, eb), m, n).tobytes(), (m, n, eb)
+
+
+@pytest.mark.parametrize("ck", ["0", "1", "16"])
+def test_chunked_fused_pass_forced(ck):
+    """Chunked fused rotation + row pass (row_chunk_kernel) forced on every fused shape
+    (IPT_ROW_CHUNK=1), chunk length cK = max(R, IPT_ROW_CHUNK_K (c-1)) rows: 0 gives chunks of
+    one row group, shorter than c - 1 (staircases and R2C blocks then span several chunks'
+    boundary copies), 1 the minimum c - 1, 16 the default.  gcd 2..32, both engines, every
+    element size, misaligned rows, lagged and unlagged column layouts, row groups, a gapped
+    batch -- all compared in full with the oracle."""
+    shapes = [(1200, 1816), (1816, 1200), (96, 40), (40, 96), (640, 32 * 33), (2 * 1009, 2 * 1013), (30 * 37, 30 * 41),
+              (4 * 99, 4 * 25), (6 * 31, 6 * 77), (64, 48), (48, 64), (2 * 7, 2 * 5), (12, 18), (62, 64)]
+    with env_var("IPT_ROW_CHUNK", "1"), env_var("IPT_ROW_CHUNK_K", ck):
+        for lag in ("1", "0"):
+            with env_var("IPT_COL_LAG", lag):
+                for eb in (4, 8, 16):
+                    for engine in ("c2r", "r2c"):
+                        run_packed(shapes, eb, ipt.c2r, "row", engine, seed=eb * 11 + len(ck))
+        with env_var("IPT_ROW_STAGE", "200000"):
+            run_packed(shapes, 4, ipt.c2r, "row", None, seed=5)
+        m, n, batch = 2 * 150, 2 * 501, 3
+        host = workloads.random_words(1 + batch * (m * n + 7), 8, seed=91)
+        hv = vwords(host, 8)
+        x = to_dev(host)
+        ipt.c2r_batched(x.data_ptr() + 8, batch, m * n + 7, m, n, elem_bytes=8)
+        got = vwords(x.cpu().numpy(), 8)
+        for k in range(batch):
+            o = 1 + k * (m * n + 7)
+            assert got[o:o + m * n].tobytes() == oracle.ipt_c2r(hv[o:o + m * n], m, n).tobytes()
+        ipt.r2c_batched(x.data_ptr() + 8, batch, m * n + 7, m, n, elem_bytes=8)
+        assert dev_bytes(x) == np.ascontiguousarray(host).tobytes()
+
+
+def test_chunked_fused_pass_each_pass():
+    """Per-pass parity of the chunked fused pass against the oracle's gather-form snapshots
+    (C2R: [r_j + d'^{-1}] then p_j o q; R2C: q^{-1} o p^{-1} then [d' + r^{-1}])."""
+    for (m, n) in [(1200, 1816), (1816, 1200), (6 * 301, 6 * 77)]:
+        host = workloads.random_words(m * n, 4, seed=m ^ n)
+        with env_var("IPT_ROW_CHUNK", "1"):
+            for engine in ("c2r", "r2c"):
+                with forced_engine(engine):
+                    if engine == "c2r":
+                        _, snaps = oracle.c2r_gather_forms(host, m, n, snapshots=True)
+                    else:
+                        _, snaps = oracle.r2c_gather_forms(host, n, m, snapshots=True)
+                    for k, e in enumerate([snaps[1], snaps[3]], start=1):
+                        x = to_dev(host)
+                        with debug_passes(k):
+                            ipt.c2r(x, m, n, elem_bytes=4)
+                        assert dev_bytes(x) == e.tobytes(), (m, n, engine, k)
+
+
+@pytest.mark.parametrize("pipe", ["0", "1"])
+def test_row_pass_kernels_both(pipe):
+    """The pipelined row pass (bulk-copy producer warp, default) and the previous kernel
+    (IPT_ROW_PIPE=0) on gcd-1 and separate-rotation shapes: rows misaligned to 16 bytes, row
+    groups, lagged side rows, single- and double-buffered rows, tiny rows (< 16 bytes)."""
+    shapes = [(1031, 97), (97, 1031), (513, 700), (700, 513), (2003, 129), (129, 2003), (333, 4099), (5, 3), (3, 5),
+              (7, 2), (2, 7), (3000, 17011)]
+    with env_var("IPT_ROW_PIPE", pipe):
+        for eb in (4, 8, 16):
+            for engine in ("c2r", "r2c"):
+                run_packed(shapes, eb, ipt.c2r, "row", engine, seed=eb + 3 * len(pipe))
+        with env_var("IPT_FUSE_ROT", "0"):
+            run_packed([(1200, 1800), (640, 32 * 33)], 4, ipt.c2r, "row", None, seed=8)
