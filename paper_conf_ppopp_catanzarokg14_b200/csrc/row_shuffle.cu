@@ -920,9 +920,11 @@ cudaError_t row_cluster_dispatch(const RowParams &P, int dir, int eb, cudaStream
 // One PRODUCER warp stages row groups with TMA bulk copies (cp.async.bulk, one per row part:
 // the 16-byte-aligned interior; the at most 3 + 3 words of ragged head / tail with 4-byte
 // cp.async) into NBUF mbarrier-tracked buffers; NW CONSUMER warps gather and write the
-// rows.  full[b]: 1 arrival (lane 0, after publishing the group id) + 32 cp.async arrivals
-// (one per producer lane, each deferred until that lane's small copies landed) + the bulk
-// bytes; empty[b]: one arrival per consumer warp once it no longer reads the buffer.  No
+// rows.  full[b]: 32 arrivals (every producer lane, after its pad-table writes) + 32 cp.async
+// arrivals (one per producer lane, each deferred until that lane's small copies landed) +
+// the bulk bytes; empty[b]: one arrival per consumer thread once it no longer reads the
+// buffer, and the producer fences the generic proxy against the async one before it
+// refills a buffer.  Every thread orders its own accesses with its own arrive / wait.  No
 // CTA-wide barrier on the data path: warps run ahead / behind independently.  Same shared-
 // memory layout as row_shuffle_kernel, so the gather (gather_row) is shared; the chunked
 // fused pass below uses the same structure.
@@ -984,8 +986,8 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
         for (int b = 0; b < NBUF; ++b) {
-            pmbar_init(smem_u32(&bar_full[b]), 33);
-            pmbar_init(smem_u32(&bar_empty[b]), NW);
+            pmbar_init(smem_u32(&bar_full[b]), 64);
+            pmbar_init(smem_u32(&bar_empty[b]), NW * 32);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -1000,7 +1002,12 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
         for (uint32_t k = 0; t < groups_total; ++k, t += gridDim.x) {
             const int b = static_cast<int>(k % NBUF);
             const uint32_t fb = smem_u32(&bar_full[b]);
-            if (k >= NBUF) pmbar_wait(smem_u32(&bar_empty[b]), ((k / NBUF) - 1) & 1);
+            if (k >= NBUF) {
+                pmbar_wait(smem_u32(&bar_empty[b]), ((k / NBUF) - 1) & 1);
+                // the consumers' generic-proxy reads of this buffer before the bulk copies'
+                // async-proxy writes into it
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            }
             const RowGroup G = row_group(P, t, gpm);
             char *mb = mat_base(G);
             const uint32_t sb0 = sbase + b * bufbytes;
@@ -1020,7 +1027,7 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
                 }
             }
             __syncwarp();
-            if (lane == 0) pmbar_arrive(fb);
+            pmbar_arrive(fb);
             pmbar_arrive_cpasync(fb);
             const uint32_t tn = t + gridDim.x;
             if (NBUF == 1 && tn < groups_total && lane == 0) {
@@ -1058,8 +1065,7 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
             if (i >= P.M - P.c + 1) gather_row<EB, DIR, true>(P, row, srow, st, i, p_begin, p_end);
             else gather_row<EB, DIR, false>(P, row, srow, st, i, p_begin, p_end);
         }
-        __syncwarp();
-        if (lane == 0) pmbar_arrive(smem_u32(&bar_empty[b]));
+        pmbar_arrive(smem_u32(&bar_empty[b]));  // every lane: its reads of the buffer are done
     }
 }
 
@@ -1088,8 +1094,8 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_chunk_kern
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
         for (int b = 0; b < NBUF; ++b) {
-            pmbar_init(smem_u32(&bar_full[b]), 33);
-            pmbar_init(smem_u32(&bar_empty[b]), NW);
+            pmbar_init(smem_u32(&bar_full[b]), 64);
+            pmbar_init(smem_u32(&bar_empty[b]), NW * 32);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -1131,7 +1137,12 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_chunk_kern
         for (uint32_t k = 0; more; ++k) {
             const int b = static_cast<int>(k % NBUF);
             const uint32_t fb = smem_u32(&bar_full[b]);
-            if (k >= NBUF) pmbar_wait(smem_u32(&bar_empty[b]), ((k / NBUF) - 1) & 1);
+            if (k >= NBUF) {
+                pmbar_wait(smem_u32(&bar_empty[b]), ((k / NBUF) - 1) & 1);
+                // the consumers' generic-proxy reads of this buffer before the bulk copies'
+                // async-proxy writes into it
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            }
             const RowGroup G = group_of(q);
             char *mb = mat_base(G.mat);
             const uint32_t sb0 = sbase + b * bufbytes;
@@ -1177,7 +1188,7 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_chunk_kern
                 }
             }
             __syncwarp();
-            if (lane == 0) pmbar_arrive(fb);  // publishes the pad tables
+            pmbar_arrive(fb);  // publishes the pad tables
             pmbar_arrive_cpasync(fb);
             more = advance(q);
             if (NBUF == 1 && more && lane == 0) {
@@ -1226,8 +1237,7 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_chunk_kern
                                         nullptr, i, p_begin, p_end);
             }
         }
-        __syncwarp();
-        if (lane == 0) pmbar_arrive(smem_u32(&bar_empty[b]));
+        pmbar_arrive(smem_u32(&bar_empty[b]));  // every lane: its reads of the buffer are done
         more = advance(q);
     }
 }

@@ -206,52 +206,6 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
         }
         asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
         __syncthreads();
-        // Fast path: every column of the block has the same floor(j/b) (always when c = 1),
-        // so each output row's base pointer and the rotation are block constants; a thread
-        // walks its columns x, x + blockDim, ... with j mod n stepped incrementally.
-        const int32_t qd0 = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b));
-        const bool uniform = qd0 == static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + cols - 1), P.fd_b));
-        if (uniform) {
-            const int32_t dstep = static_cast<int32_t>(blockDim.x % static_cast<uint32_t>(n));
-            const int32_t jm0 = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j0 + threadIdx.x), P.fd_n));
-            int32_t shift = 0;
-            if (MODE == COL_ROT) shift = P.rot_sign > 0 ? qd0 : (qd0 == 0 ? 0 : n - qd0);
-            for (int i = 0; i < n; ++i) {
-                T *orow = P.remap > 0 ? (i == n - 1 ? tmp : A + (i + 1) * pitch) : A + i * pitch;
-                if (FOLD && P.remap > 0 && i < n - 1) {
-                    int32_t L = i + 1 + qd0;
-                    L -= L >= n ? n : 0;
-                    orow = A + L * pitch;
-                }
-                orow += j0;
-                const int32_t qi = MODE == COL_C2R_SHUF ? P.q[i] : 0;
-                int32_t rs = i + shift;  // COL_ROT: the source row is the same for the whole block
-                rs -= rs >= n ? n : 0;
-                const T *brow = buf + rs * C;
-                int32_t jm = jm0;
-#pragma unroll 4
-                for (int32_t x = threadIdx.x; x < cols; x += blockDim.x) {
-                    int32_t sr;
-                    if (MODE == COL_ROT) {
-                        orow[x] = brow[x];
-                    } else {
-                        if (MODE == COL_C2R_SHUF) {
-                            sr = jm + qi;
-                            sr -= sr >= n ? n : 0;
-                        } else {
-                            int32_t u = i - jm;
-                            u += u < 0 ? n : 0;
-                            sr = qinv_s[u];
-                        }
-                        orow[x] = buf[sr * C + x];
-                    }
-                    jm += dstep;
-                    jm -= jm >= n ? n : 0;
-                }
-            }
-            __syncthreads();  // the buffer is refilled by the next column block
-            continue;
-        }
         for (int32_t x = threadIdx.x; x < cols; x += blockDim.x) {
             const int64_t j = j0 + x;  // < N < 2^31
             const uint32_t jm = fmod_(static_cast<uint32_t>(j), P.fd_n);
