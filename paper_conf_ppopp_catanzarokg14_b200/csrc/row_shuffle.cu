@@ -920,9 +920,9 @@ cudaError_t row_cluster_dispatch(const RowParams &P, int dir, int eb, cudaStream
 // One PRODUCER warp stages row groups with TMA bulk copies (cp.async.bulk, one per row part:
 // the 16-byte-aligned interior; the at most 3 + 3 words of ragged head / tail with 4-byte
 // cp.async) into NBUF mbarrier-tracked buffers; NW CONSUMER warps gather and write the
-// rows.  full[b]: 32 arrivals (every producer lane, after its pad-table writes) + 32 cp.async
-// arrivals (one per producer lane, each deferred until that lane's small copies landed) +
-// the bulk bytes; empty[b]: one arrival per consumer thread once it no longer reads the
+// rows.  full[b]: 32 arrivals (every producer lane, once its small copies have landed and its
+// pad-table entries are written) + the bulk bytes; empty[b]: one arrival per consumer
+// thread once it no longer reads the
 // buffer, and the producer fences the generic proxy against the async one before it
 // refills a buffer.  Every thread orders its own accesses with its own arrive / wait.  No
 // CTA-wide barrier on the data path: warps run ahead / behind independently.  Same shared-
@@ -936,9 +936,6 @@ __device__ __forceinline__ void pmbar_expect_tx(uint32_t bar, uint32_t bytes) {
 }
 __device__ __forceinline__ void pmbar_arrive(uint32_t bar) {
     asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" :: "r"(bar) : "memory");
-}
-__device__ __forceinline__ void pmbar_arrive_cpasync(uint32_t bar) {
-    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" :: "r"(bar) : "memory");
 }
 __device__ __forceinline__ void pmbar_wait(uint32_t bar, uint32_t parity) {
     asm volatile("{\n .reg .pred p;\n WAIT_%=:\n"
@@ -986,7 +983,7 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
         for (int b = 0; b < NBUF; ++b) {
-            pmbar_init(smem_u32(&bar_full[b]), 64);
+            pmbar_init(smem_u32(&bar_full[b]), 32);
             pmbar_init(smem_u32(&bar_empty[b]), NW * 32);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -1027,8 +1024,9 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
                 }
             }
             __syncwarp();
+            // every lane: its small copies have landed and its pad-table entries are written
+            asm volatile("cp.async.wait_all;" ::: "memory");
             pmbar_arrive(fb);
-            pmbar_arrive_cpasync(fb);
             const uint32_t tn = t + gridDim.x;
             if (NBUF == 1 && tn < groups_total && lane == 0) {
                 // single buffer: the next group's rows stream into L2 while this one is gathered
@@ -1094,7 +1092,7 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_chunk_kern
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
         for (int b = 0; b < NBUF; ++b) {
-            pmbar_init(smem_u32(&bar_full[b]), 64);
+            pmbar_init(smem_u32(&bar_full[b]), 32);
             pmbar_init(smem_u32(&bar_empty[b]), NW * 32);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
