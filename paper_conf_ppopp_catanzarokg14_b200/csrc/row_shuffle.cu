@@ -1186,8 +1186,9 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_chunk_kern
                 }
             }
             __syncwarp();
-            pmbar_arrive(fb);  // publishes the pad tables
-            pmbar_arrive_cpasync(fb);
+            // every lane: its small copies have landed and its pad-table entries are written
+            asm volatile("cp.async.wait_all;" ::: "memory");
+            pmbar_arrive(fb);
             more = advance(q);
             if (NBUF == 1 && more && lane == 0) {
                 // single buffer: the next group's rows stream into L2 while this one is gathered
