@@ -99,6 +99,8 @@ struct Plan {
     size_t side_bytes = 0;      // lagged layouts: side block bytes per matrix (M x (D TWB + pad))
     SkinnyRowParams srow{};     // skinny engine long-row shuffle
     SkinnyColParams scol{}, srot{};  // skinny engine column passes (shuffle, rotation)
+    bool chunk_force = false;   // IPT_ROW_CHUNK=1
+    int sms = 0;
     int skinny_dir = 0;         // ROW_R2C (P_{count,n}, AoS -> SoA) or ROW_C2R (P_{n,count})
 };
 
@@ -237,6 +239,30 @@ void set_lag(Plan &pl, int64_t D) {
     rp.spitch = cq.spitch;
     rp.sstride = cq.sstride;
     pl.side_bytes = static_cast<size_t>(cq.sstride);
+}
+
+// Chunk geometry of the chunked fused pass for a call on `batch` matrices: cK =
+// max(R, 8 (c-1), min(IPT_ROW_CHUNK_K (c-1), ceil(M batch / (8 SMs)))) rows -- the boundary
+// traffic 2 (c-1) / cK stays <= 25 % of a pass, and about 8 chunks per SM when the call is
+// small -- rounded to whole row groups.  Returns whether the batch has >= 2 chunks per SM
+// (always true when forced by IPT_ROW_CHUNK=1, which also uses cK = max(R, IPT_ROW_CHUNK_K (c-1))).
+bool set_chunks(Plan &pl, int64_t batch) {
+    RowParams &rp = pl.row;
+    const int64_t ckmul = env_int("IPT_ROW_CHUNK_K", 16);
+    int64_t K;
+    if (pl.chunk_force) {
+        K = std::max<int64_t>(rp.R, ckmul * (pl.c - 1));
+    } else {
+        const int64_t par_rows = (pl.M * batch + 8 * pl.sms - 1) / (8 * static_cast<int64_t>(pl.sms));
+        K = std::max<int64_t>({static_cast<int64_t>(rp.R), 8 * (pl.c - 1), std::min<int64_t>(ckmul * (pl.c - 1), par_rows)});
+    }
+    K = (K + rp.R - 1) / rp.R * rp.R;
+    const int64_t Mr = (pl.M + rp.R - 1) / rp.R * rp.R;
+    if (K > Mr) K = Mr;
+    rp.cK = static_cast<int32_t>(K);
+    rp.nch = static_cast<int32_t>((pl.M + K - 1) / K);
+    rp.fd_nch = make_fastdiv(static_cast<uint32_t>(rp.nch));
+    return pl.chunk_force || static_cast<int64_t>(rp.nch) * batch >= 2 * static_cast<int64_t>(pl.sms);
 }
 
 // Skinny engine (§6.1): P_{x,y} with min(x, y) = n <= 32 fields
@@ -417,29 +443,19 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         rsm = rowbuf * rp.R;
     }
     // Chunked fused pass (row_chunk_kernel; IPT_ROW_CHUNK=0 keeps the flag-based
-    // row_rot_kernel): chunks of cK = max(R, IPT_ROW_CHUNK_K (c-1)) rows, so the boundary copy
-    // costs 2 (c-1) / cK of a pass.
+    // row_rot_kernel): chunks of cK rows, so the boundary copy costs 2 (c-1) / cK of a pass.
     // Used where it measured faster than row_rot_kernel (tools/ab_calls.py, r02j): both row
-    // buffers fit (double buffering), the boundary traffic is <= 25 % of a pass (cK >= 8 (c-1)),
-    // and there are >= 2 chunks per SM in a single-matrix call (small c).
-    const int64_t ckmul = env_int("IPT_ROW_CHUNK_K", 16);
-    const size_t fbuf = rp.fuse ? row_fused_smem_bytes(rp, eb, pl.row_dir) : 0;
-    const int64_t par_rows = (pl.M + 8 * dev.sms - 1) / (8 * dev.sms);  // ~8 chunks per SM
-    int64_t K = std::max<int64_t>({static_cast<int64_t>(rp.R), 8 * (pl.c - 1),
-                                   std::min<int64_t>(ckmul * (pl.c - 1), par_rows)});
-    K = (K + rp.R - 1) / rp.R * rp.R;
+    // buffers fit (double buffering); cK and the ">= 2 chunks per SM" condition depend on the
+    // batch and are settled by set_chunks() (prepare_call).
     const int chunk_env = env_int("IPT_ROW_CHUNK", -1);  // -1 auto, 0 off, 1 force
-    const bool chunk_ok = 2 * rp.R * fbuf <= static_cast<size_t>(env_int("IPT_ROW_DB_MAX", 112 * 1024)) &&
-                          (pl.M + K - 1) / K >= 2 * dev.sms;
+    const size_t fbuf = rp.fuse ? row_fused_smem_bytes(rp, eb, pl.row_dir) : 0;
+    const bool chunk_ok = 2 * rp.R * fbuf <= static_cast<size_t>(env_int("IPT_ROW_DB_MAX", 112 * 1024));
     if (rp.fuse && (chunk_env == 1 || (chunk_env == -1 && chunk_ok))) {
-        if (chunk_env == 1) K = std::max<int64_t>(rp.R, ckmul * (pl.c - 1)) + rp.R - 1, K = K / rp.R * rp.R;
-        const int64_t Mr = (pl.M + rp.R - 1) / rp.R * rp.R;
-        if (K > Mr) K = Mr;
         rp.chunk = 1;
-        rp.cK = static_cast<int32_t>(K);
-        rp.nch = static_cast<int32_t>((pl.M + K - 1) / K);
-        rp.fd_nch = make_fastdiv(static_cast<uint32_t>(rp.nch));
         rp.rpitch = ((pl.N * eb + 15) & ~int64_t(15)) + 16;
+        pl.chunk_force = chunk_env == 1;
+        pl.sms = dev.sms;
+        set_chunks(pl, 1);
     }
     rp.db_max = env_int("IPT_ROW_DB_MAX", 112 * 1024);
     rp.pipe = env_int("IPT_ROW_PIPE", 1);
@@ -450,8 +466,9 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     // Lagged tile layouts (col_tile.cu "In-place hazard"; IPT_COL_LAG=0 keeps the per-tile
     // group barrier): the shuffle pass waits only for the previous tile's group, and the
     // row pass reads (R2C) / writes (C2R) the shifted layout with the side tile S of M x TWB
-    // bytes per matrix (O(max(m, n)) scratch).  Not with the cluster row pass.
-    if (env_int("IPT_COL_LAG", 1) != 0 && !use_cluster && pl.shuf.p.ntiles >= 2) {
+    // bytes per matrix (O(max(m, n)) scratch).  With the cluster row pass only in its L2 mode
+    // (row_cluster_l2_kernel reads / writes the lagged layout; the DSMEM mode does not).
+    if (env_int("IPT_COL_LAG", 1) != 0 && (!use_cluster || rp.cl_mode == 1) && pl.shuf.p.ntiles >= 2) {
         ColParams &cq = pl.shuf.p;
         cq.lag = engine == ENG_C2R ? LAG_C2R : LAG_R2C;
         // D (IPT_COL_LAGD, default 8 tiles; 0: twice the co-resident CTAs' worth of
@@ -600,6 +617,8 @@ void prepare_call(Plan &pl, int64_t batch, CallScratch &cs) {
         const int64_t dmax = static_cast<int64_t>(cap / per_tile);
         if (dmax < pl.shuf.p.lagD) set_lag(pl, dmax);
     }
+    if (pl.row.fuse && pl.row.chunk && !set_chunks(pl, batch))
+        pl.row.chunk = 0;  // too few chunks for the GPU: the flag-based fused pass
     size_t o = 0;
     cs.ctr_shuf = o;
     o += kCtrBytes;

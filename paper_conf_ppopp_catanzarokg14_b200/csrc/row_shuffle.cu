@@ -800,8 +800,8 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_cluster_kernel(RowParams P
 // of the row is done) and the segment is written back coalesced.  Shared memory is private
 // to the CTA, so one barrier per row suffices.
 template <int EB, int DIR, bool TAIL>
-__device__ __forceinline__ void gather_l2(const RowParams &P, const char *row, unsigned char *buf, int32_t p0,
-                                          int32_t p1, int32_t i) {
+__device__ __forceinline__ void gather_l2(const RowParams &P, const char *row, const char *srow, unsigned char *buf,
+                                          int32_t p0, int32_t p1, int32_t i) {
     using T = typename Word<EB>::T;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     const int32_t len = p1 - p0;
@@ -809,7 +809,9 @@ __device__ __forceinline__ void gather_l2(const RowParams &P, const char *row, u
     const int32_t p_end = min(p1, p0 + warp * per + per);
     const int32_t im = static_cast<int32_t>(fmod_(static_cast<uint32_t>(i), P.fd_N));
     const int32_t Mi = P.M - i;
-    const T *src = reinterpret_cast<const T *>(row);
+    // Lagged R2C input (P.shW > 0): logical element s < shW in the side row, else row[s - shW].
+    const T *src = reinterpret_cast<const T *>(row) - (DIR == ROW_R2C ? P.shW : 0);
+    const T *ssrc = reinterpret_cast<const T *>(srow);
     T *out = reinterpret_cast<T *>(buf) - p0;
     int32_t p = p0 + warp * per + lane;
     if (p >= p_end) return;
@@ -820,7 +822,7 @@ __device__ __forceinline__ void gather_l2(const RowParams &P, const char *row, u
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const int32_t s = w.src(P, Mi);
-                if (p + 32 * u < p_end) v[u] = __ldcg(src + s);
+                if (p + 32 * u < p_end) v[u] = __ldcg((DIR == ROW_R2C && s < P.shW ? ssrc : src) + s);
                 w.next(P);
             }
 #pragma unroll
@@ -848,21 +850,44 @@ __global__ void __launch_bounds__(kRowThreadsMax) row_cluster_l2_kernel(RowParam
         const int64_t mat = r / P.M;
         return P.base + mat * P.mat_stride_bytes + static_cast<int64_t>(r - mat * P.M) * nbytes;
     };
-    if (cid < rows_total && p1 > p0) prefetch_l2(row_of(cid) + static_cast<int64_t>(p0) * EB, (p1 - p0) * EB);
+    // Lagged layouts (P.shW > 0, shared with the column pass): R2C reads logical columns
+    // [0, shW) from the side row and [shW, N) from row[0, N - shW); C2R writes them there.
+    auto side_of = [&](int64_t r) -> char * {
+        if (!P.shW) return nullptr;
+        const int64_t mat = r / P.M;
+        return side_matrix(P.side, P.sstride, mat, P.base + mat * P.mat_stride_bytes) + (r - mat * P.M) * P.spitch;
+    };
+    // this CTA's share of the row's L2 prefetch (segment [p0, p1) of the row, its side part too)
+    auto prefetch = [&](int64_t r) {
+        if (p1 <= p0) return;
+        prefetch_l2(row_of(r) + static_cast<int64_t>(p0) * EB, (p1 - p0) * EB);
+        if (DIR == ROW_R2C && P.shW && p0 < P.shW) prefetch_l2(side_of(r) + static_cast<int64_t>(p0) * EB,
+                                                             (min(p1, P.shW) - p0) * EB);
+    };
+    if (cid < rows_total) prefetch(cid);
     for (int64_t r = cid; r < rows_total; r += ncl) {
         const int32_t i = static_cast<int32_t>(r % P.M);
         char *row = row_of(r);
-        if (r + ncl < rows_total && p1 > p0)
-            prefetch_l2(row_of(r + ncl) + static_cast<int64_t>(p0) * EB, (p1 - p0) * EB);
+        char *srow = side_of(r);
+        if (r + ncl < rows_total) prefetch(r + ncl);
         if (p1 > p0) {
-            if (i >= P.M - P.c + 1) gather_l2<EB, DIR, true>(P, row, smem, p0, p1, i);
-            else gather_l2<EB, DIR, false>(P, row, smem, p0, p1, i);
+            if (i >= P.M - P.c + 1) gather_l2<EB, DIR, true>(P, row, srow, smem, p0, p1, i);
+            else gather_l2<EB, DIR, false>(P, row, srow, smem, p0, p1, i);
         }
         // every CTA of the cluster has read the whole row (its loads have returned)
         cluster_barrier_cta_fence();
         const T *buf = reinterpret_cast<const T *>(smem);
-        T *dst = reinterpret_cast<T *>(row) + p0;
-        for (int32_t k = threadIdx.x; k < p1 - p0; k += blockDim.x) dst[k] = buf[k];
+        if (DIR == ROW_C2R && P.shW) {
+            T *dst = reinterpret_cast<T *>(row) - P.shW;
+            T *sdst = reinterpret_cast<T *>(srow);
+            for (int32_t k = threadIdx.x; k < p1 - p0; k += blockDim.x) {
+                const int32_t pp = p0 + k;
+                (pp < P.shW ? sdst : dst)[pp] = buf[k];
+            }
+        } else {
+            T *dst = reinterpret_cast<T *>(row) + p0;
+            for (int32_t k = threadIdx.x; k < p1 - p0; k += blockDim.x) dst[k] = buf[k];
+        }
         __syncthreads();  // the buffer is refilled by the next row
     }
 }
