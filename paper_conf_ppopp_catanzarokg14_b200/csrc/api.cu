@@ -737,6 +737,11 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
     pl.shuf.p.ctr = reinterpret_cast<unsigned int *>(scratch + cs.ctr_shuf);
     pl.rot.p.ctr = reinterpret_cast<unsigned int *>(scratch + cs.ctr_rot);
     pl.shuf.p.ticket = pl.rot.p.ticket = env_int("IPT_COL_TICKET", 1) != 0 ? 1 : 0;
+    // super-tiles (lagged shuffle pass only; S <= D keeps every wait on a smaller ticket, and
+    // the band-major order needs the ticket)
+    pl.shuf.p.super = 1;
+    if (pl.shuf.p.lag != LAG_NONE && pl.shuf.p.ticket && pl.shuf.p.G > 1)
+        pl.shuf.p.super = std::max(1, std::min<int>(env_int("IPT_COL_SUPER", 1), pl.shuf.p.lagD));
     if (pl.row.fuse && !pl.row.chunk) {
         pl.row.flags = reinterpret_cast<unsigned int *>(scratch + cs.flags);
         pl.row.ticket = pl.row.flags + pl.M * batch;

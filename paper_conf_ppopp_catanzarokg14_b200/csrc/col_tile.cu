@@ -465,8 +465,20 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
         }
         return;
     }
-    const uint32_t tt = fdiv(ticket, P.fd_G);                  // tile (of all matrices)
-    const int32_t r = static_cast<int32_t>(ticket - tt * P.G);  // band
+    uint32_t tt;  // tile (of all matrices)
+    int32_t r;    // band
+    if (P.lag != LAG_NONE && P.super > 1) {
+        // super-tile s = tiles [s S, s S + S'), its units band-major: ticket -> (band, tile)
+        const uint32_t per = static_cast<uint32_t>(P.G) * static_cast<uint32_t>(P.super);
+        const uint32_t s = ticket / per, rem = ticket - s * per;
+        const uint32_t t0 = s * static_cast<uint32_t>(P.super);
+        const uint32_t here = min(static_cast<uint32_t>(P.super), static_cast<uint32_t>(P.total_tiles) - t0);
+        r = static_cast<int32_t>(rem / here);
+        tt = t0 + (rem - static_cast<uint32_t>(r) * here);
+    } else {
+        tt = fdiv(ticket, P.fd_G);
+        r = static_cast<int32_t>(ticket - tt * P.G);
+    }
     col_tile_one<EB, MODE, TWB>(P, smem, tt, r);
 }
 

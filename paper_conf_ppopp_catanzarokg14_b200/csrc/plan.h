@@ -139,6 +139,9 @@ struct ColParams {
     unsigned int *ctr;  // arrival counters + dispatch ticket: kCtrSlots + 1 words of the call's
                         // stream-ordered scratch, zeroed before the launch (api.cu CallScratch)
     int32_t ticket;     // 1: units in dispatch-ticket order (an atomic per CTA); 0: block index
+    int32_t super;      // lagged layouts: units ordered band-major within super-tiles of `super`
+                        // consecutive tiles (<= lagD), so that concurrently running units read
+                        // adjacent 128-byte segments of the same rows (1: tile-major)
     int32_t rot_sign;   // COL_ROT: +1 (C2R pre-rotation) or -1 (R2C post-rotation)
     int32_t wide_a;     // a >= 2^16
     FastDiv fd_G, fd_nt;  // ticket -> (tile, band), tile -> (matrix, column tile)
