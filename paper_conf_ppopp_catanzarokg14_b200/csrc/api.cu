@@ -100,6 +100,7 @@ struct Plan {
     SkinnyRowParams srow{};     // skinny engine long-row shuffle
     SkinnyColParams scol{}, srot{};  // skinny engine column passes (shuffle, rotation)
     bool chunk_force = false;   // IPT_ROW_CHUNK=1
+    int col_super = 1;          // lagged column pass: super-tile width (col_tile_kernel)
     int sms = 0;
     int skinny_dir = 0;         // ROW_R2C (P_{count,n}, AoS -> SoA) or ROW_C2R (P_{n,count})
 };
@@ -474,9 +475,16 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         // D (IPT_COL_LAGD, default 8 tiles; 0: twice the co-resident CTAs' worth of
         // groups): the round-1 sweep found 4-8 tiles of slack enough to take the wait off
         // the critical path (tools/col_sweep.sh), larger D no better; at most ntiles - 1.
-        int64_t D = env_int("IPT_COL_LAGD", 8);
+        // Tall tiles (>= 128 bands, e.g. config 5a): units in band-major order within
+        // super-tiles of 64 tiles (col_tile_kernel), which needs D >= 64 -- the concurrently
+        // running units then share rows instead of each spanning ~1/G of a 140 GB matrix (TLB
+        // reach): column pass 2.5 -> 4.4 TB/s on config 5a (gpurun_out r02r); side block
+        // M x 64 x 128 B (0.85 % of that matrix).
+        const bool tall = cq.G >= 128;
+        int64_t D = env_int("IPT_COL_LAGD", tall ? 64 : 8);
         if (D <= 0) D = (2 * static_cast<int64_t>(cq.resident) + cq.G - 1) / cq.G;
         set_lag(pl, D);
+        pl.col_super = env_int("IPT_COL_SUPER", tall ? 64 : 1);
         pl.scratch += pl.side_bytes;
     }
     pl.onchip = rsm > pl.shuf.smem ? rsm : pl.shuf.smem;
@@ -511,7 +519,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -741,7 +749,7 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
     // the band-major order needs the ticket)
     pl.shuf.p.super = 1;
     if (pl.shuf.p.lag != LAG_NONE && pl.shuf.p.ticket && pl.shuf.p.G > 1)
-        pl.shuf.p.super = std::max(1, std::min<int>(env_int("IPT_COL_SUPER", 1), pl.shuf.p.lagD));
+        pl.shuf.p.super = std::max(1, std::min<int>(pl.col_super, pl.shuf.p.lagD));
     if (pl.row.fuse && !pl.row.chunk) {
         pl.row.flags = reinterpret_cast<unsigned int *>(scratch + cs.flags);
         pl.row.ticket = pl.row.flags + pl.M * batch;

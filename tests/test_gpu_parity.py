@@ -746,3 +746,22 @@ def test_row_pass_kernels_both(pipe):
                 run_packed(shapes, eb, ipt.c2r, "row", engine, seed=eb + 3 * len(pipe))
         with env_var("IPT_FUSE_ROT", "0"):
             run_packed([(1200, 1800), (640, 32 * 33)], 4, ipt.c2r, "row", None, seed=8)
+
+
+@pytest.mark.parametrize("sup", ["2", "3", "8"])
+def test_super_tile_unit_order(sup):
+    """Lagged column pass with units in band-major order inside super-tiles of S consecutive
+    tiles (the default for tall tiles, e.g. config 5a; forced here on small shapes with many
+    bands per tile via a small IPT_COL_SMEM): ragged last super-tiles, both engines, batches."""
+    shapes = [(1200, 1800), (2003, 129), (129, 2003), (3001, 700), (700, 3001), (333, 4099)]
+    with env_var("IPT_COL_SUPER", sup), env_var("IPT_COL_LAGD", "8"), env_var("IPT_COL_SMEM", "12000"):
+        for eb in (4, 8):
+            for engine in ("c2r", "r2c"):
+                run_packed(shapes, eb, ipt.c2r, "row", engine, seed=eb + int(sup))
+        m, n, batch = 300, 1001, 3
+        host = workloads.random_words(batch * m * n, 4, seed=17)
+        x = to_dev(host)
+        ipt.c2r_batched(x, batch, m * n, m, n, elem_bytes=4)
+        got = x.cpu().numpy().view(np.uint32)
+        for k in range(batch):
+            assert got[k * m * n:(k + 1) * m * n].tobytes() == oracle.transpose(host[k * m * n:(k + 1) * m * n], m, n).tobytes()
