@@ -288,7 +288,7 @@ ipt_status_t make_skinny_plan(const DevInfo &dev, int64_t x, int64_t y, int eb, 
     sc.b = static_cast<int32_t>(pl.b);
     sc.fd_n = make_fastdiv(static_cast<uint32_t>(n));
     sc.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
-    sc.C = std::max(32, static_cast<int>((40 * 1024) / (n * eb)) / 32 * 32);
+    sc.C = std::max(32, static_cast<int>(env_int("IPT_SKINNY_COLBYTES", 40 * 1024) / (n * eb)) / 32 * 32);
     for (int i = 0; i < n; ++i) {  // Eq. 33: q(i) = (i N - floor(i/a)) mod n; q^{-1} its inverse
         const int64_t q = ((static_cast<int64_t>(i) * (pl.N % n) - i / pl.a) % n + n) % n;
         sc.q[i] = static_cast<int32_t>(q);
@@ -520,7 +520,7 @@ struct PlanKeyHash {
 std::string tunables_key() {
     std::string s;
     for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
-                          "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
+                          "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_SKINNY_COLBYTES", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
         s += v ? v : "-";
