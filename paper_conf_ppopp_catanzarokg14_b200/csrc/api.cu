@@ -288,7 +288,10 @@ ipt_status_t make_skinny_plan(const DevInfo &dev, int64_t x, int64_t y, int eb, 
     sc.b = static_cast<int32_t>(pl.b);
     sc.fd_n = make_fastdiv(static_cast<uint32_t>(n));
     sc.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
-    sc.C = std::max(32, static_cast<int>(env_int("IPT_SKINNY_COLBYTES", 40 * 1024) / (n * eb)) / 32 * 32);
+    // Staging per CTA: >= 40 KB, and >= 3.3 KB contiguous per field row (n x 3328 B, for
+    // large n), <= 110 KB (round-2 sweep of IPT_SKINNY_COLBYTES over n = 2..32, gpurun_out r02u).
+    const int colbytes = env_int("IPT_SKINNY_COLBYTES", std::min(110000, std::max(40 * 1024, n * 3328)));
+    sc.C = std::max(32, static_cast<int>(colbytes / (n * eb)) / 32 * 32);
     for (int i = 0; i < n; ++i) {  // Eq. 33: q(i) = (i N - floor(i/a)) mod n; q^{-1} its inverse
         const int64_t q = ((static_cast<int64_t>(i) * (pl.N % n) - i / pl.a) % n + n) % n;
         sc.q[i] = static_cast<int32_t>(q);
