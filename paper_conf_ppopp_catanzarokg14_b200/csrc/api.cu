@@ -116,21 +116,26 @@ int ilog2(int v) {
 // IPT_COL_SMEM (default 54000 B, four CTAs per SM: the best of the round-1 sweeps over
 // 12-100 KiB, profiles/r01_*).  Group size G = ceil(M / B) CTAs per tile; if a group would exceed
 // the co-resident CTAs, the band grows (up to the opt-in shared-memory maximum).
-ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe);
+ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe, int nbuf_min = 2);
 
 // IPT_COL_PIPE (default 0; 1 selects it): the persistent pipelined kernel with IPT_COL_NBUF unit buffers
 // per CTA (the shared-memory target is per buffer); tiles whose group would not fit the
 // co-resident CTAs that way (very tall matrices, config 5a) take the one-unit kernel.
-ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp) {
-    if (env_int("IPT_COL_PIPE", 0) != 0 && plan_col_v(dev, pl, mode, cp, true) == IPT_OK) return IPT_OK;
+ipt_status_t plan_col(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool barrier = false) {
+    // Barrier mode (a tile's G units read before any writes: the rotation pass, unlagged
+    // shuffles) runs the persistent kernel under a cooperative launch (launch_col), so the
+    // group's co-residency is guaranteed by the launch instead of assumed.
+    if ((barrier || env_int("IPT_COL_PIPE", 0) != 0) && plan_col_v(dev, pl, mode, cp, true) == IPT_OK) return IPT_OK;
+    // very tall tiles: one unit buffer per CTA doubles the co-resident CTAs (G <= grid)
+    if (barrier && plan_col_v(dev, pl, mode, cp, true, 1) == IPT_OK) return IPT_OK;
     return plan_col_v(dev, pl, mode, cp, false);
 }
 
-ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe) {
+ipt_status_t plan_col_v(const DevInfo &dev, const Plan &pl, int mode, ColPlan &cp, bool pipe, int nbuf_min) {
     int twb = env_int("IPT_TILE_BYTES", 128);
     if (twb != 128 && twb != 256 && twb != 512) twb = 128;
     if (pl.M >= (int64_t(1) << 29)) return IPT_ERR_UNSUPPORTED;
-    const int nbuf = pipe ? std::min(std::max(env_int("IPT_COL_NBUF", 2), 2), col_max_bufs()) : 1;
+    const int nbuf = pipe ? std::min(std::max(nbuf_min == 1 ? 1 : env_int("IPT_COL_NBUF", 2), nbuf_min), col_max_bufs()) : 1;
     const int64_t target = env_int("IPT_COL_SMEM", 54000);
     const int64_t W = twb / pl.eb;
     // Largest band whose buffer fits the target (col_smem_bytes: staged rows + row indices).
@@ -490,10 +495,14 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
         pl.col_super = env_int("IPT_COL_SUPER", tall ? 64 : 1);
         pl.scratch += pl.side_bytes;
     }
+    if (pl.shuf.p.lag == LAG_NONE && pl.shuf.p.G > 1 && !pl.shuf.p.pipe) {  // unlagged shuffle: barrier mode
+        s = plan_col(dev, pl, engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.shuf, true);
+        if (s != IPT_OK) return s;
+    }
     pl.onchip = rsm > pl.shuf.smem ? rsm : pl.shuf.smem;
     pl.nlaunch = 2;
     if (pl.c > 1 && !rp.fuse) {
-        s = plan_col(dev, pl, COL_ROT, pl.rot);
+        s = plan_col(dev, pl, COL_ROT, pl.rot, true);
         if (s != IPT_OK) return s;
         pl.rot.p.rot_sign = engine == ENG_C2R ? 1 : -1;
         pl.has_rot = true;

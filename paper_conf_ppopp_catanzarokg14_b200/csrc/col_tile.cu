@@ -717,6 +717,10 @@ cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, s
     if (!P.ctr) return cudaErrorInvalidValue;
     void *args[] = {&P};
     const int threads = P.threads > 0 ? P.threads : kColThreads;
+    // The persistent kernel (barrier mode and IPT_COL_PIPE) runs as a cooperative launch: all
+    // of its CTAs (grid <= the co-resident count) are resident at once by construction, which
+    // its per-tile group barriers need; a plain launch would only assume it.
+    if (P.pipe) return cudaLaunchCooperativeKernel(kern, dim3(static_cast<unsigned>(grid)), dim3(threads), args, smem, st);
     return cudaLaunchKernel(kern, dim3(static_cast<unsigned>(grid)), dim3(threads), args, smem, st);
 }
 
