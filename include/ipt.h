@@ -6,10 +6,20 @@
  *
  * Every entry point is asynchronous on `stream` (a cudaStream_t of the current device,
  * passed as void* so that this header needs no CUDA include; NULL = legacy default
- * stream).  Arguments are validated synchronously before anything is enqueued; an
- * argument error leaves the buffer untouched.  No entry point allocates device memory
- * that outlives the call, throws, or synchronises the stream.  All entry points are
- * thread-safe and reentrant.
+ * stream).  Arguments are validated, and every step of the call planned (including the
+ * UNSUPPORTED checks of composed element sizes), synchronously before anything is
+ * enqueued; such an error leaves the buffer untouched.  No entry point allocates device
+ * memory that outlives the call, throws, or synchronises the stream.  All entry points are
+ * thread-safe and reentrant: every call owns one stream-ordered scratch allocation (its
+ * counters, flags and boundary rows), so concurrent calls from any threads on any streams
+ * (cudaStreamPerThread included) share no state.
+ *
+ * Forward progress: no kernel relies on its CTAs being co-resident or dispatched in index
+ * order.  Cross-CTA waits (the column pass's lagged-layout counters, the fused rotation's
+ * row flags) only ever target work units with a smaller dispatch ticket, taken by a CTA
+ * already running; passes whose CTAs must be co-resident (per-tile group barriers: the
+ * separate rotation pass for gcd > 32 and unlagged shuffles) are cooperative launches, which
+ * fail with IPT_ERR_CUDA instead of hanging when the GPU cannot host the whole grid.
  *
  * Memory: `ptr` is caller-owned device memory on the current device, aligned to
  * elem_bytes (16-byte alignment is NOT required).  The caller must not read or write it
