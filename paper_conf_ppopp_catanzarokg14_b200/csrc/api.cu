@@ -531,7 +531,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_SKINNY_COLBYTES", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -600,6 +600,64 @@ void profile_end(ProfRec &r, cudaStream_t st) {
     cudaEventRecord(r.stop, st);
     std::lock_guard<std::mutex> lk(g_prof_mu);
     g_prof.push_back(r);
+}
+
+// ---- TMA tensor maps of the column pass (pitch % 16 == 0; ColParams::tma) ----------------
+using EncodeTiledFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                   const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn encode_tiled() {
+    static EncodeTiledFn fn = [] {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q{};
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess) {
+            cudaGetLastError();
+            return static_cast<EncodeTiledFn>(nullptr);
+        }
+        return reinterpret_cast<EncodeTiledFn>(p);
+    }();
+    return fn;
+}
+
+// u32 view of rows of `row_bytes` at `base`, rows `pitch` apart, matrices `mstride` apart
+// (rank 3; rank 2 over `rows` rows when mstride == 0); box {32 u32 = 128 B, box_rows(, 1)}.
+bool make_map(CUtensorMap *m, const char *base, int64_t row_bytes, int64_t rows, int64_t pitch, int64_t batch,
+              int64_t mstride, uint32_t box_rows) {
+    EncodeTiledFn enc = encode_tiled();
+    if (!enc || reinterpret_cast<uintptr_t>(base) % 16 || pitch % 16 || (mstride && mstride % 16)) return false;
+    const cuuint64_t dims[3] = {static_cast<cuuint64_t>(row_bytes / 4), static_cast<cuuint64_t>(rows),
+                                static_cast<cuuint64_t>(batch)};
+    const cuuint64_t strides[2] = {static_cast<cuuint64_t>(pitch), static_cast<cuuint64_t>(mstride)};
+    const cuuint32_t box[3] = {32, box_rows, 1};
+    const cuuint32_t estr[3] = {1, 1, 1};
+    const cuuint32_t rank = mstride ? 3 : 2;
+    if (dims[0] >= (cuuint64_t(1) << 32) || dims[1] >= (cuuint64_t(1) << 32) || dims[2] >= (cuuint64_t(1) << 32))
+        return false;
+    return enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT32, rank, const_cast<char *>(base), dims, strides, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// Enable TMA staging for a shuffle / rotation pass where the layout allows (128-byte tiles,
+// 16-byte pitches and bases); otherwise the pass keeps 16-byte cp.async hulls.
+void setup_col_tma(ColParams &p, int mode, int eb) {
+    p.tma = 0;
+    if (p.pipe || p.W * eb != 128 || env_int("IPT_COL_TMA", 1) == 0) return;
+    const int64_t pitch = static_cast<int64_t>(p.N) * eb;
+    const bool packed = p.batch == 1 || p.mat_stride_bytes == static_cast<int64_t>(p.M) * pitch;
+    if (mode == COL_R2C_SHUF) {
+        if (packed && make_map(&p.tmap_g, p.base, pitch, static_cast<int64_t>(p.M) * p.batch, pitch, 1, 0, 1))
+            p.tma |= 4;
+        return;
+    }
+    const int64_t ms = p.batch == 1 ? static_cast<int64_t>(p.M) * pitch : p.mat_stride_bytes;
+    if (make_map(&p.tmap_a, p.base, pitch, p.M, pitch, p.batch, ms, kTmaBoxRows)) p.tma |= 1;
+    if (mode == COL_C2R_SHUF && p.lag == LAG_C2R && p.side && (p.tma & 1)) {  // (aligned matrix bases)
+        const char *s0 = side_matrix(p.side, p.sstride, 0, p.base);
+        if (make_map(&p.tmap_s, s0, static_cast<int64_t>(p.lagD) * 128, p.M, p.spitch, p.batch, p.sstride, kTmaBoxRows))
+            p.tma |= 2;
+    }
 }
 
 // ---- per-call global scratch (Theorem 6: O(max(m, n)) per worker) -------------------
@@ -773,6 +831,8 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
         pl.row.bnd = scratch + cs.bnd;
     }
     pl.row.side = pl.shuf.p.side = pl.side_bytes ? scratch + cs.side : nullptr;
+    setup_col_tma(pl.shuf.p, pl.engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.eb);
+    if (pl.has_rot) setup_col_tma(pl.rot.p, COL_ROT, pl.eb);
     const int64_t pitch = pl.N * pl.eb;
     const int passes = budget;
     // The rotation moves only the columns with a non-zero amount: (c - 1) / c of them.

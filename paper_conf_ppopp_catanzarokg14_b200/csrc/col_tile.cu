@@ -88,8 +88,13 @@ __host__ __device__ inline SmemLayout smem_layout(int64_t B, int W, int twb, int
     o += al16(nslots * 4);
     L.sbase = o;
     o += al16(nslots * 4);
+    o = (o + 127) & ~size_t(127);  // slot rows 128-byte aligned (TMA destinations)
     L.rows = o;
-    L.total = o + nslots * static_cast<size_t>(hull_pitch(twb));
+    // cp.async hulls: nslots x (TWB + 16); TMA: whole boxes of kTmaBoxRows x TWB (+ 3 slots of
+    // gather4 padding)
+    const size_t hull = nslots * static_cast<size_t>(hull_pitch(twb));
+    const size_t tma = ((nslots + 3 + kTmaBoxRows - 1) / kTmaBoxRows) * kTmaBoxRows * static_cast<size_t>(twb);
+    L.total = o + (hull > tma ? hull : tma);
     return L;
 }
 
@@ -391,13 +396,106 @@ __device__ __forceinline__ Dep unit_dep(const ColParams &P, uint32_t tt) {
     return d;
 }
 
+// ---- TMA staging (P.tma; 128-byte tiles, pitch % 16 == 0) -----------------------------
+// Slots at a 128-byte pitch (no hull): slot t of the unit at rows_s + 128 t.  C2R / ROT read
+// the contiguous rows rowbase .. rowbase + nslots - 1 (units whose rows wrap past M - 1 keep
+// cp.async) as 2-D boxes of kTmaBoxRows rows; R2C gathers its scattered rows 4 at a time
+// (tile::gather4).  One mbarrier per CTA counts the bytes; out-of-range rows / columns of a
+// box (the matrix's last rows, the ragged rightmost tile) are zero-filled by the TMA unit and
+// never used.
+__device__ __forceinline__ void tmbar_init(uint64_t *bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar)))
+                 : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void tmbar_expect(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.release.cta.shared::cta.b64 _, [%0], %1;"
+                 :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void tmbar_wait(uint64_t *bar, uint32_t parity) {
+    const uint32_t a = static_cast<uint32_t>(__cvta_generic_to_shared(bar));
+    asm volatile("{\n .reg .pred p;\n TW_%=:\n"
+                 " mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%0], %1;\n"
+                 " @!p bra TW_%=;\n}" :: "r"(a), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tma_box3(uint32_t dst, const CUtensorMap *map, int32_t x, int32_t y, int32_t z,
+                                         uint64_t *bar) {
+    asm volatile("cp.async.bulk.tensor.3d.shared::cta.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];"
+                 :: "r"(dst), "l"(map), "r"(x), "r"(y), "r"(z),
+                    "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))) : "memory");
+}
+__device__ __forceinline__ void tma_gather4(uint32_t dst, const CUtensorMap *map, int32_t x, int32_t r0, int32_t r1,
+                                            int32_t r2, int32_t r3, uint64_t *bar) {
+    asm volatile("cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5, %6}], [%7];"
+                 :: "r"(dst), "l"(map), "r"(x), "r"(r0), "r"(r1), "r"(r2), "r"(r3),
+                    "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))) : "memory");
+}
+
+// Whether (and from which map) unit U stages with TMA: 0 no, 1 A boxes, 2 side boxes,
+// 3 gather4.  Its x coordinate (u32 units) comes back in xcoord.
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ int tma_kind(const ColParams &P, const Unit &U, uint32_t tt, int32_t &xcoord) {
+    if (TWB != 128 || !P.tma || U.skip || U.nslots == 0) return 0;
+    const uint32_t mat = fdiv(tt, P.fd_nt);
+    const int32_t tile = U.j0 / (TWB / EB);
+    if (MODE == COL_R2C_SHUF) {
+        if (!(P.tma & 4)) return 0;
+        xcoord = U.j0 * EB / 4;
+        return 3;
+    }
+    if (MODE != COL_C2R_SHUF && MODE != COL_ROT) return 0;
+    if (U.rowbase + U.nslots > P.M) return 0;  // rows wrap past M - 1: cp.async
+    (void)mat;
+    if (MODE == COL_C2R_SHUF && P.lag == LAG_C2R && tile < P.lagD) {
+        if (!(P.tma & 2)) return 0;
+        xcoord = tile * TWB / 4;
+        return 2;
+    }
+    if (!(P.tma & 1)) return 0;
+    xcoord = (U.j0 - (MODE == COL_C2R_SHUF && P.lag == LAG_C2R ? P.lagD * (TWB / EB) : 0)) * EB / 4;
+    return 1;
+}
+
+// Issue the unit's TMA loads (warp 0: lanes split the boxes) and point sbase[] at the 128-byte
+// slots.  The caller waits on `bar` (phase `ph`).
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ void unit_load_tma(const ColParams &P, const Unit &U, uint32_t tt, int kind, int32_t xcoord,
+                                              const int32_t *srow, uint32_t *sbase, uint32_t rows_s, uint64_t *bar) {
+    const uint32_t mat = fdiv(tt, P.fd_nt);
+    const int lane = threadIdx.x & 31;
+    for (int32_t t = threadIdx.x; t < U.nslots; t += blockDim.x) sbase[t] = rows_s + static_cast<uint32_t>(t) * TWB;
+    if (threadIdx.x >= 32) return;
+    if (kind == 3) {
+        const int32_t ng = (U.nslots + 3) / 4;
+        if (lane == 0) tmbar_expect(bar, static_cast<uint32_t>(ng) * 4 * TWB);
+        __syncwarp();
+        const int32_t rbase = static_cast<int32_t>(mat) * P.M;  // packed batch: rows of all matrices
+        for (int32_t gi = lane; gi < ng; gi += 32) {
+            const int32_t t0 = 4 * gi;
+            int32_t r[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) r[e] = rbase + srow[min(t0 + e, U.nslots - 1)];
+            tma_gather4(rows_s + static_cast<uint32_t>(t0) * TWB, &P.tmap_g, xcoord, r[0], r[1], r[2], r[3], bar);
+        }
+    } else {
+        const int32_t nb = (U.nslots + kTmaBoxRows - 1) / kTmaBoxRows;
+        if (lane == 0) tmbar_expect(bar, static_cast<uint32_t>(nb) * kTmaBoxRows * TWB);
+        __syncwarp();
+        const CUtensorMap *map = kind == 2 ? &P.tmap_s : &P.tmap_a;
+        for (int32_t bi = lane; bi < nb; bi += 32)
+            tma_box3(rows_s + static_cast<uint32_t>(bi * kTmaBoxRows) * TWB, map, xcoord, U.rowbase + bi * kTmaBoxRows,
+                     static_cast<int32_t>(mat), bar);
+    }
+}
+
 // Non-persistent variant: one CTA per (tile, band).  The CTA's logical id comes from a
 // ticket counter taken at start (dispatch order), so the G members of a tile are exactly
 // G consecutive tickets: every group whose tickets are all taken is fully resident, hence
 // only the newest group can be waiting for members, and those get scheduled as older
 // groups finish.  G == 1: P.tpc consecutive tiles per CTA.
 template <int EB, int MODE, int TWB>
-__device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *smem, uint32_t tt, int32_t r) {
+__device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *smem, uint32_t tt, int32_t r,
+                                             uint64_t *tbar, uint32_t &tphase) {
     const SmemLayout L = smem_layout(P.B, TWB / EB, TWB, EB);
     int64_t *orow = reinterpret_cast<int64_t *>(smem);
     int32_t *srow = reinterpret_cast<int32_t *>(smem + L.srow);
@@ -414,12 +512,22 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
         if (P.dbg != 4) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
         __syncthreads();
     }
-    if (P.dbg != 2)  // measurement knob: 2 = skip the loads
-        unit_load<EB, MODE, TWB>(P, U, srow, sbase, static_cast<uint32_t>(__cvta_generic_to_shared(smem + L.rows)),
-                                 blockDim.x);
+    int32_t xcoord = 0;
+    const int kind = tma_kind<EB, MODE, TWB>(P, U, tt, xcoord);
+    const uint32_t rows_s = static_cast<uint32_t>(__cvta_generic_to_shared(smem + L.rows));
+    if (kind) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // earlier generic reads of the buffer
+        unit_load_tma<EB, MODE, TWB>(P, U, tt, kind, xcoord, srow, sbase, rows_s, tbar);
+    } else if (P.dbg != 2) {  // measurement knob: 2 = skip the loads
+        unit_load<EB, MODE, TWB>(P, U, srow, sbase, rows_s, blockDim.x);
+    }
     asm volatile("cp.async.commit_group;" ::: "memory");
     if (MODE != COL_R2C_SHUF && P.dbg != 4) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
     asm volatile("cp.async.wait_group 0;" ::: "memory");
+    if (kind) {
+        tmbar_wait(tbar, tphase);
+        tphase ^= 1;
+    }
     __syncthreads();  // every thread's staged data is in shared memory
     if (threadIdx.x == 0) {
         // The arrival only says "this unit's reads of its input are complete" (write-after-
@@ -441,8 +549,14 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
 }
 
 template <int EB, int MODE, int TWB>
-__global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
-    extern __shared__ __align__(16) unsigned char smem[];
+__global__ void __launch_bounds__(kColThreads) col_tile_kernel(const __grid_constant__ ColParams P) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ __align__(8) uint64_t tbar;  // TMA staging (P.tma)
+    uint32_t tphase = 0;
+    if (P.tma) {
+        if (threadIdx.x == 0) tmbar_init(&tbar);
+        __syncthreads();
+    }
     // Unit order = dispatch-ticket order (an atomic taken at start).  Barrier mode: a tile's
     // G members are G consecutive dispatches, so the whole group is co-resident.  Lagged
     // layouts only ever wait for units of smaller ticket, which were taken by CTAs already
@@ -460,7 +574,7 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
     if (P.G == 1) {
         const uint64_t t_end = min(static_cast<uint64_t>(P.total_tiles), (static_cast<uint64_t>(ticket) + 1) * P.tpc);
         for (uint64_t tt = static_cast<uint64_t>(ticket) * P.tpc; tt < t_end; ++tt) {
-            col_tile_one<EB, MODE, TWB>(P, smem, static_cast<uint32_t>(tt), 0);
+            col_tile_one<EB, MODE, TWB>(P, smem, static_cast<uint32_t>(tt), 0, &tbar, tphase);
             __syncthreads();  // shared memory is reused by the next tile
         }
         return;
@@ -479,7 +593,7 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(ColParams P) {
         tt = fdiv(ticket, P.fd_G);
         r = static_cast<int32_t>(ticket - tt * P.G);
     }
-    col_tile_one<EB, MODE, TWB>(P, smem, tt, r);
+    col_tile_one<EB, MODE, TWB>(P, smem, tt, r, &tbar, tphase);
 }
 
 // mbarrier helpers (shared::cta).
@@ -530,7 +644,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
 // two buffers both hold units of g cannot take more; all CTAs in that state would mean
 // >= 2 grid >= G taken tickets of g, i.e. none untaken.  By induction every group completes.
 template <int EB, int MODE, int TWB>
-__global__ void __launch_bounds__(kColThreads) col_pipe_kernel(ColParams P) {
+__global__ void __launch_bounds__(kColThreads) col_pipe_kernel(const __grid_constant__ ColParams P) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ unsigned int s_ticket[kMaxColBufs];
     __shared__ int s_release;  // units released so far (control -> ticket warp)

@@ -12,6 +12,7 @@
 
 #include <cstddef>
 #include <cstdint>
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include "common.cuh"
@@ -122,7 +123,15 @@ struct RowParams {
 };
 constexpr int kMaxFuseC = 32;
 
+// TMA staging of the column pass (pitch a multiple of 16 bytes): 2-D tiles of kTmaBoxRows
+// rows x 128 bytes (A and side block, 3-D maps over the batch) and R2C row gathers of 4 rows
+// (tile::gather4, a 2-D map over all rows; batches packed only).
+constexpr int kTmaBoxRows = 16;
 struct ColParams {
+    CUtensorMap tmap_a;   // 3-D {N eb / 4, M, batch} u32, box {32, kTmaBoxRows, 1}
+    CUtensorMap tmap_s;   // 3-D {spitch / 4, M, batch} u32 over the side block (lagged C2R input)
+    CUtensorMap tmap_g;   // 2-D {N eb / 4, M batch} u32, box {32, 1} (gather4)
+    int32_t tma;          // bit 0: box loads of A; bit 1: box loads of the side block; bit 2: gather4
     char *base;
     int64_t mat_stride_bytes;
     int64_t batch;
