@@ -88,13 +88,12 @@ __host__ __device__ inline SmemLayout smem_layout(int64_t B, int W, int twb, int
     o += al16(nslots * 4);
     L.sbase = o;
     o += al16(nslots * 4);
-    o = (o + 127) & ~size_t(127);  // slot rows 128-byte aligned (TMA destinations)
-    L.rows = o;
+    L.rows = o;  // the kernels round the slot region up to 128 bytes (TMA destinations): slack below
     // cp.async hulls: nslots x (TWB + 16); TMA: whole boxes of kTmaBoxRows x TWB (+ 3 slots of
     // gather4 padding)
     const size_t hull = nslots * static_cast<size_t>(hull_pitch(twb));
     const size_t tma = ((nslots + 3 + kTmaBoxRows - 1) / kTmaBoxRows) * kTmaBoxRows * static_cast<size_t>(twb);
-    L.total = o + (hull > tma ? hull : tma);
+    L.total = o + (hull > tma ? hull : tma) + 128;
     return L;
 }
 
@@ -514,7 +513,7 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     }
     int32_t xcoord = 0;
     const int kind = tma_kind<EB, MODE, TWB>(P, U, tt, xcoord);
-    const uint32_t rows_s = static_cast<uint32_t>(__cvta_generic_to_shared(smem + L.rows));
+    const uint32_t rows_s = (static_cast<uint32_t>(__cvta_generic_to_shared(smem + L.rows)) + 127u) & ~127u;
     if (kind) {
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // earlier generic reads of the buffer
         unit_load_tma<EB, MODE, TWB>(P, U, tt, kind, xcoord, srow, sbase, rows_s, tbar);
