@@ -641,19 +641,26 @@ bool make_map(CUtensorMap *m, const char *base, int64_t row_bytes, int64_t rows,
 
 // Enable TMA staging for a shuffle / rotation pass where the layout allows (128-byte tiles,
 // 16-byte pitches and bases); otherwise the pass keeps 16-byte cp.async hulls.
+// IPT_COL_TMA is a mask of the allowed kinds (default 3): 1 box loads of the matrix, 2 box loads
+// of the side block, 4 tile::gather4 for R2C (measured slower than cp.async hulls on the
+// sweep: R2C aligned shapes 4688 vs 5005 GB/s, while box loads take C2R from 5148 to 5378;
+// tools/ab_calls.py, gpurun_out r02z).
 void setup_col_tma(ColParams &p, int mode, int eb) {
     p.tma = 0;
-    if (p.pipe || p.W * eb != 128 || env_int("IPT_COL_TMA", 1) == 0) return;
+    const int allow = env_int("IPT_COL_TMA", 3);
+    if (p.pipe || p.W * eb != 128 || allow == 0) return;
     const int64_t pitch = static_cast<int64_t>(p.N) * eb;
     const bool packed = p.batch == 1 || p.mat_stride_bytes == static_cast<int64_t>(p.M) * pitch;
     if (mode == COL_R2C_SHUF) {
-        if (packed && make_map(&p.tmap_g, p.base, pitch, static_cast<int64_t>(p.M) * p.batch, pitch, 1, 0, 1))
+        if ((allow & 4) && packed &&
+            make_map(&p.tmap_g, p.base, pitch, static_cast<int64_t>(p.M) * p.batch, pitch, 1, 0, 1))
             p.tma |= 4;
         return;
     }
+    if (!(allow & 1)) return;
     const int64_t ms = p.batch == 1 ? static_cast<int64_t>(p.M) * pitch : p.mat_stride_bytes;
     if (make_map(&p.tmap_a, p.base, pitch, p.M, pitch, p.batch, ms, kTmaBoxRows)) p.tma |= 1;
-    if (mode == COL_C2R_SHUF && p.lag == LAG_C2R && p.side && (p.tma & 1)) {  // (aligned matrix bases)
+    if ((allow & 2) && mode == COL_C2R_SHUF && p.lag == LAG_C2R && p.side && (p.tma & 1)) {  // (aligned matrix bases)
         const char *s0 = side_matrix(p.side, p.sstride, 0, p.base);
         if (make_map(&p.tmap_s, s0, static_cast<int64_t>(p.lagD) * 128, p.M, p.spitch, p.batch, p.sstride, kTmaBoxRows))
             p.tma |= 2;

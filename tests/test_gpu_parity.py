@@ -765,3 +765,30 @@ def test_super_tile_unit_order(sup):
         got = x.cpu().numpy().view(np.uint32)
         for k in range(batch):
             assert got[k * m * n:(k + 1) * m * n].tobytes() == oracle.transpose(host[k * m * n:(k + 1) * m * n], m, n).tobytes()
+
+
+@pytest.mark.parametrize("mask", ["3", "7", "1", "0"])
+def test_column_tma_staging(mask):
+    """Column pass with TMA staging (IPT_COL_TMA mask: 1 box loads of the matrix, 2 of the
+    lagged side block, 4 tile::gather4 for R2C): pitches that are multiples of 16 bytes (TMA)
+    next to ones that are not (cp.async hulls), ragged rightmost tiles (zero-filled box columns),
+    last bands (zero-filled box rows), units whose rows wrap past M - 1, batches packed and
+    gapped, both engines, every element size; full comparison with the oracle."""
+    shapes = [(1200, 1800), (1801, 1200), (1200, 1801), (640, 1024), (1024, 640), (2003, 132), (132, 2003),
+              (4096, 3000), (300, 1004), (1004, 300), (96, 40), (37, 64)]
+    with env_var("IPT_COL_TMA", mask):
+        for eb in (4, 8, 16):
+            for engine in ("c2r", "r2c"):
+                run_packed(shapes, eb, ipt.c2r, "row", engine, seed=eb + int(mask))
+        for packed in (True, False):
+            m, n, batch = 400, 1204, 3
+            stride = m * n + (0 if packed else 4)
+            host = workloads.random_words(batch * stride, 4, seed=23)
+            x = to_dev(host)
+            ipt.c2r_batched(x, batch, stride, m, n, elem_bytes=4)
+            got = x.cpu().numpy().view(np.uint32)
+            for k in range(batch):
+                o = k * stride
+                assert got[o:o + m * n].tobytes() == oracle.transpose(host[o:o + m * n], m, n).tobytes(), (packed, k)
+            ipt.r2c_batched(x, batch, stride, m, n, elem_bytes=4)
+            assert dev_bytes(x) == host.tobytes()
