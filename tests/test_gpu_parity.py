@@ -779,7 +779,15 @@ def test_column_tma_staging(mask):
     with env_var("IPT_COL_TMA", mask):
         for eb in (4, 8, 16):
             for engine in ("c2r", "r2c"):
-                run_packed(shapes, eb, ipt.c2r, "row", engine, seed=eb + int(mask))
+                with forced_engine(engine):
+                    for (m, n) in shapes:  # own (256-byte-aligned) allocation per matrix: TMA-eligible
+                        host = workloads.random_words(m * n, eb, seed=m * 7 + n + eb)
+                        x = to_dev(host)
+                        ipt.c2r(x, m, n, elem_bytes=eb)
+                        assert dev_bytes(x) == oracle.transpose(vwords(host, eb), m, n).tobytes(), (m, n, eb, engine)
+                        ipt.r2c(x, m, n, elem_bytes=eb)
+                        assert dev_bytes(x) == np.ascontiguousarray(host).tobytes(), (m, n, eb, engine)
+                run_packed(shapes, eb, ipt.c2r, "row", engine, seed=eb + int(mask))  # mostly unaligned bases
         for packed in (True, False):
             m, n, batch = 400, 1204, 3
             stride = m * n + (0 if packed else 4)
