@@ -13,6 +13,12 @@ ncu)
       python bench.py --profile-only --no-cpu-baseline --no-extras > gpurun_out/ncu_launch_$TAG.log 2>&1
   timeout 600 $NCU -k regex:col_tile -c 1 -s 2 -o $REP/col_$TAG \
       python tools/one_shape.py --m 14414 --n 6565 --eb 4 --reps 3 > gpurun_out/ncu_col_$TAG.log 2>&1
+  # TMA-staged column pass: C2R shuffle of a 16-byte-pitch shape (14414 x 6564 fp32)
+  timeout 600 $NCU -k regex:col_tile -c 1 -s 2 -o $REP/coltma_$TAG \
+      python tools/one_shape.py --m 14414 --n 6564 --eb 4 --reps 3 > gpurun_out/ncu_coltma_$TAG.log 2>&1
+  # R2C shuffle (scattered source rows, cp.async hulls)
+  timeout 600 $NCU -k regex:col_tile -c 1 -s 2 -o $REP/colr2c_$TAG \
+      python tools/one_shape.py --m 6565 --n 14414 --eb 4 --reps 3 > gpurun_out/ncu_colr2c_$TAG.log 2>&1
   timeout 600 $NCU -k regex:row_pipe -c 1 -s 2 -o $REP/rowpipe_$TAG \
       python tools/one_shape.py --m 14414 --n 6565 --eb 4 --reps 3 > gpurun_out/ncu_rowpipe_$TAG.log 2>&1
   timeout 600 $NCU -k regex:row_rot -c 1 -s 2 -o $REP/rowrot_$TAG \
