@@ -685,13 +685,20 @@ struct CallScratch {
 
 size_t al256(size_t x) { return (x + 255) & ~size_t(255); }
 
+// Skinny batches: matrices per launch, each needing one tmp row of N eb bytes -- the tmp rows of
+// a launch stay within 256 MiB (at least one matrix), at most 65535 (gridDim.y).
+int64_t skinny_sub(const Plan &pl, int64_t batch) {
+    const int64_t row = std::max<int64_t>(1, pl.N * pl.eb);
+    return std::max<int64_t>(1, std::min<int64_t>({batch, (int64_t(256) << 20) / row, 65535}));
+}
+
 // Final plan of a call on `batch` matrices (batches cap the lag) and its scratch layout.
 // Pure host arithmetic: nothing is enqueued.
 void prepare_call(Plan &pl, int64_t batch, CallScratch &cs) {
     cs = CallScratch{};
     if (pl.engine == ENG_NONE || batch == 0) return;
     if (pl.engine == ENG_SKINNY) {
-        cs.total = al256(pl.scratch);
+        cs.total = al256(pl.scratch * static_cast<size_t>(skinny_sub(pl, batch)));
         return;
     }
     const double full = 2.0 * static_cast<double>(pl.M) * static_cast<double>(pl.N) * pl.eb * static_cast<double>(batch);
@@ -786,15 +793,22 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
         // shifted rows back.  A destination row is never its own source row.  With c > 1 the
         // rotation is folded in: block rho = floor(j/b) of every rolled location is shifted
         // by another rho rows (plan.h, SkinnyRowParams).
+        // Batches: every pass is one launch for a sub-batch of up to skinny_sub(...) matrices
+        // (gridDim.y = matrix, each with its own tmp row in the call's scratch).
         const int n = static_cast<int>(pl.M);
+        const int64_t sub = skinny_sub(pl, batch);
         const double rowb = 2.0 * static_cast<double>(pl.N) * pl.eb;
         char *tmp = scratch;
         s = IPT_OK;
-        for (int64_t mat = 0; mat < batch; ++mat) {
+        for (int64_t mat = 0; mat < batch; mat += sub) {
+            const int64_t nb = std::min(sub, batch - mat);
             char *A = base + mat * stride_bytes;
             SkinnyColParams shuf = pl.scol, rotp = pl.srot;
             shuf.A = rotp.A = A;
             shuf.tmp = rotp.tmp = tmp;
+            shuf.batch = rotp.batch = nb;
+            shuf.mat_stride = rotp.mat_stride = stride_bytes;
+            shuf.tmp_stride = rotp.tmp_stride = pl.N * pl.eb;
             auto rot_l = [&] { return launch_skinny_col(rotp, pl.eb, st); };
             auto shuf_l = [&] { return launch_skinny_col(shuf, pl.eb, st); };
             auto row_l = [&](int i) {
@@ -802,6 +816,9 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
                 rp.i = i;
                 rp.A = A;
                 rp.tmp = tmp;
+                rp.batch = nb;
+                rp.mat_stride = stride_bytes;
+                rp.tmp_stride = pl.N * pl.eb;
                 return [rp, &pl, st] { return launch_skinny_row(rp, pl.skinny_dir, pl.eb, st); };
             };
             if (pl.skinny_dir == ROW_R2C) {

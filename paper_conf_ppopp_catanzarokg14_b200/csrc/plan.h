@@ -189,6 +189,8 @@ struct SkinnyRowParams {
     int32_t fold;       // 1: the rotation (Eq. 23 / Eq. 36) is folded into the locations
     int32_t reg;        // 1: in-register SIMD transposition kernel (skinny_reg.cu; 4-byte fields)
     FastDiv fd_n, fd_b;
+    int64_t batch;      // matrices of the launch (gridDim.y): matrix k at A + k mat_stride,
+    int64_t mat_stride, tmp_stride;  // its tmp row at tmp + k tmp_stride (bytes)
 };
 
 // Kernel attribute / occupancy caches (api.cu): set the dynamic shared-memory limit (and
@@ -249,6 +251,8 @@ struct SkinnyColParams {
     int32_t C;          // columns per CTA (multiple of 32)
     int32_t q[32], qinv[32];  // Eq. 33 / Eq. 34 on the n rows
     FastDiv fd_n, fd_b;
+    int64_t batch;      // as SkinnyRowParams
+    int64_t mat_stride, tmp_stride;
 };
 size_t skinny_col_smem(int n, int C, int eb);
 cudaError_t launch_skinny_col(const SkinnyColParams &p, int eb, cudaStream_t st);

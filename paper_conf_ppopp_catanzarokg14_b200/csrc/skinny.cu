@@ -21,6 +21,8 @@
 //     runs of an output window [w0, w0 + nT) and writes the window (coalesced).
 // Every element is read once and written once.  In-place safety comes from the caller:
 // the destination row is never the source row (rolling rows + one tmp row, api.cu).
+#include <algorithm>
+
 #include "plan.h"
 
 namespace ipt {
@@ -82,18 +84,21 @@ __global__ void __launch_bounds__(kSkThreads) skinny_row_kernel(SkinnyRowParams 
     const uint32_t sbuf = static_cast<uint32_t>(__cvta_generic_to_shared(buf));
     const int n = P.n;
     const int64_t L = static_cast<int64_t>(n) * P.T;
+    // batches: matrix blockIdx.y of the launch, its own tmp row
+    char *const Am = P.A + static_cast<int64_t>(blockIdx.y) * P.mat_stride;
+    char *const tmpm = P.tmp + static_cast<int64_t>(blockIdx.y) * P.tmp_stride;
     const int lt = 31 - __clz(P.T);  // T is a power of two
     const int nblk = FOLD ? P.c : 1;
     if (threadIdx.x < nblk) {
         const int32_t ls = sk_src_loc(P, DIR, FOLD ? threadIdx.x : 0);
         const int32_t ld = sk_dst_loc(P, DIR, FOLD ? threadIdx.x : 0);
-        src_b[threadIdx.x] = reinterpret_cast<T *>(ls == n ? P.tmp : P.A + ls * P.N * EB);
-        dst_b[threadIdx.x] = reinterpret_cast<T *>(ld == n ? P.tmp : P.A + ld * P.N * EB);
+        src_b[threadIdx.x] = reinterpret_cast<T *>(ls == n ? tmpm : Am + ls * P.N * EB);
+        dst_b[threadIdx.x] = reinterpret_cast<T *>(ld == n ? tmpm : Am + ld * P.N * EB);
     }
     // Without folding one base serves the whole row (kept in registers).
     const int32_t l0 = sk_src_loc(P, DIR, 0), d0 = sk_dst_loc(P, DIR, 0);
-    T *const src0 = reinterpret_cast<T *>(l0 == n ? P.tmp : P.A + l0 * P.N * EB);
-    T *const dst0 = reinterpret_cast<T *>(d0 == n ? P.tmp : P.A + d0 * P.N * EB);
+    T *const src0 = reinterpret_cast<T *>(l0 == n ? tmpm : Am + l0 * P.N * EB);
+    T *const dst0 = reinterpret_cast<T *>(d0 == n ? tmpm : Am + d0 * P.N * EB);
     auto srcb = [&](int64_t x) -> T * {
         return FOLD ? src_b[fdiv(static_cast<uint32_t>(x), P.fd_b)] : src0;
     };
@@ -171,8 +176,9 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
     const uint32_t sbuf = static_cast<uint32_t>(__cvta_generic_to_shared(buf));
     const int n = P.n, C = P.C;
     const int64_t pitch = P.N;  // in elements
-    T *A = reinterpret_cast<T *>(P.A);
-    T *tmp = reinterpret_cast<T *>(P.tmp);
+    // batches: matrix blockIdx.y of the launch, its own tmp row
+    T *A = reinterpret_cast<T *>(P.A + static_cast<int64_t>(blockIdx.y) * P.mat_stride);
+    T *tmp = reinterpret_cast<T *>(P.tmp + static_cast<int64_t>(blockIdx.y) * P.tmp_stride);
     if (threadIdx.x < 32) qinv_s[threadIdx.x] = P.qinv[threadIdx.x];
     for (int64_t j0 = static_cast<int64_t>(blockIdx.x) * C; j0 < P.N; j0 += static_cast<int64_t>(gridDim.x) * C) {
         const int32_t cols = static_cast<int32_t>(min(static_cast<int64_t>(C), P.N - j0));
@@ -250,8 +256,9 @@ cudaError_t launch_col_t(const SkinnyColParams &P, cudaStream_t st) {
     const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), kSkThreads, smem);
     if (resident < 1) return cudaErrorInvalidConfiguration;
     const int64_t blocks = (P.N + P.C - 1) / P.C;
-    const int64_t grid = blocks < 4 * static_cast<int64_t>(resident) ? blocks : 4 * static_cast<int64_t>(resident);
-    kern<<<static_cast<unsigned>(grid), kSkThreads, smem, st>>>(P);
+    const int64_t per = std::max<int64_t>(1, (4 * static_cast<int64_t>(resident) + P.batch - 1) / P.batch);
+    const int64_t grid = blocks < per ? blocks : per;  // ~4 waves of CTAs over the whole batch
+    kern<<<dim3(static_cast<unsigned>(grid), static_cast<unsigned>(P.batch)), kSkThreads, smem, st>>>(P);
     return cudaGetLastError();
 }
 
@@ -275,8 +282,9 @@ cudaError_t launch_t(const SkinnyRowParams &P, cudaStream_t st) {
     if (resident < 1) return cudaErrorInvalidConfiguration;
     const int64_t L = static_cast<int64_t>(P.n) * P.T;
     const int64_t wins = (P.N + L - 1) / L;
-    const int64_t grid = wins < 4 * static_cast<int64_t>(resident) ? wins : 4 * static_cast<int64_t>(resident);
-    kern<<<static_cast<unsigned>(grid), kSkThreads, smem, st>>>(P);
+    const int64_t per = std::max<int64_t>(1, (4 * static_cast<int64_t>(resident) + P.batch - 1) / P.batch);
+    const int64_t grid = wins < per ? wins : per;
+    kern<<<dim3(static_cast<unsigned>(grid), static_cast<unsigned>(P.batch)), kSkThreads, smem, st>>>(P);
     return cudaGetLastError();
 }
 

@@ -70,8 +70,11 @@ __global__ void __launch_bounds__(kRegThreads) skinny_reg_kernel(SkinnyRowParams
     const int nblk = FOLD ? P.c : 1;
     if (threadIdx.x < nblk) {
         const int32_t ls = loc_src(P, DIR, threadIdx.x), ld = loc_dst(P, DIR, threadIdx.x);
-        s_src[threadIdx.x] = reinterpret_cast<uint32_t *>(ls == P.n ? P.tmp : P.A + ls * P.N * 4);
-        s_dst[threadIdx.x] = reinterpret_cast<uint32_t *>(ld == P.n ? P.tmp : P.A + ld * P.N * 4);
+        // batches: matrix blockIdx.y of the launch, its own tmp row
+        char *const Am = P.A + static_cast<int64_t>(blockIdx.y) * P.mat_stride;
+        char *const tmpm = P.tmp + static_cast<int64_t>(blockIdx.y) * P.tmp_stride;
+        s_src[threadIdx.x] = reinterpret_cast<uint32_t *>(ls == P.n ? tmpm : Am + ls * P.N * 4);
+        s_dst[threadIdx.x] = reinterpret_cast<uint32_t *>(ld == P.n ? tmpm : Am + ld * P.N * 4);
     }
     __syncthreads();
     auto blk = [&](int64_t x) -> int32_t {
@@ -170,9 +173,10 @@ cudaError_t launch_s(const SkinnyRowParams &P, cudaStream_t st) {
     if (resident < 1) return cudaErrorInvalidConfiguration;
     const int64_t warps = (P.N / S + 31) / 32;
     int64_t grid = (warps * 32 + kRegThreads - 1) / kRegThreads;
-    if (grid > resident) grid = resident;
+    const int64_t per = (resident + P.batch - 1) / P.batch;
+    if (grid > per) grid = per;
     if (grid < 1) grid = 1;
-    kern<<<static_cast<unsigned>(grid), kRegThreads, 0, st>>>(P);
+    kern<<<dim3(static_cast<unsigned>(grid), static_cast<unsigned>(P.batch)), kRegThreads, 0, st>>>(P);
     return cudaGetLastError();
 }
 

@@ -99,3 +99,32 @@ def test_config3_full_size_sampled(n):
         assert got[l] == host[si * n + sj]
     ipt.soa_to_aos(x, count, n, field_bytes=4)
     assert torch.equal(x, to_dev(host))
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+@pytest.mark.parametrize("fold", ["1", "0"])
+def test_batched_one_launch_per_pass(eb, fold):
+    """Skinny engine on a batch (ipt_c2r_batched / ipt_r2c_batched with a skinny shape): every
+    pass is ONE launch over the batch (gridDim.y = matrix, a tmp row per matrix), packed and
+    gapped strides, odd and even field counts (rotation folded or separate), compared in full;
+    the launch count is that of one matrix."""
+    with skinny_min(1000), fuse_rot(fold):
+        for (count, n) in [(4099, 3), (4096, 6), (3001, 8)]:
+            for gap in (0, 5):
+                batch, stride = 4, count * n + gap
+                host = workloads.random_words(batch * stride, eb, seed=count + n + gap)
+                hv = np.ascontiguousarray(host).view(np.dtype((np.void, eb))).reshape(-1)
+                x = to_dev(host)
+                assert ipt.plan_info(count, n, eb)["engine"] == "skinny"
+                l0 = ipt.launch_count()
+                ipt.c2r_batched(x, batch, stride, count, n, elem_bytes=eb)
+                torch.cuda.synchronize()
+                launches = ipt.launch_count() - l0
+                assert launches == ipt.plan_info(count, n, eb)["launches"], launches
+                got = x.cpu().numpy().view(np.uint8).view(np.dtype((np.void, eb))).reshape(-1)
+                for k in range(batch):
+                    o = k * stride
+                    assert got[o:o + count * n].tobytes() == oracle.transpose(hv[o:o + count * n], count, n).tobytes()
+                    assert got[o + count * n:o + stride].tobytes() == hv[o + count * n:o + stride].tobytes()
+                ipt.r2c_batched(x, batch, stride, count, n, elem_bytes=eb)
+                assert x.cpu().numpy().tobytes() == np.ascontiguousarray(host).tobytes()
