@@ -834,8 +834,17 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
         }
         return s;
     }
-    // Column-pass counters, fused-rotation flags + ticket: zeroed in stream order.
-    if (cs.zero_bytes && (s = check(cudaMemsetAsync(scratch, 0, cs.zero_bytes, st))) != IPT_OK) return s;
+    // Column-pass counters, fused-rotation flags + ticket: zeroed in stream order -- by the row
+    // kernel when a pipelined / chunked C2R row pass is the call's first kernel (the counters
+    // are then its only zeroed state), else by a memset.
+    const bool row_zeroes = pl.engine == ENG_C2R && !pl.has_rot && pl.row.pipe && !pl.row.cl_K &&
+                            (!pl.row.fuse || pl.row.chunk) && env_int("IPT_DEBUG_PASSES", 1 << 30) >= (1 << 30);
+    if (row_zeroes) {
+        pl.row.zero = reinterpret_cast<unsigned int *>(scratch + cs.ctr_shuf);
+        pl.row.zero_words = static_cast<int32_t>(cs.zero_bytes / 4);
+    } else if (cs.zero_bytes && (s = check(cudaMemsetAsync(scratch, 0, cs.zero_bytes, st))) != IPT_OK) {
+        return s;
+    }
     pl.shuf.p.ctr = reinterpret_cast<unsigned int *>(scratch + cs.ctr_shuf);
     pl.rot.p.ctr = reinterpret_cast<unsigned int *>(scratch + cs.ctr_rot);
     pl.shuf.p.ticket = pl.rot.p.ticket = env_int("IPT_COL_TICKET", 1) != 0 ? 1 : 0;

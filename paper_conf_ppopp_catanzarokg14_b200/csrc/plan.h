@@ -120,6 +120,10 @@ struct RowParams {
     FastDiv fd_nch;
     char *bnd;               // boundary rows: bnd_row()
     int64_t rpitch;          // bytes per boundary row slot (N eb rounded up to 16, + 16)
+    // C2R calls whose first pass is this row pass: CTA 0 zeroes the column pass's counters
+    // (zero_words words at `zero`), which saves the call's memset (api.cu launch_call).
+    unsigned int *zero;
+    int32_t zero_words;
 };
 constexpr int kMaxFuseC = 32;
 

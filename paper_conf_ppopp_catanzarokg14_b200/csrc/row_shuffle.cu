@@ -1014,6 +1014,8 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_pipe_kerne
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
+    if (P.zero && blockIdx.x == 0)
+        for (int32_t k = threadIdx.x; k < P.zero_words; k += blockDim.x) P.zero[k] = 0u;
     // Row groups in grid-stride order: CTA blockIdx.x takes groups blockIdx.x + k gridDim.x
     // (producer and consumers walk the same sequence).
     auto mat_base = [&](const RowGroup &G) { return P.base + G.mat * P.mat_stride_bytes; };
@@ -1123,6 +1125,8 @@ __global__ void __launch_bounds__(NW * 32 + 32, NW == 16 ? 2 : 4) row_chunk_kern
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
+    if (P.zero && blockIdx.x == 0)
+        for (int32_t k = threadIdx.x; k < P.zero_words; k += blockDim.x) P.zero[k] = 0u;
     // The (chunk, group) sequence of this CTA -- walked identically by producer and consumers.
     struct Seq {
         int64_t ch, mat;
