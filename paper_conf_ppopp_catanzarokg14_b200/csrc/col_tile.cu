@@ -674,7 +674,7 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(const __grid_cons
             for (int u = 0;; ++u) {
                 if (k > 0) {  // take unit u's ticket once unit u-NB is released: its buffer then
                     // frees unconditionally (the workers only have to store it)
-                    while (*reinterpret_cast<volatile int *>(&s_release) < u - NB + 1) __nanosleep(32);
+                    while (atomicAdd(&s_release, 0) < u - NB + 1) __nanosleep(32);  // (atomic: no data race)
                 }
                 const uint32_t t = atomicAdd(P.ctr + kTicketSlot, 1u);
                 if (k > 0) mbar_wait(&bar_empty[b], (k - 1) & 1);
@@ -707,7 +707,7 @@ __global__ void __launch_bounds__(kColThreads) col_pipe_kernel(const __grid_cons
                         mbar_arrive(&bar_go[rb]);
                         ++release;
                         if (++rb == NB) rb = 0;
-                        *reinterpret_cast<volatile int *>(&s_release) = release;
+                        atomicExch(&s_release, release);
                         progress = true;
                     }
                 }
