@@ -531,7 +531,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_TMA_SUPER", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_SKINNY_COLBYTES", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -621,22 +621,30 @@ EncodeTiledFn encode_tiled() {
 }
 
 // u32 view of rows of `row_bytes` at `base`, rows `pitch` apart, matrices `mstride` apart
-// (rank 3; rank 2 over `rows` rows when mstride == 0); box {32 u32 = 128 B, box_rows(, 1)}.
+// (rank 3; rank 2 when mstride == 0), grouped in super-rows of g rows (g pitch a multiple of
+// 16): dims {((g - 1) pitch + row_bytes) / 4, rows / g(, batch)}, box {32 u32 = 128 B,
+// box_rows(, 1)}.
 bool make_map(CUtensorMap *m, const char *base, int64_t row_bytes, int64_t rows, int64_t pitch, int64_t batch,
-              int64_t mstride, uint32_t box_rows) {
+              int64_t mstride, uint32_t box_rows, int g) {
     EncodeTiledFn enc = encode_tiled();
-    if (!enc || reinterpret_cast<uintptr_t>(base) % 16 || pitch % 16 || (mstride && mstride % 16)) return false;
-    const cuuint64_t dims[3] = {static_cast<cuuint64_t>(row_bytes / 4), static_cast<cuuint64_t>(rows),
-                                static_cast<cuuint64_t>(batch)};
-    const cuuint64_t strides[2] = {static_cast<cuuint64_t>(pitch), static_cast<cuuint64_t>(mstride)};
+    if (!enc || reinterpret_cast<uintptr_t>(base) % 16 || (g * pitch) % 16 || pitch % 4 || (mstride && mstride % 16))
+        return false;
+    const cuuint64_t dims[3] = {static_cast<cuuint64_t>(((g - 1) * pitch + row_bytes) / 4),
+                                static_cast<cuuint64_t>(rows / g), static_cast<cuuint64_t>(batch)};
+    const cuuint64_t strides[2] = {static_cast<cuuint64_t>(g * pitch), static_cast<cuuint64_t>(mstride)};
     const cuuint32_t box[3] = {32, box_rows, 1};
     const cuuint32_t estr[3] = {1, 1, 1};
     const cuuint32_t rank = mstride ? 3 : 2;
-    if (dims[0] >= (cuuint64_t(1) << 32) || dims[1] >= (cuuint64_t(1) << 32) || dims[2] >= (cuuint64_t(1) << 32))
+    if (dims[1] == 0 || dims[0] >= (cuuint64_t(1) << 32) || dims[1] >= (cuuint64_t(1) << 32) ||
+        dims[2] >= (cuuint64_t(1) << 32))
         return false;
     return enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT32, rank, const_cast<char *>(base), dims, strides, box, estr,
                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+int super_rows(int64_t pitch) {  // g = 16 / gcd(pitch, 16) for a pitch that is a multiple of 4
+    return pitch % 16 == 0 ? 1 : pitch % 8 == 0 ? 2 : 4;
 }
 
 // Enable TMA staging for a shuffle / rotation pass where the layout allows (128-byte tiles,
@@ -653,16 +661,26 @@ void setup_col_tma(ColParams &p, int mode, int eb) {
     const bool packed = p.batch == 1 || p.mat_stride_bytes == static_cast<int64_t>(p.M) * pitch;
     if (mode == COL_R2C_SHUF) {
         if ((allow & 4) && packed &&
-            make_map(&p.tmap_g, p.base, pitch, static_cast<int64_t>(p.M) * p.batch, pitch, 1, 0, 1))
+            make_map(&p.tmap_g, p.base, pitch, static_cast<int64_t>(p.M) * p.batch, pitch, 1, 0, 1, 1))
             p.tma |= 4;
         return;
     }
     if (!(allow & 1)) return;
-    const int64_t ms = p.batch == 1 ? static_cast<int64_t>(p.M) * pitch : p.mat_stride_bytes;
-    if (make_map(&p.tmap_a, p.base, pitch, p.M, pitch, p.batch, ms, kTmaBoxRows)) p.tma |= 1;
+    // any pitch (super-rows) unless IPT_COL_TMA_SUPER=0 restricts to 16-byte pitches
+    const bool any_pitch = env_int("IPT_COL_TMA_SUPER", 1) != 0;
+    p.tg_a = super_rows(pitch);
+    if (p.tg_a > 1 && !any_pitch) return;
+    p.trows_a = p.M / p.tg_a * p.tg_a;
+    // (rank 3 always -- the kernel issues 3-D boxes; one matrix: any 16-byte multiple serves)
+    const int64_t ms = p.batch == 1 ? ((static_cast<int64_t>(p.M) * pitch + 15) & ~int64_t(15)) : p.mat_stride_bytes;
+    if (make_map(&p.tmap_a, p.base, pitch, p.M, pitch, p.batch, ms, kTmaBoxRows, p.tg_a)) p.tma |= 1;
     if ((allow & 2) && mode == COL_C2R_SHUF && p.lag == LAG_C2R && p.side && (p.tma & 1)) {  // (aligned matrix bases)
         const char *s0 = side_matrix(p.side, p.sstride, 0, p.base);
-        if (make_map(&p.tmap_s, s0, static_cast<int64_t>(p.lagD) * 128, p.M, p.spitch, p.batch, p.sstride, kTmaBoxRows))
+        p.tg_s = super_rows(p.spitch);
+        p.trows_s = p.M / p.tg_s * p.tg_s;
+        if ((p.tg_s == 1 || any_pitch) &&
+            make_map(&p.tmap_s, s0, static_cast<int64_t>(p.lagD) * 128, p.M, p.spitch, p.batch, p.sstride,
+                     kTmaBoxRows, p.tg_s))
             p.tma |= 2;
     }
 }

@@ -92,7 +92,9 @@ __host__ __device__ inline SmemLayout smem_layout(int64_t B, int W, int twb, int
     // cp.async hulls: nslots x (TWB + 16); TMA: whole boxes of kTmaBoxRows x TWB (+ 3 slots of
     // gather4 padding)
     const size_t hull = nslots * static_cast<size_t>(hull_pitch(twb));
-    const size_t tma = ((nslots + 3 + kTmaBoxRows - 1) / kTmaBoxRows) * kTmaBoxRows * static_cast<size_t>(twb);
+    // (up to 4 phases of super-rows, each rounded up to whole boxes)
+    const size_t tma = (((nslots + 3 + kTmaBoxRows - 1) / kTmaBoxRows) * kTmaBoxRows + 4 * kTmaBoxRows) *
+                       static_cast<size_t>(twb);
     L.total = o + (hull > tma ? hull : tma) + 128;
     return L;
 }
@@ -443,14 +445,14 @@ __device__ __forceinline__ int tma_kind(const ColParams &P, const Unit &U, uint3
         return 3;
     }
     if (MODE != COL_C2R_SHUF && MODE != COL_ROT) return 0;
-    if (U.rowbase + U.nslots > P.M) return 0;  // rows wrap past M - 1: cp.async
     (void)mat;
+    // rows wrapping past M - 1, or in the last partial super-row: cp.async
     if (MODE == COL_C2R_SHUF && P.lag == LAG_C2R && tile < P.lagD) {
-        if (!(P.tma & 2)) return 0;
+        if (!(P.tma & 2) || U.rowbase + U.nslots > P.trows_s) return 0;
         xcoord = tile * TWB / 4;
         return 2;
     }
-    if (!(P.tma & 1)) return 0;
+    if (!(P.tma & 1) || U.rowbase + U.nslots > P.trows_a) return 0;
     xcoord = (U.j0 - (MODE == COL_C2R_SHUF && P.lag == LAG_C2R ? P.lagD * (TWB / EB) : 0)) * EB / 4;
     return 1;
 }
@@ -462,9 +464,9 @@ __device__ __forceinline__ void unit_load_tma(const ColParams &P, const Unit &U,
                                               const int32_t *srow, uint32_t *sbase, uint32_t rows_s, uint64_t *bar) {
     const uint32_t mat = fdiv(tt, P.fd_nt);
     const int lane = threadIdx.x & 31;
-    for (int32_t t = threadIdx.x; t < U.nslots; t += blockDim.x) sbase[t] = rows_s + static_cast<uint32_t>(t) * TWB;
-    if (threadIdx.x >= 32) return;
     if (kind == 3) {
+        for (int32_t t = threadIdx.x; t < U.nslots; t += blockDim.x) sbase[t] = rows_s + static_cast<uint32_t>(t) * TWB;
+        if (threadIdx.x >= 32) return;
         const int32_t ng = (U.nslots + 3) / 4;
         if (lane == 0) tmbar_expect(bar, static_cast<uint32_t>(ng) * 4 * TWB);
         __syncwarp();
@@ -477,13 +479,38 @@ __device__ __forceinline__ void unit_load_tma(const ColParams &P, const Unit &U,
             tma_gather4(rows_s + static_cast<uint32_t>(t0) * TWB, &P.tmap_g, xcoord, r[0], r[1], r[2], r[3], bar);
         }
     } else {
-        const int32_t nb = (U.nslots + kTmaBoxRows - 1) / kTmaBoxRows;
-        if (lane == 0) tmbar_expect(bar, static_cast<uint32_t>(nb) * kTmaBoxRows * TWB);
+        // Super-rows of g rows (g = 1 when the pitch is a multiple of 16): slot t (row rowbase
+        // + t) has phase p = row mod g; the slots of phase p, t_p, t_p + g, ..., come from the
+        // boxes of phase p (x shifted by p rows' worth of bytes, y = super-row) and sit in
+        // their own region of whole boxes, R_p.
+        const int g = kind == 2 ? P.tg_s : P.tg_a;
+        const int64_t pitch = kind == 2 ? P.spitch : static_cast<int64_t>(P.N) * EB;
+        int32_t tp[4], reg[4], nbx[4];
+        int32_t acc = 0;
+#pragma unroll
+        for (int p = 0; p < 4; ++p) {
+            if (p >= g) break;
+            tp[p] = ((p - U.rowbase) % g + g) % g;
+            const int32_t np = U.nslots > tp[p] ? (U.nslots - tp[p] + g - 1) / g : 0;
+            nbx[p] = (np + kTmaBoxRows - 1) / kTmaBoxRows;
+            reg[p] = acc;
+            acc += nbx[p] * kTmaBoxRows;
+        }
+        for (int32_t t = threadIdx.x; t < U.nslots; t += blockDim.x) {
+            const int p = (U.rowbase + t) % g;
+            sbase[t] = rows_s + static_cast<uint32_t>(reg[p] + (t - tp[p]) / g) * TWB;
+        }
+        if (threadIdx.x >= 32) return;
+        if (lane == 0) tmbar_expect(bar, static_cast<uint32_t>(acc) * TWB);
         __syncwarp();
         const CUtensorMap *map = kind == 2 ? &P.tmap_s : &P.tmap_a;
-        for (int32_t bi = lane; bi < nb; bi += 32)
-            tma_box3(rows_s + static_cast<uint32_t>(bi * kTmaBoxRows) * TWB, map, xcoord, U.rowbase + bi * kTmaBoxRows,
-                     static_cast<int32_t>(mat), bar);
+        for (int p = 0; p < g; ++p) {
+            const int32_t x = xcoord + static_cast<int32_t>(p * pitch / 4);
+            const int32_t s0 = (U.rowbase + tp[p]) / g;  // first super-row of phase p
+            for (int32_t bi = lane; bi < nbx[p]; bi += 32)
+                tma_box3(rows_s + static_cast<uint32_t>(reg[p] + bi * kTmaBoxRows) * TWB, map, x, s0 + bi * kTmaBoxRows,
+                         static_cast<int32_t>(mat), bar);
+        }
     }
 }
 

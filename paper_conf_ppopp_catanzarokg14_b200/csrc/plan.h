@@ -127,15 +127,20 @@ struct RowParams {
 };
 constexpr int kMaxFuseC = 32;
 
-// TMA staging of the column pass (pitch a multiple of 16 bytes): 2-D tiles of kTmaBoxRows
-// rows x 128 bytes (A and side block, 3-D maps over the batch) and R2C row gathers of 4 rows
-// (tile::gather4, a 2-D map over all rows; batches packed only).
+// TMA staging of the column pass: 2-D tiles of kTmaBoxRows rows x 128 bytes (A and side
+// block, 3-D maps over the batch; any pitch, via super-rows) and R2C row gathers of 4 rows
+// (tile::gather4, a 2-D map over all rows, 16-byte pitches; batches packed only).
 constexpr int kTmaBoxRows = 16;
 struct ColParams {
     CUtensorMap tmap_a;   // 3-D {N eb / 4, M, batch} u32, box {32, kTmaBoxRows, 1}
     CUtensorMap tmap_s;   // 3-D {spitch / 4, M, batch} u32 over the side block (lagged C2R input)
     CUtensorMap tmap_g;   // 2-D {N eb / 4, M batch} u32, box {32, 1} (gather4)
     int32_t tma;          // bit 0: box loads of A; bit 1: box loads of the side block; bit 2: gather4
+    // Super-rows: rows of a pitch that is not a multiple of 16 bytes are grouped g at a time
+    // (g = 16 / gcd(pitch, 16)), so that the map's row pitch g pitch is; a box at x = (phase
+    // pitch + column bytes) / 4 then loads every g-th row of one phase.  Rows of whole
+    // super-rows only (trows = g floor(M / g)).
+    int32_t tg_a, tg_s, trows_a, trows_s;
     char *base;
     int64_t mat_stride_bytes;
     int64_t batch;
