@@ -635,8 +635,9 @@ bool make_map(CUtensorMap *m, const char *base, int64_t row_bytes, int64_t rows,
     const cuuint32_t box[3] = {32, box_rows, 1};
     const cuuint32_t estr[3] = {1, 1, 1};
     const cuuint32_t rank = mstride ? 3 : 2;
-    if (dims[1] == 0 || dims[0] >= (cuuint64_t(1) << 32) || dims[1] >= (cuuint64_t(1) << 32) ||
-        dims[2] >= (cuuint64_t(1) << 32))
+    // at least one whole box in each dimension (small matrices keep cp.async)
+    if (dims[0] < box[0] || dims[1] < box[1] || dims[0] >= (cuuint64_t(1) << 32) ||
+        dims[1] >= (cuuint64_t(1) << 32) || dims[2] >= (cuuint64_t(1) << 32))
         return false;
     return enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT32, rank, const_cast<char *>(base), dims, strides, box, estr,
                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,

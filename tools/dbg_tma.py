@@ -20,3 +20,12 @@ for (m, n) in [(8, 8), (12, 20), (33, 64), (64, 64), (1200, 1800), (2000, 3000),
             except Exception as e2:
                 print("sync:", e2)
             sys.exit(1)
+# degenerate / tiny shapes (TMA maps smaller than a box must fall back)
+for (m, n) in [(1000, 10), (10, 1000), (2, 3000), (3000, 2), (4096, 64), (64, 4096), (1023, 1024), (1000, 12), (12, 1000)]:
+    for eb in (4, 8, 16):
+        x = torch.randint(0, 2**31 - 1, (m * n * eb // 4,), dtype=torch.int32, device="cuda")
+        h = x.cpu().numpy().copy()
+        ipt.c2r(x, m, n, elem_bytes=eb)
+        torch.cuda.synchronize()
+        want = oracle.transpose(h.view(np.dtype((np.void, eb))), m, n)
+        print(m, n, eb, "ok" if x.cpu().numpy().tobytes() == want.tobytes() else "MISMATCH", flush=True)
