@@ -667,8 +667,11 @@ void setup_col_tma(ColParams &p, int mode, int eb) {
         return;
     }
     if (!(allow & 1)) return;
-    // any pitch (super-rows) unless IPT_COL_TMA_SUPER=0 restricts to 16-byte pitches
-    const bool any_pitch = env_int("IPT_COL_TMA_SUPER", 1) != 0;
+    // 16-byte pitches only.  (Super-rows of g rows would make any pitch a multiple of 16, but
+    // their per-phase boxes start at x = p pitch / 4, not 16-byte aligned, and the TMA unit
+    // faults on such boxes -- cudaErrorIllegalInstruction on 1024 x 1023 fp32, gpurun_out
+    // r02aa; IPT_COL_TMA_SUPER=1 keeps that path for experiments.)
+    const bool any_pitch = env_int("IPT_COL_TMA_SUPER", 0) != 0;
     p.tg_a = super_rows(pitch);
     if (p.tg_a > 1 && !any_pitch) return;
     p.trows_a = p.M / p.tg_a * p.tg_a;
