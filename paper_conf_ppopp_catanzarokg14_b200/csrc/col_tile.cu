@@ -235,29 +235,7 @@ __device__ __forceinline__ void unit_load_t(const ColParams &P, const Unit &U, c
             }
         }
     };
-    if (MODE == COL_R2C_SHUF && P.qinc) {
-        // Source rows q^{-1}(i), i = (r0 - W + 1 + t - j0) mod M, stepped per lane (Eq. 34):
-        // with u = (c - 1 + i) mod c and w = floor((c - 1 + i) / c) b^{-1} mod a,
-        // q^{-1}(i) = w + (c - 1 - u) a; i -> i + step moves u by step mod c (one carry into
-        // floor) and w by floor(step / c) b^{-1} mod a (+ b^{-1} on the carry); i -> i - M
-        // leaves (u, w) unchanged (a b^{-1} = 0 mod a), so the walk never needs the mod M.
-        const int64_t i0 = mod_M(U.r0 - (TWB / EB - 1) + t - U.j0m, P.kshM, P.fd_M);
-        const int64_t v0 = (P.c - 1 + i0) / P.c;
-        int32_t u = static_cast<int32_t>((P.c - 1 + i0) - v0 * P.c);
-        int32_t w = static_cast<int32_t>(((v0 % P.a) * P.binv) % P.a);
-        const int32_t du = step % P.c;
-        const int32_t dw = static_cast<int32_t>(((static_cast<int64_t>(step / P.c) % P.a) * P.binv) % P.a);
-        for (; t < U.nslots; t += step, dst += dst_inc, sb += step) {
-            const int32_t q = w + (P.c - 1 - u) * P.a;
-            issue(U.inp + static_cast<int64_t>(q) * pitch + c16);
-            u += du;
-            const bool carry = u >= P.c;
-            u -= carry ? P.c : 0;
-            w += dw + (carry ? P.binv : 0);
-            w -= w >= P.a ? P.a : 0;
-            w -= w >= P.a ? P.a : 0;
-        }
-    } else if (MODE == COL_R2C_SHUF) {
+    if (MODE == COL_R2C_SHUF) {
         for (; t < U.nslots; t += step, dst += dst_inc, sb += step) issue(U.inp + static_cast<int64_t>(srow[t]) * pitch + c16);
     } else if (step <= P.M) {
         // contiguous (cyclic) input rows rowbase + t: incremental row index and pointer
@@ -556,7 +534,7 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     }
     // R2C: the loads need the scattered source rows (prepass first); otherwise the loads go
     // out first and the C2R destination rows are computed while they are in flight.
-    if (MODE == COL_R2C_SHUF && !P.qinc) {  // (the gather4 path reads srow[])
+    if (MODE == COL_R2C_SHUF) {
         if (P.dbg != 4) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
         __syncthreads();
     }
