@@ -521,7 +521,7 @@ __device__ __forceinline__ void unit_load_tma(const ColParams &P, const Unit &U,
 // groups finish.  G == 1: P.tpc consecutive tiles per CTA.
 template <int EB, int MODE, int TWB>
 __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *smem, uint32_t tt, int32_t r,
-                                             uint64_t *tbar, uint32_t &tphase) {
+                                             uint64_t *tbar, uint32_t &tphase, unsigned int *next_ticket = nullptr) {
     const SmemLayout L = smem_layout(P.B, TWB / EB, TWB, EB);
     int64_t *orow = reinterpret_cast<int64_t *>(smem);
     int32_t *srow = reinterpret_cast<int32_t *>(smem + L.srow);
@@ -530,6 +530,7 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     const Dep D = unit_dep<MODE>(P, tt);
     if (U.skip) {  // group-uniform; still arrive, later tiles sharing the counter count it
         if (D.arrive && threadIdx.x == 0) atomicAdd(P.ctr + (tt % kCtrSlots), 1u);
+        if (next_ticket && threadIdx.x == 0) *next_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
         return;
     }
     // R2C: the loads need the scattered source rows (prepass first); otherwise the loads go
@@ -569,6 +570,9 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
         }
         if (D.wait && P.dbg != 5)
             while (!ctr_reached(P, D.on)) __nanosleep(64);
+        // persistent grid: the next unit's ticket, taken now so that its latency overlaps
+        // the stores (this unit has arrived, so every ticket it could wait for is smaller)
+        if (next_ticket) *next_ticket = atomicAdd(P.ctr + kTicketSlot, 1u);
     }
     __syncthreads();
     if (P.dbg == 0 || P.dbg == 7) unit_store<EB, MODE, TWB>(P, U, orow, sbase, blockDim.x);  // 1, 3, 4, 5 = loads only
@@ -602,6 +606,35 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(const __grid_cons
         for (uint64_t tt = static_cast<uint64_t>(ticket) * P.tpc; tt < t_end; ++tt) {
             col_tile_one<EB, MODE, TWB>(P, smem, static_cast<uint32_t>(tt), 0, &tbar, tphase);
             __syncthreads();  // shared memory is reused by the next tile
+        }
+        return;
+    }
+    auto unit_of = [&](unsigned int tk, uint32_t &tt, int32_t &r) {
+        if (P.lag != LAG_NONE && P.super > 1) {
+            const uint32_t per = static_cast<uint32_t>(P.G) * static_cast<uint32_t>(P.super);
+            const uint32_t sidx = tk / per, rem = tk - sidx * per;
+            const uint32_t t0 = sidx * static_cast<uint32_t>(P.super);
+            const uint32_t here = min(static_cast<uint32_t>(P.super), static_cast<uint32_t>(P.total_tiles) - t0);
+            r = static_cast<int32_t>(rem / here);
+            tt = t0 + (rem - static_cast<uint32_t>(r) * here);
+        } else {
+            tt = fdiv(tk, P.fd_G);
+            r = static_cast<int32_t>(tk - tt * P.G);
+        }
+    };
+    if (P.persist) {
+        // Persistent grid (lagged layouts): resident CTAs loop over tickets, each unit's
+        // successor taken during its stores.  Waits still only target smaller tickets, held
+        // by running CTAs whose loads wait on nothing (col_tile_one).
+        __shared__ unsigned int s_next;
+        const uint32_t total = static_cast<uint32_t>(P.total_tiles) * static_cast<uint32_t>(P.G);
+        while (ticket < total) {
+            uint32_t ptt;
+            int32_t pr;
+            unit_of(ticket, ptt, pr);
+            col_tile_one<EB, MODE, TWB>(P, smem, ptt, pr, &tbar, tphase, &s_next);
+            __syncthreads();  // stores done (shared memory reused), s_next published
+            ticket = s_next;
         }
         return;
     }
@@ -850,8 +883,8 @@ cudaError_t launch_col(const ColParams &P0, int mode, int eb, cudaStream_t st, s
     ColParams P = P0;
     const int64_t units = P.total_tiles * P.G;
     if (units > 0xfffffff0LL) return cudaErrorInvalidConfiguration;
-    const int64_t grid = P.pipe ? std::min<int64_t>(P.resident, units)
-                                : P.G == 1 ? (P.total_tiles + P.tpc - 1) / P.tpc : units;
+    const int64_t grid = (P.pipe || P.persist) ? std::min<int64_t>(P.resident, units)
+                                               : P.G == 1 ? (P.total_tiles + P.tpc - 1) / P.tpc : units;
     if (grid > 0x7fffffffLL) return cudaErrorInvalidConfiguration;
     // Ticket + group counters: the call's own zeroed scratch (api.cu CallScratch).
     if (!P.ctr) return cudaErrorInvalidValue;
