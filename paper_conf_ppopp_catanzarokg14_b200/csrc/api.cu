@@ -888,7 +888,7 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
     pl.row.side = pl.shuf.p.side = pl.side_bytes ? scratch + cs.side : nullptr;
     setup_col_tma(pl.shuf.p, pl.engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.eb);
     pl.shuf.p.persist = pl.shuf.p.lag != LAG_NONE && pl.shuf.p.G > 1 && pl.shuf.p.ticket && !pl.shuf.p.pipe &&
-                        env_int("IPT_COL_PERSIST", 0) != 0 ? 1 : 0;
+                        env_int("IPT_COL_PERSIST", 1) != 0 ? 1 : 0;  // sweep: calls +3.1 %, R2C shuffles +13 % (r02ae)
     if (pl.has_rot) setup_col_tma(pl.rot.p, COL_ROT, pl.eb);
     const int64_t pitch = pl.N * pl.eb;
     const int passes = budget;
