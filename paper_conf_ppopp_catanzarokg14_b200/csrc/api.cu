@@ -531,7 +531,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_TMA_SUPER", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_TMA_SUPER", "IPT_COL_BULK", "IPT_COL_PERSIST", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_SKINNY_COLBYTES", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -887,6 +887,7 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
     }
     pl.row.side = pl.shuf.p.side = pl.side_bytes ? scratch + cs.side : nullptr;
     setup_col_tma(pl.shuf.p, pl.engine == ENG_C2R ? COL_C2R_SHUF : COL_R2C_SHUF, pl.eb);
+    pl.shuf.p.bulk = !pl.shuf.p.pipe && pl.shuf.p.W * pl.eb == 128 && env_int("IPT_COL_BULK", 0) != 0 ? 1 : 0;
     pl.shuf.p.persist = pl.shuf.p.lag != LAG_NONE && pl.shuf.p.G > 1 && pl.shuf.p.ticket && !pl.shuf.p.pipe &&
                         env_int("IPT_COL_PERSIST", 1) != 0 ? 1 : 0;  // sweep: calls +3.1 %, R2C shuffles +13 % (r02ae)
     if (pl.has_rot) setup_col_tma(pl.rot.p, COL_ROT, pl.eb);

@@ -514,6 +514,39 @@ __device__ __forceinline__ void unit_load_tma(const ColParams &P, const Unit &U,
     }
 }
 
+// Hull staging with 1-D bulk copies (P.bulk; any pitch, not the rightmost tile of a row):
+// one cp.async.bulk of a slot's 16-byte-aligned hull (128 or 144 bytes) per lane instead of
+// nine 16-byte cp.async; each issuing lane registers its bytes on `bar` (expect_tx), thread 0
+// arrives once every lane has issued (the caller's barrier), so the phase cannot complete
+// early.  Same slot layout as unit_load (hull pitch, sbase[t] = first tile element).
+__device__ __forceinline__ void tmbar_expect_only(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;"
+                 :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void tmbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];"
+                 :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar))) : "memory");
+}
+template <int EB, int MODE, int TWB>
+__device__ __forceinline__ void unit_load_bulk(const ColParams &P, const Unit &U, const int32_t *srow, uint32_t *sbase,
+                                               uint32_t rows_s, uint64_t *bar) {
+    constexpr int HS = hull_pitch(TWB);
+    const int64_t pitch = U.in_pitch;
+    const uint32_t bar_s = static_cast<uint32_t>(__cvta_generic_to_shared(bar));
+    const int32_t tb = U.wt * EB;
+    for (int32_t t = threadIdx.x; t < U.nslots; t += blockDim.x) {
+        const int32_t g = MODE == COL_R2C_SHUF ? srow[t] : mod_M(U.rowbase + t, P.kshM, P.fd_M);
+        const char *rp = U.inp + static_cast<int64_t>(g) * pitch;
+        const uint32_t off = static_cast<uint32_t>(reinterpret_cast<uintptr_t>(rp)) & 15u;
+        const uint32_t bytes = (off + static_cast<uint32_t>(tb) + 15u) & ~15u;
+        const uint32_t dst = rows_s + static_cast<uint32_t>(t) * HS;
+        sbase[t] = dst + off;
+        tmbar_expect_only(bar, bytes);
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                     :: "r"(dst), "l"(rp - off), "r"(bytes), "r"(bar_s) : "memory");
+    }
+}
+
 // Non-persistent variant: one CTA per (tile, band).  The CTA's logical id comes from a
 // ticket counter taken at start (dispatch order), so the G members of a tile are exactly
 // G consecutive tickets: every group whose tickets are all taken is fully resident, hence
@@ -542,16 +575,25 @@ __device__ __forceinline__ void col_tile_one(const ColParams &P, unsigned char *
     int32_t xcoord = 0;
     const int kind = tma_kind<EB, MODE, TWB>(P, U, tt, xcoord);
     const uint32_t rows_s = (static_cast<uint32_t>(__cvta_generic_to_shared(smem + L.rows)) + 127u) & ~127u;
+    // bulk hulls: not for the rightmost tile of a row (its hull may end past the buffer)
+    const bool bulk = !kind && P.bulk && !U.skip && U.j0 + U.wt < P.N && P.dbg != 2;
     if (kind) {
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // earlier generic reads of the buffer
         unit_load_tma<EB, MODE, TWB>(P, U, tt, kind, xcoord, srow, sbase, rows_s, tbar);
+    } else if (bulk) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        unit_load_bulk<EB, MODE, TWB>(P, U, srow, sbase, rows_s, tbar);
     } else if (P.dbg != 2) {  // measurement knob: 2 = skip the loads
         unit_load<EB, MODE, TWB>(P, U, srow, sbase, rows_s, blockDim.x);
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
     if (MODE != COL_R2C_SHUF && P.dbg != 4) unit_prepass<EB, MODE, TWB>(P, U, orow, srow, blockDim.x);
     asm volatile("cp.async.wait_group 0;" ::: "memory");
-    if (kind) {
+    if (bulk) {
+        __syncthreads();  // every lane has registered its bytes
+        if (threadIdx.x == 0) tmbar_arrive(tbar);
+    }
+    if (kind || bulk) {
         tmbar_wait(tbar, tphase);
         tphase ^= 1;
     }
@@ -583,7 +625,7 @@ __global__ void __launch_bounds__(kColThreads) col_tile_kernel(const __grid_cons
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ __align__(8) uint64_t tbar;  // TMA staging (P.tma)
     uint32_t tphase = 0;
-    if (P.tma) {
+    if (P.tma || P.bulk) {
         if (threadIdx.x == 0) tmbar_init(&tbar);
         __syncthreads();
     }

@@ -158,6 +158,7 @@ struct ColParams {
                         // stream-ordered scratch, zeroed before the launch (api.cu CallScratch)
     int32_t ticket;     // 1: units in dispatch-ticket order (an atomic per CTA); 0: block index
     int32_t persist;    // lagged layouts, G > 1: persistent grid of resident CTAs looping over tickets
+    int32_t bulk;       // hull staging with one 1-D bulk copy per slot (instead of 16-byte cp.async)
     int32_t super;      // lagged layouts: units ordered band-major within super-tiles of `super`
                         // consecutive tiles (<= lagD), so that concurrently running units read
                         // adjacent 128-byte segments of the same rows (1: tile-major)
