@@ -60,6 +60,8 @@ def lib() -> ctypes.CDLL:
         for name in ("oracle_c2r_source", "oracle_r2c_source"):
             getattr(L, name).restype = None
             getattr(L, name).argtypes = [_i64, _i64, _i64, _i64, ctypes.POINTER(_i64), ctypes.POINTER(_i64)]
+        L.oracle_source_many.restype = None
+        L.oracle_source_many.argtypes = [_i64, _i64, ctypes.c_int, _vp, _i64, _vp]
         for name in ("oracle_c2r_definition", "oracle_r2c_definition", "oracle_transpose"):
             getattr(L, name).restype = None
             getattr(L, name).argtypes = [_vp, _vp, _i64, _i64, ctypes.c_int]
@@ -109,6 +111,15 @@ def r2c_source(m, n, i, j):
     a, b = _i64(), _i64()
     lib().oracle_r2c_source(m, n, i, j, ctypes.byref(a), ctypes.byref(b))
     return int(a.value), int(b.value)
+
+
+def source_many(op: str, m: int, n: int, pos: np.ndarray) -> np.ndarray:
+    """Eqs. 7-10 vectorised: for linear destinations pos (i*n + j of the m x n array) the
+    linear source offsets of C2R (op="c2r", Eq. 11) or R2C (op="r2c", Eq. 12)."""
+    pos = np.ascontiguousarray(pos, dtype=np.int64)
+    out = np.empty_like(pos)
+    lib().oracle_source_many(m, n, 1 if op == "r2c" else 0, _ptr(pos), pos.size, _ptr(out))
+    return out
 
 
 def eq22_d(m, n, i, j): return int(lib().oracle_eq22_d(m, n, i, j))

@@ -800,3 +800,40 @@ def test_column_tma_staging(mask):
                 assert got[o:o + m * n].tobytes() == oracle.transpose(host[o:o + m * n], m, n).tobytes(), (packed, k)
             ipt.r2c_batched(x, batch, stride, m, n, elem_bytes=4)
             assert dev_bytes(x) == host.tobytes()
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+@pytest.mark.timeout(1800)
+def test_bench_sweep_calls_sampled_all(eb):
+    """Every call bench.py times (workloads.sweep_shapes(200) x c2r/r2c, BASELINE configs[1]),
+    in the launch configuration the bench uses. Shapes 0..47 are compared in full above; here
+    all 200 run on the index pattern (element l holds l) and each output is checked
+    (a) on 2^17 sampled destinations plus the first and last 4096, against the oracle's
+        Eqs. 7-10 (oracle.source_many), and
+    (b) in full by two properties that hold at any size: the result is a permutation of the
+        input (sum and sum of squares of the words unchanged, int64 wrap-around) and r2c
+        restores the input exactly."""
+    shapes = workloads.sweep_shapes(200)
+    dt = torch.int32 if eb == 4 else torch.int64
+    maxel = max(m * n for m, n in shapes)
+    rng = np.random.default_rng(eb)
+    base = torch.arange(maxel, dtype=torch.int64, device=DEV)
+    for k, (m, n) in enumerate(shapes):
+        total = m * n
+        x = base[:total].to(dt)
+        s1 = x.to(torch.int64).sum().item()
+        s2 = (x.to(torch.int64) * x.to(torch.int64)).sum().item()
+        for op in ("c2r", "r2c"):
+            if op == "r2c":
+                x = base[:total].to(dt)
+            pos = np.concatenate([np.arange(min(4096, total)), np.arange(max(0, total - 4096), total),
+                                  rng.integers(0, total, size=1 << 17)]).astype(np.int64)
+            getattr(ipt, op)(x, m, n, elem_bytes=eb)
+            got = x[torch.from_numpy(pos).to(DEV)].to(torch.int64).cpu().numpy()
+            want = oracle.source_many(op, m, n, pos)
+            bad = np.nonzero(got != want)[0]
+            assert bad.size == 0, (m, n, op, eb, int(pos[bad[0]]), int(got[bad[0]]), int(want[bad[0]]))
+            x64 = x.to(torch.int64)
+            assert x64.sum().item() == s1 and (x64 * x64).sum().item() == s2, (m, n, op, eb)
+            getattr(ipt, "r2c" if op == "c2r" else "c2r")(x, m, n, elem_bytes=eb)
+            assert torch.equal(x, base[:total].to(dt)), (m, n, op, eb, "round trip")

@@ -128,3 +128,31 @@ def test_batched_one_launch_per_pass(eb, fold):
                     assert got[o + count * n:o + stride].tobytes() == hv[o + count * n:o + stride].tobytes()
                 ipt.r2c_batched(x, batch, stride, count, n, elem_bytes=eb)
                 assert x.cpu().numpy().tobytes() == np.ascontiguousarray(host).tobytes()
+
+
+@pytest.mark.timeout(900)
+def test_config3_all_field_counts_sampled():
+    """Every call the bench's cfg3 key times: 2**26 structs x n = 2..32 4-byte fields,
+    aos_to_soa then soa_to_aos. Index pattern (word l holds l mod 2^32); 2^17 sampled
+    destinations plus the first and last 4096 checked against the oracle's Eqs. 7-8
+    (oracle.source_many, P_{count,n} = C2R(count, n)), the whole output checked to be a
+    permutation (sum and sum of squares), and the inverse checked to restore the input."""
+    count = 1 << 26
+    rng = np.random.default_rng(3)
+    base = torch.arange(count * 32, dtype=torch.int64, device="cuda")
+    for n in range(2, 33):
+        total = count * n
+        x = base[:total].to(torch.int32)
+        u = x.to(torch.int64) & 0xffffffff
+        s1, s2 = u.sum().item(), (u * u).sum().item()
+        ipt.aos_to_soa(x, count, n, field_bytes=4)
+        pos = np.concatenate([np.arange(4096), np.arange(total - 4096, total),
+                              rng.integers(0, total, size=1 << 17)]).astype(np.int64)
+        got = (x[torch.from_numpy(pos).cuda()].to(torch.int64) & 0xffffffff).cpu().numpy()
+        want = oracle.source_many("c2r", count, n, pos)
+        bad = np.nonzero(got != want)[0]
+        assert bad.size == 0, (n, int(pos[bad[0]]), int(got[bad[0]]), int(want[bad[0]]))
+        u = x.to(torch.int64) & 0xffffffff
+        assert u.sum().item() == s1 and (u * u).sum().item() == s2, n
+        ipt.soa_to_aos(x, count, n, field_bytes=4)
+        assert torch.equal(x, base[:total].to(torch.int32)), n

@@ -270,3 +270,17 @@ def test_aos_gather_scatter_against_numpy(S):
     ident = np.arange(nsrc, dtype=np.uint32)
     assert same(oracle.aos_gather(src, ident, S), src.reshape(-1))
     assert oracle.aos_gather(src, idx[:0], S).size == 0
+
+
+@pytest.mark.parametrize("m,n", [(1, 1), (1, 9), (9, 1), (6, 4), (7, 11), (12, 18), (64, 40), (1200, 1800)])
+def test_source_many_against_numpy(m, n):
+    """oracle.source_many (Eqs. 7-10, used by the full-size sampled GPU checks) names the
+    element numpy's out-of-place transpose puts at each destination: c2r(m, n) = P_{m,n},
+    r2c(m, n) = P_{n,m} (Theorem 1 buffer form)."""
+    pos = np.arange(m * n, dtype=np.int64)
+    idx = np.arange(m * n, dtype=np.int64)
+    assert same(oracle.source_many("c2r", m, n, pos), np_P(idx, m, n))
+    assert same(oracle.source_many("r2c", m, n, pos), np_P(idx, n, m))
+    rng = np.random.default_rng(m * 31 + n)
+    sub = rng.integers(0, m * n, size=min(500, m * n))
+    assert same(oracle.source_many("c2r", m, n, sub), np_P(idx, m, n)[sub])
