@@ -87,7 +87,7 @@ template <int TW> void run_tile(void *) {
 }
 template <int TW> void run_tile_staged(void *) {
     int ntile = G.R / TW, nb = (G.M + G.band - 1) / G.band;
-    copy_tile_staged<TW><<<ntile * nb, G.threads, G.band * TW>>>(G.a, G.M, G.R, G.band, G.grid);
+    copy_tile_staged<TW><<<ntile * nb, G.threads, (size_t)G.band * TW>>>(G.a, G.M, G.R, G.band, G.grid);
 }
 void run_contig(void *) { copy_contig<<<148 * 8, 512>>>((const uint4 *)G.a, (uint4 *)G.b, (size_t)G.M * G.R / 16); }
 
@@ -109,26 +109,27 @@ int main(int argc, char **argv) {
     G.grid = argc > 4 ? atoi(argv[4]) : 0;  // 1: tile-major block order
     float t = timeit(run_contig, nullptr, flush, fl);
     printf("{\"what\":\"contiguous\",\"GBps\":%.1f}\n", 2.0 * bytes / t / 1e6);
-    int bands[] = {128, 256, 512};
-    for (int band : bands) {
-        G.band = band;
-        t = timeit(run_tile<32>, nullptr, flush, fl);
-        printf("{\"what\":\"tile32\",\"band\":%d,\"GBps\":%.1f}\n", band, 2.0 * bytes / t / 1e6);
-        t = timeit(run_tile<64>, nullptr, flush, fl);
-        printf("{\"what\":\"tile64\",\"band\":%d,\"GBps\":%.1f}\n", band, 2.0 * bytes / t / 1e6);
-        t = timeit(run_tile<128>, nullptr, flush, fl);
-        printf("{\"what\":\"tile128\",\"band\":%d,\"GBps\":%.1f}\n", band, 2.0 * bytes / t / 1e6);
-        for (int tw : {32, 64, 128}) {
-            size_t sm = (size_t)band * tw;
-            if (sm > 200 * 1024) continue;
-            void (*f)(void *) = tw == 32 ? run_tile_staged<32> : tw == 64 ? run_tile_staged<64> : run_tile_staged<128>;
-            const void *k = tw == 32 ? (const void *)copy_tile_staged<32>
-                            : tw == 64 ? (const void *)copy_tile_staged<64> : (const void *)copy_tile_staged<128>;
+    // staged copies at a fixed shared-memory budget per CTA (the column kernel's unit size)
+    for (size_t sm : {size_t(27) << 10, size_t(54) << 10, size_t(108) << 10}) {
+        for (int tw : {128, 256, 512}) {
+            G.band = (int)(sm / tw);
+            void (*f)(void *) = tw == 128 ? run_tile_staged<128> : tw == 256 ? run_tile_staged<256> : run_tile_staged<512>;
+            const void *k = tw == 128 ? (const void *)copy_tile_staged<128>
+                            : tw == 256 ? (const void *)copy_tile_staged<256> : (const void *)copy_tile_staged<512>;
             cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
             t = timeit(f, nullptr, flush, fl);
-            printf("{\"what\":\"tile%d_staged\",\"band\":%d,\"smem\":%zu,\"GBps\":%.1f}\n", tw, band, sm,
+            printf("{\"what\":\"tile%d_staged\",\"band\":%d,\"smem\":%zu,\"GBps\":%.1f}\n", tw, G.band, sm,
                    2.0 * bytes / t / 1e6);
         }
+    }
+    for (int band : {256, 512}) {
+        G.band = band;
+        t = timeit(run_tile<128>, nullptr, flush, fl);
+        printf("{\"what\":\"tile128\",\"band\":%d,\"GBps\":%.1f}\n", band, 2.0 * bytes / t / 1e6);
+        t = timeit(run_tile<256>, nullptr, flush, fl);
+        printf("{\"what\":\"tile256\",\"band\":%d,\"GBps\":%.1f}\n", band, 2.0 * bytes / t / 1e6);
+        t = timeit(run_tile<512>, nullptr, flush, fl);
+        printf("{\"what\":\"tile512\",\"band\":%d,\"GBps\":%.1f}\n", band, 2.0 * bytes / t / 1e6);
     }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) printf("err %s\n", cudaGetErrorString(e));
