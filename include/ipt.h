@@ -115,6 +115,23 @@ ipt_status_t ipt_r2c_batched(void *base, int64_t batch, int64_t stride_elems, in
                              int64_t n, int elem_bytes, ipt_layout_t layout, void *stream);
 
 /*
+ * Host-buffer variants (the end-to-end call): the m x n matrix lives in HOST memory at
+ * `host` (pinned for asynchronous copies; pageable memory works but the copies are then
+ * synchronous); `dev` is caller-owned device memory of at least m*n*elem_bytes bytes.
+ * Stream-ordered on `stream`: copy host -> dev, ipt_c2r / ipt_r2c on dev (same semantics
+ * and arguments as above), copy dev -> host.  On return nothing has necessarily run yet;
+ * synchronise the stream before reading `host`.  Consecutive calls on two streams with two
+ * device buffers overlap one call's device->host copy with the next call's host->device
+ * copy (the two directions of the host link).  Errors: IPT_ERR_INVALID_ARGUMENT for a null
+ * host/dev pointer or the arguments ipt_c2r rejects; other codes as ipt_c2r.  On any error
+ * the host buffer is unchanged (no device->host copy is enqueued); dev is unspecified.
+ */
+ipt_status_t ipt_c2r_host(void *host, void *dev, int64_t m, int64_t n, int elem_bytes,
+                          ipt_layout_t layout, void *stream);
+ipt_status_t ipt_r2c_host(void *host, void *dev, int64_t m, int64_t n, int elem_bytes,
+                          ipt_layout_t layout, void *stream);
+
+/*
  * Skinny AoS <-> SoA conversion (§6.1).  An Array of Structures of
  * `count` structs, each of `fields` fields of field_bytes bytes, is a row-major
  * count x fields array; ipt_aos_to_soa transposes it in place into `fields` arrays of

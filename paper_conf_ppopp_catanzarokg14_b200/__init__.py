@@ -26,7 +26,7 @@ STATUS = {0: "IPT_OK", 1: "IPT_ERR_INVALID_ARGUMENT", 2: "IPT_ERR_UNSUPPORTED",
           3: "IPT_ERR_OUT_OF_MEMORY", 4: "IPT_ERR_CUDA"}
 
 # Every symbol declared in include/ipt.h.
-EXPORTS = ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
+EXPORTS = ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_c2r_host", "ipt_r2c_host", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_status_string", "ipt_plan_info",
            "ipt_launch_count", "ipt_profile_enable", "ipt_profile_read", "ipt_debug_tile_copy",
            "ipt_debug_aos_copy", "ipt_debug_aos_fill", "ipt_debug_warp_load_dump", "ipt_debug_warp_store",
@@ -52,6 +52,8 @@ _lib.ipt_c2r.argtypes = [_vp, _i64, _i64, _int, _int, _vp]
 _lib.ipt_r2c.argtypes = [_vp, _i64, _i64, _int, _int, _vp]
 _lib.ipt_c2r_batched.argtypes = [_vp, _i64, _i64, _i64, _i64, _int, _int, _vp]
 _lib.ipt_r2c_batched.argtypes = [_vp, _i64, _i64, _i64, _i64, _int, _int, _vp]
+_lib.ipt_c2r_host.argtypes = [_vp, _vp, _i64, _i64, _int, _int, _vp]
+_lib.ipt_r2c_host.argtypes = [_vp, _vp, _i64, _i64, _int, _int, _vp]
 _lib.ipt_aos_to_soa.argtypes = [_vp, _i64, _i64, _int, _vp]
 _lib.ipt_soa_to_aos.argtypes = [_vp, _i64, _i64, _int, _vp]
 _lib.ipt_scratch_bytes.argtypes = [_i64, _i64, _int, ctypes.POINTER(ctypes.c_size_t), ctypes.POINTER(ctypes.c_size_t)]
@@ -76,7 +78,7 @@ _lib.ipt_debug_aos_scatter.argtypes = [_vp, _vp, _vp, _i64, _int, _int, _vp]
 for _f in ("ipt_debug_aos_copy", "ipt_debug_aos_fill", "ipt_debug_warp_load_dump", "ipt_debug_warp_store",
            "ipt_debug_aos_gather", "ipt_debug_aos_scatter"):
     getattr(_lib, _f).restype = _int
-for _f in ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_aos_to_soa",
+for _f in ("ipt_c2r", "ipt_r2c", "ipt_c2r_batched", "ipt_r2c_batched", "ipt_c2r_host", "ipt_r2c_host", "ipt_aos_to_soa",
            "ipt_soa_to_aos", "ipt_scratch_bytes", "ipt_plan_info"):
     getattr(_lib, _f).restype = _int
 
@@ -137,6 +139,30 @@ def r2c_batched(buf, batch: int, stride_elems: int, m: int, n: int, elem_bytes: 
     p, eb, st = _ptr_eb_stream(buf, elem_bytes, stream)
     _check(_lib.ipt_r2c_batched(p, batch, stride_elems, m, n, eb, _LAYOUTS[layout], st), "ipt_r2c_batched")
     return buf
+
+
+def _host_ptr(host):
+    if isinstance(host, int):
+        return host
+    if host.is_cuda or not host.is_contiguous():
+        raise ValueError("host buffer must be a contiguous CPU tensor (pinned for asynchronous copies)")
+    return host.data_ptr()
+
+
+def c2r_host(host, dev, m: int, n: int, elem_bytes: int | None = None, layout="row", stream=None):
+    """ipt_c2r_host: host -> dev, c2r on dev, dev -> host, stream-ordered (include/ipt.h)."""
+    p, eb, st = _ptr_eb_stream(dev, elem_bytes if elem_bytes is not None else
+                               (None if isinstance(host, int) else host.element_size()), stream)
+    _check(_lib.ipt_c2r_host(_host_ptr(host), p, m, n, eb, _LAYOUTS[layout], st), "ipt_c2r_host")
+    return host
+
+
+def r2c_host(host, dev, m: int, n: int, elem_bytes: int | None = None, layout="row", stream=None):
+    """ipt_r2c_host: the inverse of c2r_host with the same arguments."""
+    p, eb, st = _ptr_eb_stream(dev, elem_bytes if elem_bytes is not None else
+                               (None if isinstance(host, int) else host.element_size()), stream)
+    _check(_lib.ipt_r2c_host(_host_ptr(host), p, m, n, eb, _LAYOUTS[layout], st), "ipt_r2c_host")
+    return host
 
 
 def aos_to_soa(buf, count: int, fields: int, field_bytes: int | None = None, stream=None):

@@ -1314,6 +1314,29 @@ ipt_status_t ipt_r2c_batched(void *base, int64_t batch, int64_t stride_elems, in
     return run_perm_any(base, batch, stride_elems, x, y, elem_bytes, stream);
 }
 
+static ipt_status_t run_host(bool c2r, void *host, void *dev, int64_t m, int64_t n, int elem_bytes,
+                             ipt_layout_t layout, void *stream) {
+    int64_t x, y;
+    if (!host || !dev || elem_bytes <= 0 || !perm_of(c2r, m, n, layout, x, y)) return IPT_ERR_INVALID_ARGUMENT;
+    if (m > 0 && n > (int64_t(1) << 62) / m / elem_bytes) return IPT_ERR_INVALID_ARGUMENT;
+    const size_t bytes = static_cast<size_t>(m) * static_cast<size_t>(n) * static_cast<size_t>(elem_bytes);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    ipt_status_t s = check(cudaMemcpyAsync(dev, host, bytes, cudaMemcpyHostToDevice, st));
+    if (s == IPT_OK) s = run_perm_any(dev, 1, -1, x, y, elem_bytes, stream);
+    if (s == IPT_OK) s = check(cudaMemcpyAsync(host, dev, bytes, cudaMemcpyDeviceToHost, st));
+    return s;
+}
+
+ipt_status_t ipt_c2r_host(void *host, void *dev, int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
+                          void *stream) {
+    return run_host(true, host, dev, m, n, elem_bytes, layout, stream);
+}
+
+ipt_status_t ipt_r2c_host(void *host, void *dev, int64_t m, int64_t n, int elem_bytes, ipt_layout_t layout,
+                          void *stream) {
+    return run_host(false, host, dev, m, n, elem_bytes, layout, stream);
+}
+
 ipt_status_t ipt_aos_to_soa(void *ptr, int64_t count, int64_t fields, int field_bytes, void *stream) {
     return run_perm_any(ptr, 1, -1, count, fields, field_bytes, stream);  // P_{count,fields}
 }

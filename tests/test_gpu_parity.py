@@ -837,3 +837,32 @@ def test_bench_sweep_calls_sampled_all(eb):
             assert x64.sum().item() == s1 and (x64 * x64).sum().item() == s2, (m, n, op, eb)
             getattr(ipt, "r2c" if op == "c2r" else "c2r")(x, m, n, elem_bytes=eb)
             assert torch.equal(x, base[:total].to(dt)), (m, n, op, eb, "round trip")
+
+
+def test_host_buffer_calls_pipelined_on_two_streams():
+    """ipt_c2r_host / ipt_r2c_host (include/ipt.h): pinned host matrix -> device -> transpose
+    -> host, stream-ordered; consecutive calls alternate two streams and two device buffers
+    (the bench's e2e pattern), every result compared in full with the oracle; invalid
+    arguments leave the host buffer untouched."""
+    shapes = [(1200, 1800, 4), (333, 4099, 8), (2003, 129, 4), (640, 1024, 16), (4096, 3000, 4), (17, 5, 8)]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    devs = [torch.empty(max(m * n * eb for m, n, eb in shapes), dtype=torch.uint8, device=DEV) for _ in range(2)]
+    hosts, wants = [], []
+    for k, (m, n, eb) in enumerate(shapes):
+        host = workloads.random_words(m * n, eb, seed=k + 40)
+        h = torch.from_numpy(np.ascontiguousarray(host).view(np.uint8).reshape(-1).copy()).pin_memory()
+        hosts.append(h)
+        wants.append(oracle.transpose(vwords(host, eb), m, n).tobytes())
+        ipt.c2r_host(h, devs[k % 2], m, n, elem_bytes=eb, stream=streams[k % 2])
+    torch.cuda.synchronize()
+    for k, (m, n, eb) in enumerate(shapes):
+        assert hosts[k].numpy().tobytes() == wants[k], (m, n, eb)
+        ipt.r2c_host(hosts[k], devs[k % 2], m, n, elem_bytes=eb, stream=streams[k % 2])
+    torch.cuda.synchronize()
+    for k, (m, n, eb) in enumerate(shapes):
+        host = workloads.random_words(m * n, eb, seed=k + 40)
+        assert hosts[k].numpy().tobytes() == np.ascontiguousarray(host).tobytes(), (m, n, eb)
+    h = hosts[0].clone()
+    with pytest.raises(ipt.IptError) as e:
+        ipt.c2r_host(h, 0, 1200, 1800, elem_bytes=4)
+    assert e.value.status == 1 and torch.equal(h, hosts[0])
