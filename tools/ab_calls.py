@@ -41,6 +41,7 @@ def main():
     p.add_argument("--eb", type=int, nargs="+", default=[4, 8])
     p.add_argument("--reps", type=int, default=3)
     p.add_argument("--quiet", action="store_true")
+    p.add_argument("--no-kernels", action="store_true", help="no per-kernel events (they separate the launches)")
     a = p.parse_args()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     summary = {}
@@ -57,7 +58,7 @@ def main():
                     set_env(env)
                     op(x, m, n, elem_bytes=eb)
                     torch.cuda.synchronize()
-                    ipt.profile_enable(True)
+                    ipt.profile_enable(not a.no_kernels)
                     ipt.profile_read()
                     ts = []
                     for _ in range(a.reps):
