@@ -99,7 +99,7 @@ struct Plan {
     size_t side_bytes = 0;      // lagged layouts: side block bytes per matrix (M x (D TWB + pad))
     SkinnyRowParams srow{};     // skinny engine long-row shuffle
     SkinnyColParams scol{}, srot{};  // skinny engine column passes (shuffle, rotation)
-    bool chunk_force = false;   // IPT_ROW_CHUNK=1
+    int chunk_force = 0;        // 1: IPT_ROW_CHUNK=1; 2: c = 5..8 (chunks of 8 (c - 1) rows)
     int col_super = 1;          // lagged column pass: super-tile width (col_tile_kernel)
     int sms = 0;
     int skinny_dir = 0;         // ROW_R2C (P_{count,n}, AoS -> SoA) or ROW_C2R (P_{n,count})
@@ -251,24 +251,32 @@ void set_lag(Plan &pl, int64_t D) {
 // max(R, 8 (c-1), min(IPT_ROW_CHUNK_K (c-1), ceil(M batch / (8 SMs)))) rows -- the boundary
 // traffic 2 (c-1) / cK stays <= 25 % of a pass, and about 8 chunks per SM when the call is
 // small -- rounded to whole row groups.  Returns whether the batch has >= 2 chunks per SM
-// (always true when forced by IPT_ROW_CHUNK=1, which also uses cK = max(R, IPT_ROW_CHUNK_K (c-1))).
+// (always true when forced: IPT_ROW_CHUNK=1 uses cK = max(R, IPT_ROW_CHUNK_K (c-1)); for c = 5..8,
+// chunk_force 2, the formula's cK when it gives 2 chunks per SM, else max(R, 8 (c-1))).
 bool set_chunks(Plan &pl, int64_t batch) {
     RowParams &rp = pl.row;
     const int64_t ckmul = env_int("IPT_ROW_CHUNK_K", 16);
-    int64_t K;
-    if (pl.chunk_force) {
-        K = std::max<int64_t>(rp.R, ckmul * (pl.c - 1));
-    } else {
-        const int64_t par_rows = (pl.M * batch + 8 * pl.sms - 1) / (8 * static_cast<int64_t>(pl.sms));
-        K = std::max<int64_t>({static_cast<int64_t>(rp.R), 8 * (pl.c - 1), std::min<int64_t>(ckmul * (pl.c - 1), par_rows)});
+    auto apply = [&](int64_t K) {
+        K = (K + rp.R - 1) / rp.R * rp.R;
+        const int64_t Mr = (pl.M + rp.R - 1) / rp.R * rp.R;
+        if (K > Mr) K = Mr;
+        rp.cK = static_cast<int32_t>(K);
+        rp.nch = static_cast<int32_t>((pl.M + K - 1) / K);
+        rp.fd_nch = make_fastdiv(static_cast<uint32_t>(rp.nch));
+        return static_cast<int64_t>(rp.nch) * batch >= 2 * static_cast<int64_t>(pl.sms);
+    };
+    if (pl.chunk_force == 1) {
+        apply(std::max<int64_t>(rp.R, ckmul * (pl.c - 1)));
+        return true;
     }
-    K = (K + rp.R - 1) / rp.R * rp.R;
-    const int64_t Mr = (pl.M + rp.R - 1) / rp.R * rp.R;
-    if (K > Mr) K = Mr;
-    rp.cK = static_cast<int32_t>(K);
-    rp.nch = static_cast<int32_t>((pl.M + K - 1) / K);
-    rp.fd_nch = make_fastdiv(static_cast<uint32_t>(rp.nch));
-    return pl.chunk_force || static_cast<int64_t>(rp.nch) * batch >= 2 * static_cast<int64_t>(pl.sms);
+    const int64_t par_rows = (pl.M * batch + 8 * pl.sms - 1) / (8 * static_cast<int64_t>(pl.sms));
+    if (apply(std::max<int64_t>({static_cast<int64_t>(rp.R), 8 * (pl.c - 1), std::min<int64_t>(ckmul * (pl.c - 1), par_rows)})))
+        return true;
+    if (pl.chunk_force == 2) {  // c = 5..8 (make_plan): chunks of 8 (c - 1) rows regardless
+        apply(std::max<int64_t>(rp.R, 8 * (pl.c - 1)));
+        return true;
+    }
+    return false;
 }
 
 // Skinny engine (§6.1): P_{x,y} with min(x, y) = n <= 32 fields
@@ -459,10 +467,16 @@ ipt_status_t make_plan(int64_t x, int64_t y, int eb, Plan &pl) {
     const int chunk_env = env_int("IPT_ROW_CHUNK", -1);  // -1 auto, 0 off, 1 force
     const size_t fbuf = rp.fuse ? row_fused_smem_bytes(rp, eb, pl.row_dir) : 0;
     const bool chunk_ok = 2 * rp.R * fbuf <= static_cast<size_t>(env_int("IPT_ROW_DB_MAX", 112 * 1024));
-    if (rp.fuse && (chunk_env == 1 || (chunk_env == -1 && chunk_ok))) {
+    // c = 5..8: the chunked pass with chunks of 8 (c - 1) rows whatever the chunk count or the
+    // row length (single-buffered rows then prefetch the next group into L2): the sweep's
+    // c = 5..8 calls 1877 -> 2093 GB/s against the flag-based pass, whose c staircase
+    // segments per row dominate; c = 2..4 and c >= 9 keep the rule below (forcing them loses
+    // 1-6 %, profiles/r02_ab_chunk_small_c.txt).
+    const bool mid_c = pl.c >= 5 && pl.c <= 8;
+    if (rp.fuse && (chunk_env == 1 || (chunk_env == -1 && (chunk_ok || mid_c)))) {
         rp.chunk = 1;
         rp.rpitch = ((pl.N * eb + 15) & ~int64_t(15)) + 16;
-        pl.chunk_force = chunk_env == 1;
+        pl.chunk_force = chunk_env == 1 ? 1 : chunk_env == -1 && mid_c ? 2 : 0;
         pl.sms = dev.sms;
         set_chunks(pl, 1);
     }
