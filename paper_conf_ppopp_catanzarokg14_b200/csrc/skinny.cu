@@ -173,6 +173,7 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
     extern __shared__ __align__(16) unsigned char smem[];
     int32_t *qinv_s = reinterpret_cast<int32_t *>(smem);  // 32 entries
     T *buf = reinterpret_cast<T *>(smem + 128);            // [n][C]
+    __shared__ T *rowp_s[32];                              // output row of each logical row
     const uint32_t sbuf = static_cast<uint32_t>(__cvta_generic_to_shared(buf));
     const int n = P.n, C = P.C;
     const int64_t pitch = P.N;  // in elements
@@ -212,35 +213,50 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
         }
         asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
         __syncthreads();
+        // Store: thread = column (coalesced per row), rows inner.  The output row of logical
+        // row i is the same for every column of the block (the folded rotation amount rho =
+        // floor(j/b) is constant within a block unless it straddles a multiple of b), so its
+        // pointer comes from a per-block shared table; the source row index steps with i.
+        auto out_row = [&](int i, int32_t rho) -> T * {
+            if (P.remap <= 0) return A + i * pitch;
+            if (i == n - 1) return tmp;
+            int32_t L = i + 1 + (FOLD ? rho : 0);
+            L -= L >= n ? n : 0;
+            return A + L * pitch;
+        };
+        auto rot_shift = [&](int32_t qd) { return P.rot_sign > 0 ? qd : (qd == 0 ? 0 : n - qd); };
+        const int32_t rho0 = (FOLD || MODE == COL_ROT) ? static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0), P.fd_b)) : 0;
+        const bool one_rho = !(FOLD || MODE == COL_ROT) ||
+                             static_cast<int32_t>(fdiv(static_cast<uint32_t>(j0 + cols - 1), P.fd_b)) == rho0;
+        if (threadIdx.x < n) rowp_s[threadIdx.x] = out_row(threadIdx.x, rho0);
+        __syncthreads();
         for (int32_t x = threadIdx.x; x < cols; x += blockDim.x) {
             const int64_t j = j0 + x;  // < N < 2^31
-            const uint32_t jm = fmod_(static_cast<uint32_t>(j), P.fd_n);
-            int32_t shift = 0;
-            const int32_t rho = FOLD ? static_cast<int32_t>(fdiv(static_cast<uint32_t>(j), P.fd_b)) : 0;
-            if (MODE == COL_ROT) {  // floor(j/b) < c <= n
-                const int32_t qd = static_cast<int32_t>(fdiv(static_cast<uint32_t>(j), P.fd_b));
-                shift = P.rot_sign > 0 ? qd : (qd == 0 ? 0 : n - qd);
-            }
+            const int32_t jm = static_cast<int32_t>(fmod_(static_cast<uint32_t>(j), P.fd_n));
+            const int32_t rho = one_rho ? rho0 : static_cast<int32_t>(fdiv(static_cast<uint32_t>(j), P.fd_b));
+            // source row of output row 0, then +1 (mod n) per row for ROT and R2C
+            int32_t s0;
+            if (MODE == COL_ROT) s0 = rot_shift(rho);
+            else if (MODE == COL_R2C_SHUF) s0 = jm == 0 ? 0 : n - jm;  // u = (0 - jm) mod n
+            else s0 = 0;
+            const T *col = buf + x;
             for (int i = 0; i < n; ++i) {
-                int32_t s;
+                int32_t src;
                 if (MODE == COL_ROT) {
-                    s = i + shift;
-                    s -= s >= n ? n : 0;
+                    src = s0;
                 } else if (MODE == COL_C2R_SHUF) {
-                    s = static_cast<int32_t>(jm) + P.q[i];
-                    s -= s >= n ? n : 0;
+                    src = jm + P.q[i];
+                    src -= src >= n ? n : 0;
                 } else {
-                    int32_t u = i - static_cast<int32_t>(jm);
-                    u += u < 0 ? n : 0;
-                    s = qinv_s[u];
+                    src = qinv_s[s0];
                 }
-                T *orow = P.remap > 0 ? (i == n - 1 ? tmp : A + (i + 1) * pitch) : A + i * pitch;
-                if (FOLD && P.remap > 0 && i < n - 1) {
-                    int32_t L = i + 1 + rho;
-                    L -= L >= n ? n : 0;
-                    orow = A + L * pitch;
+                // (plain rows: one multiply-add; rolled rows: the block's table)
+                T *orow = P.remap <= 0 ? A + i * pitch : one_rho ? rowp_s[i] : out_row(i, rho);
+                orow[j] = col[src * C];
+                if (MODE != COL_C2R_SHUF) {
+                    ++s0;
+                    s0 -= s0 >= n ? n : 0;
                 }
-                orow[j] = buf[s * C + x];
             }
         }
         __syncthreads();  // the buffer is refilled by the next column block

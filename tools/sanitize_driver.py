@@ -49,6 +49,11 @@ def main():
         roundtrip(2 * 301, 2 * 517, 4, f"fused flags {eng}")
         roundtrip(6 * 101, 6 * 77, 8, f"fused flags {eng}")
         env(IPT_ROW_CHUNK=None)
+        # c = 5..8: chunked pass chosen automatically; single-buffered rows (L2 prefetch)
+        roundtrip(6 * 101, 6 * 77, 4, f"fused c=6 auto {eng}")
+        env(IPT_ROW_DB_MAX=1024)
+        roundtrip(6 * 101, 6 * 77, 4, f"fused c=6 single-buffered {eng}")
+        env(IPT_ROW_DB_MAX=None)
         # legacy row kernel
         env(IPT_ROW_PIPE=0)
         roundtrip(301, 517, 4, f"row legacy {eng}")
@@ -69,6 +74,18 @@ def main():
     ipt.r2c_batched(x, 3, 120 * 77, 120, 77, elem_bytes=4)
     torch.cuda.synchronize()
     print("batched:", "ok" if torch.equal(x, y) else "MISMATCH", flush=True)
+    # host-buffer entry point on two streams
+    hs = [torch.randint(0, 2**31 - 1, (301 * 517,), dtype=torch.int32).pin_memory() for _ in range(2)]
+    ref = [h.clone() for h in hs]
+    ds = [torch.empty(301 * 517, dtype=torch.int32, device="cuda") for _ in range(2)]
+    sts = [torch.cuda.Stream(), torch.cuda.Stream()]
+    for k in range(2):
+        ipt.c2r_host(hs[k], ds[k], 301, 517, elem_bytes=4, stream=sts[k])
+    torch.cuda.synchronize()
+    for k in range(2):
+        ipt.r2c_host(hs[k], ds[k], 301, 517, elem_bytes=4, stream=sts[k])
+    torch.cuda.synchronize()
+    print("host API:", "ok" if all(torch.equal(hs[k], ref[k]) for k in range(2)) else "MISMATCH", flush=True)
     # skinny engine (register and shared-memory row kernels, folded rotation)
     for n, eb in ((3, 4), (8, 4), (5, 8)):
         cnt = 65536 + 96
