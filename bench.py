@@ -18,8 +18,8 @@ value   = median over all timed calls of the per-call GB/s (the paper's statisti
 moved   = the same median over the call's algorithmic bytes (4 m n s for two passes).
 extras  = cfg5b (batch of 4096 4096x3000 fp32, sharded over the ranks; strong scaling),
           cfg3 (skinny AoS<->SoA, median over n) and cfg5a (~140 GB fp64) at N = 1.
-e2e     = the same median, each call timed from a pinned-host H2D copy through ipt_c2r
-          to the D2H copy of the result (public API, host buffers).
+e2e     = Eq. 37 bytes of a step of ipt_c2r_host calls (C ABI, pinned host buffers: H2D,
+          transpose, D2H) over the step's device time, calls round-robin over 4 streams.
 roofline= the dominant kernel's algorithmic bytes / its event-timed device time against
           the measured HBM copy bandwidth (MEASURED_PEAKS.json); the per-launch events run in a
           replica of two timed steps right after the timed region (--kernel-events).
@@ -587,28 +587,32 @@ def run_ours(args, rank, world, local_rank):
 
     # ---- e2e through the public API with host buffers --------------------------------
     # ipt_c2r_host (host -> device, transpose, device -> host, stream-ordered) on every e2e
-    # shape, consecutive calls alternating two streams and two device buffers, so that one
-    # call's device->host copy overlaps the next call's host->device copy (the two directions
+    # shape, consecutive calls round-robin over NS streams and device buffers, so that one
+    # call's device->host copy overlaps the next calls' host->device copies (the two directions
     # of the host link).  E = all Eq. 37 bytes of the step / the step's device time (first
     # copy in to last copy out); median of 3 steps after one warm-up step.
     e2e_shapes = [(m, n, eb) for eb in ebs for (m, n) in shapes[:args.e2e_shapes]]
     big = max(m * n * eb for m, n, eb in e2e_shapes)
-    hosts = [torch.empty(big, dtype=torch.uint8, pin_memory=True).random_(0, 255) for _ in range(2)]
-    devs = [torch.empty(big, dtype=torch.uint8, device=dev) for _ in range(2)]
-    sts = [stream, torch.cuda.Stream(device=dev)]
+    NS = 4  # calls in flight (tools/e2e_streams.py: 1 / 2 / 3 / 4 streams -> 54 / 71 / 81 / 84 GB/s)
+    hosts = [torch.empty(big, dtype=torch.uint8, pin_memory=True).random_(0, 255) for _ in range(NS)]
+    devs = [torch.empty(big, dtype=torch.uint8, device=dev) for _ in range(NS)]
+    sts = [stream] + [torch.cuda.Stream(device=dev) for _ in range(NS - 1)]
     e2e_rates = []
     step_bytes = sum(2.0 * m * n * eb for m, n, eb in e2e_shapes)
     h2d = sum(m * n * eb for m, n, eb in e2e_shapes)
     for rep in range(4):
         torch.cuda.synchronize()
-        e0, e1, eb1 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+        e0, e1 = (torch.cuda.Event(enable_timing=True) for _ in range(2))
         e0.record(sts[0])
-        sts[1].wait_event(e0)
+        for st_ in sts[1:]:
+            st_.wait_event(e0)
         for k, (m, n, eb) in enumerate(e2e_shapes):
-            # call k + 2 reuses call k's buffers on the same stream, after its D2H
-            ipt.c2r_host(hosts[k % 2][:m * n * eb], devs[k % 2], m, n, elem_bytes=eb, stream=sts[k % 2].cuda_stream)
-        eb1.record(sts[1])
-        sts[0].wait_event(eb1)
+            # call k + NS reuses call k's buffers on the same stream, after its D2H
+            ipt.c2r_host(hosts[k % NS][:m * n * eb], devs[k % NS], m, n, elem_bytes=eb, stream=sts[k % NS].cuda_stream)
+        for st_ in sts[1:]:
+            ev = torch.cuda.Event()
+            ev.record(st_)
+            sts[0].wait_event(ev)
         e1.record(sts[0])
         e1.synchronize()
         if rep > 0:
@@ -619,8 +623,9 @@ def run_ours(args, rank, world, local_rank):
            "statistic": "all Eq. 37 bytes of the step / its device time (first H2D to last D2H), median of 3 steps, "
                         "summed over ranks",
            "note": f"ipt_c2r_host on pinned host buffers (C ABI: H2D, transpose, D2H), {len(e2e_shapes)} calls per step "
-                   f"(first {args.e2e_shapes} sweep shapes x {'/'.join('fp%d' % (8 * e) for e in ebs)}), alternating two "
-                   "streams and two device buffers so D2H of one call overlaps H2D of the next; bound by the host link"}
+                   f"(first {args.e2e_shapes} sweep shapes x {'/'.join('fp%d' % (8 * e) for e in ebs)}), round-robin over "
+                   f"{NS} streams and device buffers so D2H of one call overlaps H2D of the next; bound by the host link "
+                   "(H2D 38, D2H 52 GB/s alone)"}
     del hosts, devs
     del bufs, flush
     torch.cuda.empty_cache()
