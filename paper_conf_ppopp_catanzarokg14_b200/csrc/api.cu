@@ -103,6 +103,7 @@ struct Plan {
     int col_super = 1;          // lagged column pass: super-tile width (col_tile_kernel)
     int sms = 0;
     int skinny_dir = 0;         // ROW_R2C (P_{count,n}, AoS -> SoA) or ROW_C2R (P_{n,count})
+    bool skinny_one = false;    // register row shuffles in one cooperative launch
 };
 
 int ilog2(int v) {
@@ -342,11 +343,14 @@ ipt_status_t make_skinny_plan(const DevInfo &dev, int64_t x, int64_t y, int eb, 
     r.fd_b = make_fastdiv(static_cast<uint32_t>(pl.b));
     r.fold = fold ? 1 : 0;
     r.reg = eb == 4 && env_int("IPT_SKINNY_REG", 1) != 0 ? 1 : 0;
+    // register row shuffles: all n rows in one cooperative launch (IPT_SKINNY_ONE=0: one per row)
+    const bool one = r.reg && env_int("IPT_SKINNY_ONE", 1) != 0;
     const size_t rs = skinny_row_smem(n, r.Tp, eb);
     if (rs > static_cast<size_t>(dev.smem_optin)) return IPT_ERR_UNSUPPORTED;
     if (rs > pl.onchip) pl.onchip = rs;
     pl.scratch = static_cast<size_t>(pl.N) * eb;  // one row of the long dimension
-    pl.nlaunch = n + 1 + (pl.has_rot ? 1 : 0);
+    pl.nlaunch = (one ? 2 : n + 1) + (pl.has_rot ? 1 : 0);
+    pl.skinny_one = one;
     return IPT_OK;
 }
 
@@ -546,7 +550,7 @@ struct PlanKeyHash {
 std::string tunables_key() {
     std::string s;
     for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_TMA_SUPER", "IPT_COL_BULK", "IPT_COL_PERSIST", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
-                          "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_SKINNY_COLBYTES", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
+                          "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_SKINNY_ONE", "IPT_SKINNY_COLBYTES", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
         s += v ? v : "-";
@@ -713,6 +717,7 @@ struct CallScratch {
     size_t ctr_shuf = 0, ctr_rot = 0;  // column-pass counter blocks (kCtrBytes each)
     size_t flags = 0;                  // fused rotation: M*batch row flags + the ticket
     size_t zero_bytes = 0;             // [0, zero_bytes) is zeroed before the first pass
+    size_t gbar = 0;                   // skinny engine: grid-barrier counter of the one-launch row pass
     size_t wrap = 0, wstride = 0;      // fused rotation: per-matrix copy of rows 0..c-2
     size_t bnd = 0;                    // chunked fused pass: boundary rows
     size_t side = 0;                   // lagged layouts: side blocks
@@ -735,6 +740,10 @@ void prepare_call(Plan &pl, int64_t batch, CallScratch &cs) {
     if (pl.engine == ENG_NONE || batch == 0) return;
     if (pl.engine == ENG_SKINNY) {
         cs.total = al256(pl.scratch * static_cast<size_t>(skinny_sub(pl, batch)));
+        if (pl.skinny_one) {  // grid-barrier counter of the one-launch row shuffles (zeroed per launch)
+            cs.gbar = cs.total;
+            cs.total += 256;
+        }
         return;
     }
     const double full = 2.0 * static_cast<double>(pl.M) * static_cast<double>(pl.N) * pl.eb * static_cast<double>(batch);
@@ -847,9 +856,12 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
             shuf.tmp_stride = rotp.tmp_stride = pl.N * pl.eb;
             auto rot_l = [&] { return launch_skinny_col(rotp, pl.eb, st); };
             auto shuf_l = [&] { return launch_skinny_col(shuf, pl.eb, st); };
+            const bool one = pl.skinny_one;  // all rows in one cooperative launch
+            unsigned int *gbar = one ? reinterpret_cast<unsigned int *>(scratch + cs.gbar) : nullptr;
             auto row_l = [&](int i) {
                 SkinnyRowParams rp = pl.srow;
                 rp.i = i;
+                rp.gbar = gbar;
                 rp.A = A;
                 rp.tmp = tmp;
                 rp.batch = nb;
@@ -857,13 +869,22 @@ ipt_status_t launch_call(const Plan &pl0, const CallScratch &cs, char *base, int
                 rp.tmp_stride = pl.N * pl.eb;
                 return [rp, &pl, st] { return launch_skinny_row(rp, pl.skinny_dir, pl.eb, st); };
             };
+            auto rows = [&]() -> ipt_status_t {
+                if (!one) {
+                    ipt_status_t r = IPT_OK;
+                    for (int i = 0; i < n && r == IPT_OK; ++i) r = run(PK_SKINNY, rowb, row_l(i));
+                    return r;
+                }
+                ipt_status_t r = check(cudaMemsetAsync(gbar, 0, sizeof(unsigned int), st));
+                return r == IPT_OK ? run(PK_SKINNY, rowb * n, row_l(0)) : r;
+            };
             if (pl.skinny_dir == ROW_R2C) {
                 if ((s = run(PK_COL, rowb * n, shuf_l)) != IPT_OK) break;
-                for (int i = 0; i < n && s == IPT_OK; ++i) s = run(PK_SKINNY, rowb, row_l(i));
+                s = rows();
                 if (s == IPT_OK && pl.has_rot) s = run(PK_ROT, rowb * n, rot_l);
             } else {
                 if (pl.has_rot && (s = run(PK_ROT, rowb * n, rot_l)) != IPT_OK) break;
-                for (int i = 0; i < n && s == IPT_OK; ++i) s = run(PK_SKINNY, rowb, row_l(i));
+                s = rows();
                 if (s == IPT_OK) s = run(PK_COL, rowb * n, shuf_l);
             }
             if (s != IPT_OK) break;

@@ -199,6 +199,8 @@ struct SkinnyRowParams {
     int32_t T, Tp;      // run length per residue class; shared-memory row pitch (odd)
     int32_t fold;       // 1: the rotation (Eq. 23 / Eq. 36) is folded into the locations
     int32_t reg;        // 1: in-register SIMD transposition kernel (skinny_reg.cu; 4-byte fields)
+    unsigned int *gbar; // reg: all n rows in one cooperative launch, grid-barrier counter (zeroed
+                        // per launch); null: one launch per row
     FastDiv fd_n, fd_b;
     int64_t batch;      // matrices of the launch (gridDim.y): matrix k at A + k mat_stride,
     int64_t mat_stride, tmp_stride;  // its tmp row at tmp + k tmp_stride (bytes)

@@ -55,7 +55,7 @@ __device__ __forceinline__ int64_t dpinv_pos(const SkinnyRowParams &P, int64_t x
 }
 
 template <int S, int DIR, bool FOLD>
-__global__ void __launch_bounds__(kRegThreads) skinny_reg_kernel(SkinnyRowParams P) {
+__device__ __forceinline__ void skinny_reg_row(const SkinnyRowParams &P) {
     // U chunks per warp and iteration: all their loads are issued before any transposition
     // (memory-level parallelism for small S), U * S <= 32 data registers.
     constexpr int U = S <= 4 ? 8 : S <= 8 ? 4 : S <= 16 ? 2 : 1;
@@ -167,7 +167,56 @@ __global__ void __launch_bounds__(kRegThreads) skinny_reg_kernel(SkinnyRowParams
 }
 
 template <int S, int DIR, bool FOLD>
+__global__ void __launch_bounds__(kRegThreads) skinny_reg_kernel(SkinnyRowParams P) {
+    skinny_reg_row<S, DIR, FOLD>(P);
+}
+
+// All n long-row shuffles in ONE cooperative launch (P.gbar != nullptr): row i of the rolling
+// scheme writes the location row i - 1 (R2C) / row i + 1 (C2R) read and reads nothing another
+// row of this launch writes, so the only hazard between consecutive rows is write-after-read,
+// closed by a grid barrier: every CTA's loads of row i were consumed by its stores (complete)
+// before it arrives; no CTA writes row i + 1's destination before all have arrived.  The
+// cooperative launch guarantees the co-residency the barrier needs (or fails cleanly).
+template <int S, int DIR, bool FOLD>
+__global__ void __launch_bounds__(kRegThreads) skinny_reg_all_kernel(SkinnyRowParams P) {
+    const unsigned int nblk = gridDim.x * gridDim.y;
+    for (int32_t i = 0; i < P.n; ++i) {
+        P.i = i;
+        skinny_reg_row<S, DIR, FOLD>(P);
+        if (i + 1 == P.n) break;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            __threadfence();
+            atomicAdd(P.gbar, 1u);
+            const unsigned int target = static_cast<unsigned int>(i + 1) * nblk;
+            unsigned int v;
+            while (true) {
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(P.gbar) : "memory");
+                if (v >= target) break;
+                __nanosleep(64);
+            }
+        }
+        __syncthreads();  // also: the shared tables of row i are rebuilt for row i + 1
+    }
+}
+
+template <int S, int DIR, bool FOLD>
 cudaError_t launch_s(const SkinnyRowParams &P, cudaStream_t st) {
+    if (P.gbar) {
+        auto kern = skinny_reg_all_kernel<S, DIR, FOLD>;
+        const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), kRegThreads, 0);
+        if (resident < static_cast<int64_t>(P.batch)) return cudaErrorInvalidConfiguration;
+        const int64_t warps = (P.N / S + 31) / 32;
+        int64_t grid = (warps * 32 + kRegThreads - 1) / kRegThreads;
+        const int64_t per = resident / P.batch;  // every CTA of the launch co-resident
+        if (grid > per) grid = per;
+        if (grid < 1) grid = 1;
+        SkinnyRowParams Q = P;
+        void *args[] = {&Q};
+        return cudaLaunchCooperativeKernel(reinterpret_cast<const void *>(kern),
+                                           dim3(static_cast<unsigned>(grid), static_cast<unsigned>(P.batch)),
+                                           dim3(kRegThreads), args, 0, st);
+    }
     auto kern = skinny_reg_kernel<S, DIR, FOLD>;
     const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), kRegThreads, 0);
     if (resident < 1) return cudaErrorInvalidConfiguration;
