@@ -549,7 +549,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_TMA_SUPER", "IPT_COL_BULK", "IPT_COL_PERSIST", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_TMA_SUPER", "IPT_COL_BULK", "IPT_COL_PERSIST", "IPT_COL_SIDECAP", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_SKINNY_ONE", "IPT_SKINNY_COLBYTES", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -748,8 +748,11 @@ void prepare_call(Plan &pl, int64_t batch, CallScratch &cs) {
     }
     const double full = 2.0 * static_cast<double>(pl.M) * static_cast<double>(pl.N) * pl.eb * static_cast<double>(batch);
     if (pl.side_bytes && batch > 1) {
-        // Batches: keep the side blocks within max(256 MiB, 1/32 of the data) -- a smaller D.
-        const double cap = std::max(256.0 * (1 << 20), full / 2.0 / 32.0);
+        // Batches: keep the side blocks within max(256 MiB, 1/8 of the data) -- a smaller D
+        // beyond that.  (1/32 forced D = 2 on config 5b's 512-matrix chunks and the column pass
+        // waited on its lag: 4378 -> 4878 GB/s, call 2389 -> 2531 GB/s with 1/8;
+        // profiles/r02_batch_sidecap.txt.  D = 8 tiles of 128 B is 256 / N of the data.)
+        const double cap = std::max(256.0 * (1 << 20), full / 2.0 / static_cast<double>(env_int("IPT_COL_SIDECAP", 8)));
         const double per_tile = static_cast<double>(pl.M) * pl.shuf.p.W * pl.eb * static_cast<double>(batch);
         const int64_t dmax = static_cast<int64_t>(cap / per_tile);
         if (dmax < pl.shuf.p.lagD) set_lag(pl, dmax);
