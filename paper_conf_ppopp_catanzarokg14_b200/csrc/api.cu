@@ -256,7 +256,9 @@ void set_lag(Plan &pl, int64_t D) {
 // chunk_force 2, the formula's cK when it gives 2 chunks per SM, else max(R, 8 (c-1))).
 bool set_chunks(Plan &pl, int64_t batch) {
     RowParams &rp = pl.row;
-    const int64_t ckmul = env_int("IPT_ROW_CHUNK_K", 16);
+    // (32: large batches take chunks of up to 32 (c-1) rows -- config 5b row pass +2.5 %; single
+    // matrices rarely reach the cap, the sweep is unchanged: profiles/r02_batch_split.txt)
+    const int64_t ckmul = env_int("IPT_ROW_CHUNK_K", 32);
     auto apply = [&](int64_t K) {
         K = (K + rp.R - 1) / rp.R * rp.R;
         const int64_t Mr = (pl.M + rp.R - 1) / rp.R * rp.R;
