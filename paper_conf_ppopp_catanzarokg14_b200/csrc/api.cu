@@ -551,7 +551,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_TMA_SUPER", "IPT_COL_BULK", "IPT_COL_PERSIST", "IPT_COL_SIDECAP", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_BULK", "IPT_COL_PERSIST", "IPT_COL_SIDECAP", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_SKINNY_ONE", "IPT_SKINNY_COLBYTES", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
@@ -687,13 +687,13 @@ void setup_col_tma(ColParams &p, int mode, int eb) {
         return;
     }
     if (!(allow & 1)) return;
-    // 16-byte pitches only.  (Super-rows of g rows would make any pitch a multiple of 16, but
-    // their per-phase boxes start at x = p pitch / 4, not 16-byte aligned, and the TMA unit
-    // faults on such boxes -- cudaErrorIllegalInstruction on 1024 x 1023 fp32, gpurun_out
-    // r02aa; IPT_COL_TMA_SUPER=1 keeps that path for experiments.)
-    const bool any_pitch = env_int("IPT_COL_TMA_SUPER", 0) != 0;
+    // 16-byte pitches only.  (Super-rows of g rows make any pitch a multiple of 16, but their
+    // per-phase boxes start at x = p pitch / 4, not 16-byte aligned, and the TMA unit faults on
+    // such boxes -- cudaErrorIllegalInstruction on 1024 x 1023 fp32, gpurun_out r02aa; with the
+    // box x aligned down and 144-byte hull boxes they are correct but 5 % slower than cp.async
+    // hulls, profiles/r02_ab_tma_hull_boxes.txt.)  The kernel's phase logic stays general.
     p.tg_a = super_rows(pitch);
-    if (p.tg_a > 1 && !any_pitch) return;
+    if (p.tg_a > 1) return;
     p.trows_a = p.M / p.tg_a * p.tg_a;
     // (rank 3 always -- the kernel issues 3-D boxes; one matrix: any 16-byte multiple serves)
     const int64_t ms = p.batch == 1 ? ((static_cast<int64_t>(p.M) * pitch + 15) & ~int64_t(15)) : p.mat_stride_bytes;
@@ -702,7 +702,7 @@ void setup_col_tma(ColParams &p, int mode, int eb) {
         const char *s0 = side_matrix(p.side, p.sstride, 0, p.base);
         p.tg_s = super_rows(p.spitch);
         p.trows_s = p.M / p.tg_s * p.tg_s;
-        if ((p.tg_s == 1 || any_pitch) &&
+        if (p.tg_s == 1 &&
             make_map(&p.tmap_s, s0, static_cast<int64_t>(p.lagD) * 128, p.M, p.spitch, p.batch, p.sstride,
                      kTmaBoxRows, p.tg_s))
             p.tma |= 2;
