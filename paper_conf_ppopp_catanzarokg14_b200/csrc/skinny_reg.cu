@@ -205,7 +205,17 @@ cudaError_t launch_s(const SkinnyRowParams &P, cudaStream_t st) {
     if (P.gbar) {
         auto kern = skinny_reg_all_kernel<S, DIR, FOLD>;
         const int resident = cached_resident_blocks(reinterpret_cast<const void *>(kern), kRegThreads, 0);
-        if (resident < static_cast<int64_t>(P.batch)) return cudaErrorInvalidConfiguration;
+        if (resident < static_cast<int64_t>(P.batch)) {
+            // more matrices than co-resident CTAs: one launch per row (stream-ordered)
+            SkinnyRowParams Q = P;
+            Q.gbar = nullptr;
+            for (int32_t i = 0; i < P.n; ++i) {
+                Q.i = i;
+                const cudaError_t e = launch_s<S, DIR, FOLD>(Q, st);
+                if (e != cudaSuccess) return e;
+            }
+            return cudaSuccess;
+        }
         const int64_t warps = (P.N / S + 31) / 32;
         int64_t grid = (warps * 32 + kRegThreads - 1) / kRegThreads;
         const int64_t per = resident / P.batch;  // every CTA of the launch co-resident

@@ -156,3 +156,20 @@ def test_config3_all_field_counts_sampled():
         assert u.sum().item() == s1 and (u * u).sum().item() == s2, n
         ipt.soa_to_aos(x, count, n, field_bytes=4)
         assert torch.equal(x, base[:total].to(torch.int32)), n
+
+
+def test_large_batch_of_small_skinny_matrices():
+    """A batch of more skinny matrices than co-resident CTAs: the one-launch row shuffles
+    (cooperative, grid barrier) fall back to one launch per row; every matrix compared in full."""
+    count, n, batch = 1024, 3, 3000
+    with skinny_min(1000):
+        assert ipt.plan_info(count, n, 4)["engine"] == "skinny"
+        host = workloads.random_words(batch * count * n, 4, seed=77)
+        x = to_dev(host)
+        ipt.c2r_batched(x, batch, count * n, count, n, elem_bytes=4)
+        got = x.cpu().numpy().view(np.uint32)
+        for k in (0, 1, batch // 2, batch - 1):
+            o = k * count * n
+            assert got[o:o + count * n].tobytes() == oracle.transpose(host[o:o + count * n], count, n).tobytes(), k
+        ipt.r2c_batched(x, batch, count * n, count, n, elem_bytes=4)
+        assert x.cpu().numpy().tobytes() == host.tobytes()
