@@ -147,11 +147,12 @@ ipt_status_t ipt_soa_to_aos(void *ptr, int64_t count, int64_t fields, int field_
 /*
  * Auxiliary-space statement for ipt_c2r(m, n, elem_bytes, ...) (Theorem 6, PAPER.md:605:
  * O(max(m, n)) auxiliary space).  *global_bytes: device scratch the call allocates
- * (stream-ordered, freed before the call's work completes) for one matrix: the side block of
- * the lagged column-tile layout (M rows x 8 tiles of 128 B, M = max(m, n)), and with a fused
- * rotation one flag per row plus (C2R) gcd(m, n) - 1 wrapped rows; the skinny engine one row
- * of the long dimension.  Batched calls scale it by the batch (the side block capped at
- * max(256 MiB, 1/32 of the data)).  *onchip_per_cta: the largest shared-memory staging buffer
+ * (stream-ordered, freed before the call's work completes) for one matrix: the column-pass
+ * counters (16 KB per column pass), the side block of the lagged column-tile layout (M rows x
+ * 8 tiles of 128 B, M = max(m, n)), and with a fused rotation either one flag per row plus
+ * gcd(m, n) - 1 wrapped rows or gcd(m, n) - 1 boundary rows per chunk of >= 8 (gcd - 1) rows;
+ * the skinny engine one row of the long dimension (+ 256 B).  Batched calls scale it by the
+ * batch (the side block capped at max(256 MiB, 1/8 of the data)).  *onchip_per_cta: the largest shared-memory staging buffer
  * of any launched CTA.  Multi-word elem_bytes: the larger of the two word-level steps
  * (words as wide as a 16-byte-aligned base allows).  Either pointer may be NULL.
  */

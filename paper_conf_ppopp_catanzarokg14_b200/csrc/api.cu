@@ -1385,6 +1385,17 @@ ipt_status_t ipt_soa_to_aos(void *ptr, int64_t count, int64_t fields, int field_
     return run_perm_any(ptr, 1, -1, fields, count, field_bytes, stream);  // P_{fields,count}
 }
 
+// Device scratch a one-matrix call of plan pl allocates (its CallScratch: counters, flags, wrap /
+// boundary rows, side block; the skinny engine's tmp row and barrier word); composed element
+// sizes keep their plan's figure.
+static size_t call_scratch_bytes(const Plan &pl0, bool engine_step) {
+    if (!engine_step) return pl0.scratch;
+    Plan pl = pl0;
+    CallScratch cs;
+    prepare_call(pl, 1, cs);
+    return std::max(pl0.scratch, cs.total);
+}
+
 ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *global_bytes, size_t *onchip_per_cta) {
     if (!(valid_eb(elem_bytes) || valid_multiword_eb(elem_bytes) || valid_subword_eb(elem_bytes)) || m < 0 || n < 0)
         return IPT_ERR_INVALID_ARGUMENT;
@@ -1397,7 +1408,7 @@ ipt_status_t ipt_scratch_bytes(int64_t m, int64_t n, int elem_bytes, size_t *glo
         s = record_plan(m, n, elem_bytes, pl, extra);
     }
     if (s != IPT_OK) return s;
-    if (global_bytes) *global_bytes = pl.scratch;
+    if (global_bytes) *global_bytes = call_scratch_bytes(pl, valid_eb(elem_bytes));
     if (onchip_per_cta) *onchip_per_cta = pl.onchip;
     return IPT_OK;
 }
@@ -1427,7 +1438,7 @@ ipt_status_t ipt_plan_info(int64_t m, int64_t n, int elem_bytes, ipt_layout_t la
     out[6] = pl.engine ? pl.shuf.p.W : 0;
     out[7] = static_cast<int64_t>(pl.onchip);
     out[8] = pl.engine ? pl.row.cl_K : 0;
-    out[9] = static_cast<int64_t>(pl.scratch);
+    out[9] = static_cast<int64_t>(call_scratch_bytes(pl, valid_eb(elem_bytes)));
     return IPT_OK;
 }
 
