@@ -272,7 +272,8 @@ bool set_chunks(Plan &pl, int64_t batch) {
         apply(std::max<int64_t>(rp.R, ckmul * (pl.c - 1)));
         return true;
     }
-    const int64_t par_rows = (pl.M * batch + 8 * pl.sms - 1) / (8 * static_cast<int64_t>(pl.sms));
+    const int64_t per_sm = std::max<int64_t>(1, env_int("IPT_ROW_CHUNK_PER_SM", 8));
+    const int64_t par_rows = (pl.M * batch + per_sm * pl.sms - 1) / (per_sm * static_cast<int64_t>(pl.sms));
     if (apply(std::max<int64_t>({static_cast<int64_t>(rp.R), 8 * (pl.c - 1), std::min<int64_t>(ckmul * (pl.c - 1), par_rows)})))
         return true;
     if (pl.chunk_force == 2) {  // c = 5..8 (make_plan): chunks of 8 (c - 1) rows regardless
@@ -551,7 +552,7 @@ struct PlanKeyHash {
 
 std::string tunables_key() {
     std::string s;
-    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_BULK", "IPT_COL_PERSIST", "IPT_COL_SIDECAP", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
+    for (const char *n : {"IPT_FORCE_ENGINE", "IPT_TILE_BYTES", "IPT_COL_SMEM", "IPT_COL_PIPE", "IPT_COL_NBUF", "IPT_COL_THREADS", "IPT_COL_DEBUG", "IPT_COL_LAG", "IPT_COL_LAGD", "IPT_COL_SUPER", "IPT_COL_TMA", "IPT_COL_BULK", "IPT_COL_PERSIST", "IPT_COL_SIDECAP", "IPT_ROW_STAGE", "IPT_ROW_VEC", "IPT_ROW_DB_MAX", "IPT_ROW_PIPE", "IPT_ROW_CHUNK", "IPT_ROW_CHUNK_K", "IPT_ROW_CHUNK_PER_SM", "IPT_FUSE_ROT", "IPT_ENGINE_RULE",
                           "IPT_SKINNY_MIN", "IPT_SKINNY_REG", "IPT_SKINNY_ONE", "IPT_SKINNY_COLBYTES", "IPT_ROW_CLUSTER_MIN", "IPT_ROW_CLUSTER_K",
                           "IPT_ROW_CLUSTER_SYNC", "IPT_ROW_CLUSTER_MODE"}) {
         const char *v = std::getenv(n);
