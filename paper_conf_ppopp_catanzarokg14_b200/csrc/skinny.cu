@@ -174,6 +174,8 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
     int32_t *qinv_s = reinterpret_cast<int32_t *>(smem);  // 32 entries
     T *buf = reinterpret_cast<T *>(smem + 128);            // [n][C]
     __shared__ T *rowp_s[32];                              // output row of each logical row
+    __shared__ const T *segp_s[32];                        // the block's source segment of each row
+    __shared__ bool fast_s[32];                            // ... staged with 16-byte chunks
     const uint32_t sbuf = static_cast<uint32_t>(__cvta_generic_to_shared(buf));
     const int n = P.n, C = P.C;
     const int64_t pitch = P.N;  // in elements
@@ -195,20 +197,54 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
             }
             return A + L * pitch;
         };
-        for (int s = 0; s < n; ++s) {
+        // The block's row segments: source pointer of each row in a shared table (n threads),
+        // then every (row, 16-byte chunk) pair of the fast rows in one flattened loop -- the
+        // per-row pointer / fold / alignment work is done once per row, not once per thread.
+        if (threadIdx.x < n) {
+            const int s = threadIdx.x;
             const T *row0 = row_of(s, j0);
             const bool one_base = !FOLD || row_of(s, j0 + cols - 1) == row0;
             const T *seg = row0 + j0;
-            if (one_base && (reinterpret_cast<uintptr_t>(seg) & 15) == 0 && (cols * EB) % 16 == 0) {
-                // 16-byte chunks (cp.async.cg): 4-byte cp.async runs at ~75 % of this rate
-                const int nch = cols * EB / 16;
+            segp_s[s] = seg;
+            fast_s[s] = one_base && (reinterpret_cast<uintptr_t>(seg) & 15) == 0 && (cols * EB) % 16 == 0;
+        }
+        __syncthreads();
+        const int nch = cols * EB / 16;  // 16-byte chunks (cp.async.cg): 4-byte cp.async runs at ~75 % of this rate
+        if (nch > 2 * static_cast<int>(blockDim.x)) {
+            // long rows (small n): per row, each thread several chunks
+            for (int s = 0; s < n; ++s) {
+                if (!fast_s[s]) continue;
+                const char *seg = reinterpret_cast<const char *>(segp_s[s]);
                 for (int ch = threadIdx.x; ch < nch; ch += blockDim.x)
                     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
-                                 :: "r"(sbuf + s * C * EB + ch * 16), "l"(reinterpret_cast<const char *>(seg) + ch * 16)
+                                 :: "r"(sbuf + s * C * EB + ch * 16), "l"(seg + ch * 16) : "memory");
+            }
+        } else {
+            // short rows (large n): every (row, chunk) pair in one flattened loop
+            int s = 0, ch = threadIdx.x;
+            while (ch >= nch && s < n) {  // (nch < blockDim only for the last, narrow block)
+                ch -= nch;
+                ++s;
+            }
+            for (; s < n;) {
+                if (fast_s[s])
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
+                                 :: "r"(sbuf + s * C * EB + ch * 16), "l"(reinterpret_cast<const char *>(segp_s[s]) + ch * 16)
                                  : "memory");
-            } else {
+                ch += blockDim.x;
+                while (ch >= nch && s < n) {
+                    ch -= nch;
+                    ++s;
+                }
+            }
+        }
+        {
+            for (int s2 = 0; s2 < n; ++s2) {  // rows straddling a fold block or misaligned: per element
+                if (fast_s[s2]) continue;
+                const T *row0 = row_of(s2, j0);
+                const bool one_base = !FOLD || row_of(s2, j0 + cols - 1) == row0;
                 for (int32_t x = threadIdx.x; x < cols; x += blockDim.x)
-                    cp_async_e<EB>(sbuf + (s * C + x) * EB, (one_base ? row0 : row_of(s, j0 + x)) + j0 + x);
+                    cp_async_e<EB>(sbuf + (s2 * C + x) * EB, (one_base ? row0 : row_of(s2, j0 + x)) + j0 + x);
             }
         }
         asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
@@ -240,6 +276,7 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
             else if (MODE == COL_R2C_SHUF) s0 = jm == 0 ? 0 : n - jm;  // u = (0 - jm) mod n
             else s0 = 0;
             const T *col = buf + x;
+#pragma unroll 4
             for (int i = 0; i < n; ++i) {
                 int32_t src;
                 if (MODE == COL_ROT) {
