@@ -276,7 +276,6 @@ __global__ void __launch_bounds__(kSkThreads) skinny_col_kernel(SkinnyColParams 
             else if (MODE == COL_R2C_SHUF) s0 = jm == 0 ? 0 : n - jm;  // u = (0 - jm) mod n
             else s0 = 0;
             const T *col = buf + x;
-#pragma unroll 4
             for (int i = 0; i < n; ++i) {
                 int32_t src;
                 if (MODE == COL_ROT) {
