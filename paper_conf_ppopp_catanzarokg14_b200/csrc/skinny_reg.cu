@@ -59,13 +59,12 @@ __device__ __forceinline__ void skinny_reg_row(const SkinnyRowParams &P) {
     // U chunks per warp and iteration: all their loads are issued before any transposition
     // (memory-level parallelism for small S), U * S <= 32 data registers.
     constexpr int U = S <= 4 ? 8 : S <= 8 ? 4 : S <= 16 ? 2 : 1;
-    __shared__ int32_t s_lb[S], s_h[S];
+    __shared__ int2 s_lbh[S];  // (lb_k, h_k): one 8-byte shared load per run position
     __shared__ uint32_t *s_src[32], *s_dst[32];
     const int lane = threadIdx.x & 31;
     if (threadIdx.x < S) {
         const int64_t p = dpinv_pos(P, threadIdx.x);
-        s_lb[threadIdx.x] = static_cast<int32_t>(p - p % P.b);
-        s_h[threadIdx.x] = static_cast<int32_t>(p % P.b);
+        s_lbh[threadIdx.x] = make_int2(static_cast<int32_t>(p - p % P.b), static_cast<int32_t>(p % P.b));
     }
     const int nblk = FOLD ? P.c : 1;
     if (threadIdx.x < nblk) {
@@ -83,9 +82,10 @@ __device__ __forceinline__ void skinny_reg_row(const SkinnyRowParams &P) {
     const int32_t b = P.b;
     // run k of this row: positions lb_k + (h_k + t) mod b (t < b: one conditional subtract)
     auto run_pos = [&](int k, int32_t t) -> int32_t {
-        int32_t y = s_h[k] + t;
+        const int2 lbh = s_lbh[k];
+        int32_t y = lbh.y + t;
         y -= y >= b ? b : 0;
-        return s_lb[k] + y;
+        return lbh.x + y;
     };
     const int32_t structs = static_cast<int32_t>(P.N / S);  // whole n-element groups of the row
     const int32_t groups = structs / 32;                     // whole warps' worth
@@ -122,7 +122,7 @@ __device__ __forceinline__ void skinny_reg_row(const SkinnyRowParams &P) {
 #pragma unroll
                 for (int k = 0; k < S; ++k) {
                     const int32_t y = run_pos(k, t);
-                    (FOLD ? s_dst[blk(s_lb[k])] : dst0)[y] = r[u][k];
+                    (FOLD ? s_dst[blk(s_lbh[k].x)] : dst0)[y] = r[u][k];
                 }
             }
         } else {
@@ -132,7 +132,7 @@ __device__ __forceinline__ void skinny_reg_row(const SkinnyRowParams &P) {
                 if (g >= groups) break;
                 const int32_t t = g * 32 + lane;
 #pragma unroll
-                for (int k = 0; k < S; ++k) r[u][k] = (FOLD ? s_src[blk(s_lb[k])] : src0)[run_pos(k, t)];
+                for (int k = 0; k < S; ++k) r[u][k] = (FOLD ? s_src[blk(s_lbh[k].x)] : src0)[run_pos(k, t)];
             }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
