@@ -120,7 +120,7 @@ ipt_status_t ipt_r2c_batched(void *base, int64_t batch, int64_t stride_elems, in
  * synchronous); `dev` is caller-owned device memory of at least m*n*elem_bytes bytes.
  * Stream-ordered on `stream`: copy host -> dev, ipt_c2r / ipt_r2c on dev (same semantics
  * and arguments as above), copy dev -> host.  On return nothing has necessarily run yet;
- * synchronise the stream before reading `host`.  Consecutive calls on two streams with two
+ * synchronise the stream before reading `host`.  Consecutive calls on several streams with their own
  * device buffers overlap one call's device->host copy with the next call's host->device
  * copy (the two directions of the host link).  Errors: IPT_ERR_INVALID_ARGUMENT for a null
  * host/dev pointer or the arguments ipt_c2r rejects; other codes as ipt_c2r.  On any error
