@@ -27,7 +27,7 @@ ncu)
   timeout 600 $NCU -k regex:row_chunk -c 1 -s 2 -o $REP/rowchunk_$TAG \
       python tools/one_shape.py --m 17226 --n 6052 --eb 4 --reps 3 > gpurun_out/ncu_rowchunk_$TAG.log 2>&1
   # separate rotation pass at HBM scale (gcd 6600): col_tile_kernel<4,0,128> is COL_ROT
-  timeout 600 $NCU -k regex:col_tile_kernel -c 1 -s 2 -o $REP/colrot_$TAG \
+  timeout 600 $NCU -k regex:col_pipe_kernel -c 1 -s 1 -o $REP/colrot_$TAG \
       python tools/one_shape.py --m 19800 --n 13200 --eb 4 --reps 2 > gpurun_out/ncu_colrot_$TAG.log 2>&1
   # cluster row pass (rows of 240 KB fp64)
   timeout 600 $NCU -k regex:row_cluster -c 1 -s 1 -o $REP/rowcluster_$TAG \
