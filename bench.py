@@ -593,7 +593,9 @@ def run_ours(args, rank, world, local_rank):
     # copy in to last copy out); median of 3 steps after one warm-up step.
     e2e_shapes = [(m, n, eb) for eb in ebs for (m, n) in shapes[:args.e2e_shapes]]
     big = max(m * n * eb for m, n, eb in e2e_shapes)
-    NS = 4  # calls in flight (tools/e2e_streams.py: 1 / 2 / 3 / 4 streams -> 54 / 71 / 81 / 84 GB/s)
+    # calls in flight (tools/e2e_streams.py: 1 / 2 / 3 / 4 streams -> 54 / 71 / 81 / 84 GB/s); 2 per
+    # rank at N > 1, so that the pinned host buffers (NS x the largest matrix) stay modest per node
+    NS = 4 if world == 1 else 2
     hosts = [torch.empty(big, dtype=torch.uint8, pin_memory=True).random_(0, 255) for _ in range(NS)]
     devs = [torch.empty(big, dtype=torch.uint8, device=dev) for _ in range(NS)]
     sts = [stream] + [torch.cuda.Stream(device=dev) for _ in range(NS - 1)]
